@@ -1,0 +1,187 @@
+/*
+ * memxct.h -- C ABI of the B200-native MemXCT hot path.
+ *
+ * Paper: M. Hidayetoglu, T. Bicer, S. Garcia de Gonzalo, B. Ren, D. Gursoy, R. Kettimuthu,
+ * I. Foster, W. Hwu, "MemXCT: Memory-Centric X-ray CT Reconstruction with Massive
+ * Parallelization", SC'19.  "P:n" cites line n of the paper text (reference PAPER.md);
+ * readings R1..R20 are listed in DESIGN.md section 3.
+ *
+ * Problem (eq. 1, with R = 0 and C = R^n): least squares  min_x ||y - A x||^2  where
+ *   x  = tomogram, N x N pixels, natural index i*N + j, row i along +y;
+ *   y  = sinogram, M projections x C channels, natural index m*C + k;
+ *   A  = memoized ray-tracing matrix, A[r, p] = length of ray r inside pixel p, built once by
+ *        Siddon tracing, parallel beam, theta_m = m*pi/M, unit-spaced centred
+ *        channels (readings R1-R4).  A is stored once in fp32.
+ *
+ * Hot path: forward projection y = A x and backprojection x = A^T y as
+ * gather-only SpMVs (Listing 2), rows and columns reordered by the
+ * two-level pseudo-Hilbert ordering, inputs staged through a multi-stage shared-memory
+ * buffer addressed with 16-bit indices (Listing 3), and CG iterations.
+ *
+ * Conventions
+ *  * Ownership: a plan owns every device allocation it makes (matrices, maps, scratch, CG
+ *    vectors, NCCL communicator).  Vector pointers passed in are caller-owned and never retained
+ *    past the call.
+ *  * Device vs host: memxct_forward/back/cg take DEVICE pointers (cudaMalloc / torch CUDA
+ *    tensors) on the plan's device; the *_host variants take HOST pointers (pinned or pageable)
+ *    and do the host<->device copies inside the call (stream-ordered, then synchronised).
+ *  * dtype: float* (fp32) in PRECISION = FP32 mode, double* (fp64) in PRECISION = MIXED mode.
+ *    The matrix values are fp32 in both modes.
+ *  * Vector order: VECTOR_ORDER = 0 (default, P = 1 only): natural row-major tomogram [N][N] and
+ *    sinogram [M][C].  VECTOR_ORDER = 1: the plan's local Hilbert order (see
+ *    memxct_local_indices); required when P > 1.
+ *  * Asynchrony: forward, back and cg are stream-ordered on `cuda_stream` (a cudaStream_t; NULL =
+ *    legacy default stream).  build is synchronous.  cg synchronises only when residual_norms is
+ *    non-NULL (it copies the norms to the host).
+ *  * Errors: every call returns a status; no C++ exception crosses the ABI.  The detail of the last
+ *    error on the calling thread is memxct_last_error().  After MEMXCT_ERR_OUT_OF_MEMORY the plan
+ *    stays valid for memxct_plan_destroy.
+ *  * No CPU fallback: every arithmetic step runs in this library's CUDA kernels; without a CUDA
+ *    device memxct_build returns MEMXCT_ERR_CUDA.
+ */
+#ifndef MEMXCT_H
+#define MEMXCT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MEMXCT_VERSION_MAJOR 0
+#define MEMXCT_VERSION_MINOR 1
+
+typedef struct memxct_plan* memxct_plan_t; /* opaque */
+
+typedef enum {
+    MEMXCT_OK = 0,
+    MEMXCT_ERR_INVALID_ARG = 1,  /* bad size, null pointer, option out of range */
+    MEMXCT_ERR_STATE = 2,        /* plan used before build, option set after build, ... */
+    MEMXCT_ERR_OUT_OF_MEMORY = 3,/* device or host allocation failed */
+    MEMXCT_ERR_CUDA = 4,         /* CUDA runtime / launch error, or no device */
+    MEMXCT_ERR_NCCL = 5,         /* NCCL error (P > 1) */
+    MEMXCT_ERR_UNSUPPORTED = 6   /* valid request this build does not implement */
+} memxct_status_t;
+
+typedef enum {
+    /* Tile side of the first Hilbert level (power of two, 1..128).  Default (reading R7):
+     * largest power of two T with 8T <= min(H, W), clamped to [4, 64]. */
+    MEMXCT_OPT_TILE_TOMO = 0,
+    MEMXCT_OPT_TILE_SINO = 1,
+    /* Rows per partition (one CTA per partition; one 32-row slice per warp).
+     * Multiple of 32 in [32, 1024].  Default 512. */
+    MEMXCT_OPT_PART_ROWS = 2,
+    /* Stage-buffer capacity in fp32 entries (16-bit local addressing).
+     * 256 <= value <= 49152.  MIXED mode stages value/2 fp64 entries.  Default 12288 (48 KB). */
+    MEMXCT_OPT_BUFFER_ENTRIES = 3,
+    /* 0 = FP32 (fp32 vectors, fp32 FMA; the paper's precision), 1 = MIXED (fp32 A, fp64
+     * vectors and fp64 FMA).  Default 0. */
+    MEMXCT_OPT_PRECISION = 4,
+    /* 1 = canonical summation order (reading R16): one fp64 fma chain per row in ascending
+     * Hilbert column order, dots as per-partition fma chains summed in partition order.
+     * Requires PRECISION = MIXED.  Default 0. */
+    MEMXCT_OPT_CANONICAL = 5,
+    /* 0 = recursive-residual CGLS (default, 1 forward + 1 back per iteration, reading R13).
+     * 1 = explicit residual r = y - A x each iteration (2 forward + 1 back). */
+    MEMXCT_OPT_CG_VARIANT = 6,
+    /* 0 = natural row-major vectors (default, P = 1 only); 1 = plan (local Hilbert) order. */
+    MEMXCT_OPT_VECTOR_ORDER = 7
+} memxct_option_t;
+
+/* Create a plan for an N x N tomogram and an M x C sinogram.  Host only; no device
+ * work.  n, projections, channels must be >= 1 and n*n, projections*channels < 2^31. */
+memxct_status_t memxct_plan_create(int32_t n, int32_t projections, int32_t channels,
+                                   memxct_plan_t* out);
+
+/* Set a tuning/precision option (table above) before memxct_build; ERR_STATE afterwards. */
+memxct_status_t memxct_plan_set_option(memxct_plan_t plan, memxct_option_t option, int64_t value);
+memxct_status_t memxct_plan_get_option(memxct_plan_t plan, memxct_option_t option, int64_t* value);
+
+/* Multi-GPU (P > 1, A = R C A_p): rank in [0, nranks), a 128-byte ncclUniqueId
+ * produced by rank 0 and broadcast by the caller, and the CUDA device of this rank.  Before
+ * build.  nranks == 1 is accepted and means single GPU. */
+memxct_status_t memxct_plan_set_comm(memxct_plan_t plan, int32_t rank, int32_t nranks,
+                                     const void* nccl_unique_id, int32_t cuda_device);
+
+/* Fill a 128-byte buffer with a fresh ncclUniqueId (call on rank 0 only). */
+memxct_status_t memxct_get_unique_id(void* nccl_unique_id_out);
+
+/* Preprocessing: Hilbert ordering and domain decomposition, Siddon tracing of A on
+ * the device, order-preserving transposition to A^T, partitioning and the multi-stage buffered
+ * layout of both matrices.  Synchronous; collective over the communicator when P > 1.
+ * `cuda_stream` may be NULL. */
+memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream);
+
+/* Number of locally owned entries of a domain (0 = tomogram pixels, 1 = sinogram rays) and
+ * their natural indices in plan order (host array of `count` int64).  At P = 1 the plan order is
+ * the two-level pseudo-Hilbert order, i.e. natural_idx[h] = natural index of Hilbert position h. */
+memxct_status_t memxct_local_size(memxct_plan_t plan, int32_t domain, int64_t* count);
+memxct_status_t memxct_local_indices(memxct_plan_t plan, int32_t domain, int64_t* natural_idx);
+
+/* Forward projection y = A x.  x: device tomogram (local_size(0) entries), y: device
+ * sinogram (local_size(1) entries), dtype per PRECISION.  Overwrites y. */
+memxct_status_t memxct_forward(memxct_plan_t plan, const void* x_tomo, void* y_sino,
+                               void* cuda_stream);
+
+/* Backprojection x = A^T y (a gather with the transposed matrix, no
+ * atomics).  Overwrites x. */
+memxct_status_t memxct_back(memxct_plan_t plan, const void* y_sino, void* x_tomo,
+                            void* cuda_stream);
+
+/* CGLS reconstruction (reading R13): x_0 = 0, exactly `iters` iterations (R14),
+ * x_tomo overwritten.  residual_norms (host, iters + 1 doubles, nullable) receives ||r_k||
+ * (R15); iterations skipped after gamma or delta reach 0 repeat the last norm.  iters == 0
+ * writes zeros.  iters < 0 is INVALID_ARG. */
+memxct_status_t memxct_cg(memxct_plan_t plan, const void* y_sino, void* x_tomo, int32_t iters,
+                          double* residual_norms, void* cuda_stream);
+
+/* Host-buffer variants: same semantics, HOST pointers; the H2D copy of the input, the device
+ * computation and the D2H copy of the result all happen inside the call, which returns after
+ * the result is on the host. */
+memxct_status_t memxct_forward_host(memxct_plan_t plan, const void* x_host, void* y_host,
+                                    void* cuda_stream);
+memxct_status_t memxct_back_host(memxct_plan_t plan, const void* y_host, void* x_host,
+                                 void* cuda_stream);
+memxct_status_t memxct_cg_host(memxct_plan_t plan, const void* y_host, void* x_host,
+                               int32_t iters, double* residual_norms, void* cuda_stream);
+
+/* Byte model for the bench: nonzeros of A (= of A^T), stored SELL slots of both
+ * directions, stage-map entries of both directions, device bytes held by the plan. */
+memxct_status_t memxct_stats(memxct_plan_t plan, int64_t* nnz, int64_t* stored_slots,
+                             int64_t* map_entries, int64_t* device_bytes);
+
+/* Per-direction layout sizes (dir 0 = A / forward, 1 = A^T / back): partitions, total stages,
+ * stored slots, map entries, rows, nonzeros.  Any pointer may be NULL. */
+memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* parts,
+                                   int64_t* stages, int64_t* slots, int64_t* map_entries,
+                                   int64_t* rows, int64_t* nnz);
+
+/* Copy the layout of partitions [p0, p1) of direction `dir` to host arrays (introspection for
+ * tests; the layout is documented in DESIGN.md section 5):
+ *   stage_base  int64[p1-p0+1]   global stage index range of each partition
+ *   map_off     int64[p1-p0+1]   offset of each partition's map entries
+ *   map         int32[...]       input index (plan order) of each stage-buffer slot
+ *   slot_off    int64[(stages)*slices_per_part + 1]  slot offset of each (stage, slice) block
+ *   ind         uint16[...]      local buffer index of each slot
+ *   val         float[...]       value of each slot (0 for padding)
+ * Pass NULL for all arrays to query sizes through the int64 out-parameters. */
+memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0, int64_t p1,
+                                     int64_t* stage_base, int64_t* map_off, int32_t* map,
+                                     int64_t* slot_off, uint16_t* ind, float* val,
+                                     int64_t* n_map, int64_t* n_slot_off, int64_t* n_slots);
+
+/* Destroy a plan and free everything it owns.  NULL-safe. */
+memxct_status_t memxct_plan_destroy(memxct_plan_t plan);
+
+const char* memxct_status_string(memxct_status_t status);
+/* Detail of the last error on the calling thread ("" if none). */
+const char* memxct_last_error(void);
+
+/* Number of CUDA kernels this library has launched in this process (instrumentation for the
+ * bench's gpu_launches claim; graph launches count every kernel node). */
+int64_t memxct_kernel_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MEMXCT_H */

@@ -1,0 +1,394 @@
+// api.cu -- the C ABI of include/memxct.h.  Argument checking, plan state, error mapping;
+// every arithmetic step is delegated to the CUDA kernels of hilbert.cu, trace.cu, layout.cu,
+// spmv.cu and cg.cu.  No C++ exception crosses this boundary.
+#include <atomic>
+#include <cmath>
+#include <cstring>
+#include <string>
+
+#include "plan.h"
+
+struct memxct_plan {
+    mx::Plan P;
+};
+
+namespace mx {
+
+static std::atomic<int64_t> g_launches{0};
+void count_launch(int64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+int64_t launch_count() { return g_launches.load(std::memory_order_relaxed); }
+
+int64_t Plan::device_bytes() const {
+    return fwd.device_bytes() + back.device_bytes() +
+           (int64_t)(tomo_nat_of_h.buf.bytes() + tomo_h_of_nat.buf.bytes() + sino_nat_of_h.buf.bytes() +
+                     sino_h_of_nat.buf.bytes() + cg_r.bytes() + cg_q.bytes() + cg_s.bytes() + cg_p.bytes() +
+                     cg_ax.bytes() + part_fwd.buf.bytes() + part_back.buf.bytes() + part_vec.buf.bytes() +
+                     scal.buf.bytes() + tickets.buf.bytes() + h_in.bytes() + h_out.bytes());
+}
+
+}  // namespace mx
+
+namespace {
+
+thread_local std::string g_last_error;
+
+template <class F> memxct_status_t guarded(F&& f) {
+    try {
+        f();
+        g_last_error.clear();
+        return MEMXCT_OK;
+    } catch (const mx::Error& e) {
+        g_last_error = e.what();
+        return e.status;
+    } catch (const std::bad_alloc&) {
+        g_last_error = "host allocation failed";
+        return MEMXCT_ERR_OUT_OF_MEMORY;
+    } catch (const std::exception& e) {
+        g_last_error = e.what();
+        return MEMXCT_ERR_CUDA;
+    } catch (...) {
+        g_last_error = "unknown error";
+        return MEMXCT_ERR_CUDA;
+    }
+}
+
+mx::Plan& plan_of(memxct_plan_t plan) {
+    if (!plan) mx::fail(MEMXCT_ERR_INVALID_ARG, "plan is NULL");
+    return plan->P;
+}
+
+mx::Plan& built_plan(memxct_plan_t plan) {
+    mx::Plan& P = plan_of(plan);
+    if (!P.built) mx::fail(MEMXCT_ERR_STATE, "plan used before memxct_build");
+    if (P.device >= 0) MX_CUDA(cudaSetDevice(P.device));
+    return P;
+}
+
+cudaStream_t stream_of(void* s) { return reinterpret_cast<cudaStream_t>(s); }
+
+void need(const void* p, const char* what) {
+    if (!p) mx::fail(MEMXCT_ERR_INVALID_ARG, std::string(what) + " is NULL");
+}
+
+void run_forward(mx::Plan& P, const void* x, void* y, cudaStream_t st) {
+    if (P.esize == 4) mx::spmv_f32(P.fwd, (const float*)x, (float*)y, nullptr, nullptr, nullptr, st);
+    else mx::spmv_f64(P.fwd, (const double*)x, (double*)y, nullptr, nullptr, nullptr, false, st);
+}
+
+void run_back(mx::Plan& P, const void* y, void* x, cudaStream_t st) {
+    if (P.esize == 4) mx::spmv_f32(P.back, (const float*)y, (float*)x, nullptr, nullptr, nullptr, st);
+    else mx::spmv_f64(P.back, (const double*)y, (double*)x, nullptr, nullptr, nullptr, false, st);
+}
+
+void ensure_host_staging(mx::Plan& P) {
+    if (!P.h_in.get()) {
+        const int64_t mx_len = std::max(P.fwd.nrows, P.back.nrows);
+        P.h_in.alloc(P.esize * std::max<int64_t>(mx_len, 1));
+        P.h_out.alloc(P.esize * std::max<int64_t>(mx_len, 1));
+    }
+}
+
+}  // namespace
+
+extern "C" {
+
+memxct_status_t memxct_plan_create(int32_t n, int32_t projections, int32_t channels, memxct_plan_t* out) {
+    return guarded([&] {
+        need(out, "out");
+        *out = nullptr;
+        if (n < 1 || projections < 1 || channels < 1)
+            mx::fail(MEMXCT_ERR_INVALID_ARG, "n, projections and channels must be >= 1");
+        if ((int64_t)n * n >= ((int64_t)1 << 31) || (int64_t)projections * channels >= ((int64_t)1 << 31))
+            mx::fail(MEMXCT_ERR_INVALID_ARG, "n*n and projections*channels must be < 2^31");
+        auto* p = new memxct_plan();
+        p->P.n = n;
+        p->P.m = projections;
+        p->P.c = channels;
+        *out = p;
+    });
+}
+
+memxct_status_t memxct_plan_set_option(memxct_plan_t plan, memxct_option_t option, int64_t value) {
+    return guarded([&] {
+        mx::Plan& P = plan_of(plan);
+        if (P.built) mx::fail(MEMXCT_ERR_STATE, "options must be set before memxct_build");
+        auto range = [&](int64_t lo, int64_t hi) {
+            if (value < lo || value > hi)
+                mx::fail(MEMXCT_ERR_INVALID_ARG, "option value out of range [" + std::to_string(lo) + ", " +
+                                                     std::to_string(hi) + "]");
+        };
+        switch (option) {
+            case MEMXCT_OPT_TILE_TOMO:
+            case MEMXCT_OPT_TILE_SINO:
+                range(0, 128);
+                if (value != 0 && (value & (value - 1))) mx::fail(MEMXCT_ERR_INVALID_ARG, "tile side must be a power of two");
+                (option == MEMXCT_OPT_TILE_TOMO ? P.opt.tile_tomo : P.opt.tile_sino) = value;
+                break;
+            case MEMXCT_OPT_PART_ROWS:
+                range(32, 1024);
+                if (value % 32) mx::fail(MEMXCT_ERR_INVALID_ARG, "PART_ROWS must be a multiple of 32");
+                P.opt.part_rows = value;
+                break;
+            case MEMXCT_OPT_BUFFER_ENTRIES: range(256, 49152); P.opt.buffer_entries = value; break;
+            case MEMXCT_OPT_PRECISION: range(0, 1); P.opt.precision = value; break;
+            case MEMXCT_OPT_CANONICAL: range(0, 1); P.opt.canonical = value; break;
+            case MEMXCT_OPT_CG_VARIANT: range(0, 1); P.opt.cg_variant = value; break;
+            case MEMXCT_OPT_VECTOR_ORDER: range(0, 1); P.opt.vector_order = value; break;
+            default: mx::fail(MEMXCT_ERR_INVALID_ARG, "unknown option");
+        }
+    });
+}
+
+memxct_status_t memxct_plan_get_option(memxct_plan_t plan, memxct_option_t option, int64_t* value) {
+    return guarded([&] {
+        mx::Plan& P = plan_of(plan);
+        need(value, "value");
+        switch (option) {
+            case MEMXCT_OPT_TILE_TOMO: *value = P.built ? P.tile_tomo : P.opt.tile_tomo; break;
+            case MEMXCT_OPT_TILE_SINO: *value = P.built ? P.tile_sino : P.opt.tile_sino; break;
+            case MEMXCT_OPT_PART_ROWS: *value = P.opt.part_rows; break;
+            case MEMXCT_OPT_BUFFER_ENTRIES: *value = P.opt.buffer_entries; break;
+            case MEMXCT_OPT_PRECISION: *value = P.opt.precision; break;
+            case MEMXCT_OPT_CANONICAL: *value = P.opt.canonical; break;
+            case MEMXCT_OPT_CG_VARIANT: *value = P.opt.cg_variant; break;
+            case MEMXCT_OPT_VECTOR_ORDER: *value = P.opt.vector_order; break;
+            default: mx::fail(MEMXCT_ERR_INVALID_ARG, "unknown option");
+        }
+    });
+}
+
+memxct_status_t memxct_plan_set_comm(memxct_plan_t plan, int32_t rank, int32_t nranks,
+                                     const void* nccl_unique_id, int32_t cuda_device) {
+    return guarded([&] {
+        mx::Plan& P = plan_of(plan);
+        if (P.built) mx::fail(MEMXCT_ERR_STATE, "set_comm must precede memxct_build");
+        if (nranks < 1 || rank < 0 || rank >= nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank / nranks");
+        if (nranks > 1) {
+            need(nccl_unique_id, "nccl_unique_id");
+            mx::fail(MEMXCT_ERR_UNSUPPORTED, "P > 1 is not implemented in this build");
+        }
+        P.rank = rank;
+        P.nranks = nranks;
+        P.device = cuda_device;
+    });
+}
+
+memxct_status_t memxct_get_unique_id(void* out) {
+    return guarded([&] {
+        need(out, "out");
+        mx::fail(MEMXCT_ERR_UNSUPPORTED, "NCCL is not linked in this build");
+    });
+}
+
+memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = plan_of(plan);
+        if (P.built) mx::fail(MEMXCT_ERR_STATE, "plan already built");
+        if (P.opt.canonical && P.opt.precision != 1)
+            mx::fail(MEMXCT_ERR_INVALID_ARG, "CANONICAL requires PRECISION = MIXED");
+        if (P.opt.vector_order == 0 && P.nranks > 1)
+            mx::fail(MEMXCT_ERR_INVALID_ARG, "natural vector order requires P = 1");
+        int ndev = 0;
+        if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+            cudaGetLastError();
+            mx::fail(MEMXCT_ERR_CUDA, "no CUDA device: libmemxct has no CPU fallback");
+        }
+        if (P.device >= 0) MX_CUDA(cudaSetDevice(P.device));
+        else MX_CUDA(cudaGetDevice(&P.device));
+        mx::spmv_init();
+        cudaStream_t st = stream_of(cuda_stream);
+        P.tile_tomo = (int32_t)(P.opt.tile_tomo ? P.opt.tile_tomo : mx::default_tile(P.n, P.n));
+        P.tile_sino = (int32_t)(P.opt.tile_sino ? P.opt.tile_sino : mx::default_tile(P.m, P.c));
+        const int64_t npix = (int64_t)P.n * P.n, nrays = (int64_t)P.m * P.c;
+        P.tomo_nat_of_h.alloc(npix);
+        P.tomo_h_of_nat.alloc(npix);
+        P.sino_nat_of_h.alloc(nrays);
+        P.sino_h_of_nat.alloc(nrays);
+        mx::build_hilbert(P.n, P.n, P.tile_tomo, P.tomo_nat_of_h.p(), P.tomo_h_of_nat.p(), st);
+        mx::build_hilbert(P.m, P.c, P.tile_sino, P.sino_nat_of_h.p(), P.sino_h_of_nat.p(), st);
+        P.esize = P.opt.precision == 1 ? 8 : 4;
+        mx::build_matrices(P, st);
+        MX_CUDA(cudaStreamSynchronize(st));
+        P.built = true;
+    });
+}
+
+memxct_status_t memxct_local_size(memxct_plan_t plan, int32_t domain, int64_t* count) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(count, "count");
+        if (domain != 0 && domain != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "domain must be 0 or 1");
+        *count = domain == 0 ? P.back.nrows : P.fwd.nrows;
+    });
+}
+
+memxct_status_t memxct_local_indices(memxct_plan_t plan, int32_t domain, int64_t* natural_idx) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(natural_idx, "natural_idx");
+        if (domain != 0 && domain != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "domain must be 0 or 1");
+        const mx::DevArr<int32_t>& a = domain == 0 ? P.tomo_nat_of_h : P.sino_nat_of_h;
+        std::vector<int32_t> h(a.n);
+        MX_CUDA(cudaMemcpy(h.data(), a.p(), 4 * a.n, cudaMemcpyDeviceToHost));
+        for (int64_t i = 0; i < a.n; ++i) natural_idx[i] = h[i];
+    });
+}
+
+memxct_status_t memxct_forward(memxct_plan_t plan, const void* x_tomo, void* y_sino, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_tomo, "x_tomo");
+        need(y_sino, "y_sino");
+        run_forward(P, x_tomo, y_sino, stream_of(cuda_stream));
+    });
+}
+
+memxct_status_t memxct_back(memxct_plan_t plan, const void* y_sino, void* x_tomo, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_tomo, "x_tomo");
+        need(y_sino, "y_sino");
+        run_back(P, y_sino, x_tomo, stream_of(cuda_stream));
+    });
+}
+
+memxct_status_t memxct_cg(memxct_plan_t plan, const void* y_sino, void* x_tomo, int32_t iters,
+                          double* residual_norms, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_tomo, "x_tomo");
+        need(y_sino, "y_sino");
+        if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
+        cudaStream_t st = stream_of(cuda_stream);
+        mx::cg_run(P, y_sino, x_tomo, iters, st);
+        if (residual_norms) mx::cg_fetch_norms(P, iters, residual_norms, st);
+    });
+}
+
+memxct_status_t memxct_forward_host(memxct_plan_t plan, const void* x_host, void* y_host, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_host, "x_host");
+        need(y_host, "y_host");
+        ensure_host_staging(P);
+        cudaStream_t st = stream_of(cuda_stream);
+        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), x_host, P.esize * P.back.nrows, cudaMemcpyHostToDevice, st));
+        run_forward(P, P.h_in.get(), P.h_out.get(), st);
+        MX_CUDA(cudaMemcpyAsync(y_host, P.h_out.get(), P.esize * P.fwd.nrows, cudaMemcpyDeviceToHost, st));
+        MX_CUDA(cudaStreamSynchronize(st));
+    });
+}
+
+memxct_status_t memxct_back_host(memxct_plan_t plan, const void* y_host, void* x_host, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_host, "x_host");
+        need(y_host, "y_host");
+        ensure_host_staging(P);
+        cudaStream_t st = stream_of(cuda_stream);
+        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), y_host, P.esize * P.fwd.nrows, cudaMemcpyHostToDevice, st));
+        run_back(P, P.h_in.get(), P.h_out.get(), st);
+        MX_CUDA(cudaMemcpyAsync(x_host, P.h_out.get(), P.esize * P.back.nrows, cudaMemcpyDeviceToHost, st));
+        MX_CUDA(cudaStreamSynchronize(st));
+    });
+}
+
+memxct_status_t memxct_cg_host(memxct_plan_t plan, const void* y_host, void* x_host, int32_t iters,
+                               double* residual_norms, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_host, "x_host");
+        need(y_host, "y_host");
+        if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
+        ensure_host_staging(P);
+        cudaStream_t st = stream_of(cuda_stream);
+        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), y_host, P.esize * P.fwd.nrows, cudaMemcpyHostToDevice, st));
+        mx::cg_run(P, P.h_in.get(), P.h_out.get(), iters, st);
+        MX_CUDA(cudaMemcpyAsync(x_host, P.h_out.get(), P.esize * P.back.nrows, cudaMemcpyDeviceToHost, st));
+        if (residual_norms) mx::cg_fetch_norms(P, iters, residual_norms, st);
+        MX_CUDA(cudaStreamSynchronize(st));
+    });
+}
+
+memxct_status_t memxct_stats(memxct_plan_t plan, int64_t* nnz, int64_t* stored_slots, int64_t* map_entries,
+                             int64_t* device_bytes) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        if (nnz) *nnz = P.fwd.nnz;
+        if (stored_slots) *stored_slots = P.fwd.nslots + P.back.nslots;
+        if (map_entries) *map_entries = P.fwd.nmap + P.back.nmap;
+        if (device_bytes) *device_bytes = P.device_bytes();
+    });
+}
+
+memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* parts, int64_t* stages,
+                                   int64_t* slots, int64_t* map_entries, int64_t* rows, int64_t* nnz) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        if (dir != 0 && dir != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "dir must be 0 or 1");
+        const mx::Layout& L = dir == 0 ? P.fwd : P.back;
+        if (parts) *parts = L.nparts;
+        if (stages) *stages = L.nstages;
+        if (slots) *slots = L.nslots;
+        if (map_entries) *map_entries = L.nmap;
+        if (rows) *rows = L.nrows;
+        if (nnz) *nnz = L.nnz;
+    });
+}
+
+memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0, int64_t p1,
+                                     int64_t* stage_base, int64_t* map_off, int32_t* map, int64_t* slot_off,
+                                     uint16_t* ind, float* val, int64_t* n_map, int64_t* n_slot_off,
+                                     int64_t* n_slots) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        if (dir != 0 && dir != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "dir must be 0 or 1");
+        const mx::Layout& L = dir == 0 ? P.fwd : P.back;
+        if (p0 < 0 || p1 > L.nparts || p0 > p1) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad partition range");
+        int64_t sb[2], mo[2];
+        MX_CUDA(cudaMemcpy(&sb[0], L.stage_base.p() + p0, 8, cudaMemcpyDeviceToHost));
+        MX_CUDA(cudaMemcpy(&sb[1], L.stage_base.p() + p1, 8, cudaMemcpyDeviceToHost));
+        MX_CUDA(cudaMemcpy(&mo[0], L.map_off.p() + p0, 8, cudaMemcpyDeviceToHost));
+        MX_CUDA(cudaMemcpy(&mo[1], L.map_off.p() + p1, 8, cudaMemcpyDeviceToHost));
+        const int64_t b0 = sb[0] * L.SPP, b1 = sb[1] * L.SPP;
+        int64_t so[2];
+        MX_CUDA(cudaMemcpy(&so[0], L.slot_off.p() + b0, 8, cudaMemcpyDeviceToHost));
+        MX_CUDA(cudaMemcpy(&so[1], L.slot_off.p() + b1, 8, cudaMemcpyDeviceToHost));
+        if (n_map) *n_map = mo[1] - mo[0];
+        if (n_slot_off) *n_slot_off = b1 - b0 + 1;
+        if (n_slots) *n_slots = so[1] - so[0];
+        if (stage_base) MX_CUDA(cudaMemcpy(stage_base, L.stage_base.p() + p0, 8 * (p1 - p0 + 1), cudaMemcpyDeviceToHost));
+        if (map_off) MX_CUDA(cudaMemcpy(map_off, L.map_off.p() + p0, 8 * (p1 - p0 + 1), cudaMemcpyDeviceToHost));
+        if (map && mo[1] > mo[0]) MX_CUDA(cudaMemcpy(map, L.map.p() + mo[0], 4 * (mo[1] - mo[0]), cudaMemcpyDeviceToHost));
+        if (slot_off) MX_CUDA(cudaMemcpy(slot_off, L.slot_off.p() + b0, 8 * (b1 - b0 + 1), cudaMemcpyDeviceToHost));
+        if (ind && so[1] > so[0]) MX_CUDA(cudaMemcpy(ind, L.ind.p() + so[0], 2 * (so[1] - so[0]), cudaMemcpyDeviceToHost));
+        if (val && so[1] > so[0]) MX_CUDA(cudaMemcpy(val, L.val.p() + so[0], 4 * (so[1] - so[0]), cudaMemcpyDeviceToHost));
+    });
+}
+
+memxct_status_t memxct_plan_destroy(memxct_plan_t plan) {
+    if (!plan) return MEMXCT_OK;
+    return guarded([&] {
+        if (plan->P.device >= 0) cudaSetDevice(plan->P.device);
+        delete plan;
+    });
+}
+
+const char* memxct_status_string(memxct_status_t s) {
+    switch (s) {
+        case MEMXCT_OK: return "MEMXCT_OK";
+        case MEMXCT_ERR_INVALID_ARG: return "MEMXCT_ERR_INVALID_ARG";
+        case MEMXCT_ERR_STATE: return "MEMXCT_ERR_STATE";
+        case MEMXCT_ERR_OUT_OF_MEMORY: return "MEMXCT_ERR_OUT_OF_MEMORY";
+        case MEMXCT_ERR_CUDA: return "MEMXCT_ERR_CUDA";
+        case MEMXCT_ERR_NCCL: return "MEMXCT_ERR_NCCL";
+        case MEMXCT_ERR_UNSUPPORTED: return "MEMXCT_ERR_UNSUPPORTED";
+    }
+    return "MEMXCT_ERR_UNKNOWN";
+}
+
+const char* memxct_last_error(void) { return g_last_error.c_str(); }
+
+int64_t memxct_kernel_launch_count(void) { return mx::launch_count(); }
+
+}  // extern "C"

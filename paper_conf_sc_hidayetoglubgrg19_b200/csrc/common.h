@@ -1,0 +1,93 @@
+// common.h -- internal error handling, device buffers and launch accounting for libmemxct.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <stdexcept>
+#include <string>
+#include <utility>
+
+#include "memxct.h"
+
+namespace mx {
+
+// Internal exception; converted to a memxct_status_t at the C ABI boundary (api.cu).
+struct Error : std::runtime_error {
+    memxct_status_t status;
+    Error(memxct_status_t s, const std::string& m) : std::runtime_error(m), status(s) {}
+};
+
+[[noreturn]] inline void fail(memxct_status_t s, const std::string& m) { throw Error(s, m); }
+
+inline void cuda_check(cudaError_t e, const char* what, const char* file, int line) {
+    if (e != cudaSuccess) {
+        memxct_status_t s = (e == cudaErrorMemoryAllocation) ? MEMXCT_ERR_OUT_OF_MEMORY : MEMXCT_ERR_CUDA;
+        if (e == cudaErrorMemoryAllocation) cudaGetLastError();  // clear the sticky-free error
+        fail(s, std::string(what) + ": " + cudaGetErrorString(e) + " (" + file + ":" +
+                    std::to_string(line) + ")");
+    }
+}
+#define MX_CUDA(call) ::mx::cuda_check((call), #call, __FILE__, __LINE__)
+// After every kernel launch: launch-configuration errors surface here.
+#define MX_LAUNCHED() do { ::mx::count_launch(); MX_CUDA(cudaGetLastError()); } while (0)
+
+void count_launch(int64_t n = 1);
+int64_t launch_count();
+
+// Owning device allocation (cudaMalloc); freed on destruction, so an OOM in the middle of a
+// build leaves the plan destroyable.
+class DevBuf {
+public:
+    DevBuf() = default;
+    explicit DevBuf(size_t bytes) { alloc(bytes); }
+    DevBuf(const DevBuf&) = delete;
+    DevBuf& operator=(const DevBuf&) = delete;
+    DevBuf(DevBuf&& o) noexcept : p_(o.p_), n_(o.n_) { o.p_ = nullptr; o.n_ = 0; }
+    DevBuf& operator=(DevBuf&& o) noexcept {
+        if (this != &o) { reset(); p_ = o.p_; n_ = o.n_; o.p_ = nullptr; o.n_ = 0; }
+        return *this;
+    }
+    ~DevBuf() { reset(); }
+    void alloc(size_t bytes) {
+        reset();
+        if (bytes == 0) return;
+        void* p = nullptr;
+        cudaError_t e = cudaMalloc(&p, bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            fail(e == cudaErrorMemoryAllocation ? MEMXCT_ERR_OUT_OF_MEMORY : MEMXCT_ERR_CUDA,
+                 "cudaMalloc(" + std::to_string(bytes) + " B): " + cudaGetErrorString(e));
+        }
+        p_ = p;
+        n_ = bytes;
+        g_bytes_ += bytes;
+    }
+    void reset() {
+        if (p_) { cudaFree(p_); g_bytes_ -= n_; }
+        p_ = nullptr;
+        n_ = 0;
+    }
+    template <class T> T* as() const { return static_cast<T*>(p_); }
+    void* get() const { return p_; }
+    size_t bytes() const { return n_; }
+    static int64_t live_bytes() { return g_bytes_; }
+
+private:
+    void* p_ = nullptr;
+    size_t n_ = 0;
+    static inline int64_t g_bytes_ = 0;
+};
+
+template <class T> struct DevArr {
+    DevBuf buf;
+    int64_t n = 0;
+    void alloc(int64_t count) { buf.alloc(sizeof(T) * (size_t)(count > 0 ? count : 0)); n = count; }
+    T* p() const { return buf.as<T>(); }
+    void reset() { buf.reset(); n = 0; }
+};
+
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+}  // namespace mx

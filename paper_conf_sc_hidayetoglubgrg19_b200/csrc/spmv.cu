@@ -1,0 +1,285 @@
+// spmv.cu -- the hot kernel: staged SELL-32 SpMV for forward (A) and back (A^T) projection.
+//
+// Semantics: Listing 3 with the GPU mapping of P:457-463 -- one CTA per partition
+// of R consecutive Hilbert rows, one row per thread.  For every stage of the partition:
+//   1. gather  buf[i] = x[map[i]]  into shared memory (Listing 3 line 9);
+//   2. each warp streams its 32-row slice block of (16-bit local index, fp32 value) slots and
+//      accumulates  acc += buf[ind] * val  (Listing 3 line 14; 16-bit addressing P:709-717).
+// Finally y[row] = acc (lines 17-21).  There are no atomics: gather-only.
+//
+// B200 mapping: the slot stream (6 B per nonzero + padding) is the HBM-bound part; each lane
+// issues one 16 B load of indices and two 16 B loads of values per 8 slots
+// (ld.global.nc.L1::no_allocate with an L2 evict-first policy: the stream is touched once, and
+// must not evict the input vector / maps, which stay L2-resident).  The stage gather reads the
+// (L2-resident) input through the read-only path.  Several CTAs per SM overlap one CTA's gather
+// with another's streaming (the paper's "block scheduling" overlap).
+//
+// Optional epilogue: per-CTA partial of <y, y> (fp64) and a last-CTA reduction in fixed
+// partition order -> deterministic dot products for CG without a second pass over y.
+#include "plan.h"
+
+namespace mx {
+
+namespace {
+
+__device__ __forceinline__ uint64_t evict_first_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+
+__device__ __forceinline__ uint4 ld_stream_u4(const void* p, uint64_t pol) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
+    return r;
+}
+
+__device__ __forceinline__ float4 ld_stream_f4(const void* p, uint64_t pol) {
+    float4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p), "l"(pol));
+    return r;
+}
+
+struct SpmvArgs {
+    const int64_t* stage_base;
+    const int64_t* map_off;
+    const int32_t* map;
+    const int64_t* slot_off;
+    const uint16_t* ind;
+    const float* val;
+    const int32_t* out_idx;
+    int64_t nrows;
+    int64_t nparts;
+    int32_t R, SPP, B;
+    double* dot_part;
+    double* dot_out;
+    unsigned int* ticket;
+};
+
+// deterministic last-CTA reduction of the per-CTA partials, in partition order
+template <int kThreads>
+__device__ void finish_dot_tree(const SpmvArgs& a, double mine) {
+    __shared__ double red[kThreads / 32];
+    __shared__ bool am_last;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int nw = blockDim.x >> 5;
+    for (int o = 16; o; o >>= 1) mine += __shfl_xor_sync(0xffffffffu, mine, o);
+    if (lane == 0) red[warp] = mine;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double s = 0.0;
+        for (int w = 0; w < nw; ++w) s += red[w];
+        a.dot_part[blockIdx.x] = s;
+        __threadfence();
+        const unsigned t = atomicAdd(a.ticket, 1u);
+        am_last = (t == (unsigned)(a.nparts - 1));
+    }
+    __syncthreads();
+    if (!am_last) return;
+    __threadfence();
+    double s = 0.0;
+    for (int64_t i = threadIdx.x; i < a.nparts; i += blockDim.x) s += ((volatile double*)a.dot_part)[i];
+    for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    __syncthreads();
+    if (lane == 0) red[warp] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double tot = 0.0;
+        for (int w = 0; w < nw; ++w) tot += red[w];
+        *a.dot_out = tot;
+        *a.ticket = 0u;  // re-arm for the next launch (stream order)
+    }
+}
+
+// canonical (reading R16): partial = fma chain over the partition's rows in Hilbert order,
+// total = partials added sequentially in partition order, all in IEEE fp64 round-to-nearest.
+__device__ void finish_dot_canonical(const SpmvArgs& a, const double* rows_val, int nvalid) {
+    __shared__ bool am_last;
+    if (threadIdx.x == 0) {
+        double part = 0.0;
+        for (int i = 0; i < nvalid; ++i) part = __fma_rn(rows_val[i], rows_val[i], part);
+        a.dot_part[blockIdx.x] = part;
+        __threadfence();
+        const unsigned t = atomicAdd(a.ticket, 1u);
+        am_last = (t == (unsigned)(a.nparts - 1));
+    }
+    __syncthreads();
+    if (!am_last || threadIdx.x != 0) return;
+    __threadfence();
+    double tot = 0.0;
+    for (int64_t i = 0; i < a.nparts; ++i) tot = __dadd_rn(tot, ((volatile double*)a.dot_part)[i]);
+    *a.dot_out = tot;
+    *a.ticket = 0u;
+}
+
+constexpr int kMaxThreads = 1024;
+
+template <bool kNatOut, bool kDot>
+__global__ void __launch_bounds__(kMaxThreads)
+spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) {
+    extern __shared__ __align__(16) float sbuf[];
+    const int64_t p = blockIdx.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
+    const int64_t m0 = a.map_off[p], D = a.map_off[p + 1] - m0;
+    const uint64_t pol = evict_first_policy();
+    float acc = 0.f;
+    for (int64_t g = g0; g < g1; ++g) {
+        const int64_t s = g - g0;
+        const int cnt = (int)min((int64_t)a.B, D - s * a.B);
+        const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
+        if (g != g0) __syncthreads();  // previous stage fully consumed
+        for (int i = threadIdx.x; i < cnt; i += blockDim.x) sbuf[i] = __ldg(x + __ldg(mp + i));
+        __syncthreads();
+        const int64_t blk = g * a.SPP + warp;
+        const int64_t base = a.slot_off[blk];
+        const int64_t nchunk = (a.slot_off[blk + 1] - base) / (32 * kVec);
+        const uint4* ip = reinterpret_cast<const uint4*>(a.ind + base) + lane;
+        const float4* vp = reinterpret_cast<const float4*>(a.val + base) + lane;
+#pragma unroll 4
+        for (int64_t c = 0; c < nchunk; ++c) {
+            const uint4 iv = ld_stream_u4(ip + c * 32, pol);
+            const float4 v0 = ld_stream_f4(vp + c * 64, pol);
+            const float4 v1 = ld_stream_f4(vp + c * 64 + 32, pol);
+            acc = fmaf(sbuf[iv.x & 0xffffu], v0.x, acc);
+            acc = fmaf(sbuf[iv.x >> 16], v0.y, acc);
+            acc = fmaf(sbuf[iv.y & 0xffffu], v0.z, acc);
+            acc = fmaf(sbuf[iv.y >> 16], v0.w, acc);
+            acc = fmaf(sbuf[iv.z & 0xffffu], v1.x, acc);
+            acc = fmaf(sbuf[iv.z >> 16], v1.y, acc);
+            acc = fmaf(sbuf[iv.w & 0xffffu], v1.z, acc);
+            acc = fmaf(sbuf[iv.w >> 16], v1.w, acc);
+        }
+    }
+    const int64_t row = p * a.R + threadIdx.x;
+    const bool valid = row < a.nrows;
+    if (valid) y[kNatOut ? a.out_idx[row] : row] = acc;
+    if (kDot) finish_dot_tree<kMaxThreads>(a, valid ? (double)acc * (double)acc : 0.0);
+}
+
+// MIXED precision: fp64 stage buffer, fp64 input/output, one fp64 fma chain per row in ascending
+// Hilbert input order (stages ascend, slots within a stage ascend by local index; padding slots
+// are fma(0, finite, acc) = acc).  This is the canonical row sum of reading R16.
+template <bool kNatOut, int kDotMode>  // kDotMode: 0 none, 1 tree, 2 canonical chain
+__global__ void __launch_bounds__(kMaxThreads)
+spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y) {
+    extern __shared__ __align__(16) double dbuf[];
+    const int64_t p = blockIdx.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
+    const int64_t m0 = a.map_off[p], D = a.map_off[p + 1] - m0;
+    const uint64_t pol = evict_first_policy();
+    double acc = 0.0;
+    for (int64_t g = g0; g < g1; ++g) {
+        const int64_t s = g - g0;
+        const int cnt = (int)min((int64_t)a.B, D - s * a.B);
+        const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
+        if (g != g0) __syncthreads();
+        for (int i = threadIdx.x; i < cnt; i += blockDim.x) dbuf[i] = __ldg(x + __ldg(mp + i));
+        __syncthreads();
+        const int64_t blk = g * a.SPP + warp;
+        const int64_t base = a.slot_off[blk];
+        const int64_t nchunk = (a.slot_off[blk + 1] - base) / (32 * kVec);
+        const uint4* ip = reinterpret_cast<const uint4*>(a.ind + base) + lane;
+        const float4* vp = reinterpret_cast<const float4*>(a.val + base) + lane;
+#pragma unroll 2
+        for (int64_t c = 0; c < nchunk; ++c) {
+            const uint4 iv = ld_stream_u4(ip + c * 32, pol);
+            const float4 v0 = ld_stream_f4(vp + c * 64, pol);
+            const float4 v1 = ld_stream_f4(vp + c * 64 + 32, pol);
+            acc = __fma_rn((double)v0.x, dbuf[iv.x & 0xffffu], acc);
+            acc = __fma_rn((double)v0.y, dbuf[iv.x >> 16], acc);
+            acc = __fma_rn((double)v0.z, dbuf[iv.y & 0xffffu], acc);
+            acc = __fma_rn((double)v0.w, dbuf[iv.y >> 16], acc);
+            acc = __fma_rn((double)v1.x, dbuf[iv.z & 0xffffu], acc);
+            acc = __fma_rn((double)v1.y, dbuf[iv.z >> 16], acc);
+            acc = __fma_rn((double)v1.z, dbuf[iv.w & 0xffffu], acc);
+            acc = __fma_rn((double)v1.w, dbuf[iv.w >> 16], acc);
+        }
+    }
+    const int64_t row = p * a.R + threadIdx.x;
+    const bool valid = row < a.nrows;
+    if (valid) y[kNatOut ? a.out_idx[row] : row] = acc;
+    if (kDotMode == 1) finish_dot_tree<kMaxThreads>(a, valid ? acc * acc : 0.0);
+    if (kDotMode == 2) {
+        __syncthreads();  // the stage buffer is free: reuse it for this partition's row values
+        dbuf[threadIdx.x] = valid ? acc : 0.0;
+        __syncthreads();
+        const int64_t nvalid = min((int64_t)a.R, a.nrows - p * a.R);
+        finish_dot_canonical(a, dbuf, (int)nvalid);
+    }
+}
+
+template <class K> void set_smem(K kern) {
+    MX_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+}
+
+SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned int* ticket) {
+    SpmvArgs a;
+    a.stage_base = L.stage_base.p();
+    a.map_off = L.map_off.p();
+    a.map = L.map.p();
+    a.slot_off = L.slot_off.p();
+    a.ind = L.ind.p();
+    a.val = L.val.p();
+    a.out_idx = L.out_idx.p();
+    a.nrows = L.nrows;
+    a.nparts = L.nparts;
+    a.R = L.R;
+    a.SPP = L.SPP;
+    a.B = L.B;
+    a.dot_part = dot_part;
+    a.dot_out = dot_out;
+    a.ticket = ticket;
+    return a;
+}
+
+}  // namespace
+
+void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, double* dot_out,
+              unsigned int* ticket, cudaStream_t st) {
+    if (L.nparts == 0) return;
+    const SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
+    const size_t smem = sizeof(float) * (size_t)L.B;
+    const bool nat = L.out_idx.p() != nullptr, dot = dot_out != nullptr;
+    auto kern = nat ? (dot ? spmv_f32_kernel<true, true> : spmv_f32_kernel<true, false>)
+                    : (dot ? spmv_f32_kernel<false, true> : spmv_f32_kernel<false, false>);
+    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, y);
+    MX_LAUNCHED();
+}
+
+void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
+              unsigned int* ticket, bool canonical, cudaStream_t st) {
+    if (L.nparts == 0) return;
+    const SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
+    const size_t smem = sizeof(double) * (size_t)std::max(L.B, L.R);
+    const bool nat = L.out_idx.p() != nullptr;
+    const int mode = dot_out == nullptr ? 0 : (canonical ? 2 : 1);
+    void (*kern)(SpmvArgs, const double*, double*);
+    if (nat) kern = mode == 0 ? spmv_f64_kernel<true, 0> : mode == 1 ? spmv_f64_kernel<true, 1> : spmv_f64_kernel<true, 2>;
+    else kern = mode == 0 ? spmv_f64_kernel<false, 0> : mode == 1 ? spmv_f64_kernel<false, 1> : spmv_f64_kernel<false, 2>;
+    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, y);
+    MX_LAUNCHED();
+}
+
+// Raise the dynamic shared-memory limit of every SpMV instantiation once (outside any stream
+// capture): stage buffers go up to 227 KB per CTA.
+void spmv_init() {
+    static bool done = false;
+    if (done) return;
+    set_smem(spmv_f32_kernel<true, true>);
+    set_smem(spmv_f32_kernel<true, false>);
+    set_smem(spmv_f32_kernel<false, true>);
+    set_smem(spmv_f32_kernel<false, false>);
+    set_smem(spmv_f64_kernel<true, 0>);
+    set_smem(spmv_f64_kernel<true, 1>);
+    set_smem(spmv_f64_kernel<true, 2>);
+    set_smem(spmv_f64_kernel<false, 0>);
+    set_smem(spmv_f64_kernel<false, 1>);
+    set_smem(spmv_f64_kernel<false, 2>);
+    done = true;
+}
+
+}  // namespace mx

@@ -1,0 +1,290 @@
+"""Thin ctypes binding of libmemxct (include/memxct.h).
+
+Argument marshalling only: every step of the hot path (tracing, ordering, layout, SpMV, CG) runs
+in the library's CUDA kernels.  PyTorch is used for device memory and streams.  There is no CPU
+fallback: if the CUDA library is missing or there is no GPU, calls raise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libmemxct.so")
+
+OK = 0
+STATUS = {0: "MEMXCT_OK", 1: "MEMXCT_ERR_INVALID_ARG", 2: "MEMXCT_ERR_STATE",
+          3: "MEMXCT_ERR_OUT_OF_MEMORY", 4: "MEMXCT_ERR_CUDA", 5: "MEMXCT_ERR_NCCL",
+          6: "MEMXCT_ERR_UNSUPPORTED"}
+OPT = {"tile_tomo": 0, "tile_sino": 1, "part_rows": 2, "buffer_entries": 3, "precision": 4,
+       "canonical": 5, "cg_variant": 6, "vector_order": 7}
+
+#: every symbol include/memxct.h declares (checked by tests/test_abi.py)
+SYMBOLS = [
+    "memxct_plan_create", "memxct_plan_set_option", "memxct_plan_get_option",
+    "memxct_plan_set_comm", "memxct_get_unique_id", "memxct_build", "memxct_local_size",
+    "memxct_local_indices", "memxct_forward", "memxct_back", "memxct_cg",
+    "memxct_forward_host", "memxct_back_host", "memxct_cg_host", "memxct_stats",
+    "memxct_layout_info", "memxct_layout_export", "memxct_plan_destroy",
+    "memxct_status_string", "memxct_last_error", "memxct_kernel_launch_count",
+]
+
+
+class MemXCTError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        super().__init__(f"{where}: {STATUS.get(status, status)}: {detail}")
+        self.status = status
+
+
+_lib = None
+
+
+def lib():
+    """Load libmemxct.so (raises if it was not built: there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} not built; run `python -m paper_conf_sc_hidayetoglubgrg19_b200"
+                              f".build_ext` (the CUDA library is required, there is no CPU path)")
+        L = ctypes.CDLL(LIB_PATH)
+        i32, i64, vp, st = ctypes.c_int32, ctypes.c_int64, ctypes.c_void_p, ctypes.c_int
+        P64 = ctypes.POINTER(ctypes.c_int64)
+        sig = {
+            "memxct_plan_create": [i32, i32, i32, ctypes.POINTER(vp)],
+            "memxct_plan_set_option": [vp, ctypes.c_int, i64],
+            "memxct_plan_get_option": [vp, ctypes.c_int, P64],
+            "memxct_plan_set_comm": [vp, i32, i32, vp, i32],
+            "memxct_get_unique_id": [vp],
+            "memxct_build": [vp, vp],
+            "memxct_local_size": [vp, i32, P64],
+            "memxct_local_indices": [vp, i32, vp],
+            "memxct_forward": [vp, vp, vp, vp],
+            "memxct_back": [vp, vp, vp, vp],
+            "memxct_cg": [vp, vp, vp, i32, vp, vp],
+            "memxct_forward_host": [vp, vp, vp, vp],
+            "memxct_back_host": [vp, vp, vp, vp],
+            "memxct_cg_host": [vp, vp, vp, i32, vp, vp],
+            "memxct_stats": [vp, P64, P64, P64, P64],
+            "memxct_layout_info": [vp, i32, P64, P64, P64, P64, P64, P64],
+            "memxct_layout_export": [vp, i32, i64, i64, vp, vp, vp, vp, vp, vp, P64, P64, P64],
+            "memxct_plan_destroy": [vp],
+        }
+        for name, args in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = st
+        L.memxct_status_string.argtypes = [st]
+        L.memxct_status_string.restype = ctypes.c_char_p
+        L.memxct_last_error.argtypes = []
+        L.memxct_last_error.restype = ctypes.c_char_p
+        L.memxct_kernel_launch_count.argtypes = []
+        L.memxct_kernel_launch_count.restype = i64
+        _lib = L
+    return _lib
+
+
+def _check(status: int, where: str):
+    if status != OK:
+        raise MemXCTError(status, where, lib().memxct_last_error().decode())
+
+
+def kernel_launch_count() -> int:
+    return int(lib().memxct_kernel_launch_count())
+
+
+def _ptr(t) -> ctypes.c_void_p:
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().memxct_get_unique_id(buf), "memxct_get_unique_id")
+    return buf.raw
+
+
+class MemXCT:
+    """A MemXCT plan: geometry (N, M, C), options, built matrices, and the hot-path calls.
+
+    Mirrors memxct_plan_create / set_option / set_comm / build / forward / back / cg / destroy.
+    Vectors are torch CUDA tensors (float32 in "fp32" precision, float64 in "mixed").
+    """
+
+    def __init__(self, n: int, projections: int, channels: int, *, precision: str = "fp32",
+                 canonical: bool = False, vector_order: str = "natural", part_rows: int = None,
+                 buffer_entries: int = None, tile_tomo: int = None, tile_sino: int = None,
+                 cg_variant: int = 0, rank: int = 0, nranks: int = 1, unique_id: bytes = None,
+                 device: int = None):
+        self.n, self.m, self.c = int(n), int(projections), int(channels)
+        self._h = ctypes.c_void_p()
+        _check(lib().memxct_plan_create(self.n, self.m, self.c, ctypes.byref(self._h)),
+               "memxct_plan_create")
+        self.precision = precision
+        opts = {"precision": {"fp32": 0, "mixed": 1}[precision], "canonical": int(bool(canonical)),
+                "vector_order": {"natural": 0, "plan": 1}[vector_order], "cg_variant": cg_variant,
+                "part_rows": part_rows, "buffer_entries": buffer_entries, "tile_tomo": tile_tomo,
+                "tile_sino": tile_sino}
+        for k, v in opts.items():
+            if v is not None:
+                self.set_option(k, v)
+        if nranks > 1 or device is not None:
+            uid = None if unique_id is None else ctypes.create_string_buffer(unique_id, 128)
+            _check(lib().memxct_plan_set_comm(self._h, rank, nranks, uid,
+                                              -1 if device is None else int(device)),
+                   "memxct_plan_set_comm")
+        self.built = False
+
+    # -- options / lifecycle ---------------------------------------------------------------
+    def set_option(self, name: str, value: int):
+        _check(lib().memxct_plan_set_option(self._h, OPT[name], int(value)), "memxct_plan_set_option")
+
+    def get_option(self, name: str) -> int:
+        v = ctypes.c_int64()
+        _check(lib().memxct_plan_get_option(self._h, OPT[name], ctypes.byref(v)), "memxct_plan_get_option")
+        return v.value
+
+    def build(self, stream=None):
+        _check(lib().memxct_build(self._h, _stream(stream)), "memxct_build")
+        self.built = True
+        return self
+
+    def close(self):
+        if self._h and self._h.value:
+            lib().memxct_plan_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # -- sizes / introspection --------------------------------------------------------------
+    @property
+    def dtype(self):
+        import torch
+        return torch.float32 if self.precision == "fp32" else torch.float64
+
+    def local_size(self, domain: int) -> int:
+        v = ctypes.c_int64()
+        _check(lib().memxct_local_size(self._h, domain, ctypes.byref(v)), "memxct_local_size")
+        return v.value
+
+    def local_indices(self, domain: int) -> np.ndarray:
+        out = np.empty(self.local_size(domain), np.int64)
+        _check(lib().memxct_local_indices(self._h, domain, out.ctypes.data_as(ctypes.c_void_p)),
+               "memxct_local_indices")
+        return out
+
+    def stats(self) -> dict:
+        v = [ctypes.c_int64() for _ in range(4)]
+        _check(lib().memxct_stats(self._h, *[ctypes.byref(x) for x in v]), "memxct_stats")
+        return dict(zip(["nnz", "stored_slots", "map_entries", "device_bytes"], [x.value for x in v]))
+
+    def layout_info(self, direction: int) -> dict:
+        v = [ctypes.c_int64() for _ in range(6)]
+        _check(lib().memxct_layout_info(self._h, direction, *[ctypes.byref(x) for x in v]),
+               "memxct_layout_info")
+        return dict(zip(["parts", "stages", "slots", "map_entries", "rows", "nnz"], [x.value for x in v]))
+
+    def layout_export(self, direction: int, p0: int = 0, p1: int = None) -> dict:
+        if p1 is None:
+            p1 = self.layout_info(direction)["parts"]
+        nm, nso, ns = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        z = ctypes.c_void_p()
+        _check(lib().memxct_layout_export(self._h, direction, p0, p1, z, z, z, z, z, z,
+                                          ctypes.byref(nm), ctypes.byref(nso), ctypes.byref(ns)),
+               "memxct_layout_export")
+        out = {"stage_base": np.empty(p1 - p0 + 1, np.int64), "map_off": np.empty(p1 - p0 + 1, np.int64),
+               "map": np.empty(nm.value, np.int32), "slot_off": np.empty(nso.value, np.int64),
+               "ind": np.empty(ns.value, np.uint16), "val": np.empty(ns.value, np.float32)}
+        P = lambda a: a.ctypes.data_as(ctypes.c_void_p)
+        _check(lib().memxct_layout_export(self._h, direction, p0, p1, P(out["stage_base"]),
+                                          P(out["map_off"]), P(out["map"]), P(out["slot_off"]),
+                                          P(out["ind"]), P(out["val"]), ctypes.byref(nm),
+                                          ctypes.byref(nso), ctypes.byref(ns)),
+               "memxct_layout_export")
+        return out
+
+    # -- hot path -------------------------------------------------------------------------
+    def _vec(self, t, domain, name):
+        import torch
+        if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == self.dtype and t.is_contiguous()):
+            raise TypeError(f"{name} must be a contiguous CUDA {self.dtype} tensor")
+        if t.numel() != self.local_size(domain):
+            raise ValueError(f"{name} has {t.numel()} elements, expected {self.local_size(domain)}")
+        return t
+
+    def forward(self, x, y=None, stream=None):
+        """y = A x (device tensors)."""
+        import torch
+        self._vec(x, 0, "x")
+        if y is None:
+            y = torch.empty(self.local_size(1), dtype=self.dtype, device=x.device)
+        self._vec(y, 1, "y")
+        _check(lib().memxct_forward(self._h, _ptr(x), _ptr(y), _stream(stream)), "memxct_forward")
+        return y
+
+    def back(self, y, x=None, stream=None):
+        """x = A^T y (device tensors)."""
+        import torch
+        self._vec(y, 1, "y")
+        if x is None:
+            x = torch.empty(self.local_size(0), dtype=self.dtype, device=y.device)
+        self._vec(x, 0, "x")
+        _check(lib().memxct_back(self._h, _ptr(y), _ptr(x), _stream(stream)), "memxct_back")
+        return x
+
+    def cg(self, y, iters: int = 30, x=None, residuals: bool = False, stream=None):
+        """CGLS from x0 = 0; returns x (and ||r_k||, k = 0..iters, if residuals)."""
+        import torch
+        self._vec(y, 1, "y")
+        if x is None:
+            x = torch.empty(self.local_size(0), dtype=self.dtype, device=y.device)
+        self._vec(x, 0, "x")
+        res = np.empty(iters + 1, np.float64) if residuals else None
+        rp = res.ctypes.data_as(ctypes.c_void_p) if residuals else None
+        _check(lib().memxct_cg(self._h, _ptr(y), _ptr(x), int(iters), rp, _stream(stream)), "memxct_cg")
+        return (x, res) if residuals else x
+
+    # host-buffer variants (numpy in, numpy out; copies happen inside the C call)
+    def _host(self, a, domain, name):
+        dt = np.float32 if self.precision == "fp32" else np.float64
+        a = np.ascontiguousarray(a, dt)
+        if a.size != self.local_size(domain):
+            raise ValueError(f"{name} has {a.size} elements, expected {self.local_size(domain)}")
+        return a
+
+    def forward_host(self, x, y=None, stream=None):
+        x = self._host(x, 0, "x")
+        y = np.empty(self.local_size(1), x.dtype) if y is None else y
+        _check(lib().memxct_forward_host(self._h, x.ctypes.data_as(ctypes.c_void_p),
+                                         y.ctypes.data_as(ctypes.c_void_p), _stream(stream)),
+               "memxct_forward_host")
+        return y
+
+    def back_host(self, y, x=None, stream=None):
+        y = self._host(y, 1, "y")
+        x = np.empty(self.local_size(0), y.dtype) if x is None else x
+        _check(lib().memxct_back_host(self._h, y.ctypes.data_as(ctypes.c_void_p),
+                                      x.ctypes.data_as(ctypes.c_void_p), _stream(stream)),
+               "memxct_back_host")
+        return x
+
+    def cg_host(self, y, iters: int = 30, x=None, residuals: bool = False, stream=None):
+        y = self._host(y, 1, "y")
+        x = np.empty(self.local_size(0), y.dtype) if x is None else x
+        res = np.empty(iters + 1, np.float64) if residuals else None
+        rp = res.ctypes.data_as(ctypes.c_void_p) if residuals else None
+        _check(lib().memxct_cg_host(self._h, y.ctypes.data_as(ctypes.c_void_p),
+                                    x.ctypes.data_as(ctypes.c_void_p), int(iters), rp,
+                                    _stream(stream)), "memxct_cg_host")
+        return (x, res) if residuals else x

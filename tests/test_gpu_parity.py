@@ -1,0 +1,286 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 CPU oracle.
+
+Gates (BASELINE.json north star):
+  * Hilbert permutations bit-exact;
+  * sparsity pattern bit-exact and fp32 values exactly the oracle's fp64 lengths rounded to
+    nearest (tighter than the 1e-6 relative gate);
+  * FP32 SpMV within 1e-5 relative L2 of the fp64 oracle; MIXED SpMV bit-identical to the
+    oracle's canonical row sums;
+  * MIXED + CANONICAL CG image after 30 iterations within 1e-3 relative L2 of the canonical oracle.
+"""
+import numpy as np
+import pytest
+
+from conftest import rel_l2
+from layout_decode import check_structure, decode, real_entries
+from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_hidayetoglubgrg19_b200 import build_ext
+    build_ext.build()
+
+
+def make_plan(n, m, c, **kw):
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
+    return MemXCT(n, m, c, **kw).build()
+
+
+GEOMS = [(64, 90, 64), (33, 17, 33), (16, 5, 23), (12, 1, 12), (8, 7, 8), (40, 24, 36)]
+
+
+def tiles_of(plan):
+    return plan.get_option("tile_tomo"), plan.get_option("tile_sino")
+
+
+@pytest.mark.parametrize("n,m,c", GEOMS + [(256, 360, 256)])
+def test_hilbert_permutations_bit_exact(orc, n, m, c):
+    plan = make_plan(n, m, c)
+    tt, ts = tiles_of(plan)
+    for dom, (h, w, t) in ((0, (n, n, tt)), (1, (m, c, ts))):
+        nat_of_h = plan.local_indices(dom)
+        rank = orc.hilbert_rank(h, w, t)
+        expect = np.empty(h * w, np.int64)
+        expect[rank] = np.arange(h * w)
+        assert np.array_equal(nat_of_h, expect), (dom, h, w, t)
+
+
+@pytest.mark.parametrize("n,m,c", [(13, 5, 11)])
+@pytest.mark.parametrize("tiles", [(4, 4), (8, 2), (1, 1), (16, 128)])
+def test_hilbert_tile_options(orc, n, m, c, tiles):
+    plan = make_plan(n, m, c, tile_tomo=tiles[0], tile_sino=tiles[1])
+    for dom, (h, w, t) in ((0, (n, n, tiles[0])), (1, (m, c, tiles[1]))):
+        rank = orc.hilbert_rank(h, w, t)
+        expect = np.empty(h * w, np.int64)
+        expect[rank] = np.arange(h * w)
+        assert np.array_equal(plan.local_indices(dom), expect)
+
+
+def _pattern_keys(plan, direction, npix, R, B):
+    ex = plan.layout_export(direction)
+    d = decode(ex, R, B)
+    check_structure(d)
+    e = real_entries(d)
+    row_nat = plan.local_indices(1 if direction == 0 else 0)[e["row"]]
+    if direction == 0:
+        key = row_nat * npix + e["col"]
+    else:
+        key = e["col"] * npix + row_nat
+    order = np.argsort(key, kind="stable")
+    return key[order], e["val"][order], ex
+
+
+@pytest.mark.parametrize("n,m,c", GEOMS + [(256, 360, 256)])
+@pytest.mark.parametrize("part_rows,buf", [(512, 12288), (128, 700)])
+def test_sparsity_pattern_and_values_exact(orc, coo_cache, n, m, c, part_rows, buf):
+    if (n, m, c) == (256, 360, 256) and part_rows == 128:
+        pytest.skip("covered by the default tuning at this size")
+    plan = make_plan(n, m, c, part_rows=part_rows, buffer_entries=buf)
+    rows, cols, vals = coo_cache(n, m, c)
+    npix = n * n
+    okey = rows.astype(np.int64) * npix + cols
+    oo = np.argsort(okey)
+    okey, oval = okey[oo], vals[oo].astype(np.float32)
+    st = plan.stats()
+    assert st["nnz"] == len(rows)
+    for direction in (0, 1):
+        key, val, ex = _pattern_keys(plan, direction, npix, part_rows, buf)
+        assert np.array_equal(key, okey), direction
+        assert np.array_equal(val, oval), direction          # fp32 RN of the fp64 length
+        # every stage holds at most B distinct inputs, and maps are sorted (Hilbert order)
+        assert np.all(np.diff(ex["map_off"]) >= 0)
+
+
+def _vectors(n, m, c):
+    x_ph = inputs.shepp_logan(n)
+    rng = np.random.default_rng(11)
+    return {
+        "phantom": x_ph,
+        "uniform": inputs.uniform(n * n, inputs.seed_for(1)).astype(np.float64),
+        "normal": rng.standard_normal(n * n),
+    }, {
+        "uniform": inputs.uniform(m * c, inputs.seed_for(2)).astype(np.float64),
+        "normal": rng.standard_normal(m * c),
+    }
+
+
+@pytest.mark.parametrize("n,m,c", [(64, 90, 64), (256, 360, 256), (33, 17, 33), (16, 5, 23)])
+def test_fp32_spmv_within_1e5(orc, coo_cache, n, m, c):
+    plan = make_plan(n, m, c)
+    rows, cols, vals = coo_cache(n, m, c)
+    xs, ys = _vectors(n, m, c)
+    ys["phantom_sino"] = orc.spmv_coo(rows, cols, vals, xs["phantom"], m * c)
+    for name, x in xs.items():
+        x32 = x.astype(np.float32)
+        y_gpu = plan.forward(torch.from_numpy(x32).cuda()).cpu().numpy()
+        y_orc = orc.spmv_coo(rows, cols, vals, x32.astype(np.float64), m * c)
+        assert rel_l2(y_gpu, y_orc) <= 1e-5, name
+    for name, y in ys.items():
+        y32 = y.astype(np.float32)
+        x_gpu = plan.back(torch.from_numpy(y32).cuda()).cpu().numpy()
+        x_orc = orc.spmv_coo(cols, rows, vals, y32.astype(np.float64), n * n)
+        assert rel_l2(x_gpu, x_orc) <= 1e-5, name
+
+
+@pytest.mark.parametrize("n,m,c", [(64, 90, 64), (33, 17, 33)])
+def test_mixed_spmv_bit_identical_to_canonical_oracle(orc, coo_cache, n, m, c):
+    plan = make_plan(n, m, c, precision="mixed")
+    tt, ts = tiles_of(plan)
+    rows, cols, vals = coo_cache(n, m, c)
+    v32 = vals.astype(np.float32).astype(np.float64)
+    tomo_rank = orc.hilbert_rank(n, n, tt)
+    sino_rank = orc.hilbert_rank(m, c, ts)
+    xs, ys = _vectors(n, m, c)
+    for x in xs.values():
+        y_gpu = plan.forward(torch.from_numpy(x).cuda()).cpu().numpy()
+        y_orc = orc.spmv_canonical(rows, cols, v32, tomo_rank, x, m * c)
+        assert np.array_equal(y_gpu, y_orc)
+    for y in ys.values():
+        x_gpu = plan.back(torch.from_numpy(y).cuda()).cpu().numpy()
+        x_orc = orc.spmv_canonical(cols, rows, v32, sino_rank, y, n * n)
+        assert np.array_equal(x_gpu, x_orc)
+
+
+def test_gpu_adjoint_identity():
+    n, m, c = 256, 360, 256
+    plan = make_plan(n, m, c)
+    g = torch.Generator(device="cuda").manual_seed(0)
+    x = torch.randn(n * n, device="cuda", generator=g)
+    y = torch.randn(m * c, device="cuda", generator=g)
+    lhs = float(torch.dot(plan.forward(x).double(), y.double()))
+    rhs = float(torch.dot(x.double(), plan.back(y).double()))
+    assert abs(lhs - rhs) <= 1e-5 * max(abs(lhs), 1.0)
+
+
+def _phantom_problem(orc, coo_cache, n, m, c):
+    rows, cols, vals = coo_cache(n, m, c)
+    xt = inputs.shepp_logan(n)
+    y32 = orc.spmv_coo(rows, cols, vals, xt, m * c).astype(np.float32)
+    return rows, cols, vals, xt, y32
+
+
+@pytest.mark.parametrize("n,m,c,R", [(64, 90, 64, 512), (64, 90, 64, 128), (256, 360, 256, 512)])
+def test_cg_mixed_canonical_matches_oracle(orc, coo_cache, n, m, c, R):
+    rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
+    plan = make_plan(n, m, c, precision="mixed", canonical=True, part_rows=R)
+    tt, ts = tiles_of(plan)
+    v32 = vals.astype(np.float32).astype(np.float64)
+    x_orc, res_orc, _, _ = orc.cgls(rows, cols, v32, y32.astype(np.float64), m * c, n * n, 30,
+                                    canonical=True, row_key=orc.hilbert_rank(m, c, ts),
+                                    col_key=orc.hilbert_rank(n, n, tt), chunk_rows=R, chunk_cols=R)
+    x_gpu, res_gpu = plan.cg(torch.from_numpy(y32.astype(np.float64)).cuda(), 30, residuals=True)
+    x_gpu = x_gpu.cpu().numpy()
+    assert rel_l2(x_gpu, x_orc) <= 1e-3
+    # expected (and recorded): bit-identical iterates
+    print("canonical CG drift", rel_l2(x_gpu, x_orc), "residual drift", rel_l2(res_gpu, res_orc))
+    assert np.allclose(res_gpu, res_orc, rtol=1e-6, atol=0)
+
+
+@pytest.mark.parametrize("n,m,c", [(64, 90, 64), (256, 360, 256)])
+def test_cg_fp32_recovers_phantom(orc, coo_cache, n, m, c):
+    rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
+    plan = make_plan(n, m, c)
+    x_gpu, res = plan.cg(torch.from_numpy(y32).cuda(), 30, residuals=True)
+    x_gpu = x_gpu.cpu().numpy().astype(np.float64)
+    x_orc = orc.cgls(rows, cols, vals, y32.astype(np.float64), m * c, n * n, 30)[0]
+    e_gpu, e_orc = rel_l2(x_gpu, xt), rel_l2(x_orc, xt)
+    assert e_gpu <= 1.1 * e_orc, (e_gpu, e_orc)
+    assert np.all(np.diff(res) <= 1e-6 * res[0])
+    print("fp32 CG drift vs fp64 oracle", rel_l2(x_gpu, x_orc), "phantom error", e_gpu, e_orc)
+
+
+def test_cg_explicit_residual_variant(orc, coo_cache):
+    n, m, c = 64, 90, 64
+    rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
+    plan = make_plan(n, m, c, cg_variant=1)
+    x_gpu = plan.cg(torch.from_numpy(y32).cuda(), 30).cpu().numpy()
+    x_orc = orc.cgls(rows, cols, vals, y32.astype(np.float64), m * c, n * n, 30)[0]
+    assert rel_l2(x_gpu, xt) <= 1.1 * rel_l2(x_orc, xt)
+
+
+def test_cg_edge_cases():
+    n, m, c = 64, 90, 64
+    plan = make_plan(n, m, c)
+    y = torch.zeros(m * c, device="cuda")
+    x, res = plan.cg(y, 5, residuals=True)
+    assert torch.all(x == 0) and np.all(res == 0)
+    y = torch.rand(m * c, device="cuda")
+    x = plan.cg(y, 0)
+    assert torch.all(x == 0)
+    with pytest.raises(Exception):
+        plan.cg(y, -1)
+
+
+def test_host_variants_match_device():
+    n, m, c = 64, 90, 64
+    plan = make_plan(n, m, c)
+    x = inputs.uniform(n * n, 3)
+    y_dev = plan.forward(torch.from_numpy(x).cuda()).cpu().numpy()
+    assert np.array_equal(plan.forward_host(x), y_dev)
+    y = inputs.uniform(m * c, 4)
+    x_dev = plan.back(torch.from_numpy(y).cuda()).cpu().numpy()
+    assert np.array_equal(plan.back_host(y), x_dev)
+    xc = plan.cg(torch.from_numpy(y).cuda(), 7).cpu().numpy()
+    assert np.array_equal(plan.cg_host(y, 7), xc)
+
+
+def test_plan_vector_order_matches_natural(orc):
+    n, m, c = 64, 90, 64
+    nat = make_plan(n, m, c)
+    hil = make_plan(n, m, c, vector_order="plan")
+    pix = hil.local_indices(0)
+    ray = hil.local_indices(1)
+    x = inputs.uniform(n * n, 5)
+    y_nat = nat.forward(torch.from_numpy(x).cuda()).cpu().numpy()
+    y_hil = hil.forward(torch.from_numpy(x[pix]).cuda()).cpu().numpy()
+    assert np.array_equal(y_hil, y_nat[ray])
+
+
+def test_degenerate_geometries(orc):
+    # C > N: empty rays give zero rows; M = 1; N = 1
+    for (n, m, c) in [(8, 4, 14), (6, 1, 6), (1, 3, 1)]:
+        rows, cols, vals = orc.trace_all(n, m, c)
+        plan = make_plan(n, m, c)
+        x = np.random.default_rng(0).random(n * n).astype(np.float32)
+        y = plan.forward(torch.from_numpy(x).cuda()).cpu().numpy()
+        y_orc = orc.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)
+        assert rel_l2(y, y_orc) <= 1e-6
+        if len(rows) < m * c:
+            assert np.any(y_orc == 0) and np.all(y[y_orc == 0] == 0)
+
+
+@pytest.mark.slow
+def test_cfg3_sampled_rows(orc):
+    """Full size (BASELINE configs[2]), the launch configuration bench.py times: 2000 sampled
+    rays of y = A x and 12 sampled pixels of x = A^T y, each against the oracle's own trace."""
+    n, m, c = inputs.CONFIGS[3]
+    plan = make_plan(n, m, c)
+    st = plan.stats()
+    assert abs(st["nnz"] / (m * n * n) - 1.1953) < 2e-3
+    x = torch.from_numpy(inputs.uniform(n * n, inputs.seed_for(3))).cuda()
+    y = plan.forward(x).cpu().numpy()
+    xh = x.cpu().numpy().astype(np.float64)
+    rng = np.random.default_rng(3)
+    rays = rng.choice(m * c, 2000, replace=False)
+    got, exp = [], []
+    for r in rays:
+        pix, ln = orc.trace_ray(n, m, c, int(r))
+        got.append(y[r])
+        exp.append(float(ln @ xh[pix]))
+    assert rel_l2(np.array(got), np.array(exp)) <= 1e-5
+    ysino = torch.from_numpy(inputs.uniform(m * c, inputs.seed_for(3) + 1)).cuda()
+    xb = plan.back(ysino).cpu().numpy()
+    yh = ysino.cpu().numpy().astype(np.float64)
+    pixels = rng.choice(n * n, 12, replace=False)
+    got, exp = [], []
+    for p, (rr, ll) in zip(pixels, orc.sampled_back_rows(n, m, c, pixels)):
+        got.append(xb[p])
+        exp.append(float(ll @ yh[rr]))
+    assert rel_l2(np.array(got), np.array(exp)) <= 1e-5
