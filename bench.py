@@ -1,0 +1,376 @@
+#!/usr/bin/env python
+"""MemXCT hot-path benchmark (BASELINE.json metric: CG iter/s and SpMV GFLOP/s + HBM GB/s).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 3] [--iters 30]
+    python bench.py --impl reference ...        # the fp64 CPU oracle, timed on host cores
+
+One STEP = one CGLS reconstruction (`--iters` iterations, default 30 = the paper's count,
+P:957) of one synthetic slice: the whole hot path of SURVEY 8(a) a7-a10 (forward SpMV + back
+SpMV + fused vector steps per iteration, plus the setup backprojection), launched as one CUDA
+graph through the C ABI (memxct_cg).  The matrices are built once (memxct_build, preprocessing
+a1-a6) before timing, as in the paper.
+
+value = CG iterations per second over the whole job; inputs resident in HBM.  The 11.8 GB
+matrix stream per SpMV (cfg 3) is ~90x the L2, so no flush is needed between steps.
+e2e = the same metric through memxct_cg_host (pinned host sinogram in, host tomogram out).
+roofline = the SpMV kernel (both directions), algorithmic bytes per launch
+over its CUDA-event duration, against MEASURED_PEAKS.json's HBM copy bandwidth.
+
+N > 1 (torchrun): each rank reconstructs its own slice (independent problems, weak scaling);
+the max over ranks of the device time is taken.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback, used only if MEASURED_PEAKS.json is absent
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", type=int, default=3)
+    ap.add_argument("--iters", type=int, default=30)
+    ap.add_argument("--part-rows", type=int, default=None)
+    ap.add_argument("--buffer", type=int, default=None)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--spmv-reps", type=int, default=20)
+    return ap.parse_args()
+
+
+def workload_name(cfg, iters):
+    from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
+    n, m, c = inputs.CONFIGS[cfg]
+    return (f"cfg{cfg}: {n}x{n} tomogram, {m} projections x {c} channels, modified Shepp-Logan "
+            f"sinogram, {iters}-iteration CGLS per step")
+
+
+def peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        with open(path) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+# ------------------------------------------------------------------------------------------
+# clocks sampler (B200_PROFILING.md "clocks line")
+# ------------------------------------------------------------------------------------------
+class Clocks:
+    FIELDS = ["clocks.sm", "clocks.max.sm", "power.draw", "clocks_event_reasons.hw_slowdown",
+              "clocks_event_reasons.hw_thermal_slowdown", "clocks_event_reasons.sw_thermal_slowdown",
+              "clocks_event_reasons.sw_power_cap"]
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + ",".join(self.FIELDS),
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": float(max(mx)) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------------------
+# the oracle (CPU baseline / reference arm): bounded sample of the same workload
+# ------------------------------------------------------------------------------------------
+def oracle_sample(cfg, frac=0.02, seed=0):
+    """Trace a random `frac` of the config's rays with the oracle (untimed); returns the COO."""
+    import oracle
+    from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
+    n, m, c = inputs.CONFIGS[cfg]
+    rng = np.random.default_rng(seed)
+    rays = np.sort(rng.choice(m * c, max(1, int(frac * m * c)), replace=False))
+    rows, cols, vals = [], [], []
+    for i, r in enumerate(rays):
+        pix, ln = oracle.trace_ray(n, m, c, int(r))
+        rows.append(np.full(len(pix), i, np.int32))
+        cols.append(pix)
+        vals.append(ln)
+    return (np.concatenate(rows), np.concatenate(cols), np.concatenate(vals), len(rays), n * n)
+
+
+def oracle_step(sample, nnz_full):
+    """One oracle 'step' on the sample: forward + back SpMV (orc_spmv_coo).  Returns the
+    extrapolated CG iterations per second (1 forward + 1 back per iteration, nnz-proportional)."""
+    import oracle
+    rows, cols, vals, nr, nc = sample
+    x = np.ones(nc)
+    y = np.ones(nr)
+    t0 = time.perf_counter()
+    oracle.spmv_coo(rows, cols, vals, x, nr)
+    oracle.spmv_coo(cols, rows, vals, y, nc)
+    dt = time.perf_counter() - t0
+    t_full = dt * nnz_full / len(rows)
+    return 1.0 / t_full, dt
+
+
+def nnz_model(cfg):
+    from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
+    n, m, c = inputs.CONFIGS[cfg]
+    return int(round(1.1953 * m * n * n))
+
+
+def cpu_baseline(cfg, nnz_full, steps=3):
+    t0 = time.perf_counter()
+    sample = oracle_sample(cfg)
+    t_trace = time.perf_counter() - t0
+    vals = [oracle_step(sample, nnz_full)[0] for _ in range(steps)]
+    return {"value": float(np.median(vals)), "unit": "CG iter/s", "cores": 1, "kind": "oracle",
+            "sample": (f"oracle Siddon-traced {sample[3]} random rays (2%) of cfg{cfg} "
+                       f"({len(sample[0])} nonzeros, {t_trace:.1f} s untimed); timed orc_spmv_coo "
+                       f"forward + back on them (single thread), median of {steps}; CG iter/s "
+                       f"extrapolated by nnz_full/nnz_sample = {nnz_full / len(sample[0]):.1f}")}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    from paper_conf_sc_hidayetoglubgrg19_b200 import inputs  # noqa: F401
+    cfg = args.config
+    nnz_full = nnz_model(cfg)
+    sample = oracle_sample(cfg)
+    for _ in range(args.warmup):
+        oracle_step(sample, nnz_full)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle_step(sample, nnz_full)
+    dt = time.perf_counter() - t0
+    # each step processes nnz_sample of the 2*nnz_full work of one CG iteration
+    value = args.steps * len(sample[0]) / nnz_full / dt
+    line = {
+        "impl": "reference", "metric": "CG iter/s", "value": value, "unit": "CG iter/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": workload_name(cfg, args.iters) + " (oracle: 2% ray sample, "
+                   "forward + back SpMV per step, extrapolated to full nnz)"},
+        "cpu_baseline": {"value": value, "unit": "CG iter/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{sample[3]} random rays of cfg{cfg}, {len(sample[0])} nonzeros"},
+        "e2e": {"value": value, "unit": "CG iter/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------------------------
+# our arm
+# ------------------------------------------------------------------------------------------
+def spmv_bytes(info):
+    """Algorithmic bytes of one SpMV: 6 B per nonzero (uint16
+    local index + fp32 value), 8 B per stage-map entry (int32 map + fp32 gather),
+    4 B per output row written.  Padding slots are not counted."""
+    return 6 * info["nnz"] + 8 * info["map_entries"] + 4 * info["rows"]
+
+
+def run_ours(args, rank, world):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, inputs, kernel_launch_count
+
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    cfg = args.config
+    n, m, c = inputs.CONFIGS[cfg]
+    kw = {}
+    if args.part_rows:
+        kw["part_rows"] = args.part_rows
+    if args.buffer:
+        kw["buffer_entries"] = args.buffer
+    t0 = time.perf_counter()
+    plan = MemXCT(n, m, c, **kw).build()
+    torch.cuda.synchronize()
+    build_s = time.perf_counter() - t0
+    st = plan.stats()
+    fi, bi = plan.layout_info(0), plan.layout_info(1)
+
+    # synthetic slice: phantom sinogram from our own forward projection (values do not change
+    # the access pattern; the parity tests pin the values against the oracle)
+    x_ph = torch.from_numpy(inputs.shepp_logan(n).astype(np.float32)).to(dev)
+    y = plan.forward(x_ph)
+    x = torch.empty(n * n, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+
+    for _ in range(args.warmup):
+        plan.cg(y, args.iters, x=x, stream=stream)
+    torch.cuda.synchronize()
+
+    clocks = Clocks(local)
+    clocks.start()
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    k0 = kernel_launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for _ in range(args.steps):
+        plan.cg(y, args.iters, x=x, stream=stream)
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    launches = kernel_launch_count() - k0
+    ms = ev0.elapsed_time(ev1)
+
+    # SpMV kernels alone, each launch bracketed by events on the launching stream
+    fwd_ms, back_ms = [], []
+    yb = torch.empty_like(y)
+    xb = torch.empty_like(x)
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(2 * args.spmv_reps + 1)]
+    evs[0].record(stream)
+    for i in range(args.spmv_reps):
+        plan.forward(x, yb, stream=stream)
+        evs[2 * i + 1].record(stream)
+        plan.back(y, xb, stream=stream)
+        evs[2 * i + 2].record(stream)
+    torch.cuda.synchronize()
+    for i in range(args.spmv_reps):
+        fwd_ms.append(evs[2 * i].elapsed_time(evs[2 * i + 1]))
+        back_ms.append(evs[2 * i + 1].elapsed_time(evs[2 * i + 2]))
+    clk = clocks.stop()
+
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+
+    # e2e through the C ABI with host buffers (pinned sinogram in, tomogram out)
+    y_host = torch.empty(m * c, dtype=torch.float32, pin_memory=True)
+    y_host.copy_(y.cpu())
+    x_host = torch.empty(n * n, dtype=torch.float32, pin_memory=True)
+    plan.cg_host_ptr(y_host.data_ptr(), x_host.data_ptr(), args.iters, stream=stream)  # warm
+    if world > 1:
+        dist.barrier()
+    te0 = time.perf_counter()
+    for _ in range(args.steps):
+        plan.cg_host_ptr(y_host.data_ptr(), x_host.data_ptr(), args.iters, stream=stream)
+    te = time.perf_counter() - te0
+    te_t = torch.tensor([te], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te_t, op=dist.ReduceOp.MAX)
+    te = float(te_t.item())
+
+    if rank != 0:
+        return
+    hbm_peak, peak_src = peaks()
+    fb, bb = spmv_bytes(fi), spmv_bytes(bi)
+    tf, tb = float(np.median(fwd_ms)) * 1e-3, float(np.median(back_ms)) * 1e-3
+    achieved = (fb + bb) / (tf + tb) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", f"ncu_spmv_cfg{cfg}.json")
+    if os.path.exists(prof):
+        with open(prof) as f:
+            traffic = json.load(f).get("traffic_bytes_per_launch")
+    iters_total = args.iters * args.steps * world
+    value = iters_total / (ms_max * 1e-3)
+    line = {
+        "metric": "CG iter/s", "value": value, "unit": "CG iter/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic",
+        "config": {"workload": workload_name(cfg, args.iters),
+                   "l2": "no flush: the matrix stream per SpMV (%.1f GB) exceeds the 126 MB L2" %
+                         ((st["stored_slots"] * 3) / 2 / 1e9),
+                   "part_rows": plan.get_option("part_rows"),
+                   "buffer_entries": plan.get_option("buffer_entries"),
+                   "parallelism": "one slice per GPU" if world > 1 else "single GPU"},
+        "spmv": {"fwd_ms": tf * 1e3, "back_ms": tb * 1e3,
+                 "fwd_gflops": 2 * fi["nnz"] / tf / 1e9, "back_gflops": 2 * bi["nnz"] / tb / 1e9,
+                 "fwd_gbs": fb / tf / 1e9, "back_gbs": bb / tb / 1e9,
+                 "nnz": st["nnz"], "stored_slots_per_dir": [fi["slots"], bi["slots"]],
+                 "padding": [fi["slots"] / fi["nnz"] - 1, bi["slots"] / bi["nnz"] - 1],
+                 "map_entries": [fi["map_entries"], bi["map_entries"]],
+                 "stored_bytes_per_dir": [6 * fi["slots"] + 4 * fi["map_entries"],
+                                          6 * bi["slots"] + 4 * bi["map_entries"]]},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                     "frac": achieved / hbm_peak, "traffic": traffic, "peak_source": peak_src,
+                     "kernel": "spmv_f32_kernel (forward A + back A^T, per launch)",
+                     "algorithmic_bytes_per_launch": [fb, bb]},
+        "clocks": clk,
+        "e2e": {"value": iters_total / te, "unit": "CG iter/s",
+                "h2d_bytes_per_step": 4 * m * c, "d2h_bytes_per_step": 4 * n * n},
+        "gpu_launches": launches,
+        "build_s": build_s,
+        "device_bytes": st["device_bytes"],
+    }
+    if not args.no_cpu_baseline and world >= 1:
+        line["cpu_baseline"] = cpu_baseline(cfg, st["nnz"])
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        if args.impl == "ours":
+            import torch
+            torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", 0)))
+            dist.init_process_group("nccl")
+        else:
+            dist.init_process_group("gloo")
+    try:
+        if args.impl == "reference":
+            run_reference(args, rank, world)
+        else:
+            run_ours(args, rank, world)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

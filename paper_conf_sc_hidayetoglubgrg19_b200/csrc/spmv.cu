@@ -213,7 +213,13 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
 }
 
 template <class K> void set_smem(K kern) {
-    MX_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024));
+    int dev = 0, optin = 0;
+    MX_CUDA(cudaGetDevice(&dev));
+    MX_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    cudaFuncAttributes fa;
+    MX_CUDA(cudaFuncGetAttributes(&fa, kern));
+    MX_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 optin - (int)fa.sharedSizeBytes));
 }
 
 SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned int* ticket) {

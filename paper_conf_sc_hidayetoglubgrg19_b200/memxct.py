@@ -279,6 +279,11 @@ class MemXCT:
                "memxct_back_host")
         return x
 
+    def cg_host_ptr(self, y_ptr: int, x_ptr: int, iters: int = 30, stream=None):
+        """memxct_cg_host on raw host addresses (e.g. pinned torch CPU tensors' data_ptr())."""
+        _check(lib().memxct_cg_host(self._h, ctypes.c_void_p(y_ptr), ctypes.c_void_p(x_ptr),
+                                    int(iters), None, _stream(stream)), "memxct_cg_host")
+
     def cg_host(self, y, iters: int = 30, x=None, residuals: bool = False, stream=None):
         y = self._host(y, 1, "y")
         x = np.empty(self.local_size(0), y.dtype) if x is None else x
