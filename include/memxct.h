@@ -69,10 +69,12 @@ typedef enum {
     MEMXCT_OPT_TILE_TOMO = 0,
     MEMXCT_OPT_TILE_SINO = 1,
     /* Rows per partition (one CTA per partition; one 32-row slice per warp).
-     * Multiple of 32 in [32, 1024].  Default 512. */
+     * Multiple of 32 in [32, 1024], or 0 = auto (default): the largest of 1024/512/256/128 that
+     * leaves >= 2 partitions per SM in the smaller direction (1024 at configs 3-5). */
     MEMXCT_OPT_PART_ROWS = 2,
     /* Stage-buffer capacity in fp32 entries (16-bit local addressing).
-     * 256 <= value <= 49152.  MIXED mode stages value/2 fp64 entries.  Default 12288 (48 KB). */
+     * 256 <= value <= 57344 (224 KB), or 0 = auto (default): 36 * PART_ROWS.  MIXED mode stages
+     * value/2 fp64 entries in the same bytes. */
     MEMXCT_OPT_BUFFER_ENTRIES = 3,
     /* 0 = FP32 (fp32 vectors, fp32 FMA; the paper's precision), 1 = MIXED (fp32 A, fp64
      * vectors and fp64 FMA).  Default 0. */
@@ -164,11 +166,13 @@ memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* par
  *   slot_off    int64[(stages)*slices_per_part + 1]  slot offset of each (stage, slice) block
  *   ind         uint16[...]      local buffer index of each slot
  *   val         float[...]       value of each slot (0 for padding)
+ *   lane_chunks uint16[(n_slot_off-1)*32]  8-slot chunks of each lane of each block
  * Pass NULL for all arrays to query sizes through the int64 out-parameters. */
 memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0, int64_t p1,
                                      int64_t* stage_base, int64_t* map_off, int32_t* map,
                                      int64_t* slot_off, uint16_t* ind, float* val,
-                                     int64_t* n_map, int64_t* n_slot_off, int64_t* n_slots);
+                                     uint16_t* lane_chunks, int64_t* n_map, int64_t* n_slot_off,
+                                     int64_t* n_slots);
 
 /* Destroy a plan and free everything it owns.  NULL-safe. */
 memxct_status_t memxct_plan_destroy(memxct_plan_t plan);

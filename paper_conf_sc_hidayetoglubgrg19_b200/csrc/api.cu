@@ -3,6 +3,7 @@
 // spmv.cu and cg.cu.  No C++ exception crosses this boundary.
 #include <atomic>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -80,6 +81,28 @@ void run_back(mx::Plan& P, const void* y, void* x, cudaStream_t st) {
     else mx::spmv_f64(P.back, (const double*)y, (double*)x, nullptr, nullptr, nullptr, false, st);
 }
 
+// Default tuning (measured B200 sweep, profiles/r01_sweep.md): the largest partition (CTA) size
+// in {1024, 512, 256, 128} rows that still gives >= 2 CTAs per SM in the smaller direction, and
+// a stage buffer of 36 fp32 entries per row (144 KB at R = 1024): ~147 KB of shared memory per SM
+// at the register-limited residency of 1024/R CTAs per SM.
+void resolve_tuning(mx::Plan& P) {
+    int dev = 0, sms = 148;
+    MX_CUDA(cudaGetDevice(&dev));
+    MX_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int64_t rows = std::min<int64_t>((int64_t)P.n * P.n, (int64_t)P.m * P.c);
+    int32_t R = (int32_t)P.opt.part_rows;
+    if (R == 0) {
+        R = 128;
+        for (int32_t cand : {1024, 512, 256}) {
+            if (mx::ceil_div(rows, cand) >= 2 * (int64_t)sms) { R = cand; break; }
+        }
+    }
+    int32_t B = (int32_t)P.opt.buffer_entries;
+    if (B == 0) B = std::min<int32_t>(57344, 36 * R);
+    P.part_rows = R;
+    P.buffer_entries = B;
+}
+
 void ensure_host_staging(mx::Plan& P) {
     if (!P.h_in.get()) {
         const int64_t mx_len = std::max(P.fwd.nrows, P.back.nrows);
@@ -125,11 +148,14 @@ memxct_status_t memxct_plan_set_option(memxct_plan_t plan, memxct_option_t optio
                 (option == MEMXCT_OPT_TILE_TOMO ? P.opt.tile_tomo : P.opt.tile_sino) = value;
                 break;
             case MEMXCT_OPT_PART_ROWS:
-                range(32, 1024);
-                if (value % 32) mx::fail(MEMXCT_ERR_INVALID_ARG, "PART_ROWS must be a multiple of 32");
+                range(0, 1024);
+                if (value % 32) mx::fail(MEMXCT_ERR_INVALID_ARG, "PART_ROWS must be 0 (auto) or a multiple of 32");
                 P.opt.part_rows = value;
                 break;
-            case MEMXCT_OPT_BUFFER_ENTRIES: range(256, 49152); P.opt.buffer_entries = value; break;
+            case MEMXCT_OPT_BUFFER_ENTRIES:
+                if (value != 0) range(256, 57344);
+                P.opt.buffer_entries = value;
+                break;
             case MEMXCT_OPT_PRECISION: range(0, 1); P.opt.precision = value; break;
             case MEMXCT_OPT_CANONICAL: range(0, 1); P.opt.canonical = value; break;
             case MEMXCT_OPT_CG_VARIANT: range(0, 1); P.opt.cg_variant = value; break;
@@ -146,8 +172,8 @@ memxct_status_t memxct_plan_get_option(memxct_plan_t plan, memxct_option_t optio
         switch (option) {
             case MEMXCT_OPT_TILE_TOMO: *value = P.built ? P.tile_tomo : P.opt.tile_tomo; break;
             case MEMXCT_OPT_TILE_SINO: *value = P.built ? P.tile_sino : P.opt.tile_sino; break;
-            case MEMXCT_OPT_PART_ROWS: *value = P.opt.part_rows; break;
-            case MEMXCT_OPT_BUFFER_ENTRIES: *value = P.opt.buffer_entries; break;
+            case MEMXCT_OPT_PART_ROWS: *value = P.built ? P.part_rows : P.opt.part_rows; break;
+            case MEMXCT_OPT_BUFFER_ENTRIES: *value = P.built ? P.buffer_entries : P.opt.buffer_entries; break;
             case MEMXCT_OPT_PRECISION: *value = P.opt.precision; break;
             case MEMXCT_OPT_CANONICAL: *value = P.opt.canonical; break;
             case MEMXCT_OPT_CG_VARIANT: *value = P.opt.cg_variant; break;
@@ -207,6 +233,9 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
         mx::build_hilbert(P.n, P.n, P.tile_tomo, P.tomo_nat_of_h.p(), P.tomo_h_of_nat.p(), st);
         mx::build_hilbert(P.m, P.c, P.tile_sino, P.sino_nat_of_h.p(), P.sino_h_of_nat.p(), st);
         P.esize = P.opt.precision == 1 ? 8 : 4;
+        resolve_tuning(P);
+        const char* fd = std::getenv("MEMXCT_FUSED_DOT");
+        P.fused_dot = fd && fd[0] == '1';
         mx::build_matrices(P, st);
         MX_CUDA(cudaStreamSynchronize(st));
         P.built = true;
@@ -338,8 +367,8 @@ memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* par
 
 memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0, int64_t p1,
                                      int64_t* stage_base, int64_t* map_off, int32_t* map, int64_t* slot_off,
-                                     uint16_t* ind, float* val, int64_t* n_map, int64_t* n_slot_off,
-                                     int64_t* n_slots) {
+                                     uint16_t* ind, float* val, uint16_t* lane_chunks, int64_t* n_map,
+                                     int64_t* n_slot_off, int64_t* n_slots) {
     return guarded([&] {
         mx::Plan& P = built_plan(plan);
         if (dir != 0 && dir != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "dir must be 0 or 1");
@@ -363,6 +392,8 @@ memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0
         if (slot_off) MX_CUDA(cudaMemcpy(slot_off, L.slot_off.p() + b0, 8 * (b1 - b0 + 1), cudaMemcpyDeviceToHost));
         if (ind && so[1] > so[0]) MX_CUDA(cudaMemcpy(ind, L.ind.p() + so[0], 2 * (so[1] - so[0]), cudaMemcpyDeviceToHost));
         if (val && so[1] > so[0]) MX_CUDA(cudaMemcpy(val, L.val.p() + so[0], 4 * (so[1] - so[0]), cudaMemcpyDeviceToHost));
+        if (lane_chunks && b1 > b0)
+            MX_CUDA(cudaMemcpy(lane_chunks, L.lane_chunks.p() + b0 * 32, 2 * 32 * (b1 - b0), cudaMemcpyDeviceToHost));
     });
 }
 

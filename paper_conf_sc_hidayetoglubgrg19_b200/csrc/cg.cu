@@ -140,17 +140,39 @@ cg_update_p_kernel(T* __restrict__ p, const T* __restrict__ s, int64_t nx, Scal 
         p[i] = upd(p[i], beta, s[i]);
 }
 
+// <v, v> in fp64 over a fixed grid (deterministic: fixed element->thread map, fixed tree)
+template <class T>
+__global__ void __launch_bounds__(kVT)
+dot_kernel(const T* __restrict__ v, int64_t n, double* out, double* part, unsigned int* ticket) {
+    double acc = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < n; i += (int64_t)gridDim.x * kVT) {
+        const double e = (double)v[i];
+        acc += e * e;
+    }
+    vec_dot_finish(acc, part, out, ticket);
+}
+
 unsigned vec_blocks(int64_t n) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(kVecBlocks, ceil_div(n, kVT)));
 }
 
+// SpMV followed by the dot product of its output.  Canonical mode fuses the dot into the
+// SpMV epilogue (per-partition fma chains, reading R16).  Otherwise a separate small dot kernel
+// is used: measured on B200, the fused last-CTA epilogue slowed the 2 ms SpMV by ~0.5 ms
+// (profiles/r01a_launches.md), while the separate pass over the 4-6 MB vector costs a few us.
 template <class T>
 void spmv_dir(Plan& P, const Layout& L, const T* in, T* out, double* dot_out, cudaStream_t st) {
     double* part = (&L == &P.fwd) ? P.part_fwd.p() : P.part_back.p();
+    const bool fused = dot_out && (P.opt.canonical != 0 || P.fused_dot);
     if constexpr (sizeof(T) == 4)
-        spmv_f32(L, in, out, part, dot_out, P.tickets.p(), st);
+        spmv_f32(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), st);
     else
-        spmv_f64(L, in, out, part, dot_out, P.tickets.p(), P.opt.canonical != 0, st);
+        spmv_f64(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), P.opt.canonical != 0, st);
+    if (dot_out && !fused) {
+        dot_kernel<T><<<vec_blocks(L.nrows), kVT, 0, st>>>(out, L.nrows, dot_out, P.part_vec.p(),
+                                                           P.tickets.p() + 2);
+        MX_LAUNCHED();
+    }
 }
 
 template <class T>
@@ -186,10 +208,6 @@ void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, cudaStream_t st) {
         cg_update_p_kernel<T><<<vec_blocks(nx), kVT, 0, st>>>(p, s, nx, sc, k);
         MX_LAUNCHED();
     }
-}
-
-int64_t kernels_per_solve(const Plan& P, int32_t iters) {
-    return 3 + (int64_t)iters * (P.opt.cg_variant == 1 ? 6 : 4);
 }
 
 }  // namespace
@@ -234,9 +252,11 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
             cudaStreamDestroy(cap);
             throw;
         }
-        count_launch(-(launch_count() - before));  // captured, not launched
+        const int64_t captured = launch_count() - before;
+        count_launch(-captured);  // captured, not launched: counted at every graph launch
         MX_CUDA(cudaStreamEndCapture(cap, &g));
         auto cgg = std::make_unique<CgGraph>();
+        cgg->nkernels = captured;
         cudaError_t e = cudaGraphInstantiate(&cgg->exec, g, 0);
         cudaGraphDestroy(g);
         cudaStreamDestroy(cap);
@@ -244,7 +264,7 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
         it = P.graphs.emplace(key, std::move(cgg)).first;
     }
     MX_CUDA(cudaGraphLaunch(it->second->exec, st));
-    count_launch(kernels_per_solve(P, iters));
+    count_launch(it->second->nkernels);
     MX_CUDA(cudaGetLastError());
 }
 

@@ -164,10 +164,12 @@ __global__ void runs_kernel(const int64_t* __restrict__ row_ptr, const uint32_t*
     }
 }
 
-// one warp per (global stage, slice): slots = roundup(max run length over its 32 rows, kVec) * 32
+// one warp per (global stage, slice): chunks of each lane = ceil(run length / kVec); the block
+// stores only the chunks lanes actually have (jagged SELL, plan.h), so its size is kVec * sum.
 __global__ void width_kernel(const int32_t* __restrict__ stage_part, const int64_t* __restrict__ stage_base,
                              const int32_t* __restrict__ run_len, int64_t nstages, int32_t SPP, int64_t nrows,
-                             int32_t R, int32_t maxS, int64_t* __restrict__ blk_slots) {
+                             int32_t R, int32_t maxS, int64_t* __restrict__ blk_slots,
+                             uint16_t* __restrict__ lane_chunks) {
     const int lane = threadIdx.x & 31;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x / 32);
     for (int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32; wi < nstages * SPP; wi += warps) {
@@ -177,16 +179,36 @@ __global__ void width_kernel(const int32_t* __restrict__ stage_part, const int64
         const int64_t s = g - stage_base[p];
         const int64_t row = p * R + (int64_t)w * 32 + lane;
         const int32_t len = (row < nrows) ? run_len[row * maxS + s] : 0;
-        const int32_t mx = __reduce_max_sync(0xffffffffu, len);
-        if (lane == 0) blk_slots[wi] = (int64_t)((mx + kVec - 1) / kVec) * kVec * 32;
+        const int32_t nch = (len + kVec - 1) / kVec;
+        lane_chunks[wi * 32 + lane] = (uint16_t)nch;
+        const int32_t tot = __reduce_add_sync(0xffffffffu, nch);
+        if (lane == 0) blk_slots[wi] = (int64_t)tot * kVec;
+    }
+}
+
+// Position of chunk c of `lane` inside its block: chunks are stored chunk-index-major, and within
+// chunk c only the lanes that have it, in lane order.  prefix = slots of chunks 0..c-1 / kVec,
+// active = lanes having chunk c, rank = active lanes below `lane`.
+__device__ __forceinline__ void jagged_pos(const uint16_t* __restrict__ lc, int lane, int64_t c,
+                                           int64_t& prefix, int32_t& active, int32_t& rank) {
+    prefix = 0;
+    active = 0;
+    rank = 0;
+    for (int l = 0; l < 32; ++l) {
+        const int64_t n = lc[l];
+        prefix += n < c ? n : c;
+        const bool has = n > c;
+        active += has;
+        rank += (has && l < lane);
     }
 }
 
 __global__ void scatter_kernel(const uint32_t* __restrict__ row_ids, const float* __restrict__ vals,
                                const uint32_t* __restrict__ rank, const int64_t* __restrict__ row_ptr,
                                const int32_t* __restrict__ run_start, const int64_t* __restrict__ stage_base,
-                               const int64_t* __restrict__ slot_off, int64_t nnz, int32_t R, int32_t SPP,
-                               int32_t B, int32_t maxS, uint16_t* __restrict__ ind, float* __restrict__ val) {
+                               const int64_t* __restrict__ slot_off, const uint16_t* __restrict__ lane_chunks,
+                               int64_t nnz, int32_t R, int32_t SPP, int32_t B, int32_t maxS,
+                               uint16_t* __restrict__ ind, float* __restrict__ val) {
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x) {
         const int64_t row = row_ids[e];
         const int64_t p = row / R;
@@ -195,11 +217,15 @@ __global__ void scatter_kernel(const uint32_t* __restrict__ row_ids, const float
         const int32_t s = (int32_t)(rk / (uint32_t)B);
         const uint32_t local = rk % (uint32_t)B;
         const int64_t j = (e - row_ptr[row]) - run_start[row * maxS + s];
-        const int64_t base = slot_off[(stage_base[p] + s) * SPP + wl];
+        const int64_t blk = (stage_base[p] + s) * SPP + wl;
+        const int64_t base = slot_off[blk];
         const int64_t c = j / kVec, e8 = j % kVec;
-        const int64_t chunk = base + c * (32 * kVec);
-        ind[chunk + lane * kVec + e8] = (uint16_t)local;
-        val[chunk + (e8 >> 2) * 128 + lane * 4 + (e8 & 3)] = vals[e];
+        int64_t prefix;
+        int32_t active, rnk;
+        jagged_pos(lane_chunks + blk * 32, lane, c, prefix, active, rnk);
+        const int64_t chunk = base + prefix * kVec;
+        ind[chunk + (int64_t)rnk * kVec + e8] = (uint16_t)local;
+        val[chunk + (e8 >> 2) * ((int64_t)active * 4) + (int64_t)rnk * 4 + (e8 & 3)] = vals[e];
     }
 }
 
@@ -361,9 +387,11 @@ void build_layout(Layout& L, int64_t nrows, int64_t ncols, int64_t nnz, const ui
     DevArr<int64_t> blk_slots;
     blk_slots.alloc(nblk + 1);
     MX_CUDA(cudaMemsetAsync(blk_slots.p(), 0, 8 * (nblk + 1), st));
+    L.lane_chunks.alloc(std::max<int64_t>(nblk * 32, 1));
     if (nblk > 0) {
         width_kernel<<<blocks_for(nblk * 32), kThreads, 0, st>>>(stage_part.p(), L.stage_base.p(), run_len.p(),
-                                                                 L.nstages, L.SPP, nrows, R, maxS, blk_slots.p());
+                                                                 L.nstages, L.SPP, nrows, R, maxS, blk_slots.p(),
+                                                                 L.lane_chunks.p());
         MX_LAUNCHED();
     }
     L.slot_off.alloc(nblk + 1);
@@ -379,8 +407,8 @@ void build_layout(Layout& L, int64_t nrows, int64_t ncols, int64_t nnz, const ui
     MX_CUDA(cudaMemsetAsync(L.val.p(), 0, 4 * std::max<int64_t>(L.nslots, 1), st));
     if (nnz > 0) {
         scatter_kernel<<<blocks_for(nnz), kThreads, 0, st>>>(row_ids, vals, rank.p(), row_ptr.p(), run_start.p(),
-                                                             L.stage_base.p(), L.slot_off.p(), nnz, R, L.SPP, B,
-                                                             maxS, L.ind.p(), L.val.p());
+                                                             L.stage_base.p(), L.slot_off.p(), L.lane_chunks.p(), nnz,
+                                                             R, L.SPP, B, maxS, L.ind.p(), L.val.p());
         MX_LAUNCHED();
     }
     if (out_translate) {
@@ -432,8 +460,8 @@ void build_matrices(Plan& P, cudaStream_t st) {
     row_ptr.reset();
 
     const bool natural = (P.opt.vector_order == 0);
-    const int32_t R = (int32_t)P.opt.part_rows;
-    const int32_t B = (int32_t)(P.opt.precision == 1 ? P.opt.buffer_entries / 2 : P.opt.buffer_entries);
+    const int32_t R = P.part_rows;
+    const int32_t B = P.opt.precision == 1 ? P.buffer_entries / 2 : P.buffer_entries;
 
     // 3. A^T: stable sort by pixel (order-preserving transposition)
     DevArr<uint32_t> t_row, t_col, perm;

@@ -18,11 +18,17 @@ namespace mx {
 //   stage-buffer map           map[map_off[p] + s*B + i] = input index of buffer slot i of
 //                              local stage s (distinct inputs of p sorted by Hilbert index, cut
 //                              into chunks of B, reading R10)
-//   (stage g, slice w) block   slots [slot_off[g*SPP + w], slot_off[g*SPP + w + 1]),
-//                              width = size/32 (multiple of kVec), stored in chunks of kVec
-//                              columns: ind chunk = [32 lanes][kVec] uint16, val chunk =
-//                              [kVec/4][32 lanes][4] fp32, so each lane reads 16 B of ind and
-//                              2 x 16 B of val per chunk with fully coalesced warp loads.
+//   (stage g, slice w) block   slots [slot_off[g*SPP + w], slot_off[g*SPP + w + 1]).
+//                              Lane l (row w*32 + l) owns n_l = lane_chunks[(g*SPP + w)*32 + l]
+//                              chunks of kVec slots (its run length rounded up to kVec).
+//                              "Jagged SELL": chunk c is stored only for the a_c lanes with
+//                              n_l > c, packed in lane order; chunk c starts after
+//                              prefix_c = sum_l min(n_l, c) chunks.  Inside chunk c:
+//                                ind: [a_c lanes][kVec] uint16        (16 B per lane)
+//                                val: [kVec/4][a_c lanes][4] fp32     (2 x 16 B per lane)
+//                              so the active lanes of a warp read contiguous, fully coalesced
+//                              16 B vectors and no padding beyond the per-lane round-up to kVec
+//                              is stored or streamed (padding slots: ind 0, val 0).
 //   entries of a row in a stage ascend by local index (= ascending Hilbert input index).
 struct Layout {
     int64_t nrows = 0, ncols = 0, nnz = 0;
@@ -35,11 +41,12 @@ struct Layout {
     DevArr<int64_t> slot_off;    // nstages * SPP + 1
     DevArr<uint16_t> ind;        // nslots
     DevArr<float> val;           // nslots
+    DevArr<uint16_t> lane_chunks;  // nstages * SPP * 32
     DevArr<int32_t> out_idx;     // nrows, optional: output position of each row (natural order)
     int64_t device_bytes() const {
         return (int64_t)(stage_base.buf.bytes() + map_off.buf.bytes() + map.buf.bytes() +
                          slot_off.buf.bytes() + ind.buf.bytes() + val.buf.bytes() +
-                         out_idx.buf.bytes());
+                         lane_chunks.buf.bytes() + out_idx.buf.bytes());
     }
 };
 
@@ -48,8 +55,8 @@ constexpr int kVec = 8;  // SELL column chunk: 8 slots per lane per chunk
 struct Options {
     int64_t tile_tomo = 0;  // 0 = default rule R7
     int64_t tile_sino = 0;
-    int64_t part_rows = 512;
-    int64_t buffer_entries = 12288;
+    int64_t part_rows = 0;       // 0 = auto (resolve_tuning)
+    int64_t buffer_entries = 0;  // 0 = auto (resolve_tuning)
     int64_t precision = 0;  // 0 FP32, 1 MIXED
     int64_t canonical = 0;
     int64_t cg_variant = 0;
@@ -58,6 +65,7 @@ struct Options {
 
 struct CgGraph {
     cudaGraphExec_t exec = nullptr;
+    int64_t nkernels = 0;
     ~CgGraph() { if (exec) cudaGraphExecDestroy(exec); }
 };
 
@@ -67,6 +75,8 @@ struct Plan {
     bool built = false;
     int32_t rank = 0, nranks = 1, device = -1;
     int32_t tile_tomo = 0, tile_sino = 0;
+    bool fused_dot = false;  // MEMXCT_FUSED_DOT=1: fuse CG dots into the SpMV epilogue (tuning)
+    int32_t part_rows = 0, buffer_entries = 0;  // resolved tuning (build)
 
     // two-level pseudo-Hilbert permutations, device int32
     DevArr<int32_t> tomo_nat_of_h, tomo_h_of_nat;  // N*N

@@ -42,6 +42,31 @@ __device__ __forceinline__ float4 ld_stream_f4(const void* p, uint64_t pol) {
     return r;
 }
 
+// 8 slots of one lane: acc += buf[ind] * val in ascending slot order (one dependent chain)
+__device__ __forceinline__ void fma8(float& acc, const float* buf, const uint4& iv, const float4& v0,
+                                     const float4& v1) {
+    acc = fmaf(buf[iv.x & 0xffffu], v0.x, acc);
+    acc = fmaf(buf[iv.x >> 16], v0.y, acc);
+    acc = fmaf(buf[iv.y & 0xffffu], v0.z, acc);
+    acc = fmaf(buf[iv.y >> 16], v0.w, acc);
+    acc = fmaf(buf[iv.z & 0xffffu], v1.x, acc);
+    acc = fmaf(buf[iv.z >> 16], v1.y, acc);
+    acc = fmaf(buf[iv.w & 0xffffu], v1.z, acc);
+    acc = fmaf(buf[iv.w >> 16], v1.w, acc);
+}
+// MIXED: fp64 fma with the fp32 value widened exactly (canonical chain, reading R16)
+__device__ __forceinline__ void fma8(double& acc, const double* buf, const uint4& iv, const float4& v0,
+                                     const float4& v1) {
+    acc = __fma_rn((double)v0.x, buf[iv.x & 0xffffu], acc);
+    acc = __fma_rn((double)v0.y, buf[iv.x >> 16], acc);
+    acc = __fma_rn((double)v0.z, buf[iv.y & 0xffffu], acc);
+    acc = __fma_rn((double)v0.w, buf[iv.y >> 16], acc);
+    acc = __fma_rn((double)v1.x, buf[iv.z & 0xffffu], acc);
+    acc = __fma_rn((double)v1.y, buf[iv.z >> 16], acc);
+    acc = __fma_rn((double)v1.z, buf[iv.w & 0xffffu], acc);
+    acc = __fma_rn((double)v1.w, buf[iv.w >> 16], acc);
+}
+
 struct SpmvArgs {
     const int64_t* stage_base;
     const int64_t* map_off;
@@ -49,6 +74,7 @@ struct SpmvArgs {
     const int64_t* slot_off;
     const uint16_t* ind;
     const float* val;
+    const uint16_t* lane_chunks;
     const int32_t* out_idx;
     int64_t nrows;
     int64_t nparts;
@@ -117,11 +143,12 @@ __device__ void finish_dot_canonical(const SpmvArgs& a, const double* rows_val, 
 constexpr int kMaxThreads = 1024;
 
 template <bool kNatOut, bool kDot>
-__global__ void __launch_bounds__(kMaxThreads)
+__global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) {
     extern __shared__ __align__(16) float sbuf[];
     const int64_t p = blockIdx.x;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
     const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
     const int64_t m0 = a.map_off[p], D = a.map_off[p + 1] - m0;
     const uint64_t pol = evict_first_policy();
@@ -135,22 +162,33 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) 
         __syncthreads();
         const int64_t blk = g * a.SPP + warp;
         const int64_t base = a.slot_off[blk];
-        const int64_t nchunk = (a.slot_off[blk + 1] - base) / (32 * kVec);
-        const uint4* ip = reinterpret_cast<const uint4*>(a.ind + base) + lane;
-        const float4* vp = reinterpret_cast<const float4*>(a.val + base) + lane;
+        const int nch = a.lane_chunks[blk * 32 + lane];
+        const int maxc = __reduce_max_sync(0xffffffffu, nch);
+        const uint4* ib = reinterpret_cast<const uint4*>(a.ind + base);
+        const float4* vb = reinterpret_cast<const float4*>(a.val + base);
+        // phase 1: chunks every lane has -- plain SELL addressing, branch-free, unrolled so
+        // several 16 B loads per lane are in flight
+        const int minc = __reduce_min_sync(0xffffffffu, nch);
 #pragma unroll 4
-        for (int64_t c = 0; c < nchunk; ++c) {
-            const uint4 iv = ld_stream_u4(ip + c * 32, pol);
-            const float4 v0 = ld_stream_f4(vp + c * 64, pol);
-            const float4 v1 = ld_stream_f4(vp + c * 64 + 32, pol);
-            acc = fmaf(sbuf[iv.x & 0xffffu], v0.x, acc);
-            acc = fmaf(sbuf[iv.x >> 16], v0.y, acc);
-            acc = fmaf(sbuf[iv.y & 0xffffu], v0.z, acc);
-            acc = fmaf(sbuf[iv.y >> 16], v0.w, acc);
-            acc = fmaf(sbuf[iv.z & 0xffffu], v1.x, acc);
-            acc = fmaf(sbuf[iv.z >> 16], v1.y, acc);
-            acc = fmaf(sbuf[iv.w & 0xffffu], v1.z, acc);
-            acc = fmaf(sbuf[iv.w >> 16], v1.w, acc);
+        for (int c = 0; c < minc; ++c) {
+            const uint4 iv = ld_stream_u4(ib + c * 32 + lane, pol);
+            const float4 v0 = ld_stream_f4(vb + c * 64 + lane, pol);
+            const float4 v1 = ld_stream_f4(vb + c * 64 + 32 + lane, pol);
+            fma8(acc, sbuf, iv, v0, v1);
+        }
+        // phase 2: the ragged tail, stored only for the lanes that have it (jagged SELL)
+        int64_t pref = (int64_t)minc * 32;
+        for (int c = minc; c < maxc; ++c) {
+            const unsigned act = __ballot_sync(0xffffffffu, nch > c);
+            const int na = __popc(act);
+            if (nch > c) {
+                const int r = __popc(act & lt);
+                const uint4 iv = ld_stream_u4(ib + pref + r, pol);
+                const float4 v0 = ld_stream_f4(vb + 2 * pref + r, pol);
+                const float4 v1 = ld_stream_f4(vb + 2 * pref + na + r, pol);
+                fma8(acc, sbuf, iv, v0, v1);
+            }
+            pref += na;
         }
     }
     const int64_t row = p * a.R + threadIdx.x;
@@ -163,11 +201,12 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) 
 // Hilbert input order (stages ascend, slots within a stage ascend by local index; padding slots
 // are fma(0, finite, acc) = acc).  This is the canonical row sum of reading R16.
 template <bool kNatOut, int kDotMode>  // kDotMode: 0 none, 1 tree, 2 canonical chain
-__global__ void __launch_bounds__(kMaxThreads)
+__global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y) {
     extern __shared__ __align__(16) double dbuf[];
     const int64_t p = blockIdx.x;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
     const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
     const int64_t m0 = a.map_off[p], D = a.map_off[p + 1] - m0;
     const uint64_t pol = evict_first_policy();
@@ -181,22 +220,33 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
         __syncthreads();
         const int64_t blk = g * a.SPP + warp;
         const int64_t base = a.slot_off[blk];
-        const int64_t nchunk = (a.slot_off[blk + 1] - base) / (32 * kVec);
-        const uint4* ip = reinterpret_cast<const uint4*>(a.ind + base) + lane;
-        const float4* vp = reinterpret_cast<const float4*>(a.val + base) + lane;
-#pragma unroll 2
-        for (int64_t c = 0; c < nchunk; ++c) {
-            const uint4 iv = ld_stream_u4(ip + c * 32, pol);
-            const float4 v0 = ld_stream_f4(vp + c * 64, pol);
-            const float4 v1 = ld_stream_f4(vp + c * 64 + 32, pol);
-            acc = __fma_rn((double)v0.x, dbuf[iv.x & 0xffffu], acc);
-            acc = __fma_rn((double)v0.y, dbuf[iv.x >> 16], acc);
-            acc = __fma_rn((double)v0.z, dbuf[iv.y & 0xffffu], acc);
-            acc = __fma_rn((double)v0.w, dbuf[iv.y >> 16], acc);
-            acc = __fma_rn((double)v1.x, dbuf[iv.z & 0xffffu], acc);
-            acc = __fma_rn((double)v1.y, dbuf[iv.z >> 16], acc);
-            acc = __fma_rn((double)v1.z, dbuf[iv.w & 0xffffu], acc);
-            acc = __fma_rn((double)v1.w, dbuf[iv.w >> 16], acc);
+        const int nch = a.lane_chunks[blk * 32 + lane];
+        const int maxc = __reduce_max_sync(0xffffffffu, nch);
+        const uint4* ib = reinterpret_cast<const uint4*>(a.ind + base);
+        const float4* vb = reinterpret_cast<const float4*>(a.val + base);
+        // phase 1: chunks every lane has -- plain SELL addressing, branch-free, unrolled so
+        // several 16 B loads per lane are in flight
+        const int minc = __reduce_min_sync(0xffffffffu, nch);
+#pragma unroll 4
+        for (int c = 0; c < minc; ++c) {
+            const uint4 iv = ld_stream_u4(ib + c * 32 + lane, pol);
+            const float4 v0 = ld_stream_f4(vb + c * 64 + lane, pol);
+            const float4 v1 = ld_stream_f4(vb + c * 64 + 32 + lane, pol);
+            fma8(acc, dbuf, iv, v0, v1);
+        }
+        // phase 2: the ragged tail, stored only for the lanes that have it (jagged SELL)
+        int64_t pref = (int64_t)minc * 32;
+        for (int c = minc; c < maxc; ++c) {
+            const unsigned act = __ballot_sync(0xffffffffu, nch > c);
+            const int na = __popc(act);
+            if (nch > c) {
+                const int r = __popc(act & lt);
+                const uint4 iv = ld_stream_u4(ib + pref + r, pol);
+                const float4 v0 = ld_stream_f4(vb + 2 * pref + r, pol);
+                const float4 v1 = ld_stream_f4(vb + 2 * pref + na + r, pol);
+                fma8(acc, dbuf, iv, v0, v1);
+            }
+            pref += na;
         }
     }
     const int64_t row = p * a.R + threadIdx.x;
@@ -230,6 +280,7 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.slot_off = L.slot_off.p();
     a.ind = L.ind.p();
     a.val = L.val.p();
+    a.lane_chunks = L.lane_chunks.p();
     a.out_idx = L.out_idx.p();
     a.nrows = L.nrows;
     a.nparts = L.nparts;

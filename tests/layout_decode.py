@@ -1,7 +1,8 @@
-"""Test-side decoder of the staged SELL-32 layout exported by memxct_layout_export.
+"""Test-side decoder of the jagged SELL-32 layout exported by memxct_layout_export.
 
-Pure index bookkeeping in numpy (documented layout); no arithmetic of the
-method.  Returns every stored slot as (plan row, input index, value, local index, j, stage).
+Pure index bookkeeping in numpy (documented layout: plan.h / DESIGN.md section 5); no arithmetic
+of the method.  Returns every stored slot as (plan row, input index, value, local index, j,
+stage).
 """
 import numpy as np
 
@@ -15,27 +16,44 @@ def decode(ex, R, B, p0=0):
     SPP = R // 32
     g0 = sb[0]
     nblk = len(so) - 1
+    n = ex["lane_chunks"].reshape(nblk, 32).astype(np.int64)
     sizes = np.diff(so)
-    assert np.all(sizes % (32 * KVEC) == 0)
-    slot = np.arange(so[-1] - so[0], dtype=np.int64)
-    blk = np.repeat(np.arange(nblk, dtype=np.int64), sizes)
-    off = slot - (so[blk] - so[0])
-    c, r = off // 256, off % 256
-    lane, e8 = r // KVEC, r % KVEC
-    j = c * KVEC + e8
-    val_pos = (so[blk] - so[0]) + c * 256 + (e8 // 4) * 128 + lane * 4 + (e8 % 4)
-    ind = ex["ind"].astype(np.int64)
-    val = ex["val"][val_pos]
-    g = blk // SPP + g0
-    w = blk % SPP
+    assert np.array_equal(sizes, n.sum(1) * KVEC)
+    # one record per (block, lane, chunk)
+    cnt = n.ravel()
+    bl = np.repeat(np.arange(nblk * 32, dtype=np.int64), cnt)
+    b, l = bl // 32, bl % 32
+    start = np.repeat(np.cumsum(cnt) - cnt, cnt)
+    c = np.arange(len(bl), dtype=np.int64) - start
+    prefix = np.zeros_like(c)
+    active = np.zeros_like(c)
+    rank = np.zeros_like(c)
+    for lp in range(32):
+        nl = n[b, lp]
+        prefix += np.minimum(nl, c)
+        has = nl > c
+        active += has
+        rank += has & (lp < l)
+    base = so[b] - so[0]
+    e8 = np.arange(KVEC, dtype=np.int64)[None, :]
+    ind_pos = (base + (prefix + rank) * KVEC)[:, None] + e8
+    val_pos = (base + prefix * KVEC)[:, None] + (e8 // 4) * (active * 4)[:, None] + (rank * 4)[:, None] + e8 % 4
+    ind = ex["ind"][ind_pos].astype(np.int64).ravel()
+    val = ex["val"][val_pos].ravel()
+    assert len(np.unique(ind_pos)) == ind_pos.size and len(np.unique(val_pos)) == val_pos.size
+    j = (c[:, None] * KVEC + e8).ravel()
+    b = np.repeat(b, KVEC)
+    lane = np.repeat(l, KVEC)
+    g = b // SPP + g0
+    w = b % SPP
     part = np.searchsorted(sb, g, side="right") - 1
     s = g - sb[part]
     row = (part + p0) * R + w * 32 + lane
-    cnt = np.minimum(B, (mo[part + 1] - mo[part]) - s * B)
-    assert np.all(ind < np.maximum(cnt, 1))
+    cnt_stage = np.minimum(B, (mo[part + 1] - mo[part]) - s * B)
+    assert np.all(ind < np.maximum(cnt_stage, 1))
     map_pos = (mo[part] - mo[0]) + s * B + ind
     col = ex["map"][np.minimum(map_pos, len(ex["map"]) - 1)] if len(ex["map"]) else np.zeros_like(ind)
-    return dict(row=row, col=col.astype(np.int64), val=val, ind=ind, j=j, stage=g, blk=blk, lane=lane)
+    return dict(row=row, col=col.astype(np.int64), val=val, ind=ind, j=j, stage=g, blk=b, lane=lane)
 
 
 def real_entries(d):
@@ -45,8 +63,8 @@ def real_entries(d):
 
 
 def check_structure(d):
-    """Padding is (ind 0, val 0); inside each (row, stage) the real slots come first and
-    ascend by local index (canonical order, reading R16)."""
+    """Padding is (ind 0, val 0) and only fills the last chunk of a lane's run; inside each
+    (row, stage) the real slots come first and ascend by local index (canonical order, R16)."""
     pad = d["val"] == 0
     assert np.all(d["ind"][pad] == 0)
     key = (d["stage"] * 1_000_000_007 + d["row"]).astype(np.int64)
@@ -58,3 +76,6 @@ def check_structure(d):
     # ascending local index among consecutive real slots
     both = same & real[:-1] & real[1:]
     assert np.all(ind2[1:][both] > ind2[:-1][both])
+    # at most KVEC-1 padding slots per (row, stage) run
+    runs, counts = np.unique(k2[~real], return_counts=True)
+    assert counts.size == 0 or counts.max() < KVEC
