@@ -105,8 +105,36 @@ memxct_status_t memxct_plan_get_option(memxct_plan_t plan, memxct_option_t optio
 memxct_status_t memxct_plan_set_comm(memxct_plan_t plan, int32_t rank, int32_t nranks,
                                      const void* nccl_unique_id, int32_t cuda_device);
 
-/* Fill a 128-byte buffer with a fresh ncclUniqueId (call on rank 0 only). */
+/* Fill a 128-byte buffer with a fresh ncclUniqueId (call on rank 0 only).  NCCL is loaded at
+ * run time (dlopen of libnccl.so.2); MEMXCT_ERR_NCCL if it is unavailable. */
 memxct_status_t memxct_get_unique_id(void* nccl_unique_id_out);
+
+/* Virtual ranks (testing the multi-GPU path on one device): a group of `nranks` plans in one
+ * process, each built and driven from its own host thread, whose collectives are device copies
+ * instead of NCCL.  Same decomposition, maps, kernels and results as NCCL ranks; not graph
+ * captured.  The group must outlive its plans. */
+typedef struct memxct_group* memxct_group_t;
+memxct_status_t memxct_local_group_create(int32_t nranks, memxct_group_t* out);
+memxct_status_t memxct_local_group_destroy(memxct_group_t group);
+memxct_status_t memxct_plan_set_comm_local(memxct_plan_t plan, memxct_group_t group, int32_t rank);
+
+/* Domain decomposition helper (host only, reading R12): split `count` tiles with
+ * nonnegative `weights` (nonzeros per tile, in Hilbert order) into `parts` contiguous ranges
+ * with about equal weight; bounds[0..parts] (host) receives the range boundaries, every range
+ * non-empty when count >= parts.  memxct_build uses it for both domains. */
+memxct_status_t memxct_partition_ranges(const int64_t* weights, int64_t count, int32_t parts,
+                                        int64_t* bounds);
+
+/* After build: the Hilbert-index ranges owned by every rank (bounds[0..nranks]) for domain 0
+ * (tomogram pixels) or 1 (sinogram rays). */
+memxct_status_t memxct_domain_ranges(memxct_plan_t plan, int32_t domain, int64_t* bounds);
+
+/* After build (P > 1): this rank's footprint rays (rows of A_p), the partial-sinogram entries it
+ * sends per forward exchange and receives (the back exchange is the reverse), and the number of
+ * peers it talks to.  Any pointer may be NULL. */
+memxct_status_t memxct_exchange_info(memxct_plan_t plan, int64_t* footprint_rays,
+                                     int64_t* sent_entries, int64_t* received_entries,
+                                     int32_t* peers);
 
 /* Preprocessing: Hilbert ordering and domain decomposition, Siddon tracing of A on
  * the device, order-preserving transposition to A^T, partitioning and the multi-stage buffered

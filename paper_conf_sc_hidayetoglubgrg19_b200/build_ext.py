@@ -21,10 +21,24 @@ INCLUDE = os.path.join(ROOT, "include")
 OUT = os.path.join(PKG, "libmemxct.so")
 BUILD = os.path.join(PKG, "build")
 
-SOURCES = ["api.cu", "hilbert.cu", "trace.cu", "layout.cu", "spmv.cu", "cg.cu"]
+SOURCES = ["api.cu", "hilbert.cu", "trace.cu", "layout.cu", "spmv.cu", "cg.cu", "comm.cu", "exchange.cu"]
 EXTRA = {"trace.cu": ["--fmad=false"]}
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+
+
+def _nccl_include() -> str:
+    """nccl.h for the declarations only: libnccl.so.2 is dlopen'ed at run time (the one torch
+    already loaded), so the library has no link-time NCCL dependency."""
+    try:
+        import importlib.util
+        spec = importlib.util.find_spec("nvidia.nccl")
+        for loc in (spec.submodule_search_locations or []):
+            if os.path.exists(os.path.join(loc, "include", "nccl.h")):
+                return os.path.join(loc, "include")
+    except Exception:
+        pass
+    return "/usr/include"
 
 
 def _deps_mtime() -> float:
@@ -39,7 +53,7 @@ def up_to_date() -> bool:
 def _compile(src: str) -> str:
     obj = os.path.join(BUILD, src.replace(".cu", ".o"))
     cmd = [NVCC, "-c", "-O3", "-lineinfo", "-std=c++17", *ARCH, "-Xcompiler", "-fPIC",
-           "-Xptxas", "-v", "-I", INCLUDE, "-I", CSRC, *EXTRA.get(src, []),
+           "-Xptxas", "-v", "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(), *EXTRA.get(src, []),
            os.path.join(CSRC, src), "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
@@ -56,7 +70,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     with cf.ThreadPoolExecutor(max_workers=min(len(SOURCES), os.cpu_count() or 4)) as ex:
         objs = list(ex.map(_compile, SOURCES))
     tmp = OUT + f".{os.getpid()}.tmp"
-    cmd = [NVCC, "-shared", *ARCH, "-o", tmp, *objs, "-cudart", "static"]
+    cmd = [NVCC, "-shared", *ARCH, "-o", tmp, *objs, "-cudart", "static", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")

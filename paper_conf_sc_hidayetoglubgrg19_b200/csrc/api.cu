@@ -13,6 +13,10 @@ struct memxct_plan {
     mx::Plan P;
 };
 
+struct memxct_group {
+    std::shared_ptr<mx::LocalGroup> g;
+};
+
 namespace mx {
 
 static std::atomic<int64_t> g_launches{0};
@@ -24,7 +28,9 @@ int64_t Plan::device_bytes() const {
            (int64_t)(tomo_nat_of_h.buf.bytes() + tomo_h_of_nat.buf.bytes() + sino_nat_of_h.buf.bytes() +
                      sino_h_of_nat.buf.bytes() + cg_r.bytes() + cg_q.bytes() + cg_s.bytes() + cg_p.bytes() +
                      cg_ax.bytes() + part_fwd.buf.bytes() + part_back.buf.bytes() + part_vec.buf.bytes() +
-                     scal.buf.bytes() + tickets.buf.bytes() + h_in.bytes() + h_out.bytes());
+                     scal.buf.bytes() + tickets.buf.bytes() + h_in.bytes() + h_out.bytes() +
+                     fp_rays.buf.bytes()) +
+           ex.device_bytes();
 }
 
 }  // namespace mx
@@ -71,15 +77,9 @@ void need(const void* p, const char* what) {
     if (!p) mx::fail(MEMXCT_ERR_INVALID_ARG, std::string(what) + " is NULL");
 }
 
-void run_forward(mx::Plan& P, const void* x, void* y, cudaStream_t st) {
-    if (P.esize == 4) mx::spmv_f32(P.fwd, (const float*)x, (float*)y, nullptr, nullptr, nullptr, st);
-    else mx::spmv_f64(P.fwd, (const double*)x, (double*)y, nullptr, nullptr, nullptr, false, st);
-}
+void run_forward(mx::Plan& P, const void* x, void* y, cudaStream_t st) { mx::apply_forward(P, x, y, st); }
 
-void run_back(mx::Plan& P, const void* y, void* x, cudaStream_t st) {
-    if (P.esize == 4) mx::spmv_f32(P.back, (const float*)y, (float*)x, nullptr, nullptr, nullptr, st);
-    else mx::spmv_f64(P.back, (const double*)y, (double*)x, nullptr, nullptr, nullptr, false, st);
-}
+void run_back(mx::Plan& P, const void* y, void* x, cudaStream_t st) { mx::apply_back(P, y, x, st); }
 
 // Default tuning (measured B200 sweep, profiles/r01_sweep.md): the largest partition (CTA) size
 // in {1024, 512, 256, 128} rows that still gives >= 2 CTAs per SM in the smaller direction, and
@@ -89,7 +89,7 @@ void resolve_tuning(mx::Plan& P) {
     int dev = 0, sms = 148;
     MX_CUDA(cudaGetDevice(&dev));
     MX_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-    const int64_t rows = std::min<int64_t>((int64_t)P.n * P.n, (int64_t)P.m * P.c);
+    const int64_t rows = std::min<int64_t>((int64_t)P.n * P.n, (int64_t)P.m * P.c) / P.nranks;
     int32_t R = (int32_t)P.opt.part_rows;
     if (R == 0) {
         R = 128;
@@ -105,7 +105,7 @@ void resolve_tuning(mx::Plan& P) {
 
 void ensure_host_staging(mx::Plan& P) {
     if (!P.h_in.get()) {
-        const int64_t mx_len = std::max(P.fwd.nrows, P.back.nrows);
+        const int64_t mx_len = std::max(P.local_len(0), P.local_len(1));
         P.h_in.alloc(P.esize * std::max<int64_t>(mx_len, 1));
         P.h_out.alloc(P.esize * std::max<int64_t>(mx_len, 1));
     }
@@ -191,18 +191,85 @@ memxct_status_t memxct_plan_set_comm(memxct_plan_t plan, int32_t rank, int32_t n
         if (nranks < 1 || rank < 0 || rank >= nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank / nranks");
         if (nranks > 1) {
             need(nccl_unique_id, "nccl_unique_id");
-            mx::fail(MEMXCT_ERR_UNSUPPORTED, "P > 1 is not implemented in this build");
+            P.unique_id.assign((const uint8_t*)nccl_unique_id, (const uint8_t*)nccl_unique_id + 128);
         }
         P.rank = rank;
         P.nranks = nranks;
         P.device = cuda_device;
+        P.local_group.reset();
     });
 }
 
 memxct_status_t memxct_get_unique_id(void* out) {
     return guarded([&] {
         need(out, "out");
-        mx::fail(MEMXCT_ERR_UNSUPPORTED, "NCCL is not linked in this build");
+        mx::nccl_unique_id(out);
+    });
+}
+
+memxct_status_t memxct_local_group_create(int32_t nranks, memxct_group_t* out) {
+    return guarded([&] {
+        need(out, "out");
+        if (nranks < 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "nranks < 1");
+        *out = new memxct_group{std::make_shared<mx::LocalGroup>(nranks)};
+    });
+}
+
+memxct_status_t memxct_local_group_destroy(memxct_group_t group) {
+    return guarded([&] { delete group; });
+}
+
+memxct_status_t memxct_plan_set_comm_local(memxct_plan_t plan, memxct_group_t group, int32_t rank) {
+    return guarded([&] {
+        mx::Plan& P = plan_of(plan);
+        need(group, "group");
+        if (P.built) mx::fail(MEMXCT_ERR_STATE, "set_comm must precede memxct_build");
+        if (rank < 0 || rank >= group->g->nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank");
+        P.rank = rank;
+        P.nranks = group->g->nranks;
+        P.local_group = group->g;
+    });
+}
+
+memxct_status_t memxct_partition_ranges(const int64_t* weights, int64_t count, int32_t parts, int64_t* bounds) {
+    return guarded([&] {
+        need(bounds, "bounds");
+        if (count < 0 || parts < 1 || (count > 0 && !weights)) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad arguments");
+        std::vector<int64_t> w(weights, weights + count);
+        for (int64_t v : w)
+            if (v < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "negative weight");
+        const auto b = mx::partition_ranges(w, parts);
+        for (int32_t g = 0; g <= parts; ++g) bounds[g] = b[g];
+    });
+}
+
+memxct_status_t memxct_domain_ranges(memxct_plan_t plan, int32_t domain, int64_t* bounds) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(bounds, "bounds");
+        if (domain != 0 && domain != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "domain must be 0 or 1");
+        const auto& b = domain == 0 ? P.tomo_bounds : P.sino_bounds;
+        for (size_t g = 0; g < b.size(); ++g) bounds[g] = b[g];
+    });
+}
+
+memxct_status_t memxct_exchange_info(memxct_plan_t plan, int64_t* footprint_rays, int64_t* sent_entries,
+                                     int64_t* received_entries, int32_t* peers) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        int64_t sent = 0, np = 0;
+        for (int q = 0; q < (int)P.ex.scount.size(); ++q)
+            if (q != P.rank) {
+                sent += P.ex.scount[q];
+                np += (P.ex.scount[q] > 0 || P.ex.rcount[q] > 0);
+            }
+        int64_t recv = 0;
+        for (int q = 0; q < (int)P.ex.rcount.size(); ++q)
+            if (q != P.rank) recv += P.ex.rcount[q];
+        if (footprint_rays) *footprint_rays = P.nfp;
+        if (sent_entries) *sent_entries = sent;
+        if (received_entries) *received_entries = recv;
+        if (peers) *peers = (int32_t)np;
     });
 }
 
@@ -230,9 +297,14 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
         P.tomo_h_of_nat.alloc(npix);
         P.sino_nat_of_h.alloc(nrays);
         P.sino_h_of_nat.alloc(nrays);
-        mx::build_hilbert(P.n, P.n, P.tile_tomo, P.tomo_nat_of_h.p(), P.tomo_h_of_nat.p(), st);
-        mx::build_hilbert(P.m, P.c, P.tile_sino, P.sino_nat_of_h.p(), P.sino_h_of_nat.p(), st);
+        mx::build_hilbert(P.n, P.n, P.tile_tomo, P.tomo_nat_of_h.p(), P.tomo_h_of_nat.p(), &P.tomo_tile_off, st);
+        mx::build_hilbert(P.m, P.c, P.tile_sino, P.sino_nat_of_h.p(), P.sino_h_of_nat.p(), &P.sino_tile_off, st);
         P.esize = P.opt.precision == 1 ? 8 : 4;
+        if (P.nranks > 1) {
+            if (P.opt.canonical) mx::fail(MEMXCT_ERR_UNSUPPORTED, "CANONICAL mode is single-GPU only");
+            if (P.local_group) P.comm = mx::make_local_comm(P.local_group, P.rank);
+            else P.comm = mx::make_nccl_comm(P.rank, P.nranks, P.unique_id.data());
+        }
         resolve_tuning(P);
         const char* fd = std::getenv("MEMXCT_FUSED_DOT");
         P.fused_dot = fd && fd[0] == '1';
@@ -247,7 +319,7 @@ memxct_status_t memxct_local_size(memxct_plan_t plan, int32_t domain, int64_t* c
         mx::Plan& P = built_plan(plan);
         need(count, "count");
         if (domain != 0 && domain != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "domain must be 0 or 1");
-        *count = domain == 0 ? P.back.nrows : P.fwd.nrows;
+        *count = P.local_len(domain);
     });
 }
 
@@ -257,9 +329,10 @@ memxct_status_t memxct_local_indices(memxct_plan_t plan, int32_t domain, int64_t
         need(natural_idx, "natural_idx");
         if (domain != 0 && domain != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "domain must be 0 or 1");
         const mx::DevArr<int32_t>& a = domain == 0 ? P.tomo_nat_of_h : P.sino_nat_of_h;
-        std::vector<int32_t> h(a.n);
-        MX_CUDA(cudaMemcpy(h.data(), a.p(), 4 * a.n, cudaMemcpyDeviceToHost));
-        for (int64_t i = 0; i < a.n; ++i) natural_idx[i] = h[i];
+        const int64_t lo = domain == 0 ? P.t0 : P.s0, cnt = P.local_len(domain);
+        std::vector<int32_t> h(cnt);
+        if (cnt > 0) MX_CUDA(cudaMemcpy(h.data(), a.p() + lo, 4 * cnt, cudaMemcpyDeviceToHost));
+        for (int64_t i = 0; i < cnt; ++i) natural_idx[i] = h[i];
     });
 }
 
@@ -301,9 +374,9 @@ memxct_status_t memxct_forward_host(memxct_plan_t plan, const void* x_host, void
         need(y_host, "y_host");
         ensure_host_staging(P);
         cudaStream_t st = stream_of(cuda_stream);
-        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), x_host, P.esize * P.back.nrows, cudaMemcpyHostToDevice, st));
+        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), x_host, P.esize * P.local_len(0), cudaMemcpyHostToDevice, st));
         run_forward(P, P.h_in.get(), P.h_out.get(), st);
-        MX_CUDA(cudaMemcpyAsync(y_host, P.h_out.get(), P.esize * P.fwd.nrows, cudaMemcpyDeviceToHost, st));
+        MX_CUDA(cudaMemcpyAsync(y_host, P.h_out.get(), P.esize * P.local_len(1), cudaMemcpyDeviceToHost, st));
         MX_CUDA(cudaStreamSynchronize(st));
     });
 }
@@ -315,9 +388,9 @@ memxct_status_t memxct_back_host(memxct_plan_t plan, const void* y_host, void* x
         need(y_host, "y_host");
         ensure_host_staging(P);
         cudaStream_t st = stream_of(cuda_stream);
-        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), y_host, P.esize * P.fwd.nrows, cudaMemcpyHostToDevice, st));
+        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), y_host, P.esize * P.local_len(1), cudaMemcpyHostToDevice, st));
         run_back(P, P.h_in.get(), P.h_out.get(), st);
-        MX_CUDA(cudaMemcpyAsync(x_host, P.h_out.get(), P.esize * P.back.nrows, cudaMemcpyDeviceToHost, st));
+        MX_CUDA(cudaMemcpyAsync(x_host, P.h_out.get(), P.esize * P.local_len(0), cudaMemcpyDeviceToHost, st));
         MX_CUDA(cudaStreamSynchronize(st));
     });
 }
@@ -331,9 +404,9 @@ memxct_status_t memxct_cg_host(memxct_plan_t plan, const void* y_host, void* x_h
         if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
         ensure_host_staging(P);
         cudaStream_t st = stream_of(cuda_stream);
-        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), y_host, P.esize * P.fwd.nrows, cudaMemcpyHostToDevice, st));
+        MX_CUDA(cudaMemcpyAsync(P.h_in.get(), y_host, P.esize * P.local_len(1), cudaMemcpyHostToDevice, st));
         mx::cg_run(P, P.h_in.get(), P.h_out.get(), iters, st);
-        MX_CUDA(cudaMemcpyAsync(x_host, P.h_out.get(), P.esize * P.back.nrows, cudaMemcpyDeviceToHost, st));
+        MX_CUDA(cudaMemcpyAsync(x_host, P.h_out.get(), P.esize * P.local_len(0), cudaMemcpyDeviceToHost, st));
         if (residual_norms) mx::cg_fetch_norms(P, iters, residual_norms, st);
         MX_CUDA(cudaStreamSynchronize(st));
     });

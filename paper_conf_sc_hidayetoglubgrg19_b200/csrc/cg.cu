@@ -24,7 +24,8 @@ struct Scal {
     double* gam;   // [iters + 1]
     double* del;   // [iters + 1]
     double* res2;  // [iters + 1]
-    int* stop;     // [1]
+    int* stop;     // [1]  iterations stopped (gamma or delta reached 0)
+    int* stop_at;  // [1]  first iteration that did not run
 };
 
 Scal scal_of(Plan& P, int32_t iters) {
@@ -33,6 +34,7 @@ Scal scal_of(Plan& P, int32_t iters) {
     s.del = s.gam + (iters + 1);
     s.res2 = s.del + (iters + 1);
     s.stop = reinterpret_cast<int*>(s.res2 + (iters + 1));
+    s.stop_at = s.stop + 1;
     return s;
 }
 
@@ -74,7 +76,7 @@ cg_init_kernel(const T* __restrict__ y, T* __restrict__ r, int64_t nr, T* __rest
         acc += (double)v * (double)v;
     }
     for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < nx; i += (int64_t)gridDim.x * kVT) x[i] = T(0);
-    if (blockIdx.x == 0 && threadIdx.x == 0) *sc.stop = 0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) { *sc.stop = 0; *sc.stop_at = 0x7fffffff; }
     vec_dot_finish(acc, part, sc.res2, ticket);
 }
 
@@ -95,7 +97,7 @@ cg_update_xr_kernel(T* __restrict__ x, const T* __restrict__ p, int64_t nx, T* _
                     unsigned int* ticket) {
     const double g = sc.gam[k - 1], d = sc.del[k];
     if (*sc.stop || g == 0.0 || d == 0.0) {
-        if (blockIdx.x == 0 && threadIdx.x == 0) { *sc.stop = 1; sc.res2[k] = sc.res2[k - 1]; }
+        if (blockIdx.x == 0 && threadIdx.x == 0 && !*sc.stop) { *sc.stop = 1; *sc.stop_at = k; }
         return;
     }
     const double alpha = __ddiv_rn(g, d);
@@ -117,10 +119,7 @@ template <class T>
 __global__ void __launch_bounds__(kVT)
 cg_explicit_r_kernel(const T* __restrict__ y, const T* __restrict__ ax, T* __restrict__ r, int64_t nr,
                      Scal sc, int32_t k, double* part, unsigned int* ticket) {
-    if (*sc.stop) {
-        if (blockIdx.x == 0 && threadIdx.x == 0) sc.res2[k] = sc.res2[k - 1];
-        return;
-    }
+    if (*sc.stop) return;
     double acc = 0.0;
     for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < nr; i += (int64_t)gridDim.x * kVT) {
         const T v = y[i] - ax[i];
@@ -156,28 +155,45 @@ unsigned vec_blocks(int64_t n) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(kVecBlocks, ceil_div(n, kVT)));
 }
 
-// SpMV followed by the dot product of its output.  Canonical mode fuses the dot into the
+// Projection followed by the dot product of its output.  Canonical mode fuses the dot into the
 // SpMV epilogue (per-partition fma chains, reading R16).  Otherwise a separate small dot kernel
 // is used: measured on B200, the fused last-CTA epilogue slowed the 2 ms SpMV by ~0.5 ms
 // (profiles/r01a_launches.md), while the separate pass over the 4-6 MB vector costs a few us.
+// P > 1: the projection includes the exchange (A = R C A_p), and the local dot is allreduced.
 template <class T>
-void spmv_dir(Plan& P, const Layout& L, const T* in, T* out, double* dot_out, cudaStream_t st) {
-    double* part = (&L == &P.fwd) ? P.part_fwd.p() : P.part_back.p();
-    const bool fused = dot_out && (P.opt.canonical != 0 || P.fused_dot);
-    if constexpr (sizeof(T) == 4)
-        spmv_f32(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), st);
-    else
-        spmv_f64(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), P.opt.canonical != 0, st);
-    if (dot_out && !fused) {
-        dot_kernel<T><<<vec_blocks(L.nrows), kVT, 0, st>>>(out, L.nrows, dot_out, P.part_vec.p(),
-                                                           P.tickets.p() + 2);
-        MX_LAUNCHED();
+void op_dir(Plan& P, bool forward, const T* in, T* out, double* dot_out, cudaStream_t st) {
+    const Layout& L = forward ? P.fwd : P.back;
+    if (P.nranks == 1) {
+        double* part = forward ? P.part_fwd.p() : P.part_back.p();
+        const bool fused = dot_out && (P.opt.canonical != 0 || P.fused_dot);
+        if constexpr (sizeof(T) == 4)
+            spmv_f32(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), st);
+        else
+            spmv_f64(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), P.opt.canonical != 0, st);
+        if (dot_out && !fused) {
+            dot_kernel<T><<<vec_blocks(L.nrows), kVT, 0, st>>>(out, L.nrows, dot_out, P.part_vec.p(),
+                                                               P.tickets.p() + 2);
+            MX_LAUNCHED();
+        }
+        return;
     }
+    if (forward) apply_forward(P, in, out, st);
+    else apply_back(P, in, out, st);
+    if (dot_out) {
+        const int64_t n = P.local_len(forward ? 1 : 0);
+        dot_kernel<T><<<vec_blocks(n), kVT, 0, st>>>(out, n, dot_out, P.part_vec.p(), P.tickets.p() + 2);
+        MX_LAUNCHED();
+        P.comm->allreduce_sum(dot_out, 1, DType::F64, st);
+    }
+}
+
+void allreduce_scalar(Plan& P, double* v, cudaStream_t st) {
+    if (P.nranks > 1) P.comm->allreduce_sum(v, 1, DType::F64, st);
 }
 
 template <class T>
 void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, cudaStream_t st) {
-    const int64_t nx = P.back.nrows, nr = P.fwd.nrows;
+    const int64_t nx = P.local_len(0), nr = P.local_len(1);
     T* r = P.cg_r.as<T>();
     T* q = P.cg_q.as<T>();
     T* s = P.cg_s.as<T>();
@@ -189,31 +205,38 @@ void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, cudaStream_t st) {
     const unsigned gb = vec_blocks(std::max(nx, nr));
     cg_init_kernel<T><<<gb, kVT, 0, st>>>(y, r, nr, x, nx, sc, vpart, tick);
     MX_LAUNCHED();
-    spmv_dir<T>(P, P.back, r, s, sc.gam, st);                  // s = A^T r, gamma_0
+    allreduce_scalar(P, sc.res2, st);
+    op_dir<T>(P, false, r, s, sc.gam, st);                      // s = A^T r, gamma_0
     copy_kernel<T><<<vec_blocks(nx), kVT, 0, st>>>(s, p, nx);  // p = s
     MX_LAUNCHED();
     for (int32_t k = 1; k <= iters; ++k) {
-        spmv_dir<T>(P, P.fwd, p, q, sc.del + k, st);           // q = A p, delta_k
+        op_dir<T>(P, true, p, q, sc.del + k, st);               // q = A p, delta_k
         if (P.opt.cg_variant == 1) {
             cg_update_xr_kernel<T, false><<<vec_blocks(nx), kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k, vpart, tick);
             MX_LAUNCHED();
-            spmv_dir<T>(P, P.fwd, x, ax, nullptr, st);           // ax = A x
+            op_dir<T>(P, true, x, ax, nullptr, st);              // ax = A x
             cg_explicit_r_kernel<T><<<vec_blocks(nr), kVT, 0, st>>>(y, ax, r, nr, sc, k, vpart, tick);
             MX_LAUNCHED();
         } else {
             cg_update_xr_kernel<T, true><<<gb, kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k, vpart, tick);
             MX_LAUNCHED();
         }
-        spmv_dir<T>(P, P.back, r, s, sc.gam + k, st);          // s = A^T r, gamma_k
+        allreduce_scalar(P, sc.res2 + k, st);
+        op_dir<T>(P, false, r, s, sc.gam + k, st);              // s = A^T r, gamma_k
         cg_update_p_kernel<T><<<vec_blocks(nx), kVT, 0, st>>>(p, s, nx, sc, k);
         MX_LAUNCHED();
     }
 }
 
+void cg_enqueue_any(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
+    if (P.esize == 4) cg_enqueue<float>(P, (const float*)y, (float*)x, iters, st);
+    else cg_enqueue<double>(P, (const double*)y, (double*)x, iters, st);
+}
+
 }  // namespace
 
 void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
-    const int64_t nx = P.back.nrows, nr = P.fwd.nrows;
+    const int64_t nx = P.local_len(0), nr = P.local_len(1);
     if (!P.cg_r.get()) {
         P.cg_r.alloc(P.esize * std::max<int64_t>(nr, 1));
         P.cg_q.alloc(P.esize * std::max<int64_t>(nr, 1));
@@ -233,6 +256,10 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
         MX_CUDA(cudaMemsetAsync(P.scal.p(), 0, 8 * (3 * ((int64_t)iters + 1) + 1), st));
         P.scal_iters = iters;
     }
+    if (P.nranks > 1 && !P.comm->capturable()) {  // virtual ranks: eager launches
+        cg_enqueue_any(P, y, x, iters, st);
+        return;
+    }
     auto key = std::make_tuple(y, x, iters, st);
     auto it = P.graphs.find(key);
     if (it == P.graphs.end()) {
@@ -244,8 +271,7 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
         MX_CUDA(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
         const int64_t before = launch_count();
         try {
-            if (P.esize == 4) cg_enqueue<float>(P, (const float*)y, (float*)x, iters, cap);
-            else cg_enqueue<double>(P, (const double*)y, (double*)x, iters, cap);
+            cg_enqueue_any(P, y, x, iters, cap);
         } catch (...) {
             cudaStreamEndCapture(cap, &g);
             if (g) cudaGraphDestroy(g);
@@ -269,10 +295,15 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
 }
 
 void cg_fetch_norms(Plan& P, int32_t iters, double* out, cudaStream_t st) {
-    const Scal sc = scal_of(P, P.scal_iters);
+    const Scal sc = scal_of(P, (int32_t)P.scal_iters);
+    int stop_at = 0;
     MX_CUDA(cudaMemcpyAsync(out, sc.res2, 8 * ((int64_t)iters + 1), cudaMemcpyDeviceToHost, st));
+    MX_CUDA(cudaMemcpyAsync(&stop_at, sc.stop_at, sizeof(int), cudaMemcpyDeviceToHost, st));
     MX_CUDA(cudaStreamSynchronize(st));
-    for (int32_t k = 0; k <= iters; ++k) out[k] = std::sqrt(out[k]);
+    for (int32_t k = 0; k <= iters; ++k) {
+        if (k >= stop_at) out[k] = out[k - 1];  // iterations that did not run repeat the last norm
+        else out[k] = std::sqrt(out[k]);
+    }
 }
 
 }  // namespace mx

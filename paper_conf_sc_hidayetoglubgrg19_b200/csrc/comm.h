@@ -1,0 +1,64 @@
+// comm.h -- the multi-GPU transport of the domain decomposition A = R C A_p.
+//
+// Two implementations of one interface:
+//   * NcclComm  -- one process per GPU; NCCL (dlopen'ed libnccl.so.2) grouped ncclSend/ncclRecv
+//                  as the sparse all-to-allv of P:731-756, ncclAllReduce for CG dot products.
+//                  All calls are stream-ordered and CUDA-graph capturable.
+//   * LocalComm -- P "virtual ranks" (plans) in one process on one device, one host thread
+//                  each; the same collectives done with device-to-device copies and a small
+//                  device reduction kernel.  A test shim: it lets the whole multi-rank path run
+//                  and be checked against the oracle on a single GPU.  Not graph-capturable.
+#pragma once
+
+#include <condition_variable>
+#include <memory>
+#include <mutex>
+#include <vector>
+
+#include "common.h"
+
+namespace mx {
+
+enum class DType { I32, I64, F32, F64 };
+size_t dtype_size(DType t);
+
+class Comm {
+public:
+    virtual ~Comm() = default;
+    int rank = 0, nranks = 1;
+    virtual bool capturable() const = 0;
+    // in-place elementwise sum over ranks (device buffer)
+    virtual void allreduce_sum(void* buf, int64_t count, DType t, cudaStream_t st) = 0;
+    // sparse all-to-allv: to peer q send `scount[q]` elements at send + sdispl[q], from peer q
+    // receive `rcount[q]` elements into recv + rdispl[q] (host count/displacement arrays).
+    virtual void alltoallv(const void* send, const int64_t* scount, const int64_t* sdispl, void* recv,
+                           const int64_t* rcount, const int64_t* rdispl, DType t, cudaStream_t st) = 0;
+    // gather one int64 per rank on the host (build-time bookkeeping)
+    virtual std::vector<int64_t> allgather_host(int64_t v, cudaStream_t st) = 0;
+};
+
+std::unique_ptr<Comm> make_nccl_comm(int rank, int nranks, const void* unique_id);
+void nccl_unique_id(void* out);
+
+// shared state of a group of virtual ranks
+struct LocalGroup {
+    explicit LocalGroup(int n) : nranks(n), posts(n) {}
+    int nranks;
+    std::mutex mu;
+    std::condition_variable cv;
+    int arrived = 0;
+    int64_t generation = 0;
+    struct Post {
+        const void* send = nullptr;
+        const int64_t* sdispl = nullptr;
+        const int64_t* scount = nullptr;
+        void* buf = nullptr;
+        int64_t value = 0;
+    };
+    std::vector<Post> posts;
+    void barrier();
+};
+
+std::unique_ptr<Comm> make_local_comm(std::shared_ptr<LocalGroup> g, int rank);
+
+}  // namespace mx

@@ -1,0 +1,262 @@
+// exchange.cu -- domain decomposition over P GPUs (sec. 3.4, Table 1):
+//   a3  both domains split into contiguous Hilbert tile ranges balanced on nonzeros;
+//   a6  exchange maps of the sparse communication;
+//   a8  forward  y = R C A_p x: partial projection on the footprint rays, all-to-allv of the
+//       partials to the ray owners, reduction in fixed peer order;
+//   a9  back     x = A_p^T C^T R^T y: owners duplicate their ray values to every interacting
+//       rank (the transposed communication), then the partial backprojection.
+// The footprint rays of a rank are kept in Hilbert order; since ray ownership is a contiguous
+// Hilbert range, that is also (owner, Hilbert) order, so the forward partials bound for each
+// owner are one contiguous slice of the SpMV output (zero-copy send), and the backprojection
+// receives straight into the same slices.
+#include <cub/device/device_segmented_reduce.cuh>
+
+#include <algorithm>
+#include <vector>
+
+#include "comm.h"
+#include "plan.h"
+
+namespace mx {
+
+std::vector<int64_t> partition_ranges(const std::vector<int64_t>& w, int32_t parts) {
+    const int64_t k = (int64_t)w.size();
+    std::vector<int64_t> pre(k + 1, 0);
+    for (int64_t i = 0; i < k; ++i) pre[i + 1] = pre[i] + w[i];
+    const int64_t total = pre[k];
+    std::vector<int64_t> b(parts + 1, 0);
+    b[parts] = k;
+    for (int32_t g = 1; g < parts; ++g) {
+        // first boundary whose prefix reaches g/P of the total (ties: the nearer of the two)
+        const int64_t target = (int64_t)((long double)total * g / parts + 0.5L);
+        int64_t i = std::lower_bound(pre.begin(), pre.end(), target) - pre.begin();
+        if (i > 0 && i <= k && (target - pre[i - 1]) < (pre[i] - target)) --i;
+        i = std::max(i, b[g - 1]);
+        if (k >= parts) i = std::max<int64_t>(i, b[g - 1] + 1);       // every rank gets a tile
+        if (k >= parts) i = std::min<int64_t>(i, k - (parts - g));
+        b[g] = std::min(i, k);
+    }
+    return b;
+}
+
+namespace {
+
+constexpr int kT = 256;
+
+unsigned nblocks(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 1 << 20)); }
+
+template <class T>
+__global__ void reduce_kernel(const T* __restrict__ recv, const int64_t* __restrict__ ptr,
+                              const int32_t* __restrict__ pos, int64_t nown, T* __restrict__ y) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nown; i += (int64_t)gridDim.x * blockDim.x) {
+        T acc = T(0);
+        for (int64_t k = ptr[i]; k < ptr[i + 1]; ++k) acc += recv[pos[k]];  // peer order
+        y[i] = acc;
+    }
+}
+
+template <class T>
+__global__ void pack_kernel(const T* __restrict__ y, const int32_t* __restrict__ idx, int64_t n, T* __restrict__ out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = y[idx[i]];
+}
+
+__global__ void flag_kernel(const int32_t* __restrict__ len, int64_t n, int32_t* __restrict__ flag) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        flag[i] = len[i] > 0;
+}
+
+__global__ void compact_kernel(const int32_t* __restrict__ len, const int64_t* __restrict__ pos, int64_t n,
+                               int32_t* __restrict__ fp_rays, int32_t* __restrict__ fp_len) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        if (len[i] > 0) {
+            fp_rays[pos[i]] = (int32_t)i;
+            fp_len[pos[i]] = len[i];
+        }
+}
+
+std::vector<int64_t> tile_sums(const int32_t* w, const std::vector<int64_t>& tile_off, cudaStream_t st) {
+    const int64_t nt = (int64_t)tile_off.size() - 1;
+    DevArr<int64_t> off, out;
+    off.alloc(nt + 1);
+    out.alloc(nt);
+    MX_CUDA(cudaMemcpyAsync(off.p(), tile_off.data(), 8 * (nt + 1), cudaMemcpyHostToDevice, st));
+    size_t tb = 0;
+    MX_CUDA(cub::DeviceSegmentedReduce::Sum(nullptr, tb, w, out.p(), nt, off.p(), off.p() + 1, st));
+    DevBuf tmp(tb);
+    MX_CUDA(cub::DeviceSegmentedReduce::Sum(tmp.get(), tb, w, out.p(), nt, off.p(), off.p() + 1, st));
+    MX_LAUNCHED();
+    std::vector<int64_t> h(nt);
+    MX_CUDA(cudaMemcpyAsync(h.data(), out.p(), 8 * nt, cudaMemcpyDeviceToHost, st));
+    MX_CUDA(cudaStreamSynchronize(st));
+    return h;
+}
+
+}  // namespace
+
+// a3: tomogram and sinogram ranges of this rank
+void decompose(Plan& P, const Geometry& G, cudaStream_t st) {
+    const int64_t npix = (int64_t)P.n * P.n, nrays = (int64_t)P.m * P.c;
+    if (P.nranks == 1) {
+        P.t0 = 0; P.t1 = npix; P.s0 = 0; P.s1 = nrays;
+        P.tomo_bounds = {0, npix};
+        P.sino_bounds = {0, nrays};
+        return;
+    }
+    Comm& C = *P.comm;
+    // per-pixel nonzeros (column counts of A): each rank traces 1/P of the rays, then allreduce
+    DevArr<int32_t> hist;
+    hist.alloc(npix);
+    MX_CUDA(cudaMemsetAsync(hist.p(), 0, 4 * npix, st));
+    trace_hist(P, G, nrays * P.rank / P.nranks, nrays * (P.rank + 1) / P.nranks, hist.p(), st);
+    C.allreduce_sum(hist.p(), npix, DType::I32, st);
+    const auto tw = tile_sums(hist.p(), P.tomo_tile_off, st);
+    hist.reset();
+    // per-ray nonzeros (row lengths of A)
+    DevArr<int32_t> rl;
+    rl.alloc(nrays);
+    trace_count(P, G, nullptr, nrays, 0, 0, false, rl.p(), st);
+    const auto sw = tile_sums(rl.p(), P.sino_tile_off, st);
+    const auto bt = partition_ranges(tw, P.nranks), bs = partition_ranges(sw, P.nranks);
+    P.tomo_bounds.resize(P.nranks + 1);
+    P.sino_bounds.resize(P.nranks + 1);
+    for (int g = 0; g <= P.nranks; ++g) {
+        P.tomo_bounds[g] = P.tomo_tile_off[bt[g]];
+        P.sino_bounds[g] = P.sino_tile_off[bs[g]];
+    }
+    P.t0 = P.tomo_bounds[P.rank];
+    P.t1 = P.tomo_bounds[P.rank + 1];
+    P.s0 = P.sino_bounds[P.rank];
+    P.s1 = P.sino_bounds[P.rank + 1];
+}
+
+// footprint rays of the local tomogram subdomain (all rays at P = 1) and their row lengths
+int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStream_t st) {
+    const int64_t nrays = (int64_t)P.m * P.c;
+    if (P.nranks == 1) {
+        fp_len.alloc(nrays);
+        trace_count(P, G, nullptr, nrays, 0, 0, false, fp_len.p(), st);
+        P.fp_rays.reset();
+        return nrays;
+    }
+    DevArr<int32_t> len;
+    len.alloc(nrays);
+    trace_count(P, G, nullptr, nrays, P.t0, P.t1, true, len.p(), st);
+    DevArr<int32_t> flag;
+    DevArr<int64_t> flag64, pos;
+    flag.alloc(nrays);
+    flag64.alloc(nrays + 1);
+    pos.alloc(nrays + 1);
+    flag_kernel<<<nblocks(nrays), kT, 0, st>>>(len.p(), nrays, flag.p());
+    MX_LAUNCHED();
+    widen_i32_to_i64(flag.p(), flag64.p(), nrays, st);
+    MX_CUDA(cudaMemsetAsync(flag64.p() + nrays, 0, 8, st));
+    exclusive_scan_i64(flag64.p(), pos.p(), nrays + 1, st);
+    int64_t nfp = 0;
+    MX_CUDA(cudaMemcpyAsync(&nfp, pos.p() + nrays, 8, cudaMemcpyDeviceToHost, st));
+    MX_CUDA(cudaStreamSynchronize(st));
+    P.fp_rays.alloc(std::max<int64_t>(nfp, 1));
+    fp_len.alloc(std::max<int64_t>(nfp, 1));
+    compact_kernel<<<nblocks(nrays), kT, 0, st>>>(len.p(), pos.p(), nrays, P.fp_rays.p(), fp_len.p());
+    MX_LAUNCHED();
+    MX_CUDA(cudaStreamSynchronize(st));
+    return nfp;
+}
+
+// a6: exchange maps (P > 1)
+void build_exchange(Plan& P, cudaStream_t st) {
+    if (P.nranks == 1) return;
+    Comm& C = *P.comm;
+    Exchange& X = P.ex;
+    const int np = P.nranks;
+    std::vector<int32_t> fp(P.nfp);
+    if (P.nfp > 0) MX_CUDA(cudaMemcpy(fp.data(), P.fp_rays.p(), 4 * P.nfp, cudaMemcpyDeviceToHost));
+    X.sdispl.assign(np + 1, 0);
+    for (int h = 0; h <= np; ++h)
+        X.sdispl[h] = std::lower_bound(fp.begin(), fp.end(), (int32_t)std::min<int64_t>(P.sino_bounds[h], INT32_MAX)) - fp.begin();
+    X.sdispl[np] = P.nfp;
+    X.scount.assign(np, 0);
+    for (int h = 0; h < np; ++h) X.scount[h] = X.sdispl[h + 1] - X.sdispl[h];
+    X.rcount.assign(np, 0);
+    for (int h = 0; h < np; ++h) {
+        const auto v = C.allgather_host(X.scount[h], st);  // v[q] = what rank q sends to owner h
+        if (h == P.rank) X.rcount = v;
+    }
+    X.rdispl.assign(np + 1, 0);
+    for (int q = 0; q < np; ++q) X.rdispl[q + 1] = X.rdispl[q] + X.rcount[q];
+    X.nrecv = X.rdispl[np];
+    // index lists: owned-local index of each footprint ray, by owner
+    std::vector<int32_t> idx(std::max<int64_t>(P.nfp, 1));
+    for (int h = 0; h < np; ++h)
+        for (int64_t i = X.sdispl[h]; i < X.sdispl[h + 1]; ++i) idx[i] = (int32_t)(fp[i] - P.sino_bounds[h]);
+    DevArr<int32_t> send_idx;
+    send_idx.alloc(std::max<int64_t>(P.nfp, 1));
+    MX_CUDA(cudaMemcpy(send_idx.p(), idx.data(), 4 * P.nfp, cudaMemcpyHostToDevice));
+    X.recv_idx.alloc(std::max<int64_t>(X.nrecv, 1));
+    C.alltoallv(send_idx.p(), X.scount.data(), X.sdispl.data(), X.recv_idx.p(), X.rcount.data(), X.rdispl.data(),
+                DType::I32, st);
+    MX_CUDA(cudaStreamSynchronize(st));
+    // reduction map R: for every owned ray, its received partials in peer order (stable sort)
+    const int64_t nown = P.s1 - P.s0;
+    DevArr<uint32_t> keys_out, perm;
+    keys_out.alloc(std::max<int64_t>(X.nrecv, 1));
+    perm.alloc(std::max<int64_t>(X.nrecv, 1));
+    if (X.nrecv > 0)
+        stable_sort_by_key(reinterpret_cast<const uint32_t*>(X.recv_idx.p()), keys_out.p(), perm.p(), X.nrecv,
+                           std::max<int64_t>(nown, 1), st);
+    X.red_ptr.alloc(nown + 1);
+    row_ptr_from_sorted(keys_out.p(), X.nrecv, nown, X.red_ptr.p(), st);
+    X.red_pos.alloc(std::max<int64_t>(X.nrecv, 1));
+    if (X.nrecv > 0)
+        MX_CUDA(cudaMemcpyAsync(X.red_pos.p(), perm.p(), 4 * X.nrecv, cudaMemcpyDeviceToDevice, st));
+    X.y_fp.alloc(P.esize * std::max<int64_t>(P.nfp, 1));
+    X.recv_buf.alloc(P.esize * std::max<int64_t>(X.nrecv, 1));
+    MX_CUDA(cudaStreamSynchronize(st));
+}
+
+template <class T>
+static void forward_t(Plan& P, const T* x, T* y, cudaStream_t st) {
+    if (P.nranks == 1) {
+        spmv_any(P, P.fwd, x, y, st);
+        return;
+    }
+    Exchange& X = P.ex;
+    T* yfp = X.y_fp.as<T>();
+    T* rb = X.recv_buf.as<T>();
+    spmv_any(P, P.fwd, x, yfp, st);                                         // A_p
+    P.comm->alltoallv(yfp, X.scount.data(), X.sdispl.data(), rb, X.rcount.data(), X.rdispl.data(),
+                      sizeof(T) == 4 ? DType::F32 : DType::F64, st);        // C
+    const int64_t nown = P.s1 - P.s0;
+    reduce_kernel<T><<<nblocks(nown), kT, 0, st>>>(rb, X.red_ptr.p(), X.red_pos.p(), nown, y);  // R
+    MX_LAUNCHED();
+}
+
+template <class T>
+static void back_t(Plan& P, const T* y, T* x, cudaStream_t st) {
+    if (P.nranks == 1) {
+        spmv_any(P, P.back, y, x, st);
+        return;
+    }
+    Exchange& X = P.ex;
+    T* yfp = X.y_fp.as<T>();
+    T* rb = X.recv_buf.as<T>();
+    if (X.nrecv > 0) {
+        pack_kernel<T><<<nblocks(X.nrecv), kT, 0, st>>>(y, X.recv_idx.p(), X.nrecv, rb);   // R^T
+        MX_LAUNCHED();
+    }
+    P.comm->alltoallv(rb, X.rcount.data(), X.rdispl.data(), yfp, X.scount.data(), X.sdispl.data(),
+                      sizeof(T) == 4 ? DType::F32 : DType::F64, st);        // C^T
+    spmv_any(P, P.back, yfp, x, st);                                        // A_p^T
+}
+
+void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st) {
+    if (P.esize == 4) forward_t<float>(P, (const float*)x, (float*)y, st);
+    else forward_t<double>(P, (const double*)x, (double*)y, st);
+}
+
+void apply_back(Plan& P, const void* y, void* x, cudaStream_t st) {
+    if (P.esize == 4) back_t<float>(P, (const float*)y, (float*)x, st);
+    else back_t<double>(P, (const double*)y, (double*)x, st);
+}
+
+}  // namespace mx

@@ -143,7 +143,7 @@ int32_t default_tile(int32_t h, int32_t w) {
 }
 
 void build_hilbert(int32_t H, int32_t W, int32_t T, int32_t* nat_of_h, int32_t* h_of_nat,
-                   cudaStream_t st) {
+                   std::vector<int64_t>* tile_off, cudaStream_t st) {
     if (T < 1 || T > 128 || (T & (T - 1))) fail(MEMXCT_ERR_INVALID_ARG, "tile side must be a power of two in [1, 128]");
     const int32_t rt = (H + T - 1) / T, ct = (W + T - 1) / T;
     std::vector<int32_t> tx, ty;
@@ -186,6 +186,10 @@ void build_hilbert(int32_t H, int32_t W, int32_t T, int32_t* nat_of_h, int32_t* 
     MX_CUDA(cudaMemcpyAsync(dty.p(), ty.data(), nt * 4, cudaMemcpyHostToDevice, st));
     MX_CUDA(cudaMemcpyAsync(dor.p(), orient.data(), nt, cudaMemcpyHostToDevice, st));
     MX_CUDA(cudaMemcpyAsync(doff.p(), off.data(), nt * 8, cudaMemcpyHostToDevice, st));
+    if (tile_off) {
+        *tile_off = off;
+        tile_off->push_back(acc);
+    }
     hilbert_cells_kernel<<<(unsigned)nt, kHilThreads, 0, st>>>(H, W, T, dtx.p(), dty.p(), dor.p(),
                                                                 doff.p(), nat_of_h, h_of_nat);
     MX_LAUNCHED();

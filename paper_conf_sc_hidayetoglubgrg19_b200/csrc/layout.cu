@@ -246,6 +246,14 @@ template <class T> T read_scalar(const T* dptr, cudaStream_t st) {
     return v;
 }
 
+int bits_for(int64_t n) {
+    int b = 1;
+    while (b < 32 && ((int64_t)1 << b) < n) ++b;
+    return b;
+}
+
+}  // namespace
+
 void exclusive_scan_i64(const int64_t* in, int64_t* out, int64_t n, cudaStream_t st) {
     size_t tb = 0;
     MX_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, in, out, n, st));
@@ -255,10 +263,15 @@ void exclusive_scan_i64(const int64_t* in, int64_t* out, int64_t n, cudaStream_t
     MX_CUDA(cudaStreamSynchronize(st));
 }
 
-int bits_for(int64_t n) {
-    int b = 1;
-    while (b < 32 && ((int64_t)1 << b) < n) ++b;
-    return b;
+void widen_i32_to_i64(const int32_t* in, int64_t* out, int64_t n, cudaStream_t st) {
+    if (n == 0) return;
+    widen_kernel<<<blocks_for(n), kThreads, 0, st>>>(in, out, n);
+    MX_LAUNCHED();
+}
+
+void row_ptr_from_sorted(const uint32_t* row_ids, int64_t nnz, int64_t nrows, int64_t* row_ptr, cudaStream_t st) {
+    row_ptr_kernel<<<blocks_for(nrows + 1), kThreads, 0, st>>>(row_ids, nnz, nrows, row_ptr);
+    MX_LAUNCHED();
 }
 
 // stable radix sort of (key, index) pairs: perm_out[i] = original index of the i-th smallest key
@@ -276,8 +289,6 @@ void stable_sort_by_key(const uint32_t* keys_in, uint32_t* keys_out, uint32_t* p
     MX_LAUNCHED();
     MX_CUDA(cudaStreamSynchronize(st));
 }
-
-}  // namespace
 
 void build_layout(Layout& L, int64_t nrows, int64_t ncols, int64_t nnz, const uint32_t* row_ids,
                   const uint32_t* cols, const float* vals, int32_t R, int32_t B,
@@ -419,7 +430,6 @@ void build_layout(Layout& L, int64_t nrows, int64_t ncols, int64_t nnz, const ui
 }
 
 void build_matrices(Plan& P, cudaStream_t st) {
-    const int64_t nrays = (int64_t)P.m * P.c, npix = (int64_t)P.n * P.n;
     // angle tables (reading R1), the same expression as the paper's geometry in DESIGN.md
     std::vector<double> hc(P.m), hs(P.m);
     for (int32_t m = 0; m < P.m; ++m) {
@@ -432,43 +442,49 @@ void build_matrices(Plan& P, cudaStream_t st) {
     ds.alloc(P.m);
     MX_CUDA(cudaMemcpyAsync(dc.p(), hc.data(), 8 * P.m, cudaMemcpyHostToDevice, st));
     MX_CUDA(cudaMemcpyAsync(ds.p(), hs.data(), 8 * P.m, cudaMemcpyHostToDevice, st));
+    Geometry G;
+    G.cos_t = dc.p();
+    G.sin_t = ds.p();
 
-    // 1. count pass + scan
+    // a3: this rank's tomogram and sinogram subdomains (whole domains at P = 1)
+    decompose(P, G, st);
+    const int64_t npix = P.t1 - P.t0;
+
+    // 1. rows of A_p = footprint rays (every ray at P = 1), count pass + scan
     DevArr<int32_t> row_len;
-    row_len.alloc(nrays);
-    trace_count(P, dc.p(), ds.p(), nrays, row_len.p(), st);
+    const int64_t nrows = P.nfp = footprint(P, G, row_len, st);
     DevArr<int64_t> len64, row_ptr;
-    len64.alloc(nrays + 1);
-    row_ptr.alloc(nrays + 1);
-    widen_kernel<<<blocks_for(nrays), kThreads, 0, st>>>(row_len.p(), len64.p(), nrays);
-    MX_LAUNCHED();
-    MX_CUDA(cudaMemsetAsync(len64.p() + nrays, 0, 8, st));
-    exclusive_scan_i64(len64.p(), row_ptr.p(), nrays + 1, st);
+    len64.alloc(nrows + 1);
+    row_ptr.alloc(nrows + 1);
+    widen_i32_to_i64(row_len.p(), len64.p(), nrows, st);
+    MX_CUDA(cudaMemsetAsync(len64.p() + nrows, 0, 8, st));
+    exclusive_scan_i64(len64.p(), row_ptr.p(), nrows + 1, st);
     len64.reset();
     row_len.reset();
-    const int64_t nnz = read_scalar(row_ptr.p() + nrays, st);
+    const int64_t nnz = read_scalar(row_ptr.p() + nrows, st);
     if (nnz >= ((int64_t)1 << 32))
         fail(MEMXCT_ERR_UNSUPPORTED, "nnz >= 2^32 on one GPU; shard the problem over more GPUs");
 
-    // 2. emit (Hilbert pixel, length, Hilbert ray)
+    // 2. emit (local Hilbert pixel, length, row) for the segments inside this rank's pixels
     DevArr<uint32_t> a_col, a_row;
     DevArr<float> a_val;
     a_col.alloc(nnz);
     a_row.alloc(nnz);
     a_val.alloc(nnz);
-    trace_emit(P, dc.p(), ds.p(), nrays, row_ptr.p(), a_col.p(), a_val.p(), a_row.p(), st);
+    trace_emit(P, G, P.nranks == 1 ? nullptr : P.fp_rays.p(), nrows, P.t0, P.t1, row_ptr.p(), a_col.p(),
+               a_val.p(), a_row.p(), st);
     row_ptr.reset();
 
-    const bool natural = (P.opt.vector_order == 0);
+    const bool natural = (P.opt.vector_order == 0);  // P = 1 only
     const int32_t R = P.part_rows;
     const int32_t B = P.opt.precision == 1 ? P.buffer_entries / 2 : P.buffer_entries;
 
-    // 3. A^T: stable sort by pixel (order-preserving transposition)
+    // 3. A_p^T: stable sort by pixel (order-preserving transposition)
     DevArr<uint32_t> t_row, t_col, perm;
     DevArr<float> t_val;
     t_row.alloc(nnz);
     perm.alloc(nnz);
-    stable_sort_by_key(a_col.p(), t_row.p(), perm.p(), nnz, npix, st);
+    stable_sort_by_key(a_col.p(), t_row.p(), perm.p(), nnz, std::max<int64_t>(npix, 1), st);
     a_col.reset();
     t_col.alloc(nnz);
     t_val.alloc(nnz);
@@ -478,15 +494,15 @@ void build_matrices(Plan& P, cudaStream_t st) {
     a_row.reset();
     a_val.reset();
     perm.reset();
-    build_layout(P.back, npix, nrays, nnz, t_row.p(), t_col.p(), t_val.p(), R, B,
+    build_layout(P.back, npix, nrows, nnz, t_row.p(), t_col.p(), t_val.p(), R, B,
                  natural ? P.sino_nat_of_h.p() : nullptr, natural ? P.tomo_nat_of_h.p() : nullptr, st);
 
-    // 4. A with ascending pixels inside each ray: stable sort of the A^T entries by ray
+    // 4. A_p with ascending pixels inside each row: stable sort of the A_p^T entries by row
     DevArr<uint32_t> f_row, f_col;
     DevArr<float> f_val;
     f_row.alloc(nnz);
     perm.alloc(nnz);
-    stable_sort_by_key(t_col.p(), f_row.p(), perm.p(), nnz, nrays, st);
+    stable_sort_by_key(t_col.p(), f_row.p(), perm.p(), nnz, std::max<int64_t>(nrows, 1), st);
     t_col.reset();
     f_col.alloc(nnz);
     f_val.alloc(nnz);
@@ -496,8 +512,11 @@ void build_matrices(Plan& P, cudaStream_t st) {
     t_row.reset();
     t_val.reset();
     perm.reset();
-    build_layout(P.fwd, nrays, npix, nnz, f_row.p(), f_col.p(), f_val.p(), R, B,
+    build_layout(P.fwd, nrows, npix, nnz, f_row.p(), f_col.p(), f_val.p(), R, B,
                  natural ? P.tomo_nat_of_h.p() : nullptr, natural ? P.sino_nat_of_h.p() : nullptr, st);
+
+    // a6: exchange maps of the sparse all-to-allv (P > 1)
+    build_exchange(P, st);
 }
 
 }  // namespace mx

@@ -6,6 +6,7 @@
 #include <tuple>
 #include <vector>
 
+#include "comm.h"
 #include "common.h"
 
 namespace mx {
@@ -63,6 +64,28 @@ struct Options {
     int64_t vector_order = 0;  // 0 natural, 1 plan
 };
 
+// host-side angle tables on the device (reading R1)
+struct Geometry {
+    const double* cos_t = nullptr;
+    const double* sin_t = nullptr;
+};
+
+// sparse all-to-allv plan of this rank (P > 1)
+struct Exchange {
+    // forward: partials of footprint slice [sdispl[h], sdispl[h+1]) go to ray owner h;
+    // partials from peer q land in recv_buf[rdispl[q] .. + rcount[q]).  Back reverses both.
+    std::vector<int64_t> scount, sdispl, rcount, rdispl;
+    int64_t nrecv = 0;
+    DevArr<int32_t> recv_idx;  // owned-local ray of every received partial (peer order)
+    DevArr<int64_t> red_ptr;   // reduction map R: CSR over owned rays ...
+    DevArr<int32_t> red_pos;   // ... of positions in recv_buf, ascending peer order
+    DevBuf y_fp, recv_buf;     // footprint partials, receive / pack buffer
+    int64_t device_bytes() const {
+        return (int64_t)(recv_idx.buf.bytes() + red_ptr.buf.bytes() + red_pos.buf.bytes() + y_fp.bytes() +
+                         recv_buf.bytes());
+    }
+};
+
 struct CgGraph {
     cudaGraphExec_t exec = nullptr;
     int64_t nkernels = 0;
@@ -77,6 +100,17 @@ struct Plan {
     int32_t tile_tomo = 0, tile_sino = 0;
     bool fused_dot = false;  // MEMXCT_FUSED_DOT=1: fuse CG dots into the SpMV epilogue (tuning)
     int32_t part_rows = 0, buffer_entries = 0;  // resolved tuning (build)
+
+    // domain decomposition: this rank owns Hilbert pixels [t0, t1) and rays [s0, s1)
+    std::unique_ptr<Comm> comm;
+    std::shared_ptr<LocalGroup> local_group;
+    std::vector<uint8_t> unique_id;
+    int64_t t0 = 0, t1 = 0, s0 = 0, s1 = 0;
+    std::vector<int64_t> tomo_bounds, sino_bounds;      // per rank, Hilbert index ranges
+    std::vector<int64_t> tomo_tile_off, sino_tile_off;  // Hilbert offset of every tile (+ total)
+    int64_t nfp = 0;                                    // footprint rays (rows of A_p)
+    DevArr<int32_t> fp_rays;                            // their Hilbert ray indices (P > 1)
+    Exchange ex;
 
     // two-level pseudo-Hilbert permutations, device int32
     DevArr<int32_t> tomo_nat_of_h, tomo_h_of_nat;  // N*N
@@ -96,27 +130,41 @@ struct Plan {
     DevBuf h_in, h_out;
     std::map<std::tuple<const void*, void*, int32_t, cudaStream_t>, std::unique_ptr<CgGraph>> graphs;
 
-    int64_t vec_len(int domain) const { return domain == 0 ? (int64_t)n * n : (int64_t)m * c; }
+    int64_t local_len(int domain) const { return domain == 0 ? t1 - t0 : s1 - s0; }
     int64_t device_bytes() const;
 };
 
 // hilbert.cu
 void build_hilbert(int32_t h, int32_t w, int32_t t, int32_t* nat_of_h, int32_t* h_of_nat,
-                   cudaStream_t st);
+                   std::vector<int64_t>* tile_off, cudaStream_t st);
 int32_t default_tile(int32_t h, int32_t w);
 
-// trace.cu: Siddon count / emit over rays listed in plan (Hilbert) order
-void trace_count(const Plan& P, const double* cos_t, const double* sin_t, int64_t nrays,
-                 int32_t* row_len, cudaStream_t st);
-void trace_emit(const Plan& P, const double* cos_t, const double* sin_t, int64_t nrays,
-                const int64_t* row_ptr, uint32_t* cols, float* vals, uint32_t* row_ids,
-                cudaStream_t st);
+// trace.cu: Siddon count / emit over rays (row r = Hilbert ray hray[r], or r if hray is null);
+// with `filter`, only segments in Hilbert pixels [lo, hi) count (emit writes pixel - lo)
+void trace_count(const Plan& P, const Geometry& G, const int32_t* hray, int64_t nrows, int64_t lo, int64_t hi,
+                 bool filter, int32_t* row_len, cudaStream_t st);
+void trace_emit(const Plan& P, const Geometry& G, const int32_t* hray, int64_t nrows, int64_t lo, int64_t hi,
+                const int64_t* row_ptr, uint32_t* cols, float* vals, uint32_t* row_ids, cudaStream_t st);
+void trace_hist(const Plan& P, const Geometry& G, int64_t r0, int64_t r1, int32_t* hist, cudaStream_t st);
 
 // layout.cu: staged SELL-32 layout from entries sorted by (row, col)
 void build_layout(Layout& L, int64_t nrows, int64_t ncols, int64_t nnz, const uint32_t* row_ids,
                   const uint32_t* cols, const float* vals, int32_t R, int32_t B,
                   const int32_t* in_translate, const int32_t* out_translate, cudaStream_t st);
 void build_matrices(Plan& P, cudaStream_t st);
+void widen_i32_to_i64(const int32_t* in, int64_t* out, int64_t n, cudaStream_t st);
+void exclusive_scan_i64(const int64_t* in, int64_t* out, int64_t n, cudaStream_t st);
+void stable_sort_by_key(const uint32_t* keys_in, uint32_t* keys_out, uint32_t* perm_out, int64_t n,
+                        int64_t key_range, cudaStream_t st);
+void row_ptr_from_sorted(const uint32_t* row_ids, int64_t nnz, int64_t nrows, int64_t* row_ptr, cudaStream_t st);
+
+// exchange.cu: domain decomposition and the A = R C A_p operators
+std::vector<int64_t> partition_ranges(const std::vector<int64_t>& w, int32_t parts);
+void decompose(Plan& P, const Geometry& G, cudaStream_t st);
+int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStream_t st);
+void build_exchange(Plan& P, cudaStream_t st);
+void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
+void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);
 
 // spmv.cu
 void spmv_init();
@@ -124,6 +172,13 @@ void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, doubl
               unsigned int* ticket, cudaStream_t st);
 void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
               unsigned int* ticket, bool canonical, cudaStream_t st);
+
+inline void spmv_any(Plan&, const Layout& L, const float* in, float* out, cudaStream_t st) {
+    spmv_f32(L, in, out, nullptr, nullptr, nullptr, st);
+}
+inline void spmv_any(Plan&, const Layout& L, const double* in, double* out, cudaStream_t st) {
+    spmv_f64(L, in, out, nullptr, nullptr, nullptr, false, st);
+}
 
 // cg.cu
 void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st);

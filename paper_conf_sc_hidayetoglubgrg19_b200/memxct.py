@@ -29,6 +29,8 @@ SYMBOLS = [
     "memxct_forward_host", "memxct_back_host", "memxct_cg_host", "memxct_stats",
     "memxct_layout_info", "memxct_layout_export", "memxct_plan_destroy",
     "memxct_status_string", "memxct_last_error", "memxct_kernel_launch_count",
+    "memxct_local_group_create", "memxct_local_group_destroy", "memxct_plan_set_comm_local",
+    "memxct_partition_ranges", "memxct_domain_ranges", "memxct_exchange_info",
 ]
 
 
@@ -70,6 +72,12 @@ def lib():
             "memxct_layout_info": [vp, i32, P64, P64, P64, P64, P64, P64],
             "memxct_layout_export": [vp, i32, i64, i64, vp, vp, vp, vp, vp, vp, vp, P64, P64, P64],
             "memxct_plan_destroy": [vp],
+            "memxct_local_group_create": [i32, ctypes.POINTER(vp)],
+            "memxct_local_group_destroy": [vp],
+            "memxct_plan_set_comm_local": [vp, vp, i32],
+            "memxct_partition_ranges": [vp, i64, i32, vp],
+            "memxct_domain_ranges": [vp, i32, vp],
+            "memxct_exchange_info": [vp, P64, P64, P64, ctypes.POINTER(i32)],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -111,6 +119,46 @@ def get_unique_id() -> bytes:
     return buf.raw
 
 
+def partition_ranges(weights, parts: int) -> np.ndarray:
+    """Host helper of the domain decomposition (memxct_partition_ranges): contiguous ranges of
+    about equal weight; returns bounds[0..parts]."""
+    w = np.ascontiguousarray(weights, np.int64)
+    out = np.empty(parts + 1, np.int64)
+    _check(lib().memxct_partition_ranges(w.ctypes.data_as(ctypes.c_void_p), len(w), int(parts),
+                                         out.ctypes.data_as(ctypes.c_void_p)), "memxct_partition_ranges")
+    return out
+
+
+class LocalGroup:
+    """Virtual ranks in one process (memxct_local_group_create): P plans on one device, each
+    driven from its own thread, collectives done by device copies.  For testing the multi-GPU
+    path on a single GPU."""
+
+    def __init__(self, nranks: int):
+        self.nranks = int(nranks)
+        self._h = ctypes.c_void_p()
+        _check(lib().memxct_local_group_create(self.nranks, ctypes.byref(self._h)), "memxct_local_group_create")
+
+    def close(self):
+        if self._h and self._h.value:
+            lib().memxct_local_group_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def bootstrap_unique_id(rank: int, group=None) -> bytes:
+    """Rank 0 makes an ncclUniqueId; every rank receives it through torch.distributed."""
+    import torch.distributed as dist
+    obj = [get_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
 class MemXCT:
     """A MemXCT plan: geometry (N, M, C), options, built matrices, and the hot-path calls.
 
@@ -122,7 +170,7 @@ class MemXCT:
                  canonical: bool = False, vector_order: str = "natural", part_rows: int = None,
                  buffer_entries: int = None, tile_tomo: int = None, tile_sino: int = None,
                  cg_variant: int = 0, rank: int = 0, nranks: int = 1, unique_id: bytes = None,
-                 device: int = None):
+                 device: int = None, group: "LocalGroup" = None):
         self.n, self.m, self.c = int(n), int(projections), int(channels)
         self._h = ctypes.c_void_p()
         _check(lib().memxct_plan_create(self.n, self.m, self.c, ctypes.byref(self._h)),
@@ -135,7 +183,12 @@ class MemXCT:
         for k, v in opts.items():
             if v is not None:
                 self.set_option(k, v)
-        if nranks > 1 or device is not None:
+        self._group = group  # keep the virtual-rank group alive as long as the plan
+        self.rank = int(rank)
+        self.nranks = group.nranks if group is not None else int(nranks)
+        if group is not None:
+            _check(lib().memxct_plan_set_comm_local(self._h, group._h, int(rank)), "memxct_plan_set_comm_local")
+        elif nranks > 1 or device is not None:
             uid = None if unique_id is None else ctypes.create_string_buffer(unique_id, 128)
             _check(lib().memxct_plan_set_comm(self._h, rank, nranks, uid,
                                               -1 if device is None else int(device)),
@@ -188,6 +241,20 @@ class MemXCT:
         v = [ctypes.c_int64() for _ in range(4)]
         _check(lib().memxct_stats(self._h, *[ctypes.byref(x) for x in v]), "memxct_stats")
         return dict(zip(["nnz", "stored_slots", "map_entries", "device_bytes"], [x.value for x in v]))
+
+    def domain_ranges(self, domain: int) -> np.ndarray:
+        """Hilbert-index range boundaries of every rank for domain 0 (pixels) / 1 (rays)."""
+        out = np.empty(self.nranks + 1, np.int64)
+        _check(lib().memxct_domain_ranges(self._h, domain, out.ctypes.data_as(ctypes.c_void_p)),
+               "memxct_domain_ranges")
+        return out
+
+    def exchange_info(self) -> dict:
+        a, b, c = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        d = ctypes.c_int32()
+        _check(lib().memxct_exchange_info(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c),
+                                          ctypes.byref(d)), "memxct_exchange_info")
+        return {"footprint_rays": a.value, "sent": b.value, "received": c.value, "peers": d.value}
 
     def layout_info(self, direction: int) -> dict:
         v = [ctypes.c_int64() for _ in range(6)]

@@ -1,0 +1,134 @@
+"""Multi-GPU path (A = R C A_p) on ONE device through virtual ranks: P plans in one
+process, each driven from its own thread; the collectives are device copies instead of NCCL,
+everything else (decomposition, footprints, exchange maps, reduce-R, pack-R^T, kernels, CG) is
+the code NCCL ranks run.  Results are assembled through memxct_local_indices and compared with
+the single-GPU plan and the fp64 oracle."""
+import threading
+
+import numpy as np
+import pytest
+
+from conftest import rel_l2
+from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sc_hidayetoglubgrg19_b200 import build_ext
+    build_ext.build()
+
+
+def run_ranks(nranks, fn):
+    out, err = [None] * nranks, [None] * nranks
+
+    def body(r):
+        try:
+            with torch.cuda.stream(torch.cuda.Stream()):
+                out[r] = fn(r)
+                torch.cuda.current_stream().synchronize()
+        except BaseException as e:  # noqa: BLE001
+            err[r] = e
+    ts = [threading.Thread(target=body, args=(r,)) for r in range(nranks)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(timeout=600)
+    for e in err:
+        if e is not None:
+            raise e
+    return out
+
+
+def build_group(n, m, c, nranks, **kw):
+    from paper_conf_sc_hidayetoglubgrg19_b200 import LocalGroup, MemXCT
+    g = LocalGroup(nranks)
+    plans = run_ranks(nranks, lambda r: MemXCT(n, m, c, group=g, rank=r, vector_order="plan", **kw).build())
+    return g, plans
+
+
+def scatter(plans, vec, domain, dtype):
+    return [torch.from_numpy(np.ascontiguousarray(vec[p.local_indices(domain)]).astype(dtype)).cuda()
+            for p in plans]
+
+
+def gather(plans, parts, domain, size):
+    out = np.zeros(size)
+    for p, v in zip(plans, parts):
+        out[p.local_indices(domain)] = v.cpu().numpy()
+    return out
+
+
+@pytest.mark.parametrize("nranks", [2, 3, 4])
+@pytest.mark.parametrize("geom", [(64, 90, 64), (256, 360, 256)])
+def test_decomposition_and_fp32_projections(orc, coo_cache, nranks, geom):
+    n, m, c = geom
+    g, plans = build_group(n, m, c, nranks)
+    # both domains are covered exactly once, identically on every rank
+    for dom, size in ((0, n * n), (1, m * c)):
+        b = plans[0].domain_ranges(dom)
+        assert b[0] == 0 and b[-1] == size and np.all(np.diff(b) > 0)
+        for p in plans[1:]:
+            assert np.array_equal(p.domain_ranges(dom), b)
+        idx = np.concatenate([p.local_indices(dom) for p in plans])
+        assert np.array_equal(np.sort(idx), np.arange(size))
+    # nonzeros of A_p sum to nnz(A) and are balanced
+    rows, cols, vals = coo_cache(n, m, c)
+    nnz = [p.layout_info(0)["nnz"] for p in plans]
+    assert sum(nnz) == len(rows)
+    assert max(nnz) / np.mean(nnz) < 1.25, nnz
+    info = [p.exchange_info() for p in plans]
+    assert sum(i["sent"] for i in info) == sum(i["received"] for i in info)
+    # forward / back against the oracle
+    x = inputs.shepp_logan(n).astype(np.float32)
+    xs = scatter(plans, x, 0, np.float32)
+    ys = run_ranks(nranks, lambda r: plans[r].forward(xs[r]))
+    y = gather(plans, ys, 1, m * c)
+    y_orc = orc.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)
+    assert rel_l2(y, y_orc) <= 1e-5
+    yv = inputs.uniform(m * c, 7)
+    yss = scatter(plans, yv, 1, np.float32)
+    xb = run_ranks(nranks, lambda r: plans[r].back(yss[r]))
+    xbg = gather(plans, xb, 0, n * n)
+    x_orc = orc.spmv_coo(cols, rows, vals, yv.astype(np.float64), n * n)
+    assert rel_l2(xbg, x_orc) <= 1e-5
+
+
+@pytest.mark.parametrize("nranks", [2, 4])
+def test_mixed_projections_and_cg(orc, coo_cache, nranks):
+    n, m, c = 64, 90, 64
+    g, plans = build_group(n, m, c, nranks, precision="mixed")
+    rows, cols, vals = coo_cache(n, m, c)
+    v32 = vals.astype(np.float32).astype(np.float64)
+    x = inputs.normal(n * n, 3)
+    xs = scatter(plans, x, 0, np.float64)
+    y = gather(plans, run_ranks(nranks, lambda r: plans[r].forward(xs[r])), 1, m * c)
+    assert rel_l2(y, orc.spmv_coo(rows, cols, v32, x, m * c)) <= 1e-13
+    xt = inputs.shepp_logan(n)
+    ysino = orc.spmv_coo(rows, cols, vals, xt, m * c).astype(np.float32).astype(np.float64)
+    yss = scatter(plans, ysino, 1, np.float64)
+    res = run_ranks(nranks, lambda r: plans[r].cg(yss[r], 10, residuals=True))
+    xr = gather(plans, [r[0] for r in res], 0, n * n)
+    x_orc, res_orc, _, _ = orc.cgls(rows, cols, v32, ysino, m * c, n * n, 10)
+    assert rel_l2(xr, x_orc) <= 1e-6
+    for r in res:
+        assert np.allclose(r[1], res_orc, rtol=1e-9)
+
+
+def test_fp32_cg_multirank_recovers_phantom(orc, coo_cache):
+    n, m, c = 256, 360, 256
+    nranks = 4
+    g, plans = build_group(n, m, c, nranks)
+    rows, cols, vals = coo_cache(n, m, c)
+    xt = inputs.shepp_logan(n)
+    y32 = orc.spmv_coo(rows, cols, vals, xt, m * c).astype(np.float32)
+    yss = scatter(plans, y32, 1, np.float32)
+    res = run_ranks(nranks, lambda r: plans[r].cg(yss[r], 30, residuals=True))
+    xr = gather(plans, [r[0] for r in res], 0, n * n)
+    x_orc = orc.cgls(rows, cols, vals, y32.astype(np.float64), m * c, n * n, 30)[0]
+    assert rel_l2(xr, xt) <= 1.1 * rel_l2(x_orc, xt)
+    assert np.all(np.diff(res[0][1]) <= 1e-6 * res[0][1][0])
