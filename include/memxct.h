@@ -87,7 +87,11 @@ typedef enum {
      * 1 = explicit residual r = y - A x each iteration (2 forward + 1 back). */
     MEMXCT_OPT_CG_VARIANT = 6,
     /* 0 = natural row-major vectors (default, P = 1 only); 1 = plan (local Hilbert) order. */
-    MEMXCT_OPT_VECTOR_ORDER = 7
+    MEMXCT_OPT_VECTOR_ORDER = 7,
+    /* 1..8: slices per matrix stream the batched calls are tuned for (multi-slice reconstruction,
+     * P:943-947).  The automatic stage buffer becomes 36 * PART_ROWS / 2^ceil(log2(SLICES))
+     * entries so that many slices' inputs fit in shared memory.  Default 1. */
+    MEMXCT_OPT_SLICES = 8
 } memxct_option_t;
 
 /* Create a plan for an N x N tomogram and an M x C sinogram.  Host only; no device
@@ -164,6 +168,20 @@ memxct_status_t memxct_back(memxct_plan_t plan, const void* y_sino, void* x_tomo
  * writes zeros.  iters < 0 is INVALID_ARG. */
 memxct_status_t memxct_cg(memxct_plan_t plan, const void* y_sino, void* x_tomo, int32_t iters,
                           double* residual_norms, void* cuda_stream);
+
+/* Multi-slice variants (the paper reuses the memoized matrices for every
+ * slice): `slices` independent slices with the same geometry, vectors slice-major
+ * (x[s * local_size(0) + i], y[s * local_size(1) + r]), FP32 only.  The slices are processed in
+ * groups of up to 8 that share one stream of the matrix from HBM (an SpMM), each slice's
+ * arithmetic identical to the single-slice call (bit-identical results).  memxct_cg_batch runs
+ * `slices` (<= 32) independent CGLS solves; residual_norms (nullable) is [slices][iters + 1]. */
+memxct_status_t memxct_forward_batch(memxct_plan_t plan, int32_t slices, const void* x_tomo,
+                                     void* y_sino, void* cuda_stream);
+memxct_status_t memxct_back_batch(memxct_plan_t plan, int32_t slices, const void* y_sino,
+                                  void* x_tomo, void* cuda_stream);
+memxct_status_t memxct_cg_batch(memxct_plan_t plan, int32_t slices, const void* y_sino,
+                                void* x_tomo, int32_t iters, double* residual_norms,
+                                void* cuda_stream);
 
 /* Host-buffer variants: same semantics, HOST pointers; the H2D copy of the input, the device
  * computation and the D2H copy of the result all happen inside the call, which returns after

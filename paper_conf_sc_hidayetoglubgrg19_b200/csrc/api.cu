@@ -98,7 +98,11 @@ void resolve_tuning(mx::Plan& P) {
         }
     }
     int32_t B = (int32_t)P.opt.buffer_entries;
-    if (B == 0) B = std::min<int32_t>(57344, 36 * R);
+    if (B == 0) {
+        int32_t k = 1;
+        while (k < P.opt.slices) k *= 2;  // batched calls stage k slices per buffer entry
+        B = std::max<int32_t>(256, std::min<int32_t>(57344, 36 * R) / k);
+    }
     P.part_rows = R;
     P.buffer_entries = B;
 }
@@ -160,6 +164,7 @@ memxct_status_t memxct_plan_set_option(memxct_plan_t plan, memxct_option_t optio
             case MEMXCT_OPT_CANONICAL: range(0, 1); P.opt.canonical = value; break;
             case MEMXCT_OPT_CG_VARIANT: range(0, 1); P.opt.cg_variant = value; break;
             case MEMXCT_OPT_VECTOR_ORDER: range(0, 1); P.opt.vector_order = value; break;
+            case MEMXCT_OPT_SLICES: range(1, 8); P.opt.slices = value; break;
             default: mx::fail(MEMXCT_ERR_INVALID_ARG, "unknown option");
         }
     });
@@ -178,6 +183,7 @@ memxct_status_t memxct_plan_get_option(memxct_plan_t plan, memxct_option_t optio
             case MEMXCT_OPT_CANONICAL: *value = P.opt.canonical; break;
             case MEMXCT_OPT_CG_VARIANT: *value = P.opt.cg_variant; break;
             case MEMXCT_OPT_VECTOR_ORDER: *value = P.opt.vector_order; break;
+            case MEMXCT_OPT_SLICES: *value = P.opt.slices; break;
             default: mx::fail(MEMXCT_ERR_INVALID_ARG, "unknown option");
         }
     });
@@ -362,8 +368,8 @@ memxct_status_t memxct_cg(memxct_plan_t plan, const void* y_sino, void* x_tomo, 
         need(y_sino, "y_sino");
         if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
         cudaStream_t st = stream_of(cuda_stream);
-        mx::cg_run(P, y_sino, x_tomo, iters, st);
-        if (residual_norms) mx::cg_fetch_norms(P, iters, residual_norms, st);
+        mx::cg_run(P, y_sino, x_tomo, iters, 1, st);
+        if (residual_norms) mx::cg_fetch_norms(P, iters, 1, residual_norms, st);
     });
 }
 
@@ -405,10 +411,49 @@ memxct_status_t memxct_cg_host(memxct_plan_t plan, const void* y_host, void* x_h
         ensure_host_staging(P);
         cudaStream_t st = stream_of(cuda_stream);
         MX_CUDA(cudaMemcpyAsync(P.h_in.get(), y_host, P.esize * P.local_len(1), cudaMemcpyHostToDevice, st));
-        mx::cg_run(P, P.h_in.get(), P.h_out.get(), iters, st);
+        mx::cg_run(P, P.h_in.get(), P.h_out.get(), iters, 1, st);
         MX_CUDA(cudaMemcpyAsync(x_host, P.h_out.get(), P.esize * P.local_len(0), cudaMemcpyDeviceToHost, st));
-        if (residual_norms) mx::cg_fetch_norms(P, iters, residual_norms, st);
+        if (residual_norms) mx::cg_fetch_norms(P, iters, 1, residual_norms, st);
         MX_CUDA(cudaStreamSynchronize(st));
+    });
+}
+
+memxct_status_t memxct_forward_batch(memxct_plan_t plan, int32_t slices, const void* x_tomo, void* y_sino,
+                                     void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_tomo, "x_tomo");
+        need(y_sino, "y_sino");
+        if (slices < 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "slices < 1");
+        if (P.esize != 4) mx::fail(MEMXCT_ERR_UNSUPPORTED, "batched projections are FP32 only");
+        mx::apply_forward_batch(P, slices, (const float*)x_tomo, (float*)y_sino, stream_of(cuda_stream));
+    });
+}
+
+memxct_status_t memxct_back_batch(memxct_plan_t plan, int32_t slices, const void* y_sino, void* x_tomo,
+                                  void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_tomo, "x_tomo");
+        need(y_sino, "y_sino");
+        if (slices < 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "slices < 1");
+        if (P.esize != 4) mx::fail(MEMXCT_ERR_UNSUPPORTED, "batched projections are FP32 only");
+        mx::apply_back_batch(P, slices, (const float*)y_sino, (float*)x_tomo, stream_of(cuda_stream));
+    });
+}
+
+memxct_status_t memxct_cg_batch(memxct_plan_t plan, int32_t slices, const void* y_sino, void* x_tomo,
+                                int32_t iters, double* residual_norms, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_tomo, "x_tomo");
+        need(y_sino, "y_sino");
+        if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
+        if (slices < 1 || slices > 32) mx::fail(MEMXCT_ERR_INVALID_ARG, "slices must be in [1, 32]");
+        if (slices > 1 && P.esize != 4) mx::fail(MEMXCT_ERR_UNSUPPORTED, "multi-slice CG is FP32 only");
+        cudaStream_t st = stream_of(cuda_stream);
+        mx::cg_run(P, y_sino, x_tomo, iters, slices, st);
+        if (residual_norms) mx::cg_fetch_norms(P, iters, slices, residual_norms, st);
     });
 }
 

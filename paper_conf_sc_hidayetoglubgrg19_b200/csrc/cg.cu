@@ -1,15 +1,19 @@
-// cg.cu -- CGLS driver (sec. 3.5.2; readings R13-R16).
+// cg.cu -- CGLS driver (sec. 3.5.2; readings R13-R16), for one slice or a batch of K
+// slices that share the memoized matrices.
 //
-// Recursive-residual CGLS, x0 = 0 (reading R14), exactly `iters` iterations:
+// Recursive-residual CGLS per slice, x0 = 0 (reading R14), exactly `iters` iterations:
 //   setup:  r = y;  s = A^T r;  p = s;  gamma_0 = <s,s>;  res_0 = ||r||
-//   iter k: q = A p, delta_k = <q,q>          (dot fused into the forward SpMV epilogue)
+//   iter k: q = A p, delta_k = <q,q>
 //           alpha = gamma_{k-1} / delta_k;  x = fma(alpha, p, x);  r = fma(-alpha, q, r)
-//           s = A^T r, gamma_k = <s,s>        (dot fused into the back SpMV epilogue)
+//           s = A^T r, gamma_k = <s,s>
 //           beta = gamma_k / gamma_{k-1};  p = fma(beta, p, s)
 // CG_VARIANT = 1 recomputes the residual explicitly, r = y - A x (2 forward + 1 back).
-// Scalars live on the device (one slot per iteration), so the whole solve is one CUDA graph:
-// no host round trip per iteration.  Iterations after gamma or delta reach 0 are no-ops, like
-// the oracle's early exit.
+// Vectors of a batch are slice-major ([K][n]); every vector kernel runs a grid of
+// (blocks, K) with slice = blockIdx.y, and the per-slice arithmetic (including the reduction
+// order of the dots) is exactly the single-slice one, so slice s of a batch reproduces a
+// single-slice solve bit for bit.  Scalars live on the device (one slot per slice and
+// iteration), so the whole solve is one CUDA graph.  Iterations after gamma or delta reach 0 are
+// no-ops, like the oracle's early exit.
 #include "plan.h"
 
 namespace mx {
@@ -19,30 +23,37 @@ namespace {
 constexpr int kVT = 256;
 constexpr int kVecBlocks = 296;  // 2 x 148 SMs
 
-// scalar slots
+// scalar slots of slice s: gam[s*n1 + k], del[...], res2[...]; stop flags per slice
 struct Scal {
-    double* gam;   // [iters + 1]
-    double* del;   // [iters + 1]
-    double* res2;  // [iters + 1]
-    int* stop;     // [1]  iterations stopped (gamma or delta reached 0)
-    int* stop_at;  // [1]  first iteration that did not run
+    double* gam;
+    double* del;
+    double* res2;
+    int* stop;     // [K]  iterations stopped (gamma or delta reached 0)
+    int* stop_at;  // [K]  first iteration that did not run
+    int32_t n1;    // iters + 1
 };
 
-Scal scal_of(Plan& P, int32_t iters) {
+int64_t scal_doubles(int32_t iters, int32_t K) { return 3 * (int64_t)(iters + 1) * K + K; }
+
+Scal scal_of(Plan& P) {
+    const int32_t n1 = (int32_t)P.scal_iters + 1, K = P.scal_slices;
     Scal s;
+    s.n1 = n1;
     s.gam = P.scal.p();
-    s.del = s.gam + (iters + 1);
-    s.res2 = s.del + (iters + 1);
-    s.stop = reinterpret_cast<int*>(s.res2 + (iters + 1));
-    s.stop_at = s.stop + 1;
+    s.del = s.gam + (int64_t)n1 * K;
+    s.res2 = s.del + (int64_t)n1 * K;
+    s.stop = reinterpret_cast<int*>(s.res2 + (int64_t)n1 * K);
+    s.stop_at = s.stop + K;
     return s;
 }
 
-// block-wide deterministic reduction + last-block finish (fixed order)
+// block-wide deterministic reduction + last-block finish (fixed order); per slice blockIdx.y
 __device__ void vec_dot_finish(double mine, double* part, double* out, unsigned int* ticket) {
     __shared__ double red[kVT / 32];
     __shared__ bool am_last;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    part += (int64_t)blockIdx.y * gridDim.x;
+    ticket += blockIdx.y;
     for (int o = 16; o; o >>= 1) mine += __shfl_xor_sync(0xffffffffu, mine, o);
     if (lane == 0) red[warp] = mine;
     __syncthreads();
@@ -64,26 +75,30 @@ __device__ void vec_dot_finish(double mine, double* part, double* out, unsigned 
     }
 }
 
+#define MX_GRID_LOOP(i, n) for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < (n); i += (int64_t)gridDim.x * kVT)
+
 // r = y ; x = 0 ; res2[0] = <r, r> ; stop = 0
 template <class T>
 __global__ void __launch_bounds__(kVT)
 cg_init_kernel(const T* __restrict__ y, T* __restrict__ r, int64_t nr, T* __restrict__ x, int64_t nx,
                Scal sc, double* part, unsigned int* ticket) {
+    const int s = blockIdx.y;
+    y += s * nr; r += s * nr; x += s * nx;
     double acc = 0.0;
-    for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < nr; i += (int64_t)gridDim.x * kVT) {
+    MX_GRID_LOOP(i, nr) {
         const T v = y[i];
         r[i] = v;
         acc += (double)v * (double)v;
     }
-    for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < nx; i += (int64_t)gridDim.x * kVT) x[i] = T(0);
-    if (blockIdx.x == 0 && threadIdx.x == 0) { *sc.stop = 0; *sc.stop_at = 0x7fffffff; }
-    vec_dot_finish(acc, part, sc.res2, ticket);
+    MX_GRID_LOOP(i, nx) x[i] = T(0);
+    if (blockIdx.x == 0 && threadIdx.x == 0) { sc.stop[s] = 0; sc.stop_at[s] = 0x7fffffff; }
+    vec_dot_finish(acc, part, sc.res2 + (int64_t)s * sc.n1, ticket);
 }
 
 template <class T>
-__global__ void copy_kernel(const T* __restrict__ a, T* __restrict__ b, int64_t n) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        b[i] = a[i];
+__global__ void __launch_bounds__(kVT) copy_kernel(const T* __restrict__ a, T* __restrict__ b, int64_t n) {
+    a += blockIdx.y * n; b += blockIdx.y * n;
+    MX_GRID_LOOP(i, n) b[i] = a[i];
 }
 
 __device__ __forceinline__ float upd(float a, double s, float b) { return (float)__fma_rn(s, (double)a, (double)b); }
@@ -95,22 +110,24 @@ __global__ void __launch_bounds__(kVT)
 cg_update_xr_kernel(T* __restrict__ x, const T* __restrict__ p, int64_t nx, T* __restrict__ r,
                     const T* __restrict__ q, int64_t nr, Scal sc, int32_t k, double* part,
                     unsigned int* ticket) {
-    const double g = sc.gam[k - 1], d = sc.del[k];
-    if (*sc.stop || g == 0.0 || d == 0.0) {
-        if (blockIdx.x == 0 && threadIdx.x == 0 && !*sc.stop) { *sc.stop = 1; *sc.stop_at = k; }
+    const int s = blockIdx.y;
+    const int64_t o = (int64_t)s * sc.n1;
+    x += s * nx; p += s * nx; r += s * nr; q += s * nr;
+    const double g = sc.gam[o + k - 1], d = sc.del[o + k];
+    if (sc.stop[s] || g == 0.0 || d == 0.0) {
+        if (blockIdx.x == 0 && threadIdx.x == 0 && !sc.stop[s]) { sc.stop[s] = 1; sc.stop_at[s] = k; }
         return;
     }
     const double alpha = __ddiv_rn(g, d);
-    for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < nx; i += (int64_t)gridDim.x * kVT)
-        x[i] = upd(p[i], alpha, x[i]);
-    double acc = 0.0;
+    MX_GRID_LOOP(i, nx) x[i] = upd(p[i], alpha, x[i]);
     if (kUpdateR) {
-        for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < nr; i += (int64_t)gridDim.x * kVT) {
+        double acc = 0.0;
+        MX_GRID_LOOP(i, nr) {
             const T v = upd(q[i], -alpha, r[i]);
             r[i] = v;
             acc += (double)v * (double)v;
         }
-        vec_dot_finish(acc, part, sc.res2 + k, ticket);
+        vec_dot_finish(acc, part, sc.res2 + o + k, ticket);
     }
 }
 
@@ -119,148 +136,169 @@ template <class T>
 __global__ void __launch_bounds__(kVT)
 cg_explicit_r_kernel(const T* __restrict__ y, const T* __restrict__ ax, T* __restrict__ r, int64_t nr,
                      Scal sc, int32_t k, double* part, unsigned int* ticket) {
-    if (*sc.stop) return;
+    const int s = blockIdx.y;
+    if (sc.stop[s]) return;
+    y += s * nr; ax += s * nr; r += s * nr;
     double acc = 0.0;
-    for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < nr; i += (int64_t)gridDim.x * kVT) {
+    MX_GRID_LOOP(i, nr) {
         const T v = y[i] - ax[i];
         r[i] = v;
         acc += (double)v * (double)v;
     }
-    vec_dot_finish(acc, part, sc.res2 + k, ticket);
+    vec_dot_finish(acc, part, sc.res2 + (int64_t)s * sc.n1 + k, ticket);
 }
 
 // beta = gam[k] / gam[k-1]; p = fma(beta, p, s)
 template <class T>
 __global__ void __launch_bounds__(kVT)
-cg_update_p_kernel(T* __restrict__ p, const T* __restrict__ s, int64_t nx, Scal sc, int32_t k) {
-    if (*sc.stop) return;
-    const double beta = __ddiv_rn(sc.gam[k], sc.gam[k - 1]);
-    for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < nx; i += (int64_t)gridDim.x * kVT)
-        p[i] = upd(p[i], beta, s[i]);
+cg_update_p_kernel(T* __restrict__ p, const T* __restrict__ sv, int64_t nx, Scal sc, int32_t k) {
+    const int s = blockIdx.y;
+    if (sc.stop[s]) return;
+    const int64_t o = (int64_t)s * sc.n1;
+    p += s * nx; sv += s * nx;
+    const double beta = __ddiv_rn(sc.gam[o + k], sc.gam[o + k - 1]);
+    MX_GRID_LOOP(i, nx) p[i] = upd(p[i], beta, sv[i]);
 }
 
-// <v, v> in fp64 over a fixed grid (deterministic: fixed element->thread map, fixed tree)
+// <v, v> in fp64 over a fixed grid (deterministic: fixed element->thread map, fixed tree);
+// out[s * stride] for slice s = blockIdx.y
 template <class T>
 __global__ void __launch_bounds__(kVT)
-dot_kernel(const T* __restrict__ v, int64_t n, double* out, double* part, unsigned int* ticket) {
+dot_kernel(const T* __restrict__ v, int64_t n, double* out, int64_t stride, double* part, unsigned int* ticket) {
+    v += blockIdx.y * n;
     double acc = 0.0;
-    for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < n; i += (int64_t)gridDim.x * kVT) {
+    MX_GRID_LOOP(i, n) {
         const double e = (double)v[i];
         acc += e * e;
     }
-    vec_dot_finish(acc, part, out, ticket);
+    vec_dot_finish(acc, part, out + blockIdx.y * stride, ticket);
 }
 
 unsigned vec_blocks(int64_t n) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(kVecBlocks, ceil_div(n, kVT)));
 }
 
-// Projection followed by the dot product of its output.  Canonical mode fuses the dot into the
-// SpMV epilogue (per-partition fma chains, reading R16).  Otherwise a separate small dot kernel
-// is used: measured on B200, the fused last-CTA epilogue slowed the 2 ms SpMV by ~0.5 ms
-// (profiles/r01a_launches.md), while the separate pass over the 4-6 MB vector costs a few us.
-// P > 1: the projection includes the exchange (A = R C A_p), and the local dot is allreduced.
+// Projection of K slices followed by the per-slice dot of the output.  Canonical mode (K = 1,
+// P = 1) fuses the dot into the SpMV epilogue (per-partition fma chains, reading R16).
+// Otherwise a separate small dot kernel is used: measured on B200, the fused last-CTA epilogue
+// slowed the 2 ms SpMV by ~0.5 ms (profiles/r01a_launches.md), while the separate pass over the
+// 4-6 MB vector costs a few us.  P > 1: the projection includes the exchange (A = R C A_p) and
+// the local dots are allreduced.
 template <class T>
-void op_dir(Plan& P, bool forward, const T* in, T* out, double* dot_out, cudaStream_t st) {
-    const Layout& L = forward ? P.fwd : P.back;
-    if (P.nranks == 1) {
+void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, int64_t dot_stride,
+            cudaStream_t st) {
+    const bool fused = dot_out && K == 1 && P.nranks == 1 && (P.opt.canonical != 0 || P.fused_dot);
+    if (P.nranks == 1 && K == 1) {
+        const Layout& L = forward ? P.fwd : P.back;
         double* part = forward ? P.part_fwd.p() : P.part_back.p();
-        const bool fused = dot_out && (P.opt.canonical != 0 || P.fused_dot);
         if constexpr (sizeof(T) == 4)
             spmv_f32(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), st);
         else
             spmv_f64(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), P.opt.canonical != 0, st);
-        if (dot_out && !fused) {
-            dot_kernel<T><<<vec_blocks(L.nrows), kVT, 0, st>>>(out, L.nrows, dot_out, P.part_vec.p(),
-                                                               P.tickets.p() + 2);
-            MX_LAUNCHED();
+    } else if (K == 1) {
+        if (forward) apply_forward(P, in, out, st);
+        else apply_back(P, in, out, st);
+    } else {
+        if constexpr (sizeof(T) == 4) {
+            if (forward) apply_forward_batch(P, K, in, out, st);
+            else apply_back_batch(P, K, in, out, st);
+        } else {
+            fail(MEMXCT_ERR_UNSUPPORTED, "multi-slice CG is FP32 only");
         }
-        return;
     }
-    if (forward) apply_forward(P, in, out, st);
-    else apply_back(P, in, out, st);
-    if (dot_out) {
+    if (dot_out && !fused) {
         const int64_t n = P.local_len(forward ? 1 : 0);
-        dot_kernel<T><<<vec_blocks(n), kVT, 0, st>>>(out, n, dot_out, P.part_vec.p(), P.tickets.p() + 2);
+        dot_kernel<T><<<dim3(vec_blocks(n), K), kVT, 0, st>>>(out, n, dot_out, dot_stride, P.part_vec.p(),
+                                                              P.tickets.p() + 64);
         MX_LAUNCHED();
-        P.comm->allreduce_sum(dot_out, 1, DType::F64, st);
+        if (P.nranks > 1)
+            for (int s = 0; s < K; ++s) P.comm->allreduce_sum(dot_out + s * dot_stride, 1, DType::F64, st);
     }
 }
 
-void allreduce_scalar(Plan& P, double* v, cudaStream_t st) {
-    if (P.nranks > 1) P.comm->allreduce_sum(v, 1, DType::F64, st);
+void allreduce_slices(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) {
+    if (P.nranks > 1)
+        for (int s = 0; s < K; ++s) P.comm->allreduce_sum(v + s * stride, 1, DType::F64, st);
 }
 
 template <class T>
-void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, cudaStream_t st) {
+void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, int K, cudaStream_t st) {
     const int64_t nx = P.local_len(0), nr = P.local_len(1);
     T* r = P.cg_r.as<T>();
     T* q = P.cg_q.as<T>();
     T* s = P.cg_s.as<T>();
     T* p = P.cg_p.as<T>();
     T* ax = P.cg_ax.as<T>();
-    const Scal sc = scal_of(P, (int32_t)P.scal_iters);
+    const Scal sc = scal_of(P);
     double* vpart = P.part_vec.p();
-    unsigned int* tick = P.tickets.p() + 1;
+    unsigned int* tick = P.tickets.p() + 32;
     const unsigned gb = vec_blocks(std::max(nx, nr));
-    cg_init_kernel<T><<<gb, kVT, 0, st>>>(y, r, nr, x, nx, sc, vpart, tick);
+    cg_init_kernel<T><<<dim3(gb, K), kVT, 0, st>>>(y, r, nr, x, nx, sc, vpart, tick);
     MX_LAUNCHED();
-    allreduce_scalar(P, sc.res2, st);
-    op_dir<T>(P, false, r, s, sc.gam, st);                      // s = A^T r, gamma_0
-    copy_kernel<T><<<vec_blocks(nx), kVT, 0, st>>>(s, p, nx);  // p = s
+    allreduce_slices(P, sc.res2, K, sc.n1, st);
+    op_dir<T>(P, false, K, r, s, sc.gam, sc.n1, st);                    // s = A^T r, gamma_0
+    copy_kernel<T><<<dim3(vec_blocks(nx), K), kVT, 0, st>>>(s, p, nx);  // p = s
     MX_LAUNCHED();
     for (int32_t k = 1; k <= iters; ++k) {
-        op_dir<T>(P, true, p, q, sc.del + k, st);               // q = A p, delta_k
+        op_dir<T>(P, true, K, p, q, sc.del + k, sc.n1, st);             // q = A p, delta_k
         if (P.opt.cg_variant == 1) {
-            cg_update_xr_kernel<T, false><<<vec_blocks(nx), kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k, vpart, tick);
+            cg_update_xr_kernel<T, false><<<dim3(vec_blocks(nx), K), kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k,
+                                                                                    vpart, tick);
             MX_LAUNCHED();
-            op_dir<T>(P, true, x, ax, nullptr, st);              // ax = A x
-            cg_explicit_r_kernel<T><<<vec_blocks(nr), kVT, 0, st>>>(y, ax, r, nr, sc, k, vpart, tick);
+            op_dir<T>(P, true, K, x, ax, nullptr, 0, st);                // ax = A x
+            cg_explicit_r_kernel<T><<<dim3(vec_blocks(nr), K), kVT, 0, st>>>(y, ax, r, nr, sc, k, vpart, tick);
             MX_LAUNCHED();
         } else {
-            cg_update_xr_kernel<T, true><<<gb, kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k, vpart, tick);
+            cg_update_xr_kernel<T, true><<<dim3(gb, K), kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k, vpart, tick);
             MX_LAUNCHED();
         }
-        allreduce_scalar(P, sc.res2 + k, st);
-        op_dir<T>(P, false, r, s, sc.gam + k, st);              // s = A^T r, gamma_k
-        cg_update_p_kernel<T><<<vec_blocks(nx), kVT, 0, st>>>(p, s, nx, sc, k);
+        allreduce_slices(P, sc.res2 + k, K, sc.n1, st);
+        op_dir<T>(P, false, K, r, s, sc.gam + k, sc.n1, st);            // s = A^T r, gamma_k
+        cg_update_p_kernel<T><<<dim3(vec_blocks(nx), K), kVT, 0, st>>>(p, s, nx, sc, k);
         MX_LAUNCHED();
     }
 }
 
-void cg_enqueue_any(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
-    if (P.esize == 4) cg_enqueue<float>(P, (const float*)y, (float*)x, iters, st);
-    else cg_enqueue<double>(P, (const double*)y, (double*)x, iters, st);
+void cg_enqueue_any(Plan& P, const void* y, void* x, int32_t iters, int K, cudaStream_t st) {
+    if (P.esize == 4) cg_enqueue<float>(P, (const float*)y, (float*)x, iters, K, st);
+    else cg_enqueue<double>(P, (const double*)y, (double*)x, iters, K, st);
 }
 
 }  // namespace
 
-void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
+void cg_run(Plan& P, const void* y, void* x, int32_t iters, int32_t K, cudaStream_t st) {
+    if (K < 1 || K > 64) fail(MEMXCT_ERR_INVALID_ARG, "slices must be in [1, 64]");
+    if (K > 1 && P.esize != 4) fail(MEMXCT_ERR_UNSUPPORTED, "multi-slice CG is FP32 only");
     const int64_t nx = P.local_len(0), nr = P.local_len(1);
-    if (!P.cg_r.get()) {
-        P.cg_r.alloc(P.esize * std::max<int64_t>(nr, 1));
-        P.cg_q.alloc(P.esize * std::max<int64_t>(nr, 1));
-        P.cg_s.alloc(P.esize * std::max<int64_t>(nx, 1));
-        P.cg_p.alloc(P.esize * std::max<int64_t>(nx, 1));
-        if (P.opt.cg_variant == 1) P.cg_ax.alloc(P.esize * std::max<int64_t>(nr, 1));
-        P.part_fwd.alloc(std::max<int64_t>(P.fwd.nparts, 1));
-        P.part_back.alloc(std::max<int64_t>(P.back.nparts, 1));
-        P.part_vec.alloc(kVecBlocks);
-        P.tickets.alloc(4);
-        MX_CUDA(cudaMemsetAsync(P.tickets.p(), 0, 4 * sizeof(unsigned int), st));
-    }
-    if (iters > P.scal_iters) {
+    if (K > P.cg_slices) {
         MX_CUDA(cudaStreamSynchronize(st));
         P.graphs.clear();
-        P.scal.alloc(3 * ((int64_t)iters + 1) + 1);
-        MX_CUDA(cudaMemsetAsync(P.scal.p(), 0, 8 * (3 * ((int64_t)iters + 1) + 1), st));
-        P.scal_iters = iters;
+        P.cg_r.alloc(P.esize * std::max<int64_t>(nr, 1) * K);
+        P.cg_q.alloc(P.esize * std::max<int64_t>(nr, 1) * K);
+        P.cg_s.alloc(P.esize * std::max<int64_t>(nx, 1) * K);
+        P.cg_p.alloc(P.esize * std::max<int64_t>(nx, 1) * K);
+        if (P.opt.cg_variant == 1) P.cg_ax.alloc(P.esize * std::max<int64_t>(nr, 1) * K);
+        P.part_fwd.alloc(std::max<int64_t>(P.fwd.nparts, 1));
+        P.part_back.alloc(std::max<int64_t>(P.back.nparts, 1));
+        P.part_vec.alloc((int64_t)kVecBlocks * K);
+        P.tickets.alloc(128);
+        MX_CUDA(cudaMemsetAsync(P.tickets.p(), 0, 128 * sizeof(unsigned int), st));
+        P.cg_slices = K;
+    }
+    if (iters > P.scal_iters || K > P.scal_slices) {
+        MX_CUDA(cudaStreamSynchronize(st));
+        P.graphs.clear();
+        P.scal_iters = std::max<int64_t>(iters, P.scal_iters);
+        P.scal_slices = std::max<int32_t>(K, P.scal_slices);
+        const int64_t nd = scal_doubles((int32_t)P.scal_iters, P.scal_slices);
+        P.scal.alloc(nd);
+        MX_CUDA(cudaMemsetAsync(P.scal.p(), 0, 8 * nd, st));
     }
     if (P.nranks > 1 && !P.comm->capturable()) {  // virtual ranks: eager launches
-        cg_enqueue_any(P, y, x, iters, st);
+        cg_enqueue_any(P, y, x, iters, K, st);
         return;
     }
-    auto key = std::make_tuple(y, x, iters, st);
+    auto key = std::make_tuple(y, x, iters * 64 + K, st);
     auto it = P.graphs.find(key);
     if (it == P.graphs.end()) {
         // capture the whole solve once on a private stream, replay it on the caller's stream
@@ -271,7 +309,7 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
         MX_CUDA(cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal));
         const int64_t before = launch_count();
         try {
-            cg_enqueue_any(P, y, x, iters, cap);
+            cg_enqueue_any(P, y, x, iters, K, cap);
         } catch (...) {
             cudaStreamEndCapture(cap, &g);
             if (g) cudaGraphDestroy(g);
@@ -294,15 +332,19 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st) {
     MX_CUDA(cudaGetLastError());
 }
 
-void cg_fetch_norms(Plan& P, int32_t iters, double* out, cudaStream_t st) {
-    const Scal sc = scal_of(P, (int32_t)P.scal_iters);
-    int stop_at = 0;
-    MX_CUDA(cudaMemcpyAsync(out, sc.res2, 8 * ((int64_t)iters + 1), cudaMemcpyDeviceToHost, st));
-    MX_CUDA(cudaMemcpyAsync(&stop_at, sc.stop_at, sizeof(int), cudaMemcpyDeviceToHost, st));
+void cg_fetch_norms(Plan& P, int32_t iters, int32_t K, double* out, cudaStream_t st) {
+    const Scal sc = scal_of(P);
+    std::vector<double> res2((size_t)sc.n1 * K);
+    std::vector<int> stop_at(K);
+    MX_CUDA(cudaMemcpyAsync(res2.data(), sc.res2, 8 * (size_t)sc.n1 * K, cudaMemcpyDeviceToHost, st));
+    MX_CUDA(cudaMemcpyAsync(stop_at.data(), sc.stop_at, sizeof(int) * K, cudaMemcpyDeviceToHost, st));
     MX_CUDA(cudaStreamSynchronize(st));
-    for (int32_t k = 0; k <= iters; ++k) {
-        if (k >= stop_at) out[k] = out[k - 1];  // iterations that did not run repeat the last norm
-        else out[k] = std::sqrt(out[k]);
+    for (int s = 0; s < K; ++s) {
+        double* o = out + (int64_t)s * (iters + 1);
+        for (int32_t k = 0; k <= iters; ++k) {
+            if (k >= stop_at[s]) o[k] = o[k - 1];  // iterations that did not run repeat the last norm
+            else o[k] = std::sqrt(res2[(size_t)s * sc.n1 + k]);
+        }
     }
 }
 

@@ -249,6 +249,81 @@ static void back_t(Plan& P, const T* y, T* x, cudaStream_t st) {
     spmv_any(P, P.back, yfp, x, st);                                        // A_p^T
 }
 
+// ---- K slices at once (slice-major vectors): one matrix stream per group of <= 8 slices -----
+namespace {
+
+// largest power of two <= min(remaining, what the stage buffer admits)
+int group_size(const Plan& P, int remaining) {
+    const int kmax = std::min(spmm_max_slices(P.fwd), spmm_max_slices(P.back));
+    int k = 1;
+    while (k * 2 <= std::min(remaining, kmax)) k *= 2;
+    return k;
+}
+
+void ensure_batch_buffers(Plan& P, int k) {
+    Exchange& X = P.ex;
+    if (k <= X.batch_cap) return;
+    X.y_fp_b.alloc(sizeof(float) * std::max<int64_t>(P.nfp, 1) * k);
+    X.recv_b.alloc(sizeof(float) * std::max<int64_t>(X.nrecv, 1) * k);
+    X.batch_cap = k;
+}
+
+}  // namespace
+
+void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t st) {
+    const int64_t nx = P.local_len(0), ny = P.local_len(1);
+    for (int s0 = 0; s0 < K;) {
+        const int k = group_size(P, K - s0);
+        const float* xs = x + s0 * nx;
+        float* ys = y + s0 * ny;
+        if (P.nranks == 1) {
+            spmm_f32(P.fwd, k, xs, nx, ys, ny, st);
+        } else {
+            ensure_batch_buffers(P, k);
+            Exchange& X = P.ex;
+            float* yfp = X.y_fp_b.as<float>();
+            float* rb = X.recv_b.as<float>();
+            spmm_f32(P.fwd, k, xs, nx, yfp, P.nfp, st);                       // A_p, k slices
+            for (int s = 0; s < k; ++s) {
+                P.comm->alltoallv(yfp + s * P.nfp, X.scount.data(), X.sdispl.data(), rb + s * X.nrecv,
+                                  X.rcount.data(), X.rdispl.data(), DType::F32, st);          // C
+                reduce_kernel<float><<<nblocks(ny), kT, 0, st>>>(rb + s * X.nrecv, X.red_ptr.p(), X.red_pos.p(),
+                                                                 ny, ys + s * ny);            // R
+                MX_LAUNCHED();
+            }
+        }
+        s0 += k;
+    }
+}
+
+void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st) {
+    const int64_t nx = P.local_len(0), ny = P.local_len(1);
+    for (int s0 = 0; s0 < K;) {
+        const int k = group_size(P, K - s0);
+        const float* ys = y + s0 * ny;
+        float* xs = x + s0 * nx;
+        if (P.nranks == 1) {
+            spmm_f32(P.back, k, ys, ny, xs, nx, st);
+        } else {
+            ensure_batch_buffers(P, k);
+            Exchange& X = P.ex;
+            float* yfp = X.y_fp_b.as<float>();
+            float* rb = X.recv_b.as<float>();
+            for (int s = 0; s < k; ++s) {
+                if (X.nrecv > 0) {
+                    pack_kernel<float><<<nblocks(X.nrecv), kT, 0, st>>>(ys + s * ny, X.recv_idx.p(), X.nrecv,
+                                                                        rb + s * X.nrecv);  // R^T
+                    MX_LAUNCHED();
+                }
+                P.comm->alltoallv(rb + s * X.nrecv, X.rcount.data(), X.rdispl.data(), yfp + s * P.nfp,
+                                  X.scount.data(), X.sdispl.data(), DType::F32, st);        // C^T
+            }
+            spmm_f32(P.back, k, yfp, P.nfp, xs, nx, st);                      // A_p^T, k slices
+        }
+        s0 += k;
+    }
+}
+
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st) {
     if (P.esize == 4) forward_t<float>(P, (const float*)x, (float*)y, st);
     else forward_t<double>(P, (const double*)x, (double*)y, st);

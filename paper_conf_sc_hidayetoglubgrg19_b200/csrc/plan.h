@@ -62,6 +62,7 @@ struct Options {
     int64_t canonical = 0;
     int64_t cg_variant = 0;
     int64_t vector_order = 0;  // 0 natural, 1 plan
+    int64_t slices = 1;        // slices per batched call the stage buffer is sized for
 };
 
 // host-side angle tables on the device (reading R1)
@@ -80,9 +81,11 @@ struct Exchange {
     DevArr<int64_t> red_ptr;   // reduction map R: CSR over owned rays ...
     DevArr<int32_t> red_pos;   // ... of positions in recv_buf, ascending peer order
     DevBuf y_fp, recv_buf;     // footprint partials, receive / pack buffer
+    DevBuf y_fp_b, recv_b;     // the same for batched (multi-slice) calls
+    int32_t batch_cap = 0;
     int64_t device_bytes() const {
         return (int64_t)(recv_idx.buf.bytes() + red_ptr.buf.bytes() + red_pos.buf.bytes() + y_fp.bytes() +
-                         recv_buf.bytes());
+                         recv_buf.bytes() + y_fp_b.bytes() + recv_b.bytes());
     }
 };
 
@@ -126,6 +129,7 @@ struct Plan {
     DevArr<double> scal;                            // per-iteration scalars
     DevArr<unsigned int> tickets;                   // last-block counters
     int64_t scal_iters = -1;
+    int32_t scal_slices = 0, cg_slices = 0;
     // staging for *_host calls
     DevBuf h_in, h_out;
     std::map<std::tuple<const void*, void*, int32_t, cudaStream_t>, std::unique_ptr<CgGraph>> graphs;
@@ -165,6 +169,9 @@ int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStrea
 void build_exchange(Plan& P, cudaStream_t st);
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
 void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);
+// K slices, slice-major [K][local_len] fp32 vectors
+void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t st);
+void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st);
 
 // spmv.cu
 void spmv_init();
@@ -172,6 +179,9 @@ void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, doubl
               unsigned int* ticket, cudaStream_t st);
 void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
               unsigned int* ticket, bool canonical, cudaStream_t st);
+// K in {1, 2, 4, 8} slices at once: x[s*ldx + i], y[s*ldy + r]
+void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int64_t ldy, cudaStream_t st);
+int spmm_max_slices(const Layout& L);
 
 inline void spmv_any(Plan&, const Layout& L, const float* in, float* out, cudaStream_t st) {
     spmv_f32(L, in, out, nullptr, nullptr, nullptr, st);
@@ -181,7 +191,7 @@ inline void spmv_any(Plan&, const Layout& L, const double* in, double* out, cuda
 }
 
 // cg.cu
-void cg_run(Plan& P, const void* y, void* x, int32_t iters, cudaStream_t st);
-void cg_fetch_norms(Plan& P, int32_t iters, double* out, cudaStream_t st);
+void cg_run(Plan& P, const void* y, void* x, int32_t iters, int32_t slices, cudaStream_t st);
+void cg_fetch_norms(Plan& P, int32_t iters, int32_t slices, double* out, cudaStream_t st);
 
 }  // namespace mx

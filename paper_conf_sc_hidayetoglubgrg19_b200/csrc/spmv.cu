@@ -293,7 +293,146 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     return a;
 }
 
+// ---- multi-slice SpMM (k slices share the memoized A) --------
+// Same layout and stage structure as the single-slice kernel; the stage buffer holds the K
+// slices' inputs interleaved ([B][K] fp32), so every slot read from HBM feeds K fmas and one
+// matrix stream serves K slices.  Each slice's fma sequence is exactly the single-slice kernel's,
+// so every slice's result is bit-identical to spmv_f32 on the same plan.
+template <int K>
+__device__ __forceinline__ void load_k(const float* __restrict__ buf, uint32_t i, float (&b)[K]) {
+    if constexpr (K == 2) {
+        const float2 v = reinterpret_cast<const float2*>(buf)[i];
+        b[0] = v.x; b[1] = v.y;
+    } else if constexpr (K == 4) {
+        const float4 v = reinterpret_cast<const float4*>(buf)[i];
+        b[0] = v.x; b[1] = v.y; b[2] = v.z; b[3] = v.w;
+    } else {
+        const float4 u = reinterpret_cast<const float4*>(buf)[2 * i];
+        const float4 v = reinterpret_cast<const float4*>(buf)[2 * i + 1];
+        b[0] = u.x; b[1] = u.y; b[2] = u.z; b[3] = u.w; b[4] = v.x; b[5] = v.y; b[6] = v.z; b[7] = v.w;
+    }
+}
+
+template <int K>
+__device__ __forceinline__ void fma_k(float (&acc)[K], const float* buf, uint32_t i, float w) {
+    float b[K];
+    load_k<K>(buf, i, b);
+#pragma unroll
+    for (int s = 0; s < K; ++s) acc[s] = fmaf(b[s], w, acc[s]);
+}
+
+template <int K>
+__device__ __forceinline__ void fma8_k(float (&acc)[K], const float* buf, const uint4& iv, const float4& v0,
+                                       const float4& v1) {
+    fma_k<K>(acc, buf, iv.x & 0xffffu, v0.x);
+    fma_k<K>(acc, buf, iv.x >> 16, v0.y);
+    fma_k<K>(acc, buf, iv.y & 0xffffu, v0.z);
+    fma_k<K>(acc, buf, iv.y >> 16, v0.w);
+    fma_k<K>(acc, buf, iv.z & 0xffffu, v1.x);
+    fma_k<K>(acc, buf, iv.z >> 16, v1.y);
+    fma_k<K>(acc, buf, iv.w & 0xffffu, v1.z);
+    fma_k<K>(acc, buf, iv.w >> 16, v1.w);
+}
+
+template <int K, bool kNatOut>
+__global__ void __launch_bounds__(kMaxThreads, 1)
+spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __restrict__ y, int64_t ldy) {
+    extern __shared__ __align__(16) float kbuf[];  // [B][K]
+    const int64_t p = blockIdx.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
+    const int64_t m0 = a.map_off[p], D = a.map_off[p + 1] - m0;
+    const uint64_t pol = evict_first_policy();
+    float acc[K];
+#pragma unroll
+    for (int s = 0; s < K; ++s) acc[s] = 0.f;
+    for (int64_t g = g0; g < g1; ++g) {
+        const int64_t st = g - g0;
+        const int cnt = (int)min((int64_t)a.B, D - st * a.B);
+        const int32_t* __restrict__ mp = a.map + m0 + st * a.B;
+        if (g != g0) __syncthreads();
+        for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
+            const int64_t col = __ldg(mp + i);
+            float v[K];
+#pragma unroll
+            for (int s = 0; s < K; ++s) v[s] = __ldg(x + s * ldx + col);
+            if constexpr (K == 2) {
+                reinterpret_cast<float2*>(kbuf)[i] = make_float2(v[0], v[1]);
+            } else if constexpr (K == 4) {
+                reinterpret_cast<float4*>(kbuf)[i] = make_float4(v[0], v[1], v[2], v[3]);
+            } else {
+                reinterpret_cast<float4*>(kbuf)[2 * i] = make_float4(v[0], v[1], v[2], v[3]);
+                reinterpret_cast<float4*>(kbuf)[2 * i + 1] = make_float4(v[4], v[5], v[6], v[7]);
+            }
+        }
+        __syncthreads();
+        const int64_t blk = g * a.SPP + warp;
+        const int64_t base = a.slot_off[blk];
+        const int nch = a.lane_chunks[blk * 32 + lane];
+        const int maxc = __reduce_max_sync(0xffffffffu, nch);
+        const int minc = __reduce_min_sync(0xffffffffu, nch);
+        const uint4* ib = reinterpret_cast<const uint4*>(a.ind + base);
+        const float4* vb = reinterpret_cast<const float4*>(a.val + base);
+#pragma unroll (K >= 8 ? 1 : 2)
+        for (int c = 0; c < minc; ++c) {
+            const uint4 iv = ld_stream_u4(ib + c * 32 + lane, pol);
+            const float4 v0 = ld_stream_f4(vb + c * 64 + lane, pol);
+            const float4 v1 = ld_stream_f4(vb + c * 64 + 32 + lane, pol);
+            fma8_k<K>(acc, kbuf, iv, v0, v1);
+        }
+        int64_t pref = (int64_t)minc * 32;
+        for (int c = minc; c < maxc; ++c) {
+            const unsigned act = __ballot_sync(0xffffffffu, nch > c);
+            const int na = __popc(act);
+            if (nch > c) {
+                const int r = __popc(act & lt);
+                const uint4 iv = ld_stream_u4(ib + pref + r, pol);
+                const float4 v0 = ld_stream_f4(vb + 2 * pref + r, pol);
+                const float4 v1 = ld_stream_f4(vb + 2 * pref + na + r, pol);
+                fma8_k<K>(acc, kbuf, iv, v0, v1);
+            }
+            pref += na;
+        }
+    }
+    const int64_t row = p * a.R + threadIdx.x;
+    if (row < a.nrows) {
+        const int64_t o = kNatOut ? a.out_idx[row] : row;
+#pragma unroll
+        for (int s = 0; s < K; ++s) y[s * ldy + o] = acc[s];
+    }
+}
+
+template <int K>
+void launch_spmm(const Layout& L, const float* x, int64_t ldx, float* y, int64_t ldy, cudaStream_t st) {
+    const SpmvArgs a = make_args(L, nullptr, nullptr, nullptr);
+    const size_t smem = sizeof(float) * (size_t)L.B * K;
+    auto kern = L.out_idx.p() ? spmm_f32_kernel<K, true> : spmm_f32_kernel<K, false>;
+    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, ldx, y, ldy);
+    MX_LAUNCHED();
+}
+
 }  // namespace
+
+int spmm_max_slices(const Layout& L) {
+    int dev = 0, optin = 0;
+    MX_CUDA(cudaGetDevice(&dev));
+    MX_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    int k = 1;
+    while (k < 8 && (size_t)L.B * 4 * (2 * k) <= (size_t)optin) k *= 2;
+    return k;
+}
+
+void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int64_t ldy, cudaStream_t st) {
+    if (L.nparts == 0) return;
+    switch (k) {
+        case 1: spmv_f32(L, x, y, nullptr, nullptr, nullptr, st); break;
+        case 2: launch_spmm<2>(L, x, ldx, y, ldy, st); break;
+        case 4: launch_spmm<4>(L, x, ldx, y, ldy, st); break;
+        case 8: launch_spmm<8>(L, x, ldx, y, ldy, st); break;
+        default: fail(MEMXCT_ERR_INVALID_ARG, "internal: slice group must be 1, 2, 4 or 8");
+    }
+}
 
 void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, double* dot_out,
               unsigned int* ticket, cudaStream_t st) {
@@ -336,6 +475,12 @@ void spmv_init() {
     set_smem(spmv_f64_kernel<false, 0>);
     set_smem(spmv_f64_kernel<false, 1>);
     set_smem(spmv_f64_kernel<false, 2>);
+    set_smem(spmm_f32_kernel<2, true>);
+    set_smem(spmm_f32_kernel<2, false>);
+    set_smem(spmm_f32_kernel<4, true>);
+    set_smem(spmm_f32_kernel<4, false>);
+    set_smem(spmm_f32_kernel<8, true>);
+    set_smem(spmm_f32_kernel<8, false>);
     done = true;
 }
 

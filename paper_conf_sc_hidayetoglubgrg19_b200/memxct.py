@@ -19,7 +19,7 @@ STATUS = {0: "MEMXCT_OK", 1: "MEMXCT_ERR_INVALID_ARG", 2: "MEMXCT_ERR_STATE",
           3: "MEMXCT_ERR_OUT_OF_MEMORY", 4: "MEMXCT_ERR_CUDA", 5: "MEMXCT_ERR_NCCL",
           6: "MEMXCT_ERR_UNSUPPORTED"}
 OPT = {"tile_tomo": 0, "tile_sino": 1, "part_rows": 2, "buffer_entries": 3, "precision": 4,
-       "canonical": 5, "cg_variant": 6, "vector_order": 7}
+       "canonical": 5, "cg_variant": 6, "vector_order": 7, "slices": 8}
 
 #: every symbol include/memxct.h declares (checked by tests/test_abi.py)
 SYMBOLS = [
@@ -31,6 +31,7 @@ SYMBOLS = [
     "memxct_status_string", "memxct_last_error", "memxct_kernel_launch_count",
     "memxct_local_group_create", "memxct_local_group_destroy", "memxct_plan_set_comm_local",
     "memxct_partition_ranges", "memxct_domain_ranges", "memxct_exchange_info",
+    "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch",
 ]
 
 
@@ -78,6 +79,9 @@ def lib():
             "memxct_partition_ranges": [vp, i64, i32, vp],
             "memxct_domain_ranges": [vp, i32, vp],
             "memxct_exchange_info": [vp, P64, P64, P64, ctypes.POINTER(i32)],
+            "memxct_forward_batch": [vp, i32, vp, vp, vp],
+            "memxct_back_batch": [vp, i32, vp, vp, vp],
+            "memxct_cg_batch": [vp, i32, vp, vp, i32, vp, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -170,7 +174,7 @@ class MemXCT:
                  canonical: bool = False, vector_order: str = "natural", part_rows: int = None,
                  buffer_entries: int = None, tile_tomo: int = None, tile_sino: int = None,
                  cg_variant: int = 0, rank: int = 0, nranks: int = 1, unique_id: bytes = None,
-                 device: int = None, group: "LocalGroup" = None):
+                 device: int = None, group: "LocalGroup" = None, slices: int = None):
         self.n, self.m, self.c = int(n), int(projections), int(channels)
         self._h = ctypes.c_void_p()
         _check(lib().memxct_plan_create(self.n, self.m, self.c, ctypes.byref(self._h)),
@@ -179,7 +183,7 @@ class MemXCT:
         opts = {"precision": {"fp32": 0, "mixed": 1}[precision], "canonical": int(bool(canonical)),
                 "vector_order": {"natural": 0, "plan": 1}[vector_order], "cg_variant": cg_variant,
                 "part_rows": part_rows, "buffer_entries": buffer_entries, "tile_tomo": tile_tomo,
-                "tile_sino": tile_sino}
+                "tile_sino": tile_sino, "slices": slices}
         for k, v in opts.items():
             if v is not None:
                 self.set_option(k, v)
@@ -321,6 +325,49 @@ class MemXCT:
         res = np.empty(iters + 1, np.float64) if residuals else None
         rp = res.ctypes.data_as(ctypes.c_void_p) if residuals else None
         _check(lib().memxct_cg(self._h, _ptr(y), _ptr(x), int(iters), rp, _stream(stream)), "memxct_cg")
+        return (x, res) if residuals else x
+
+    # -- multi-slice (slice-major [K, n] tensors) ---------------------------------------------
+    def _batch(self, t, domain, name):
+        import torch
+        if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == self.dtype and t.is_contiguous()
+                and t.dim() == 2 and t.shape[1] == self.local_size(domain)):
+            raise TypeError(f"{name} must be a contiguous CUDA [slices, {self.local_size(domain)}] tensor")
+        return t
+
+    def forward_batch(self, x, y=None, stream=None):
+        """y[s] = A x[s] for every slice s (one matrix stream per group of up to 8 slices)."""
+        import torch
+        self._batch(x, 0, "x")
+        k = x.shape[0]
+        if y is None:
+            y = torch.empty(k, self.local_size(1), dtype=self.dtype, device=x.device)
+        self._batch(y, 1, "y")
+        _check(lib().memxct_forward_batch(self._h, k, _ptr(x), _ptr(y), _stream(stream)), "memxct_forward_batch")
+        return y
+
+    def back_batch(self, y, x=None, stream=None):
+        import torch
+        self._batch(y, 1, "y")
+        k = y.shape[0]
+        if x is None:
+            x = torch.empty(k, self.local_size(0), dtype=self.dtype, device=y.device)
+        self._batch(x, 0, "x")
+        _check(lib().memxct_back_batch(self._h, k, _ptr(y), _ptr(x), _stream(stream)), "memxct_back_batch")
+        return x
+
+    def cg_batch(self, y, iters: int = 30, x=None, residuals: bool = False, stream=None):
+        """Independent CGLS solves of every slice of y ([K, local_size(1)])."""
+        import torch
+        self._batch(y, 1, "y")
+        k = y.shape[0]
+        if x is None:
+            x = torch.empty(k, self.local_size(0), dtype=self.dtype, device=y.device)
+        self._batch(x, 0, "x")
+        res = np.empty((k, iters + 1), np.float64) if residuals else None
+        rp = res.ctypes.data_as(ctypes.c_void_p) if residuals else None
+        _check(lib().memxct_cg_batch(self._h, k, _ptr(y), _ptr(x), int(iters), rp, _stream(stream)),
+               "memxct_cg_batch")
         return (x, res) if residuals else x
 
     # host-buffer variants (numpy in, numpy out; copies happen inside the C call)

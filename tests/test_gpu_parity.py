@@ -284,3 +284,38 @@ def test_cfg3_sampled_rows(orc):
         got.append(xb[p])
         exp.append(float(ll @ yh[rr]))
     assert rel_l2(np.array(got), np.array(exp)) <= 1e-5
+
+
+# ---- multi-slice ---------------------------------------------------------
+@pytest.mark.parametrize("k", [1, 2, 3, 4, 8, 11])
+def test_batched_projections_bit_identical_to_single(orc, coo_cache, k):
+    n, m, c = 64, 90, 64
+    plan = make_plan(n, m, c, slices=4)
+    rng = np.random.default_rng(k)
+    X = torch.from_numpy(rng.random((k, n * n), dtype=np.float32)).cuda()
+    Y = plan.forward_batch(X)
+    for s in range(k):
+        assert torch.equal(Y[s], plan.forward(X[s].contiguous()))
+    rows, cols, vals = coo_cache(n, m, c)
+    y0 = orc.spmv_coo(rows, cols, vals, X[0].cpu().numpy().astype(np.float64), m * c)
+    assert rel_l2(Y[0].cpu().numpy(), y0) <= 1e-5
+    Yin = torch.from_numpy(rng.random((k, m * c), dtype=np.float32)).cuda()
+    XB = plan.back_batch(Yin)
+    for s in range(k):
+        assert torch.equal(XB[s], plan.back(Yin[s].contiguous()))
+
+
+def test_batched_cg_bit_identical_to_single(orc, coo_cache):
+    n, m, c = 64, 90, 64
+    plan = make_plan(n, m, c, slices=4)
+    rows, cols, vals = coo_cache(n, m, c)
+    xs = [inputs.shepp_logan(n), inputs.uniform(n * n, 5).astype(np.float64),
+          np.roll(inputs.shepp_logan(n), 100), 0 * inputs.shepp_logan(n), inputs.shepp_logan(n)[::-1].copy()]
+    Y = np.stack([orc.spmv_coo(rows, cols, vals, x, m * c) for x in xs]).astype(np.float32)
+    Yt = torch.from_numpy(Y).cuda()
+    X, R = plan.cg_batch(Yt, 12, residuals=True)
+    for s in range(len(xs)):
+        xs1, r1 = plan.cg(Yt[s].contiguous(), 12, residuals=True)
+        assert torch.equal(X[s], xs1), s
+        assert np.array_equal(R[s], r1)
+    assert torch.all(X[3] == 0)   # the zero sinogram stops at once
