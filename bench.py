@@ -361,6 +361,14 @@ def run_ours(args, rank, world):
         dist.all_reduce(te_t, op=dist.ReduceOp.MAX)
     te = float(te_t.item())
 
+    exch_t = None
+    if world > 1:
+        exch_t = plan.exchange_time(20, stream=stream)
+        et = torch.tensor([exch_t["fwd_us"], exch_t["back_us"]], dtype=torch.float64, device=dev)
+        dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        exch_t = {"fwd_us": float(et[0]), "back_us": float(et[1]),
+                  "per_cg_iter_us": float(et[0] + et[1]), "how": "max over ranks, CUDA events, 20 reps"}
+
     multislice = None
     if args.slices > 1 and world == 1:
         multislice = bench_multislice(args, plan, y, n, m, c, stream)
@@ -411,7 +419,7 @@ def run_ours(args, rank, world):
         "device_bytes": st["device_bytes"],
     }
     if world > 1:
-        line["exchange"] = plan.exchange_info()
+        line["exchange"] = {**plan.exchange_info(), **exch_t}
     if multislice is not None:
         line["multislice"] = multislice
     if not args.no_cpu_baseline and world == 1:

@@ -169,6 +169,20 @@ memxct_status_t memxct_back(memxct_plan_t plan, const void* y_sino, void* x_tomo
 memxct_status_t memxct_cg(memxct_plan_t plan, const void* y_sino, void* x_tomo, int32_t iters,
                           double* residual_norms, void* cuda_stream);
 
+/* SIRT on the same operators (the paper's comparison solver, 45 iterations,
+ * P:907-912): x_0 = 0, x_{k+1} = x_k + C A^T R (y - A x_k) with R = 1 / row sums of A and
+ * C = 1 / column sums (0 where a sum is 0).  residual_norms (host, iters + 1, nullable) receives
+ * ||y - A x_k||, k = 0..iters.  Synchronous.  Same dtypes and vector order as memxct_cg. */
+memxct_status_t memxct_sirt(memxct_plan_t plan, const void* y_sino, void* x_tomo, int32_t iters,
+                            double* residual_norms, void* cuda_stream);
+
+/* Collective (P > 1): device time, in microseconds, of one forward exchange (all-to-allv of the
+ * partial sinograms + reduction R) and one back exchange (duplication R^T + reverse
+ * all-to-allv), averaged over `reps` back-to-back repetitions timed with CUDA events on
+ * `cuda_stream`.  Writes 0 at P = 1. */
+memxct_status_t memxct_exchange_time(memxct_plan_t plan, int32_t reps, double* us_forward,
+                                     double* us_back, void* cuda_stream);
+
 /* Multi-slice variants (the paper reuses the memoized matrices for every
  * slice): `slices` independent slices with the same geometry, vectors slice-major
  * (x[s * local_size(0) + i], y[s * local_size(1) + r]), FP32 only.  The slices are processed in

@@ -76,6 +76,12 @@ int orc_cgls(int64_t nrows, int64_t ncols, int64_t nnz, const int32_t* rows, con
              const int64_t* row_key, const int64_t* col_key, int64_t chunk_rows, int64_t chunk_cols,
              double* x, double* res, double* true_res);
 
+/* SIRT: x_0 = 0, x_{k+1} = x_k + C A^T R (y - A x_k), R = 1/row
+ * sums, C = 1/column sums (0 for empty rows/columns).  res[k] = ||y - A x_k||, k = 0..iters
+ * (nullable).  Pinned by the weighted least-squares fixed point and the closed-form x_1. */
+int orc_sirt(int64_t nrows, int64_t ncols, int64_t nnz, const int32_t* rows, const int32_t* cols,
+             const double* vals, const double* y, int32_t iters, double* x, double* res);
+
 /* Canonical dot (reading R16): elements visited in ascending key order, fma chains over chunks
  * of `chunk` elements, chunk partials summed sequentially. */
 double orc_dot_canonical(int64_t n, const double* a, const double* b, const int64_t* key,

@@ -18,7 +18,7 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 __all__ = [
     "build_oracle", "lib", "trace_ray", "count_nnz", "row_lengths", "trace_all", "gilbert2d",
     "d2xy", "hilbert_rank", "spmv_coo", "spmv_canonical", "cgls", "dot_canonical",
-    "coo_to_csr", "sampled_back_rows",
+    "coo_to_csr", "sampled_back_rows", "sirt",
 ]
 
 
@@ -61,6 +61,8 @@ def lib():
         L.orc_spmv_canonical.argtypes = [i64, vp, vp, vp, vp, vp, vp]
         L.orc_cgls.restype = ctypes.c_int
         L.orc_cgls.argtypes = [i64, i64, i64, vp, vp, vp, vp, i32, i32, vp, vp, i64, i64, vp, vp, vp]
+        L.orc_sirt.restype = ctypes.c_int
+        L.orc_sirt.argtypes = [i64, i64, i64, vp, vp, vp, vp, i32, vp, vp]
         L.orc_dot_canonical.restype = dbl
         L.orc_dot_canonical.argtypes = [i64, vp, vp, vp, i64]
         _lib = L
@@ -180,6 +182,18 @@ def cgls(rows, cols, vals, y, nrows: int, ncols: int, iters: int, canonical: boo
                           1 if canonical else 0, rk, ck, chunk_rows, chunk_cols,
                           _p(x), _p(res), _p(tres))
     return x, res, tres, int(done)
+
+
+def sirt(rows, cols, vals, y, nrows: int, ncols: int, iters: int):
+    """SIRT from x0 = 0.  Returns (x, res[iters+1] = ||y - A x_k||)."""
+    rows = np.ascontiguousarray(rows, np.int32)
+    cols = np.ascontiguousarray(cols, np.int32)
+    vals = np.ascontiguousarray(vals, np.float64)
+    y = np.ascontiguousarray(y, np.float64)
+    x = np.empty(ncols, np.float64)
+    res = np.empty(iters + 1, np.float64)
+    lib().orc_sirt(nrows, ncols, len(rows), _p(rows), _p(cols), _p(vals), _p(y), iters, _p(x), _p(res))
+    return x, res
 
 
 def sampled_back_rows(n: int, m: int, c: int, pixels):

@@ -21,7 +21,8 @@ INCLUDE = os.path.join(ROOT, "include")
 OUT = os.path.join(PKG, "libmemxct.so")
 BUILD = os.path.join(PKG, "build")
 
-SOURCES = ["api.cu", "hilbert.cu", "trace.cu", "layout.cu", "spmv.cu", "cg.cu", "comm.cu", "exchange.cu"]
+SOURCES = ["api.cu", "hilbert.cu", "trace.cu", "layout.cu", "spmv.cu", "cg.cu", "comm.cu", "exchange.cu",
+           "sirt.cu"]
 EXTRA = {"trace.cu": ["--fmad=false"]}
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

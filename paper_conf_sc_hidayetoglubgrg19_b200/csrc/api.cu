@@ -418,6 +418,27 @@ memxct_status_t memxct_cg_host(memxct_plan_t plan, const void* y_host, void* x_h
     });
 }
 
+memxct_status_t memxct_sirt(memxct_plan_t plan, const void* y_sino, void* x_tomo, int32_t iters,
+                            double* residual_norms, void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(x_tomo, "x_tomo");
+        need(y_sino, "y_sino");
+        if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
+        mx::sirt_run(P, y_sino, x_tomo, iters, residual_norms, stream_of(cuda_stream));
+    });
+}
+
+memxct_status_t memxct_exchange_time(memxct_plan_t plan, int32_t reps, double* us_forward, double* us_back,
+                                     void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(us_forward, "us_forward");
+        need(us_back, "us_back");
+        mx::time_exchange(P, reps, us_forward, us_back, stream_of(cuda_stream));
+    });
+}
+
 memxct_status_t memxct_forward_batch(memxct_plan_t plan, int32_t slices, const void* x_tomo, void* y_sino,
                                      void* cuda_stream) {
     return guarded([&] {

@@ -324,6 +324,60 @@ void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st)
     }
 }
 
+// Device time of the communication steps alone (C + R forward, R^T + C^T back), averaged over
+// `reps` back-to-back repetitions with CUDA events on `st` -- the "exchange time per iteration"
+// of the north star (one forward + one back exchange per CG iteration).
+void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st) {
+    *us_fwd = *us_back = 0.0;
+    if (P.nranks == 1 || reps < 1) return;
+    Exchange& X = P.ex;
+    const DType t = P.esize == 4 ? DType::F32 : DType::F64;
+    const int64_t nown = P.s1 - P.s0;
+    DevBuf own(P.esize * std::max<int64_t>(nown, 1));
+    MX_CUDA(cudaMemsetAsync(own.get(), 0, P.esize * std::max<int64_t>(nown, 1), st));
+    MX_CUDA(cudaMemsetAsync(X.y_fp.get(), 0, P.esize * std::max<int64_t>(P.nfp, 1), st));
+    cudaEvent_t e[3];
+    for (auto& ev : e) MX_CUDA(cudaEventCreate(&ev));
+    auto fwd = [&] {
+        P.comm->alltoallv(X.y_fp.get(), X.scount.data(), X.sdispl.data(), X.recv_buf.get(), X.rcount.data(),
+                          X.rdispl.data(), t, st);
+        if (P.esize == 4)
+            reduce_kernel<float><<<nblocks(nown), kT, 0, st>>>(X.recv_buf.as<float>(), X.red_ptr.p(), X.red_pos.p(),
+                                                               nown, own.as<float>());
+        else
+            reduce_kernel<double><<<nblocks(nown), kT, 0, st>>>(X.recv_buf.as<double>(), X.red_ptr.p(),
+                                                                X.red_pos.p(), nown, own.as<double>());
+        MX_LAUNCHED();
+    };
+    auto back = [&] {
+        if (X.nrecv > 0) {
+            if (P.esize == 4)
+                pack_kernel<float><<<nblocks(X.nrecv), kT, 0, st>>>(own.as<float>(), X.recv_idx.p(), X.nrecv,
+                                                                    X.recv_buf.as<float>());
+            else
+                pack_kernel<double><<<nblocks(X.nrecv), kT, 0, st>>>(own.as<double>(), X.recv_idx.p(), X.nrecv,
+                                                                     X.recv_buf.as<double>());
+            MX_LAUNCHED();
+        }
+        P.comm->alltoallv(X.recv_buf.get(), X.rcount.data(), X.rdispl.data(), X.y_fp.get(), X.scount.data(),
+                          X.sdispl.data(), t, st);
+    };
+    fwd();
+    back();  // warm-up
+    MX_CUDA(cudaEventRecord(e[0], st));
+    for (int i = 0; i < reps; ++i) fwd();
+    MX_CUDA(cudaEventRecord(e[1], st));
+    for (int i = 0; i < reps; ++i) back();
+    MX_CUDA(cudaEventRecord(e[2], st));
+    MX_CUDA(cudaEventSynchronize(e[2]));
+    float a = 0.f, b = 0.f;
+    MX_CUDA(cudaEventElapsedTime(&a, e[0], e[1]));
+    MX_CUDA(cudaEventElapsedTime(&b, e[1], e[2]));
+    for (auto& ev : e) cudaEventDestroy(ev);
+    *us_fwd = 1e3 * a / reps;
+    *us_back = 1e3 * b / reps;
+}
+
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st) {
     if (P.esize == 4) forward_t<float>(P, (const float*)x, (float*)y, st);
     else forward_t<double>(P, (const double*)x, (double*)y, st);

@@ -89,6 +89,17 @@ struct Exchange {
     }
 };
 
+// SIRT scratch (sirt.cu): inverse row / column sums and work vectors
+struct SirtState {
+    bool ready = false;
+    DevBuf rinv, cinv, r, ax, s, ones;
+    DevArr<double> part;
+    int64_t device_bytes() const {
+        return (int64_t)(rinv.bytes() + cinv.bytes() + r.bytes() + ax.bytes() + s.bytes() + ones.bytes() +
+                         part.buf.bytes());
+    }
+};
+
 struct CgGraph {
     cudaGraphExec_t exec = nullptr;
     int64_t nkernels = 0;
@@ -114,6 +125,7 @@ struct Plan {
     int64_t nfp = 0;                                    // footprint rays (rows of A_p)
     DevArr<int32_t> fp_rays;                            // their Hilbert ray indices (P > 1)
     Exchange ex;
+    SirtState sirt;
 
     // two-level pseudo-Hilbert permutations, device int32
     DevArr<int32_t> tomo_nat_of_h, tomo_h_of_nat;  // N*N
@@ -169,6 +181,7 @@ int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStrea
 void build_exchange(Plan& P, cudaStream_t st);
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
 void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);
+void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 // K slices, slice-major [K][local_len] fp32 vectors
 void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t st);
 void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st);
@@ -193,5 +206,8 @@ inline void spmv_any(Plan&, const Layout& L, const double* in, double* out, cuda
 // cg.cu
 void cg_run(Plan& P, const void* y, void* x, int32_t iters, int32_t slices, cudaStream_t st);
 void cg_fetch_norms(Plan& P, int32_t iters, int32_t slices, double* out, cudaStream_t st);
+
+// sirt.cu
+void sirt_run(Plan& P, const void* y, void* x, int32_t iters, double* residual_norms, cudaStream_t st);
 
 }  // namespace mx

@@ -31,7 +31,8 @@ SYMBOLS = [
     "memxct_status_string", "memxct_last_error", "memxct_kernel_launch_count",
     "memxct_local_group_create", "memxct_local_group_destroy", "memxct_plan_set_comm_local",
     "memxct_partition_ranges", "memxct_domain_ranges", "memxct_exchange_info",
-    "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch",
+    "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
+    "memxct_sirt",
 ]
 
 
@@ -82,6 +83,9 @@ def lib():
             "memxct_forward_batch": [vp, i32, vp, vp, vp],
             "memxct_back_batch": [vp, i32, vp, vp, vp],
             "memxct_cg_batch": [vp, i32, vp, vp, i32, vp, vp],
+            "memxct_sirt": [vp, vp, vp, i32, vp, vp],
+            "memxct_exchange_time": [vp, i32, ctypes.POINTER(ctypes.c_double),
+                                     ctypes.POINTER(ctypes.c_double), vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -260,6 +264,13 @@ class MemXCT:
                                           ctypes.byref(d)), "memxct_exchange_info")
         return {"footprint_rays": a.value, "sent": b.value, "received": c.value, "peers": d.value}
 
+    def exchange_time(self, reps: int = 20, stream=None) -> dict:
+        """Collective: device microseconds of one forward and one back exchange (P > 1)."""
+        f, b = ctypes.c_double(), ctypes.c_double()
+        _check(lib().memxct_exchange_time(self._h, int(reps), ctypes.byref(f), ctypes.byref(b),
+                                          _stream(stream)), "memxct_exchange_time")
+        return {"fwd_us": f.value, "back_us": b.value}
+
     def layout_info(self, direction: int) -> dict:
         v = [ctypes.c_int64() for _ in range(6)]
         _check(lib().memxct_layout_info(self._h, direction, *[ctypes.byref(x) for x in v]),
@@ -325,6 +336,18 @@ class MemXCT:
         res = np.empty(iters + 1, np.float64) if residuals else None
         rp = res.ctypes.data_as(ctypes.c_void_p) if residuals else None
         _check(lib().memxct_cg(self._h, _ptr(y), _ptr(x), int(iters), rp, _stream(stream)), "memxct_cg")
+        return (x, res) if residuals else x
+
+    def sirt(self, y, iters: int = 45, x=None, residuals: bool = False, stream=None):
+        """SIRT from x0 = 0 (memxct_sirt); returns x (and ||y - A x_k||, k = 0..iters)."""
+        import torch
+        self._vec(y, 1, "y")
+        if x is None:
+            x = torch.empty(self.local_size(0), dtype=self.dtype, device=y.device)
+        self._vec(x, 0, "x")
+        res = np.empty(iters + 1, np.float64)
+        _check(lib().memxct_sirt(self._h, _ptr(y), _ptr(x), int(iters), res.ctypes.data_as(ctypes.c_void_p),
+                                 _stream(stream)), "memxct_sirt")
         return (x, res) if residuals else x
 
     # -- multi-slice (slice-major [K, n] tensors) ---------------------------------------------
