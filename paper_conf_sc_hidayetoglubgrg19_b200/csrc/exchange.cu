@@ -108,14 +108,15 @@ void decompose(Plan& P, const Geometry& G, cudaStream_t st) {
     DevArr<int32_t> hist;
     hist.alloc(npix);
     MX_CUDA(cudaMemsetAsync(hist.p(), 0, 4 * npix, st));
-    trace_hist(P, G, nrays * P.rank / P.nranks, nrays * (P.rank + 1) / P.nranks, hist.p(), st);
+    const int64_t ra = nrays * P.rank / P.nranks, rb = nrays * (P.rank + 1) / P.nranks;
+    trace_hist(P, G, nullptr, ra, rb - ra, 0, 0, false, hist.p(), st);
     C.allreduce_sum(hist.p(), npix, DType::I32, st);
     const auto tw = tile_sums(hist.p(), P.tomo_tile_off, st);
     hist.reset();
     // per-ray nonzeros (row lengths of A)
     DevArr<int32_t> rl;
     rl.alloc(nrays);
-    trace_count(P, G, nullptr, nrays, 0, 0, false, rl.p(), st);
+    trace_count(P, G, nullptr, 0, nrays, 0, 0, false, rl.p(), st);
     const auto sw = tile_sums(rl.p(), P.sino_tile_off, st);
     const auto bt = partition_ranges(tw, P.nranks), bs = partition_ranges(sw, P.nranks);
     P.tomo_bounds.resize(P.nranks + 1);
@@ -135,13 +136,13 @@ int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStrea
     const int64_t nrays = (int64_t)P.m * P.c;
     if (P.nranks == 1) {
         fp_len.alloc(nrays);
-        trace_count(P, G, nullptr, nrays, 0, 0, false, fp_len.p(), st);
+        trace_count(P, G, nullptr, 0, nrays, 0, 0, false, fp_len.p(), st);
         P.fp_rays.reset();
         return nrays;
     }
     DevArr<int32_t> len;
     len.alloc(nrays);
-    trace_count(P, G, nullptr, nrays, P.t0, P.t1, true, len.p(), st);
+    trace_count(P, G, nullptr, 0, nrays, P.t0, P.t1, true, len.p(), st);
     DevArr<int32_t> flag;
     DevArr<int64_t> flag64, pos;
     flag.alloc(nrays);

@@ -1,29 +1,34 @@
-// layout.cu -- preprocessing: Siddon-traced A, order-preserving transposition to
-// A^T, and the multi-stage buffered layout of both matrices, all on the device.
+// layout.cu -- preprocessing: Siddon-traced A_p, its order-preserving transposition,
+// and the multi-stage buffered layout of both directions, all on the device, built
+// in CHUNKS of whole partitions so the temporaries stay within a memory budget (configs 4-5
+// exceed 2^32 nonzeros per direction; the finished layouts alone take most of the 180 GB).
 //
-// Pipeline (build_matrices):
-//   1. count pass: row lengths of A over rays in Hilbert order (trace.cu), exclusive scan;
-//   2. emit pass: (Hilbert pixel, fp32 length, Hilbert ray) per entry, rows in Hilbert order;
-//   3. A^T by a STABLE radix sort on the pixel key: entries of each pixel keep ascending ray
-//      order -- the scan-based, order-preserving transposition of P:847-858 (no atomics);
-//   4. A with ascending pixel order inside each ray by a second stable sort (on the ray key) of
-//      the A^T entries;
-//   5. build_layout for each direction.
+// Per direction, rows are generated chunk by chunk, sorted by (row, input):
+//   A   (rows = footprint rays):   emit the chunk's rays (trace.cu), then a segmented sort of
+//                                  every ray's entries by pixel;
+//   A^T (rows = local pixels):     re-trace the footprint rays with a pixel-range filter for the
+//                                  chunk's pixels, then a STABLE radix sort on the pixel key --
+//                                  entries of a pixel keep ascending ray order: the scan-based,
+//                                  order-preserving transposition of P:847-858 (no atomics).
+// Two passes over the chunks: pass 1 sizes everything (distinct inputs, stages and slots per
+// partition), the exact final arrays are allocated, pass 2 regenerates the chunk (unless there
+// is only one, which is kept) and scatters it.
 //
-// build_layout (per direction), reading R10/R11:
-//   * partition p = R consecutive Hilbert rows (one CTA); its distinct inputs are found with a
-//     per-partition bitmap over the input domain; a popcount prefix over the bitmap gives every
-//     entry the rank of its input among the partition's distinct inputs, in ascending Hilbert
-//     order (the stage map order);
-//   * stage s of p = ranks [s*B, (s+1)*B): map[s*B + i] = input index (P:598-599, 16-bit local
-//     index i = rank % B);
-//   * per 32-row slice and stage: width = max entries of its rows in that stage, rounded up to
-//     kVec; slots stored column-chunk-major (plan.h) and padded with (ind 0, val 0).
+// Layout per partition p = R consecutive rows (one CTA), readings R10/R11:
+//   * distinct inputs of p by a per-partition bitmap over the input domain; a popcount prefix
+//     gives every entry the rank of its input among them, in ascending Hilbert order (the stage
+//     map order);
+//   * stage s = ranks [s*B, (s+1)*B): map[s*B + i] = input index, 16-bit local index
+//     i = rank % B;
+//   * per (stage, 32-row slice) block: jagged SELL-32 (plan.h): each lane's run rounded up to
+//     kVec slots, chunk c stored only for the lanes that have it.
 #include <cub/block/block_scan.cuh>
 #include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
+#include <cub/device/device_segmented_sort.cuh>
 
 #include <cmath>
+#include <functional>
 #include <vector>
 
 #include "plan.h"
@@ -38,30 +43,26 @@ inline unsigned blocks_for(int64_t n, int threads = kThreads) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, threads), 1 << 30));
 }
 
-template <class T> __global__ void iota_kernel(T* out, int64_t n) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        out[i] = (T)i;
-}
+#define MX_LOOP(i, n) for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < (n); i += (int64_t)gridDim.x * blockDim.x)
 
-__global__ void widen_kernel(const int32_t* in, int64_t* out, int64_t n) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        out[i] = in[i];
-}
+template <class T> __global__ void iota_kernel(T* out, int64_t n) { MX_LOOP(i, n) out[i] = (T)i; }
 
-// row_ptr[r] = first entry with row_ids >= r (row_ids sorted ascending), r in [0, nrows]
-__global__ void row_ptr_kernel(const uint32_t* __restrict__ row_ids, int64_t nnz, int64_t nrows,
+__global__ void widen_kernel(const int32_t* in, int64_t* out, int64_t n) { MX_LOOP(i, n) out[i] = in[i]; }
+
+// row_ptr[r] = first entry with row_ids >= r0 + r (row_ids sorted ascending), r in [0, nrows]
+__global__ void row_ptr_kernel(const uint32_t* __restrict__ row_ids, int64_t nnz, int64_t r0, int64_t nrows,
                                int64_t* __restrict__ row_ptr) {
-    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r <= nrows; r += (int64_t)gridDim.x * blockDim.x) {
+    MX_LOOP(r, nrows + 1) {
         int64_t lo = 0, hi = nnz;
         while (lo < hi) {
             const int64_t mid = (lo + hi) >> 1;
-            if ((int64_t)row_ids[mid] < r) lo = mid + 1; else hi = mid;
+            if ((int64_t)row_ids[mid] < r0 + r) lo = mid + 1; else hi = mid;
         }
         row_ptr[r] = lo;
     }
 }
 
-// mark the input of every entry of partitions [pa, pb) in the chunk bitmap
+// mark the input of every entry of partitions [pa, ...) in the sub-chunk bitmap
 __global__ void mark_kernel(const uint32_t* __restrict__ row_ids, const uint32_t* __restrict__ cols,
                             int64_t e0, int64_t e1, int32_t R, int64_t pa, int64_t words,
                             uint32_t* __restrict__ bitmap) {
@@ -109,10 +110,9 @@ __global__ void rank_kernel(const uint32_t* __restrict__ row_ids, const uint32_t
 
 // map[map_off[p] + rank] = translated input of every set bit of partition p's bitmap
 __global__ void map_kernel(const uint32_t* __restrict__ bitmap, const uint32_t* __restrict__ word_prefix,
-                           int64_t words, int64_t nchunk, int64_t pa, const int64_t* __restrict__ map_off,
+                           int64_t words, int64_t nsub, int64_t pa, const int64_t* __restrict__ map_off,
                            const int32_t* __restrict__ translate, int32_t* __restrict__ map) {
-    const int64_t total = nchunk * words;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    MX_LOOP(i, nsub * words) {
         uint32_t b = bitmap[i];
         if (!b) continue;
         const int64_t p = i / words, w = i % words;
@@ -126,30 +126,26 @@ __global__ void map_kernel(const uint32_t* __restrict__ bitmap, const uint32_t* 
     }
 }
 
-__global__ void stages_kernel(const int64_t* __restrict__ distinct, int64_t nparts, int32_t B,
-                              int64_t* __restrict__ nst) {
-    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < nparts; p += (int64_t)gridDim.x * blockDim.x)
-        nst[p] = (distinct[p] + B - 1) / B;
+__global__ void stages_kernel(const int64_t* __restrict__ distinct, int64_t n, int32_t B, int64_t* __restrict__ nst) {
+    MX_LOOP(p, n) nst[p] = (distinct[p] + B - 1) / B;
 }
 
 __global__ void stage_part_kernel(const int64_t* __restrict__ stage_base, int64_t nparts,
                                   int32_t* __restrict__ stage_part) {
-    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < nparts; p += (int64_t)gridDim.x * blockDim.x)
-        for (int64_t g = stage_base[p]; g < stage_base[p + 1]; ++g) stage_part[g] = (int32_t)p;
+    MX_LOOP(p, nparts)
+    for (int64_t g = stage_base[p]; g < stage_base[p + 1]; ++g) stage_part[g] = (int32_t)p;
 }
 
-// per (row, local stage): start of the stage's run inside the row and its length
+// per (chunk row, local stage): start of the stage's run inside the row and its length
 __global__ void runs_kernel(const int64_t* __restrict__ row_ptr, const uint32_t* __restrict__ rank,
-                            const int64_t* __restrict__ stage_base, int64_t nrows, int32_t R, int32_t B,
+                            const int64_t* __restrict__ nst, int64_t ra, int64_t nr, int32_t R, int32_t B,
                             int32_t maxS, int32_t* __restrict__ run_start, int32_t* __restrict__ run_len) {
-    const int64_t total = nrows * maxS;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t row = i / maxS;
+    MX_LOOP(i, nr * maxS) {
+        const int64_t r = i / maxS;
         const int32_t s = (int32_t)(i % maxS);
-        const int64_t p = row / R;
-        const int64_t S = stage_base[p + 1] - stage_base[p];
+        const int64_t S = nst[(ra + r) / R];
         if (s >= S) { run_start[i] = 0; run_len[i] = 0; continue; }
-        const int64_t b = row_ptr[row], e = row_ptr[row + 1];
+        const int64_t b = row_ptr[r], e = row_ptr[r + 1];
         auto lower = [&](uint64_t key) {
             int64_t lo = b, hi = e;
             while (lo < hi) {
@@ -164,21 +160,21 @@ __global__ void runs_kernel(const int64_t* __restrict__ row_ptr, const uint32_t*
     }
 }
 
-// one warp per (global stage, slice): chunks of each lane = ceil(run length / kVec); the block
-// stores only the chunks lanes actually have (jagged SELL, plan.h), so its size is kVec * sum.
-__global__ void width_kernel(const int32_t* __restrict__ stage_part, const int64_t* __restrict__ stage_base,
-                             const int32_t* __restrict__ run_len, int64_t nstages, int32_t SPP, int64_t nrows,
-                             int32_t R, int32_t maxS, int64_t* __restrict__ blk_slots,
+// one warp per chunk block (local stage, slice): chunks of each lane = ceil(run / kVec); the
+// block stores only the chunks lanes actually have (jagged SELL, plan.h)
+__global__ void width_kernel(const int32_t* __restrict__ stage_part, const int64_t* __restrict__ cs_base,
+                             const int32_t* __restrict__ run_len, int64_t nblk, int32_t SPP, int64_t pa,
+                             int64_t ra, int64_t nrows, int32_t R, int32_t maxS, int64_t* __restrict__ blk_slots,
                              uint16_t* __restrict__ lane_chunks) {
     const int lane = threadIdx.x & 31;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x / 32);
-    for (int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32; wi < nstages * SPP; wi += warps) {
+    for (int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32; wi < nblk; wi += warps) {
         const int64_t g = wi / SPP;
         const int32_t w = (int32_t)(wi % SPP);
-        const int64_t p = stage_part[g];
-        const int64_t s = g - stage_base[p];
-        const int64_t row = p * R + (int64_t)w * 32 + lane;
-        const int32_t len = (row < nrows) ? run_len[row * maxS + s] : 0;
+        const int64_t pl = stage_part[g];
+        const int64_t s = g - cs_base[pl];
+        const int64_t row = (pa + pl) * R + (int64_t)w * 32 + lane;
+        const int32_t len = (row < nrows) ? run_len[(row - ra) * maxS + s] : 0;
         const int32_t nch = (len + kVec - 1) / kVec;
         lane_chunks[wi * 32 + lane] = (uint16_t)nch;
         const int32_t tot = __reduce_add_sync(0xffffffffu, nch);
@@ -186,8 +182,22 @@ __global__ void width_kernel(const int32_t* __restrict__ stage_part, const int64
     }
 }
 
+// pass 1: slots of every partition of the chunk
+__global__ void part_slots_kernel(const int64_t* __restrict__ blk_slots, const int64_t* __restrict__ cs_base,
+                                  int64_t np, int32_t SPP, int64_t pa, int64_t* __restrict__ slots_p) {
+    MX_LOOP(p, np) {
+        int64_t s = 0;
+        for (int64_t b = cs_base[p] * SPP; b < cs_base[p + 1] * SPP; ++b) s += blk_slots[b];
+        slots_p[pa + p] = s;
+    }
+}
+
+__global__ void add_offset_kernel(const int64_t* __restrict__ in, int64_t n, int64_t off, int64_t* __restrict__ out) {
+    MX_LOOP(i, n) out[i] = in[i] + off;
+}
+
 // Position of chunk c of `lane` inside its block: chunks are stored chunk-index-major, and within
-// chunk c only the lanes that have it, in lane order.  prefix = slots of chunks 0..c-1 / kVec,
+// chunk c only the lanes that have it, in lane order.  prefix = chunks stored before chunk c,
 // active = lanes having chunk c, rank = active lanes below `lane`.
 __device__ __forceinline__ void jagged_pos(const uint16_t* __restrict__ lc, int lane, int64_t c,
                                            int64_t& prefix, int32_t& active, int32_t& rank) {
@@ -207,16 +217,17 @@ __global__ void scatter_kernel(const uint32_t* __restrict__ row_ids, const float
                                const uint32_t* __restrict__ rank, const int64_t* __restrict__ row_ptr,
                                const int32_t* __restrict__ run_start, const int64_t* __restrict__ stage_base,
                                const int64_t* __restrict__ slot_off, const uint16_t* __restrict__ lane_chunks,
-                               int64_t nnz, int32_t R, int32_t SPP, int32_t B, int32_t maxS,
+                               int64_t nnz, int64_t ra, int32_t R, int32_t SPP, int32_t B, int32_t maxS,
                                uint16_t* __restrict__ ind, float* __restrict__ val) {
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x) {
+    MX_LOOP(e, nnz) {
         const int64_t row = row_ids[e];
+        const int64_t r = row - ra;
         const int64_t p = row / R;
         const int32_t wl = (int32_t)((row % R) >> 5), lane = (int32_t)(row & 31);
         const uint32_t rk = rank[e];
         const int32_t s = (int32_t)(rk / (uint32_t)B);
         const uint32_t local = rk % (uint32_t)B;
-        const int64_t j = (e - row_ptr[row]) - run_start[row * maxS + s];
+        const int64_t j = (e - row_ptr[r]) - run_start[r * maxS + s];
         const int64_t blk = (stage_base[p] + s) * SPP + wl;
         const int64_t base = slot_off[blk];
         const int64_t c = j / kVec, e8 = j % kVec;
@@ -232,10 +243,23 @@ __global__ void scatter_kernel(const uint32_t* __restrict__ row_ids, const float
 __global__ void gather_u32_f32(const uint32_t* __restrict__ perm, const uint32_t* __restrict__ src_u,
                                const float* __restrict__ src_f, uint32_t* __restrict__ dst_u,
                                float* __restrict__ dst_f, int64_t n) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    MX_LOOP(i, n) {
         const uint32_t q = perm[i];
         dst_u[i] = src_u[q];
         dst_f[i] = src_f[q];
+    }
+}
+
+__global__ void offset_u32_kernel(uint32_t* v, int64_t n, uint32_t add) { MX_LOOP(i, n) v[i] += add; }
+
+// per partition of R rows: sum of 32-bit per-row counts
+__global__ void part_sum_kernel(const int32_t* __restrict__ cnt, int64_t nrows, int32_t R, int64_t np,
+                                int64_t* __restrict__ out) {
+    MX_LOOP(p, np) {
+        int64_t s = 0;
+        const int64_t r1 = min(nrows, (p + 1) * (int64_t)R);
+        for (int64_t r = p * R; r < r1; ++r) s += cnt[r];
+        out[p] = s;
     }
 }
 
@@ -244,6 +268,13 @@ template <class T> T read_scalar(const T* dptr, cudaStream_t st) {
     MX_CUDA(cudaMemcpyAsync(&v, dptr, sizeof(T), cudaMemcpyDeviceToHost, st));
     MX_CUDA(cudaStreamSynchronize(st));
     return v;
+}
+
+template <class T> std::vector<T> to_host(const T* d, int64_t n, cudaStream_t st) {
+    std::vector<T> h(std::max<int64_t>(n, 0));
+    if (n > 0) MX_CUDA(cudaMemcpyAsync(h.data(), d, sizeof(T) * n, cudaMemcpyDeviceToHost, st));
+    MX_CUDA(cudaStreamSynchronize(st));
+    return h;
 }
 
 int bits_for(int64_t n) {
@@ -270,7 +301,7 @@ void widen_i32_to_i64(const int32_t* in, int64_t* out, int64_t n, cudaStream_t s
 }
 
 void row_ptr_from_sorted(const uint32_t* row_ids, int64_t nnz, int64_t nrows, int64_t* row_ptr, cudaStream_t st) {
-    row_ptr_kernel<<<blocks_for(nrows + 1), kThreads, 0, st>>>(row_ids, nnz, nrows, row_ptr);
+    row_ptr_kernel<<<blocks_for(nrows + 1), kThreads, 0, st>>>(row_ids, nnz, 0, nrows, row_ptr);
     MX_LAUNCHED();
 }
 
@@ -290,137 +321,222 @@ void stable_sort_by_key(const uint32_t* keys_in, uint32_t* keys_out, uint32_t* p
     MX_CUDA(cudaStreamSynchronize(st));
 }
 
-void build_layout(Layout& L, int64_t nrows, int64_t ncols, int64_t nnz, const uint32_t* row_ids,
-                  const uint32_t* cols, const float* vals, int32_t R, int32_t B,
-                  const int32_t* in_translate, const int32_t* out_translate, cudaStream_t st) {
+// ---- chunked layout builder ------------------------------------------------------------------
+namespace {
+
+struct Entries {            // one chunk of a direction, sorted by (row, input)
+    DevArr<uint32_t> row;   // absolute row ids
+    DevArr<uint32_t> col;   // input index (plan order, local to the rank)
+    DevArr<float> val;
+    int64_t n = 0;
+    void reset() { row.reset(); col.reset(); val.reset(); n = 0; }
+};
+using Generator = std::function<void(int64_t ra, int64_t rb, Entries& out, cudaStream_t st)>;
+
+struct Builder {
+    Layout& L;
+    int64_t nrows, ncols;
+    int32_t R, B, SPP;
+    const int32_t* in_translate;
+    int64_t words;
+    int64_t bitmap_parts;   // partitions per bitmap sub-chunk
+    DevArr<int64_t> distinct, nst, slots_p;
+    std::vector<int64_t> h_stage_base, h_part_slot;
+
+    // ranks of one chunk's entries (and, in pass 2, the stage maps)
+    void ranks(const Entries& E, int64_t pa, int64_t pb, const std::vector<int64_t>& h_row_ptr, int64_t ra,
+               DevArr<uint32_t>& rank, bool write_map, cudaStream_t st) {
+        DevArr<uint32_t> bitmap, wprefix;
+        const int64_t q = std::min<int64_t>(bitmap_parts, pb - pa);
+        bitmap.alloc(q * words);
+        wprefix.alloc(q * words);
+        for (int64_t qa = pa; qa < pb; qa += q) {
+            const int64_t qb = std::min(pb, qa + q);
+            const int64_t e0 = h_row_ptr[std::min<int64_t>(qa * R, nrows) - ra];
+            const int64_t e1 = h_row_ptr[std::min<int64_t>(qb * R, nrows) - ra];
+            MX_CUDA(cudaMemsetAsync(bitmap.p(), 0, 4 * (qb - qa) * words, st));
+            if (e1 > e0) {
+                mark_kernel<<<blocks_for(e1 - e0), kThreads, 0, st>>>(E.row.p(), E.col.p(), e0, e1, R, qa, words,
+                                                                      bitmap.p());
+                MX_LAUNCHED();
+            }
+            prefix_kernel<<<(unsigned)(qb - qa), kScanThreads, 0, st>>>(bitmap.p(), words, qa, wprefix.p(),
+                                                                        distinct.p());
+            MX_LAUNCHED();
+            if (e1 > e0) {
+                rank_kernel<<<blocks_for(e1 - e0), kThreads, 0, st>>>(E.row.p(), E.col.p(), e0, e1, R, qa, words,
+                                                                      bitmap.p(), wprefix.p(), rank.p());
+                MX_LAUNCHED();
+            }
+            if (write_map) {
+                map_kernel<<<blocks_for((qb - qa) * words), kThreads, 0, st>>>(bitmap.p(), wprefix.p(), words,
+                                                                                qb - qa, qa, L.map_off.p(),
+                                                                                in_translate, L.map.p());
+                MX_LAUNCHED();
+            }
+        }
+    }
+
+    void process(const Entries& E, int64_t pa, int64_t pb, int pass, cudaStream_t st) {
+        const int64_t ra = pa * R, rb = std::min<int64_t>(pb * R, nrows), nr = rb - ra, np = pb - pa;
+        DevArr<int64_t> row_ptr;
+        row_ptr.alloc(nr + 1);
+        row_ptr_kernel<<<blocks_for(nr + 1), kThreads, 0, st>>>(E.row.p(), E.n, ra, nr, row_ptr.p());
+        MX_LAUNCHED();
+        const auto h_row_ptr = to_host(row_ptr.p(), nr + 1, st);
+        DevArr<uint32_t> rank;
+        rank.alloc(std::max<int64_t>(E.n, 1));
+        ranks(E, pa, pb, h_row_ptr, ra, rank, pass == 2, st);
+        stages_kernel<<<blocks_for(np), kThreads, 0, st>>>(distinct.p() + pa, np, B, nst.p() + pa);
+        MX_LAUNCHED();
+        const auto h_nst = to_host(nst.p() + pa, np, st);
+        int64_t maxS = 1;
+        std::vector<int64_t> h_cs(np + 1, 0);
+        for (int64_t p = 0; p < np; ++p) {
+            maxS = std::max(maxS, h_nst[p]);
+            h_cs[p + 1] = h_cs[p] + h_nst[p];
+        }
+        const int64_t ns = h_cs[np], nblk = ns * SPP;
+        DevArr<int64_t> cs;
+        cs.alloc(np + 1);
+        MX_CUDA(cudaMemcpyAsync(cs.p(), h_cs.data(), 8 * (np + 1), cudaMemcpyHostToDevice, st));
+        DevArr<int32_t> run_start, run_len, stage_part;
+        run_start.alloc(std::max<int64_t>(nr * maxS, 1));
+        run_len.alloc(std::max<int64_t>(nr * maxS, 1));
+        if (nr > 0) {
+            runs_kernel<<<blocks_for(nr * maxS), kThreads, 0, st>>>(row_ptr.p(), rank.p(), nst.p(), ra, nr, R, B,
+                                                                    (int32_t)maxS, run_start.p(), run_len.p());
+            MX_LAUNCHED();
+        }
+        stage_part.alloc(std::max<int64_t>(ns, 1));
+        stage_part_kernel<<<blocks_for(np), kThreads, 0, st>>>(cs.p(), np, stage_part.p());
+        MX_LAUNCHED();
+        DevArr<int64_t> blk_slots;
+        DevArr<uint16_t> lanes;
+        blk_slots.alloc(nblk + 1);
+        MX_CUDA(cudaMemsetAsync(blk_slots.p(), 0, 8 * (nblk + 1), st));
+        // pass 2 writes the lane counts straight into the final array
+        uint16_t* lane_out = nullptr;
+        if (pass == 2) lane_out = L.lane_chunks.p() + h_stage_base[pa] * SPP * 32;
+        else { lanes.alloc(std::max<int64_t>(nblk * 32, 1)); lane_out = lanes.p(); }
+        if (nblk > 0) {
+            width_kernel<<<blocks_for(nblk * 32), kThreads, 0, st>>>(stage_part.p(), cs.p(), run_len.p(), nblk, SPP,
+                                                                     pa, ra, nrows, R, (int32_t)maxS, blk_slots.p(),
+                                                                     lane_out);
+            MX_LAUNCHED();
+        }
+        run_len.reset();
+        if (pass == 1) {
+            part_slots_kernel<<<blocks_for(np), kThreads, 0, st>>>(blk_slots.p(), cs.p(), np, SPP, pa, slots_p.p());
+            MX_LAUNCHED();
+            MX_CUDA(cudaStreamSynchronize(st));
+            return;
+        }
+        // pass 2: block offsets = partition slot base + scan of the chunk's block sizes
+        DevArr<int64_t> boff;
+        boff.alloc(nblk + 1);
+        exclusive_scan_i64(blk_slots.p(), boff.p(), nblk + 1, st);
+        if (nblk > 0) {
+            add_offset_kernel<<<blocks_for(nblk), kThreads, 0, st>>>(boff.p(), nblk, h_part_slot[pa],
+                                                                     L.slot_off.p() + h_stage_base[pa] * SPP);
+            MX_LAUNCHED();
+        }
+        if (E.n > 0) {
+            scatter_kernel<<<blocks_for(E.n), kThreads, 0, st>>>(E.row.p(), E.val.p(), rank.p(), row_ptr.p(),
+                                                                 run_start.p(), L.stage_base.p(), L.slot_off.p(),
+                                                                 L.lane_chunks.p(), E.n, ra, R, SPP, B, (int32_t)maxS,
+                                                                 L.ind.p(), L.val.p());
+            MX_LAUNCHED();
+        }
+        MX_CUDA(cudaStreamSynchronize(st));
+    }
+};
+
+// budget of chunk entries: what is free after the finished layouts of both directions
+int64_t chunk_budget(int64_t nnz_both_dirs_remaining) {
+    size_t fr = 0, tot = 0;
+    MX_CUDA(cudaMemGetInfo(&fr, &tot));
+    const double reserve = 6.3 * (double)nnz_both_dirs_remaining + 3e9;
+    const double avail = (double)fr - reserve;
+    const int64_t cap = ((int64_t)1 << 31) - 1;  // CUB segmented sort: int item counts
+    if (const char* e = std::getenv("MEMXCT_BUILD_CHUNK")) return std::max<int64_t>(1, std::min<int64_t>(cap, atoll(e)));
+    return std::max<int64_t>(1 << 24, std::min<int64_t>(cap, (int64_t)(avail / 48.0)));
+}
+
+void build_direction(Layout& L, int64_t nrows, int64_t ncols, const std::vector<int64_t>& part_nnz, int32_t R,
+                     int32_t B, const Generator& gen, const int32_t* in_translate, const int32_t* out_translate,
+                     int64_t budget, cudaStream_t st) {
     L = Layout{};
     L.nrows = nrows;
     L.ncols = ncols;
-    L.nnz = nnz;
     L.R = R;
     L.SPP = R / 32;
     L.B = B;
     L.nparts = ceil_div(nrows, R);
     const int64_t nparts = L.nparts;
-
-    DevArr<int64_t> row_ptr;
-    row_ptr.alloc(nrows + 1);
-    row_ptr_kernel<<<blocks_for(nrows + 1), kThreads, 0, st>>>(row_ids, nnz, nrows, row_ptr.p());
-    MX_LAUNCHED();
-    std::vector<int64_t> h_row_ptr(nrows + 1);
-    MX_CUDA(cudaMemcpyAsync(h_row_ptr.data(), row_ptr.p(), 8 * (nrows + 1), cudaMemcpyDeviceToHost, st));
-    MX_CUDA(cudaStreamSynchronize(st));
-
-    // ---- distinct inputs per partition via chunked bitmaps --------------------------------
-    const int64_t words = std::max<int64_t>(1, ceil_div(ncols, 32));
-    const int64_t budget = (int64_t)2 << 30;  // bytes for bitmap + word prefix per chunk
-    const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(nparts, budget / (words * 8)));
-    const int64_t nchunks = ceil_div(nparts, chunk);
-    DevArr<uint32_t> bitmap, wprefix, rank;
-    bitmap.alloc(chunk * words);
-    wprefix.alloc(chunk * words);
-    rank.alloc(nnz);
-    DevArr<int64_t> distinct;
-    distinct.alloc(nparts);
-
-    auto chunk_entries = [&](int64_t pa, int64_t pb, int64_t& e0, int64_t& e1) {
-        e0 = h_row_ptr[std::min<int64_t>(pa * R, nrows)];
-        e1 = h_row_ptr[std::min<int64_t>(pb * R, nrows)];
-    };
-    auto do_bitmap = [&](int64_t pa, int64_t pb) {
-        int64_t e0, e1;
-        chunk_entries(pa, pb, e0, e1);
-        MX_CUDA(cudaMemsetAsync(bitmap.p(), 0, 4 * (pb - pa) * words, st));
-        if (e1 > e0) {
-            mark_kernel<<<blocks_for(e1 - e0), kThreads, 0, st>>>(row_ids, cols, e0, e1, R, pa, words, bitmap.p());
-            MX_LAUNCHED();
-        }
-        prefix_kernel<<<(unsigned)(pb - pa), kScanThreads, 0, st>>>(bitmap.p(), words, pa, wprefix.p(), distinct.p());
-        MX_LAUNCHED();
-        if (e1 > e0) {
-            rank_kernel<<<blocks_for(e1 - e0), kThreads, 0, st>>>(row_ids, cols, e0, e1, R, pa, words,
-                                                                   bitmap.p(), wprefix.p(), rank.p());
-            MX_LAUNCHED();
-        }
-    };
-    for (int64_t ci = 0; ci < nchunks; ++ci) do_bitmap(ci * chunk, std::min(nparts, (ci + 1) * chunk));
-
-    // ---- stages and map offsets --------------------------------------------------------------
-    DevArr<int64_t> nst, dtmp;
-    nst.alloc(nparts + 1);
-    dtmp.alloc(nparts + 1);
-    MX_CUDA(cudaMemsetAsync(nst.p() + nparts, 0, 8, st));
-    stages_kernel<<<blocks_for(nparts), kThreads, 0, st>>>(distinct.p(), nparts, B, nst.p());
-    MX_LAUNCHED();
+    Builder b{L, nrows, ncols, R, B, R / 32, in_translate};
+    b.words = std::max<int64_t>(1, ceil_div(ncols, 32));
+    b.bitmap_parts = std::max<int64_t>(1, ((int64_t)2 << 30) / (b.words * 8));
+    b.distinct.alloc(nparts + 1);
+    b.nst.alloc(nparts + 1);
+    b.slots_p.alloc(nparts + 1);
+    MX_CUDA(cudaMemsetAsync(b.distinct.p(), 0, 8 * (nparts + 1), st));
+    MX_CUDA(cudaMemsetAsync(b.nst.p(), 0, 8 * (nparts + 1), st));
+    MX_CUDA(cudaMemsetAsync(b.slots_p.p(), 0, 8 * (nparts + 1), st));
+    L.nnz = 0;
+    for (int64_t v : part_nnz) L.nnz += v;
+    // chunks of whole partitions under the entry budget
+    std::vector<std::pair<int64_t, int64_t>> chunks;
+    for (int64_t pa = 0; pa < nparts;) {
+        int64_t pb = pa, acc = 0;
+        while (pb < nparts && (pb == pa || acc + part_nnz[pb] <= budget)) acc += part_nnz[pb++];
+        chunks.emplace_back(pa, pb);
+        pa = pb;
+    }
+    Entries keep;
+    // pass 1: sizes
+    for (auto& c : chunks) {
+        Entries E;
+        gen(c.first * R, std::min<int64_t>(c.second * R, nrows), E, st);
+        b.process(E, c.first, c.second, 1, st);
+        if (chunks.size() == 1) keep = std::move(E);
+    }
     L.stage_base.alloc(nparts + 1);
-    exclusive_scan_i64(nst.p(), L.stage_base.p(), nparts + 1, st);
-    MX_CUDA(cudaMemcpyAsync(dtmp.p(), distinct.p(), 8 * nparts, cudaMemcpyDeviceToDevice, st));
-    MX_CUDA(cudaMemsetAsync(dtmp.p() + nparts, 0, 8, st));
     L.map_off.alloc(nparts + 1);
-    exclusive_scan_i64(dtmp.p(), L.map_off.p(), nparts + 1, st);
-    L.nstages = read_scalar(L.stage_base.p() + nparts, st);
+    DevArr<int64_t> part_slot;
+    part_slot.alloc(nparts + 1);
+    exclusive_scan_i64(b.nst.p(), L.stage_base.p(), nparts + 1, st);
+    exclusive_scan_i64(b.distinct.p(), L.map_off.p(), nparts + 1, st);
+    exclusive_scan_i64(b.slots_p.p(), part_slot.p(), nparts + 1, st);
+    b.h_stage_base = to_host(L.stage_base.p(), nparts + 1, st);
+    b.h_part_slot = to_host(part_slot.p(), nparts + 1, st);
+    L.nstages = b.h_stage_base[nparts];
     L.nmap = read_scalar(L.map_off.p() + nparts, st);
+    L.nslots = b.h_part_slot[nparts];
     {
-        std::vector<int64_t> h_nst(nparts);
-        MX_CUDA(cudaMemcpyAsync(h_nst.data(), nst.p(), 8 * nparts, cudaMemcpyDeviceToHost, st));
-        MX_CUDA(cudaStreamSynchronize(st));
-        int64_t mx = 0;
+        const auto h_nst = to_host(b.nst.p(), nparts, st);
+        int64_t mx = 1;
         for (int64_t v : h_nst) mx = std::max(mx, v);
-        L.max_stages = (int32_t)std::max<int64_t>(mx, 1);
+        L.max_stages = (int32_t)mx;
     }
-    const int32_t maxS = L.max_stages;
-
-    // ---- map ------------------------------------------------------------------------------
-    L.map.alloc(std::max<int64_t>(L.nmap, 1));
-    for (int64_t ci = 0; ci < nchunks; ++ci) {
-        const int64_t pa = ci * chunk, pb = std::min(nparts, (ci + 1) * chunk);
-        if (nchunks > 1) do_bitmap(pa, pb);  // single chunk: bitmap still holds it
-        map_kernel<<<blocks_for((pb - pa) * words), kThreads, 0, st>>>(bitmap.p(), wprefix.p(), words, pb - pa, pa,
-                                                                        L.map_off.p(), in_translate, L.map.p());
-        MX_LAUNCHED();
-    }
-    bitmap.reset();
-    wprefix.reset();
-
-    // ---- per (row, stage) runs, slice widths, slot offsets ----------------------------------
-    DevArr<int32_t> run_start, run_len, stage_part;
-    run_start.alloc(nrows * maxS);
-    run_len.alloc(nrows * maxS);
-    if (nrows > 0) {
-        runs_kernel<<<blocks_for(nrows * maxS), kThreads, 0, st>>>(row_ptr.p(), rank.p(), L.stage_base.p(), nrows, R,
-                                                                   B, maxS, run_start.p(), run_len.p());
-        MX_LAUNCHED();
-    }
-    stage_part.alloc(std::max<int64_t>(L.nstages, 1));
-    stage_part_kernel<<<blocks_for(nparts), kThreads, 0, st>>>(L.stage_base.p(), nparts, stage_part.p());
-    MX_LAUNCHED();
     const int64_t nblk = L.nstages * L.SPP;
-    DevArr<int64_t> blk_slots;
-    blk_slots.alloc(nblk + 1);
-    MX_CUDA(cudaMemsetAsync(blk_slots.p(), 0, 8 * (nblk + 1), st));
-    L.lane_chunks.alloc(std::max<int64_t>(nblk * 32, 1));
-    if (nblk > 0) {
-        width_kernel<<<blocks_for(nblk * 32), kThreads, 0, st>>>(stage_part.p(), L.stage_base.p(), run_len.p(),
-                                                                 L.nstages, L.SPP, nrows, R, maxS, blk_slots.p(),
-                                                                 L.lane_chunks.p());
-        MX_LAUNCHED();
-    }
+    L.map.alloc(std::max<int64_t>(L.nmap, 1));
     L.slot_off.alloc(nblk + 1);
-    exclusive_scan_i64(blk_slots.p(), L.slot_off.p(), nblk + 1, st);
-    L.nslots = read_scalar(L.slot_off.p() + nblk, st);
-    blk_slots.reset();
-    run_len.reset();
-
-    // ---- scatter entries into the slots ---------------------------------------------------
+    MX_CUDA(cudaMemcpyAsync(L.slot_off.p() + nblk, &L.nslots, 8, cudaMemcpyHostToDevice, st));
+    L.lane_chunks.alloc(std::max<int64_t>(nblk * 32, 1));
     L.ind.alloc(std::max<int64_t>(L.nslots, 1));
     L.val.alloc(std::max<int64_t>(L.nslots, 1));
     MX_CUDA(cudaMemsetAsync(L.ind.p(), 0, 2 * std::max<int64_t>(L.nslots, 1), st));
     MX_CUDA(cudaMemsetAsync(L.val.p(), 0, 4 * std::max<int64_t>(L.nslots, 1), st));
-    if (nnz > 0) {
-        scatter_kernel<<<blocks_for(nnz), kThreads, 0, st>>>(row_ids, vals, rank.p(), row_ptr.p(), run_start.p(),
-                                                             L.stage_base.p(), L.slot_off.p(), L.lane_chunks.p(), nnz,
-                                                             R, L.SPP, B, maxS, L.ind.p(), L.val.p());
-        MX_LAUNCHED();
+    // pass 2: scatter (regenerating each chunk unless there was only one)
+    for (auto& c : chunks) {
+        if (chunks.size() == 1) {
+            b.process(keep, c.first, c.second, 2, st);
+        } else {
+            Entries E;
+            gen(c.first * R, std::min<int64_t>(c.second * R, nrows), E, st);
+            b.process(E, c.first, c.second, 2, st);
+        }
     }
     if (out_translate) {
         L.out_idx.alloc(std::max<int64_t>(nrows, 1));
@@ -428,6 +544,19 @@ void build_layout(Layout& L, int64_t nrows, int64_t ncols, int64_t nnz, const ui
     }
     MX_CUDA(cudaStreamSynchronize(st));
 }
+
+std::vector<int64_t> partition_sums(const int32_t* cnt, int64_t nrows, int32_t R, cudaStream_t st) {
+    const int64_t np = ceil_div(nrows, R);
+    DevArr<int64_t> out;
+    out.alloc(std::max<int64_t>(np, 1));
+    if (np > 0) {
+        part_sum_kernel<<<blocks_for(np), kThreads, 0, st>>>(cnt, nrows, R, np, out.p());
+        MX_LAUNCHED();
+    }
+    return to_host(out.p(), np, st);
+}
+
+}  // namespace
 
 void build_matrices(Plan& P, cudaStream_t st) {
     // angle tables (reading R1), the same expression as the paper's geometry in DESIGN.md
@@ -450,70 +579,97 @@ void build_matrices(Plan& P, cudaStream_t st) {
     decompose(P, G, st);
     const int64_t npix = P.t1 - P.t0;
 
-    // 1. rows of A_p = footprint rays (every ray at P = 1), count pass + scan
-    DevArr<int32_t> row_len;
-    const int64_t nrows = P.nfp = footprint(P, G, row_len, st);
-    DevArr<int64_t> len64, row_ptr;
-    len64.alloc(nrows + 1);
-    row_ptr.alloc(nrows + 1);
-    widen_i32_to_i64(row_len.p(), len64.p(), nrows, st);
-    MX_CUDA(cudaMemsetAsync(len64.p() + nrows, 0, 8, st));
-    exclusive_scan_i64(len64.p(), row_ptr.p(), nrows + 1, st);
-    len64.reset();
-    row_len.reset();
-    const int64_t nnz = read_scalar(row_ptr.p() + nrows, st);
-    if (nnz >= ((int64_t)1 << 32))
-        fail(MEMXCT_ERR_UNSUPPORTED, "nnz >= 2^32 on one GPU; shard the problem over more GPUs");
-
-    // 2. emit (local Hilbert pixel, length, row) for the segments inside this rank's pixels
-    DevArr<uint32_t> a_col, a_row;
-    DevArr<float> a_val;
-    a_col.alloc(nnz);
-    a_row.alloc(nnz);
-    a_val.alloc(nnz);
-    trace_emit(P, G, P.nranks == 1 ? nullptr : P.fp_rays.p(), nrows, P.t0, P.t1, row_ptr.p(), a_col.p(),
-               a_val.p(), a_row.p(), st);
-    row_ptr.reset();
-
+    // rows of A_p = footprint rays (every ray at P = 1) and their lengths
+    DevArr<int32_t> fp_len;
+    const int64_t nrows = P.nfp = footprint(P, G, fp_len, st);
+    const int32_t* hray = P.nranks == 1 ? nullptr : P.fp_rays.p();
     const bool natural = (P.opt.vector_order == 0);  // P = 1 only
     const int32_t R = P.part_rows;
     const int32_t B = P.opt.precision == 1 ? P.buffer_entries / 2 : P.buffer_entries;
 
-    // 3. A_p^T: stable sort by pixel (order-preserving transposition)
-    DevArr<uint32_t> t_row, t_col, perm;
-    DevArr<float> t_val;
-    t_row.alloc(nnz);
-    perm.alloc(nnz);
-    stable_sort_by_key(a_col.p(), t_row.p(), perm.p(), nnz, std::max<int64_t>(npix, 1), st);
-    a_col.reset();
-    t_col.alloc(nnz);
-    t_val.alloc(nnz);
-    gather_u32_f32<<<blocks_for(nnz), kThreads, 0, st>>>(perm.p(), a_row.p(), a_val.p(), t_col.p(), t_val.p(), nnz);
-    MX_LAUNCHED();
-    MX_CUDA(cudaStreamSynchronize(st));
-    a_row.reset();
-    a_val.reset();
-    perm.reset();
-    build_layout(P.back, npix, nrows, nnz, t_row.p(), t_col.p(), t_val.p(), R, B,
-                 natural ? P.sino_nat_of_h.p() : nullptr, natural ? P.tomo_nat_of_h.p() : nullptr, st);
+    const auto fwd_part_nnz = partition_sums(fp_len.p(), nrows, R, st);
+    int64_t nnz = 0;
+    for (int64_t v : fwd_part_nnz) nnz += v;
+    const int64_t budget = chunk_budget(2 * nnz);
 
-    // 4. A_p with ascending pixels inside each row: stable sort of the A_p^T entries by row
-    DevArr<uint32_t> f_row, f_col;
-    DevArr<float> f_val;
-    f_row.alloc(nnz);
-    perm.alloc(nnz);
-    stable_sort_by_key(t_col.p(), f_row.p(), perm.p(), nnz, std::max<int64_t>(nrows, 1), st);
-    t_col.reset();
-    f_col.alloc(nnz);
-    f_val.alloc(nnz);
-    gather_u32_f32<<<blocks_for(nnz), kThreads, 0, st>>>(perm.p(), t_row.p(), t_val.p(), f_col.p(), f_val.p(), nnz);
-    MX_LAUNCHED();
-    MX_CUDA(cudaStreamSynchronize(st));
-    t_row.reset();
-    t_val.reset();
-    perm.reset();
-    build_layout(P.fwd, nrows, npix, nnz, f_row.p(), f_col.p(), f_val.p(), R, B,
-                 natural ? P.tomo_nat_of_h.p() : nullptr, natural ? P.sino_nat_of_h.p() : nullptr, st);
+    // ---- A_p: rows = footprint rays; entries of each ray sorted by local pixel --------------
+    Generator gen_fwd = [&](int64_t ra, int64_t rb, Entries& E, cudaStream_t s) {
+        const int64_t nr = rb - ra;
+        DevArr<int64_t> len64, rp;
+        len64.alloc(nr + 1);
+        rp.alloc(nr + 1);
+        widen_i32_to_i64(fp_len.p() + ra, len64.p(), nr, s);
+        MX_CUDA(cudaMemsetAsync(len64.p() + nr, 0, 8, s));
+        exclusive_scan_i64(len64.p(), rp.p(), nr + 1, s);
+        E.n = read_scalar(rp.p() + nr, s);
+        DevArr<uint32_t> col;
+        DevArr<float> val;
+        col.alloc(std::max<int64_t>(E.n, 1));
+        val.alloc(std::max<int64_t>(E.n, 1));
+        E.row.alloc(std::max<int64_t>(E.n, 1));
+        trace_emit(P, G, hray, ra, nr, P.t0, P.t1, rp.p(), col.p(), val.p(), E.row.p(), s);
+        E.col.alloc(std::max<int64_t>(E.n, 1));
+        E.val.alloc(std::max<int64_t>(E.n, 1));
+        if (E.n > 0) {
+            size_t tb = 0;
+            MX_CUDA(cub::DeviceSegmentedSort::SortPairs(nullptr, tb, col.p(), E.col.p(), val.p(), E.val.p(),
+                                                        (int)E.n, (int)nr, rp.p(), rp.p() + 1, s));
+            DevBuf tmp(tb);
+            MX_CUDA(cub::DeviceSegmentedSort::SortPairs(tmp.get(), tb, col.p(), E.col.p(), val.p(), E.val.p(),
+                                                        (int)E.n, (int)nr, rp.p(), rp.p() + 1, s));
+            MX_LAUNCHED();
+        }
+        MX_CUDA(cudaStreamSynchronize(s));
+    };
+    build_direction(P.fwd, nrows, npix, fwd_part_nnz, R, B, gen_fwd, natural ? P.tomo_nat_of_h.p() : nullptr,
+                    natural ? P.sino_nat_of_h.p() : nullptr, budget, st);
+
+    // ---- A_p^T: rows = local pixels; every footprint ray re-traced with the chunk's pixel range,
+    // then the order-preserving (stable) sort by pixel -------------------------------------------
+    DevArr<int32_t> pix_cnt;
+    pix_cnt.alloc(std::max<int64_t>(npix, 1));
+    MX_CUDA(cudaMemsetAsync(pix_cnt.p(), 0, 4 * std::max<int64_t>(npix, 1), st));
+    trace_hist(P, G, hray, 0, nrows, P.t0, P.t1, true, pix_cnt.p(), st);
+    const auto back_part_nnz = partition_sums(pix_cnt.p(), npix, R, st);
+    pix_cnt.reset();
+    Generator gen_back = [&](int64_t ra, int64_t rb, Entries& E, cudaStream_t s) {
+        const int64_t lo = P.t0 + ra, hi = P.t0 + rb;
+        DevArr<int32_t> len;
+        len.alloc(std::max<int64_t>(nrows, 1));
+        trace_count(P, G, hray, 0, nrows, lo, hi, true, len.p(), s);
+        DevArr<int64_t> len64, rp;
+        len64.alloc(nrows + 1);
+        rp.alloc(nrows + 1);
+        widen_i32_to_i64(len.p(), len64.p(), nrows, s);
+        MX_CUDA(cudaMemsetAsync(len64.p() + nrows, 0, 8, s));
+        exclusive_scan_i64(len64.p(), rp.p(), nrows + 1, s);
+        len.reset();
+        len64.reset();
+        E.n = read_scalar(rp.p() + nrows, s);
+        DevArr<uint32_t> pix, ray;
+        DevArr<float> val;
+        pix.alloc(std::max<int64_t>(E.n, 1));
+        ray.alloc(std::max<int64_t>(E.n, 1));
+        val.alloc(std::max<int64_t>(E.n, 1));
+        trace_emit(P, G, hray, 0, nrows, lo, hi, rp.p(), pix.p(), val.p(), ray.p(), s);
+        rp.reset();
+        DevArr<uint32_t> perm;
+        E.row.alloc(std::max<int64_t>(E.n, 1));
+        perm.alloc(std::max<int64_t>(E.n, 1));
+        if (E.n > 0) stable_sort_by_key(pix.p(), E.row.p(), perm.p(), E.n, std::max<int64_t>(rb - ra, 1), s);
+        pix.reset();
+        E.col.alloc(std::max<int64_t>(E.n, 1));
+        E.val.alloc(std::max<int64_t>(E.n, 1));
+        if (E.n > 0) {
+            gather_u32_f32<<<blocks_for(E.n), kThreads, 0, s>>>(perm.p(), ray.p(), val.p(), E.col.p(), E.val.p(), E.n);
+            MX_LAUNCHED();
+            offset_u32_kernel<<<blocks_for(E.n), kThreads, 0, s>>>(E.row.p(), E.n, (uint32_t)ra);
+            MX_LAUNCHED();
+        }
+        MX_CUDA(cudaStreamSynchronize(s));
+    };
+    build_direction(P.back, npix, nrows, back_part_nnz, R, B, gen_back, natural ? P.sino_nat_of_h.p() : nullptr,
+                    natural ? P.tomo_nat_of_h.p() : nullptr, chunk_budget(nnz), st);
 
     // a6: exchange maps of the sparse all-to-allv (P > 1)
     build_exchange(P, st);

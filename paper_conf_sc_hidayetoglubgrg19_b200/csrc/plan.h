@@ -155,18 +155,19 @@ void build_hilbert(int32_t h, int32_t w, int32_t t, int32_t* nat_of_h, int32_t* 
                    std::vector<int64_t>* tile_off, cudaStream_t st);
 int32_t default_tile(int32_t h, int32_t w);
 
-// trace.cu: Siddon count / emit over rays (row r = Hilbert ray hray[r], or r if hray is null);
-// with `filter`, only segments in Hilbert pixels [lo, hi) count (emit writes pixel - lo)
-void trace_count(const Plan& P, const Geometry& G, const int32_t* hray, int64_t nrows, int64_t lo, int64_t hi,
-                 bool filter, int32_t* row_len, cudaStream_t st);
-void trace_emit(const Plan& P, const Geometry& G, const int32_t* hray, int64_t nrows, int64_t lo, int64_t hi,
-                const int64_t* row_ptr, uint32_t* cols, float* vals, uint32_t* row_ids, cudaStream_t st);
-void trace_hist(const Plan& P, const Geometry& G, int64_t r0, int64_t r1, int32_t* hist, cudaStream_t st);
+// trace.cu: Siddon passes over rows [r0, r0 + nrows) (absolute row r = Hilbert ray hray[r], or r
+// if hray is null); with `filter`, only segments in Hilbert pixels [lo, hi) count.
+//   count: row_len[r - r0];  emit: cols = pixel - lo, row_ids = r (row_ptr chunk-local);
+//   hist: atomicAdd(hist[pixel - lo], 1) (lo = 0 without filter)
+void trace_count(const Plan& P, const Geometry& G, const int32_t* hray, int64_t r0, int64_t nrows, int64_t lo,
+                 int64_t hi, bool filter, int32_t* row_len, cudaStream_t st);
+void trace_emit(const Plan& P, const Geometry& G, const int32_t* hray, int64_t r0, int64_t nrows, int64_t lo,
+                int64_t hi, const int64_t* row_ptr, uint32_t* cols, float* vals, uint32_t* row_ids,
+                cudaStream_t st);
+void trace_hist(const Plan& P, const Geometry& G, const int32_t* hray, int64_t r0, int64_t nrows, int64_t lo,
+                int64_t hi, bool filter, int32_t* hist, cudaStream_t st);
 
-// layout.cu: staged SELL-32 layout from entries sorted by (row, col)
-void build_layout(Layout& L, int64_t nrows, int64_t ncols, int64_t nnz, const uint32_t* row_ids,
-                  const uint32_t* cols, const float* vals, int32_t R, int32_t B,
-                  const int32_t* in_translate, const int32_t* out_translate, cudaStream_t st);
+// layout.cu: chunked device build of both directions' staged jagged-SELL layouts
 void build_matrices(Plan& P, cudaStream_t st);
 void widen_i32_to_i64(const int32_t* in, int64_t* out, int64_t n, cudaStream_t st);
 void exclusive_scan_i64(const int64_t* in, int64_t* out, int64_t n, cudaStream_t st);

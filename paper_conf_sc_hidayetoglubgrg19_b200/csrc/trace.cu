@@ -111,7 +111,7 @@ __device__ int64_t trace_one(int32_t n, int32_t c_chan, int64_t ray, double cs, 
                         cols[cnt] = (uint32_t)(h - lo);
                         vals[cnt] = __double2float_rn(seg);
                     }
-                    if (kMode == kHist) atomicAdd(hist + h, 1);
+                    if (kMode == kHist) atomicAdd(hist + (h - lo), 1);
                     ++cnt;
                 }
             }
@@ -122,83 +122,93 @@ __device__ int64_t trace_one(int32_t n, int32_t c_chan, int64_t ray, double cs, 
     return cnt;
 }
 
-// rows: Hilbert ray index of row r = hray ? hray[r] : r0 + r; natural ray = nat_of_h[...]
-__device__ __forceinline__ int64_t natural_ray(const int32_t* __restrict__ hray, int64_t r0, int64_t r,
+// absolute row r: Hilbert ray hray[r] (footprint list) or r itself; natural ray = nat_of_h[...]
+__device__ __forceinline__ int64_t natural_ray(const int32_t* __restrict__ hray, int64_t, int64_t r,
                                                const int32_t* __restrict__ nat_of_h) {
-    return nat_of_h[hray ? (int64_t)hray[r] : r0 + r];
+    return nat_of_h[hray ? (int64_t)hray[r] : r];
 }
 
 template <bool kFilter>
-__global__ void trace_count_kernel(int32_t n, int32_t c_chan, int64_t nrows, const int32_t* __restrict__ hray,
-                                   const int32_t* __restrict__ nat_of_h, const double* __restrict__ cos_t,
-                                   const double* __restrict__ sin_t, const int32_t* __restrict__ pix_rank,
-                                   int64_t lo, int64_t hi, int32_t* __restrict__ row_len) {
+__global__ void trace_count_kernel(int32_t n, int32_t c_chan, int64_t r0, int64_t nrows,
+                                   const int32_t* __restrict__ hray, const int32_t* __restrict__ nat_of_h,
+                                   const double* __restrict__ cos_t, const double* __restrict__ sin_t,
+                                   const int32_t* __restrict__ pix_rank, int64_t lo, int64_t hi,
+                                   int32_t* __restrict__ row_len) {
     const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= nrows) return;
-    const int64_t ray = natural_ray(hray, 0, r, nat_of_h);
+    const int64_t ray = natural_ray(hray, r0, r0 + r, nat_of_h);
     const int64_t m = ray / c_chan;
     row_len[r] = (int32_t)trace_one<kCount, kFilter>(n, c_chan, ray, cos_t[m], sin_t[m], pix_rank, lo, hi,
                                                       nullptr, nullptr, nullptr);
 }
 
-__global__ void trace_emit_kernel(int32_t n, int32_t c_chan, int64_t nrows, const int32_t* __restrict__ hray,
-                                  const int32_t* __restrict__ nat_of_h, const double* __restrict__ cos_t,
-                                  const double* __restrict__ sin_t, const int32_t* __restrict__ pix_rank,
-                                  int64_t lo, int64_t hi, const int64_t* __restrict__ row_ptr,
-                                  uint32_t* __restrict__ cols, float* __restrict__ vals,
-                                  uint32_t* __restrict__ row_ids) {
+__global__ void trace_emit_kernel(int32_t n, int32_t c_chan, int64_t r0, int64_t nrows,
+                                  const int32_t* __restrict__ hray, const int32_t* __restrict__ nat_of_h,
+                                  const double* __restrict__ cos_t, const double* __restrict__ sin_t,
+                                  const int32_t* __restrict__ pix_rank, int64_t lo, int64_t hi,
+                                  const int64_t* __restrict__ row_ptr, uint32_t* __restrict__ cols,
+                                  float* __restrict__ vals, uint32_t* __restrict__ row_ids) {
     const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (r >= nrows) return;
-    const int64_t ray = natural_ray(hray, 0, r, nat_of_h);
+    const int64_t ray = natural_ray(hray, r0, r0 + r, nat_of_h);
     const int64_t m = ray / c_chan;
     const int64_t b = row_ptr[r];
     const int64_t cnt = trace_one<kEmit, true>(n, c_chan, ray, cos_t[m], sin_t[m], pix_rank, lo, hi, cols + b,
                                                vals + b, nullptr);
-    for (int64_t e = 0; e < cnt; ++e) row_ids[b + e] = (uint32_t)r;
+    for (int64_t e = 0; e < cnt; ++e) row_ids[b + e] = (uint32_t)(r0 + r);
 }
 
-__global__ void trace_hist_kernel(int32_t n, int32_t c_chan, int64_t r0, int64_t r1,
-                                  const int32_t* __restrict__ nat_of_h, const double* __restrict__ cos_t,
-                                  const double* __restrict__ sin_t, const int32_t* __restrict__ pix_rank,
+template <bool kFilter>
+__global__ void trace_hist_kernel(int32_t n, int32_t c_chan, int64_t r0, int64_t nrows,
+                                  const int32_t* __restrict__ hray, const int32_t* __restrict__ nat_of_h,
+                                  const double* __restrict__ cos_t, const double* __restrict__ sin_t,
+                                  const int32_t* __restrict__ pix_rank, int64_t lo, int64_t hi,
                                   int32_t* __restrict__ hist) {
-    const int64_t r = r0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (r >= r1) return;
-    const int64_t ray = nat_of_h[r];
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= nrows) return;
+    const int64_t ray = natural_ray(hray, r0, r0 + r, nat_of_h);
     const int64_t m = ray / c_chan;
-    trace_one<kHist, false>(n, c_chan, ray, cos_t[m], sin_t[m], pix_rank, 0, 0, nullptr, nullptr, hist);
+    trace_one<kHist, kFilter>(n, c_chan, ray, cos_t[m], sin_t[m], pix_rank, lo, hi, nullptr, nullptr, hist);
 }
 
 }  // namespace
 
-void trace_count(const Plan& P, const Geometry& G, const int32_t* hray, int64_t nrows, int64_t lo, int64_t hi,
-                 bool filter, int32_t* row_len, cudaStream_t st) {
+void trace_count(const Plan& P, const Geometry& G, const int32_t* hray, int64_t r0, int64_t nrows, int64_t lo,
+                 int64_t hi, bool filter, int32_t* row_len, cudaStream_t st) {
     if (nrows == 0) return;
     const int threads = 128;
     const unsigned blocks = (unsigned)ceil_div(nrows, threads);
     if (filter)
-        trace_count_kernel<true><<<blocks, threads, 0, st>>>(P.n, P.c, nrows, hray, P.sino_nat_of_h.p(), G.cos_t,
-                                                             G.sin_t, P.tomo_h_of_nat.p(), lo, hi, row_len);
+        trace_count_kernel<true><<<blocks, threads, 0, st>>>(P.n, P.c, r0, nrows, hray, P.sino_nat_of_h.p(),
+                                                             G.cos_t, G.sin_t, P.tomo_h_of_nat.p(), lo, hi, row_len);
     else
-        trace_count_kernel<false><<<blocks, threads, 0, st>>>(P.n, P.c, nrows, hray, P.sino_nat_of_h.p(), G.cos_t,
-                                                              G.sin_t, P.tomo_h_of_nat.p(), lo, hi, row_len);
+        trace_count_kernel<false><<<blocks, threads, 0, st>>>(P.n, P.c, r0, nrows, hray, P.sino_nat_of_h.p(),
+                                                              G.cos_t, G.sin_t, P.tomo_h_of_nat.p(), lo, hi, row_len);
     MX_LAUNCHED();
 }
 
-void trace_emit(const Plan& P, const Geometry& G, const int32_t* hray, int64_t nrows, int64_t lo, int64_t hi,
-                const int64_t* row_ptr, uint32_t* cols, float* vals, uint32_t* row_ids, cudaStream_t st) {
+void trace_emit(const Plan& P, const Geometry& G, const int32_t* hray, int64_t r0, int64_t nrows, int64_t lo,
+                int64_t hi, const int64_t* row_ptr, uint32_t* cols, float* vals, uint32_t* row_ids,
+                cudaStream_t st) {
     if (nrows == 0) return;
     const int threads = 128;
     trace_emit_kernel<<<(unsigned)ceil_div(nrows, threads), threads, 0, st>>>(
-        P.n, P.c, nrows, hray, P.sino_nat_of_h.p(), G.cos_t, G.sin_t, P.tomo_h_of_nat.p(), lo, hi, row_ptr, cols,
-        vals, row_ids);
+        P.n, P.c, r0, nrows, hray, P.sino_nat_of_h.p(), G.cos_t, G.sin_t, P.tomo_h_of_nat.p(), lo, hi, row_ptr,
+        cols, vals, row_ids);
     MX_LAUNCHED();
 }
 
-void trace_hist(const Plan& P, const Geometry& G, int64_t r0, int64_t r1, int32_t* hist, cudaStream_t st) {
-    if (r1 <= r0) return;
+void trace_hist(const Plan& P, const Geometry& G, const int32_t* hray, int64_t r0, int64_t nrows, int64_t lo,
+                int64_t hi, bool filter, int32_t* hist, cudaStream_t st) {
+    if (nrows <= 0) return;
     const int threads = 128;
-    trace_hist_kernel<<<(unsigned)ceil_div(r1 - r0, threads), threads, 0, st>>>(
-        P.n, P.c, r0, r1, P.sino_nat_of_h.p(), G.cos_t, G.sin_t, P.tomo_h_of_nat.p(), hist);
+    const unsigned blocks = (unsigned)ceil_div(nrows, threads);
+    if (filter)
+        trace_hist_kernel<true><<<blocks, threads, 0, st>>>(P.n, P.c, r0, nrows, hray, P.sino_nat_of_h.p(), G.cos_t,
+                                                            G.sin_t, P.tomo_h_of_nat.p(), lo, hi, hist);
+    else
+        trace_hist_kernel<false><<<blocks, threads, 0, st>>>(P.n, P.c, r0, nrows, hray, P.sino_nat_of_h.p(),
+                                                             G.cos_t, G.sin_t, P.tomo_h_of_nat.p(), 0, 0, hist);
     MX_LAUNCHED();
 }
 
