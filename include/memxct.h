@@ -90,7 +90,9 @@ typedef enum {
     MEMXCT_OPT_VECTOR_ORDER = 7,
     /* 1..8: slices per matrix stream the batched calls are tuned for (multi-slice reconstruction,
      * P:943-947).  The automatic stage buffer becomes 36 * PART_ROWS / 2^ceil(log2(SLICES))
-     * entries so that many slices' inputs fit in shared memory.  Default 1. */
+     * entries so that many slices' inputs fit in shared memory, and (FP32) the entries of every
+     * row are stored in a shared-memory-bank-aware order instead of ascending input order (same
+     * sums up to fp32 rounding order).  Default 1. */
     MEMXCT_OPT_SLICES = 8
 } memxct_option_t;
 

@@ -182,6 +182,57 @@ __global__ void width_kernel(const int32_t* __restrict__ stage_part, const int64
     }
 }
 
+// Bank-aware order inside every (row, stage) run (FP32 plans tuned for K >= 2 slices, where the
+// shared-memory gather of K-wide entries, not HBM, limits the SpMM): entries are ordered by
+// bank class c = ((local index) - lane) mod C, then by local index, so at a given slot position the
+// lanes of one shared-memory phase (C lanes: 8 for 16 B entries, 16 for 8 B) mostly read
+// different banks.  jnew[e] = position of entry e inside its run.  A stable counting sort on C
+// classes done by one warp per run.
+__global__ void bank_order_kernel(const uint32_t* __restrict__ rank, const int64_t* __restrict__ row_ptr,
+                                  const int32_t* __restrict__ run_start, const int32_t* __restrict__ run_len,
+                                  int64_t nr, int32_t maxS, int64_t ra, int32_t B, int32_t C,
+                                  int32_t* __restrict__ jnew) {
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    const int64_t warps = (int64_t)gridDim.x * (blockDim.x / 32);
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32; i < nr * maxS; i += warps) {
+        const int32_t len = run_len[i];
+        if (len == 0) continue;
+        const int64_t r = i / maxS;
+        const int64_t b = row_ptr[r] + run_start[i];
+        const int32_t shift = (int32_t)((ra + r) & (C - 1));
+        // class counts: lane c holds count of class c
+        int32_t cnt = 0;
+        for (int32_t k0 = 0; k0 < len; k0 += 32) {
+            const int32_t k = k0 + lane;
+            const int32_t cls = k < len ? (int32_t)(((rank[b + k] % (uint32_t)B) - shift) & (C - 1)) : 32;
+            for (int32_t c = 0; c < C; ++c) {
+                const unsigned m = __ballot_sync(0xffffffffu, cls == c);
+                if (lane == c) cnt += __popc(m);
+            }
+        }
+        // exclusive scan over classes -> base of each class; running offset per class
+        int32_t incl = cnt;
+        for (int o = 1; o < 32; o <<= 1) {
+            const int32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += v;
+        }
+        int32_t next = incl - cnt;  // lane c: next free position of class c
+        for (int32_t k0 = 0; k0 < len; k0 += 32) {
+            const int32_t k = k0 + lane;
+            const bool valid = k < len;
+            const int32_t cls = valid ? (int32_t)(((rank[b + k] % (uint32_t)B) - shift) & (C - 1)) : 32;
+            const unsigned same = __match_any_sync(0xffffffffu, cls);
+            const int32_t pos = __shfl_sync(0xffffffffu, next, cls & 31) + __popc(same & lt);
+            if (valid) jnew[b + k] = pos;
+            for (int32_t c = 0; c < C; ++c) {
+                const unsigned m = __ballot_sync(0xffffffffu, cls == c);
+                if (lane == c) next += __popc(m);
+            }
+        }
+    }
+}
+
 // pass 1: slots of every partition of the chunk
 __global__ void part_slots_kernel(const int64_t* __restrict__ blk_slots, const int64_t* __restrict__ cs_base,
                                   int64_t np, int32_t SPP, int64_t pa, int64_t* __restrict__ slots_p) {
@@ -217,8 +268,8 @@ __global__ void scatter_kernel(const uint32_t* __restrict__ row_ids, const float
                                const uint32_t* __restrict__ rank, const int64_t* __restrict__ row_ptr,
                                const int32_t* __restrict__ run_start, const int64_t* __restrict__ stage_base,
                                const int64_t* __restrict__ slot_off, const uint16_t* __restrict__ lane_chunks,
-                               int64_t nnz, int64_t ra, int32_t R, int32_t SPP, int32_t B, int32_t maxS,
-                               uint16_t* __restrict__ ind, float* __restrict__ val) {
+                               const int32_t* __restrict__ jnew, int64_t nnz, int64_t ra, int32_t R, int32_t SPP,
+                               int32_t B, int32_t maxS, uint16_t* __restrict__ ind, float* __restrict__ val) {
     MX_LOOP(e, nnz) {
         const int64_t row = row_ids[e];
         const int64_t r = row - ra;
@@ -227,7 +278,7 @@ __global__ void scatter_kernel(const uint32_t* __restrict__ row_ids, const float
         const uint32_t rk = rank[e];
         const int32_t s = (int32_t)(rk / (uint32_t)B);
         const uint32_t local = rk % (uint32_t)B;
-        const int64_t j = (e - row_ptr[r]) - run_start[r * maxS + s];
+        const int64_t j = jnew ? (int64_t)jnew[e] : (e - row_ptr[r]) - run_start[r * maxS + s];
         const int64_t blk = (stage_base[p] + s) * SPP + wl;
         const int64_t base = slot_off[blk];
         const int64_t c = j / kVec, e8 = j % kVec;
@@ -340,6 +391,7 @@ struct Builder {
     const int32_t* in_translate;
     int64_t words;
     int64_t bitmap_parts;   // partitions per bitmap sub-chunk
+    int32_t bank_classes;   // 0 = ascending local index in every run; else bank-aware order
     DevArr<int64_t> distinct, nst, slots_p;
     std::vector<int64_t> h_stage_base, h_part_slot;
 
@@ -425,6 +477,14 @@ struct Builder {
                                                                      lane_out);
             MX_LAUNCHED();
         }
+        DevArr<int32_t> jnew;
+        if (pass == 2 && bank_classes > 0 && E.n > 0 && nr > 0) {
+            jnew.alloc(E.n);
+            bank_order_kernel<<<blocks_for(nr * maxS * 32), kThreads, 0, st>>>(rank.p(), row_ptr.p(), run_start.p(),
+                                                                              run_len.p(), nr, (int32_t)maxS, ra, B,
+                                                                              bank_classes, jnew.p());
+            MX_LAUNCHED();
+        }
         run_len.reset();
         if (pass == 1) {
             part_slots_kernel<<<blocks_for(np), kThreads, 0, st>>>(blk_slots.p(), cs.p(), np, SPP, pa, slots_p.p());
@@ -444,8 +504,8 @@ struct Builder {
         if (E.n > 0) {
             scatter_kernel<<<blocks_for(E.n), kThreads, 0, st>>>(E.row.p(), E.val.p(), rank.p(), row_ptr.p(),
                                                                  run_start.p(), L.stage_base.p(), L.slot_off.p(),
-                                                                 L.lane_chunks.p(), E.n, ra, R, SPP, B, (int32_t)maxS,
-                                                                 L.ind.p(), L.val.p());
+                                                                 L.lane_chunks.p(), jnew.p(), E.n, ra, R, SPP, B,
+                                                                 (int32_t)maxS, L.ind.p(), L.val.p());
             MX_LAUNCHED();
         }
         MX_CUDA(cudaStreamSynchronize(st));
@@ -465,7 +525,7 @@ int64_t chunk_budget(int64_t nnz_both_dirs_remaining) {
 
 void build_direction(Layout& L, int64_t nrows, int64_t ncols, const std::vector<int64_t>& part_nnz, int32_t R,
                      int32_t B, const Generator& gen, const int32_t* in_translate, const int32_t* out_translate,
-                     int64_t budget, cudaStream_t st) {
+                     int64_t budget, int32_t bank_classes, cudaStream_t st) {
     L = Layout{};
     L.nrows = nrows;
     L.ncols = ncols;
@@ -473,8 +533,10 @@ void build_direction(Layout& L, int64_t nrows, int64_t ncols, const std::vector<
     L.SPP = R / 32;
     L.B = B;
     L.nparts = ceil_div(nrows, R);
+    L.bank_ordered = bank_classes > 0;
     const int64_t nparts = L.nparts;
     Builder b{L, nrows, ncols, R, B, R / 32, in_translate};
+    b.bank_classes = bank_classes;
     b.words = std::max<int64_t>(1, ceil_div(ncols, 32));
     b.bitmap_parts = std::max<int64_t>(1, ((int64_t)2 << 30) / (b.words * 8));
     b.distinct.alloc(nparts + 1);
@@ -591,6 +653,9 @@ void build_matrices(Plan& P, cudaStream_t st) {
     int64_t nnz = 0;
     for (int64_t v : fwd_part_nnz) nnz += v;
     const int64_t budget = chunk_budget(2 * nnz);
+    // bank-aware run order for FP32 plans tuned for batched calls (16 B entries: 8 lanes per
+    // shared-memory phase; 8 B: 16); canonical order (ascending) otherwise
+    const int32_t bank = (P.opt.precision == 0 && P.opt.slices > 1) ? (P.opt.slices > 2 ? 8 : 16) : 0;
 
     // ---- A_p: rows = footprint rays; entries of each ray sorted by local pixel --------------
     Generator gen_fwd = [&](int64_t ra, int64_t rb, Entries& E, cudaStream_t s) {
@@ -622,7 +687,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
         MX_CUDA(cudaStreamSynchronize(s));
     };
     build_direction(P.fwd, nrows, npix, fwd_part_nnz, R, B, gen_fwd, natural ? P.tomo_nat_of_h.p() : nullptr,
-                    natural ? P.sino_nat_of_h.p() : nullptr, budget, st);
+                    natural ? P.sino_nat_of_h.p() : nullptr, budget, bank, st);
 
     // ---- A_p^T: rows = local pixels; every footprint ray re-traced with the chunk's pixel range,
     // then the order-preserving (stable) sort by pixel -------------------------------------------
@@ -669,7 +734,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
         MX_CUDA(cudaStreamSynchronize(s));
     };
     build_direction(P.back, npix, nrows, back_part_nnz, R, B, gen_back, natural ? P.sino_nat_of_h.p() : nullptr,
-                    natural ? P.tomo_nat_of_h.p() : nullptr, chunk_budget(nnz), st);
+                    natural ? P.tomo_nat_of_h.p() : nullptr, chunk_budget(nnz), bank, st);
 
     // a6: exchange maps of the sparse all-to-allv (P > 1)
     build_exchange(P, st);

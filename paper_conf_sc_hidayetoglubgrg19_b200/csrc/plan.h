@@ -36,6 +36,7 @@ struct Layout {
     int64_t nparts = 0, nstages = 0, nslots = 0, nmap = 0;
     int32_t R = 0, SPP = 0, B = 0;
     int32_t max_stages = 0;
+    bool bank_ordered = false;   // runs in bank-aware order instead of ascending local index
     DevArr<int64_t> stage_base;  // nparts + 1
     DevArr<int64_t> map_off;     // nparts + 1
     DevArr<int32_t> map;         // nmap

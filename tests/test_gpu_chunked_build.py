@@ -48,6 +48,36 @@ def test_chunked_layout_identical(geom, chunk):
     assert torch.equal(a.back(y), b.back(y))
 
 
+@pytest.mark.parametrize("slices,classes", [(2, 16), (4, 8)])
+def test_bank_ordered_layout_same_matrix(orc, coo_cache, slices, classes):
+    """SLICES > 1 (FP32) stores every run in bank-aware order: same multiset of (row, input,
+    value) as the oracle's A, each run a permutation of its ascending order with bank classes
+    ((local - lane) mod C) non-decreasing, projections within 1e-5."""
+    from conftest import rel_l2
+    from layout_decode import check_structure, decode, real_entries
+    n, m, c = 64, 90, 64
+    plan = _build(n, m, c, part_rows=128, buffer_entries=4096, slices=slices)
+    rows, cols, vals = coo_cache(n, m, c)
+    okey = np.sort(rows.astype(np.int64) * n * n + cols)
+    for direction in (0, 1):
+        ex = plan.layout_export(direction)
+        d = decode(ex, 128, plan.get_option("buffer_entries"))
+        check_structure(d, ordered=False)
+        e = real_entries(d)
+        row_nat = plan.local_indices(1 if direction == 0 else 0)[e["row"]]
+        key = row_nat * n * n + e["col"] if direction == 0 else e["col"] * n * n + row_nat
+        assert np.array_equal(np.sort(key), okey)
+        # inside every (row, stage) run the bank class is non-decreasing along the slots
+        cls = (e["ind"] - e["row"]) % classes
+        k = e["stage"] * 10**9 + e["row"]
+        o = np.lexsort((e["j"], k))
+        same = k[o][1:] == k[o][:-1]
+        assert np.all(cls[o][1:][same] >= cls[o][:-1][same])
+    x = inputs.uniform(n * n, 4)
+    y = plan.forward(torch.from_numpy(x).cuda()).cpu().numpy()
+    assert rel_l2(y, orc.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)) <= 1e-5
+
+
 def test_chunked_build_virtual_ranks():
     from test_gpu_multirank import build_group, gather, run_ranks, scatter
     n, m, c = 64, 90, 64
