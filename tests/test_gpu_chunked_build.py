@@ -51,8 +51,8 @@ def test_chunked_layout_identical(geom, chunk):
 @pytest.mark.parametrize("slices,classes", [(2, 16), (4, 8)])
 def test_bank_ordered_layout_same_matrix(orc, coo_cache, slices, classes):
     """SLICES > 1 (FP32) stores every run in bank-aware order: same multiset of (row, input,
-    value) as the oracle's A, each run a permutation of its ascending order with bank classes
-    ((local - lane) mod C) non-decreasing, projections within 1e-5."""
+    value) as the oracle's A, and at every slot position the C lanes of one shared-memory phase
+    mostly read distinct bank groups (local index mod C); projections within 1e-5."""
     from conftest import rel_l2
     from layout_decode import check_structure, decode, real_entries
     n, m, c = 64, 90, 64
@@ -67,12 +67,16 @@ def test_bank_ordered_layout_same_matrix(orc, coo_cache, slices, classes):
         row_nat = plan.local_indices(1 if direction == 0 else 0)[e["row"]]
         key = row_nat * n * n + e["col"] if direction == 0 else e["col"] * n * n + row_nat
         assert np.array_equal(np.sort(key), okey)
-        # inside every (row, stage) run the bank class is non-decreasing along the slots
-        cls = (e["ind"] - e["row"]) % classes
-        k = e["stage"] * 10**9 + e["row"]
-        o = np.lexsort((e["j"], k))
-        same = k[o][1:] == k[o][:-1]
-        assert np.all(cls[o][1:][same] >= cls[o][:-1][same])
+        # bank conflicts: max multiplicity of a bank group among the lanes of a phase at each
+        # (block, slot position); ascending order gives ~2.4 on such runs, the schedule ~1.1
+        grp = e["blk"] * 10**6 + e["j"] * 4 + e["lane"] // classes
+        key = grp * classes + e["ind"] % classes
+        u, cnt = np.unique(key, return_counts=True)
+        gu = u // classes
+        mult = np.zeros(gu.max() + 1, np.int64)
+        np.maximum.at(mult, gu, cnt)
+        mean_mult = mult[np.unique(gu)].mean()
+        assert mean_mult < 1.35, mean_mult
     x = inputs.uniform(n * n, 4)
     y = plan.forward(torch.from_numpy(x).cuda()).cpu().numpy()
     assert rel_l2(y, orc.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)) <= 1e-5
