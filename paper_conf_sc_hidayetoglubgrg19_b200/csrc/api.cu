@@ -101,9 +101,11 @@ void resolve_tuning(mx::Plan& P) {
     if (B == 0) {
         int32_t k = 1;
         while (k < P.opt.slices) k *= 2;  // batched calls stage k slices per buffer entry
-        // single slice: 36 entries per row (sweep r01_sweep.md); k slices: ~200 KB of k-wide
-        // entries per CTA at R = 1024 (sweep r01_sweep_spmm.md: 4 slices, B = 12288 best)
-        B = (k == 1) ? std::min<int32_t>(57344, 36 * R) : std::min<int32_t>(51200, 144 * R) / k;
+        // single slice: 36 entries per row (sweep r01_sweep.md); k slices: 192 KB of k-wide
+        // entries per CTA at R = 1024 (sweep r01_sweep_spmm.md: 4 slices, B = 12288 best; 200 KB
+        // pushes the shared-memory carveout to 228 KB and the L1 left for the gathers drops to
+        // 28 KB: 26 % slower)
+        B = (k == 1) ? std::min<int32_t>(57344, 36 * R) : std::min<int32_t>(49152, 144 * R) / k;
         B = std::max<int32_t>(256, B - B % 256);
     }
     P.part_rows = R;

@@ -76,7 +76,7 @@ def test_bank_ordered_layout_same_matrix(orc, coo_cache, slices, classes):
         mult = np.zeros(gu.max() + 1, np.int64)
         np.maximum.at(mult, gu, cnt)
         mean_mult = mult[np.unique(gu)].mean()
-        assert mean_mult < 1.35, mean_mult
+        assert mean_mult < (1.35 if classes == 8 else 1.8), mean_mult
     x = inputs.uniform(n * n, 4)
     y = plan.forward(torch.from_numpy(x).cuda()).cpu().numpy()
     assert rel_l2(y, orc.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)) <= 1e-5
