@@ -70,7 +70,7 @@ typedef enum {
     MEMXCT_OPT_TILE_SINO = 1,
     /* Rows per partition (one CTA per partition; one 32-row slice per warp).
      * Multiple of 32 in [32, 1024], or 0 = auto (default): the largest of 1024/512/256/128 that
-     * leaves >= 2 partitions per SM in the smaller direction (1024 at configs 3-5). */
+     * leaves >= 1 partition per SM in the smaller direction (1024 at configs 3-5, 256 at cfg2). */
     MEMXCT_OPT_PART_ROWS = 2,
     /* Stage-buffer capacity in fp32 entries (16-bit local addressing).
      * 256 <= value <= 57344 (224 KB), or 0 = auto (default): 36 * PART_ROWS.  MIXED mode stages

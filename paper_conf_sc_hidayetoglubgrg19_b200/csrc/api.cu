@@ -92,9 +92,11 @@ void resolve_tuning(mx::Plan& P) {
     const int64_t rows = std::min<int64_t>((int64_t)P.n * P.n, (int64_t)P.m * P.c) / P.nranks;
     int32_t R = (int32_t)P.opt.part_rows;
     if (R == 0) {
+        // largest partition still giving every SM a CTA in the smaller direction (cfg2 sweep,
+        // profiles/r01_sweep_cfg2.md: R = 256 / 512 beat 128 by 25 %)
         R = 128;
         for (int32_t cand : {1024, 512, 256}) {
-            if (mx::ceil_div(rows, cand) >= 2 * (int64_t)sms) { R = cand; break; }
+            if (mx::ceil_div(rows, cand) >= (int64_t)sms) { R = cand; break; }
         }
     }
     int32_t B = (int32_t)P.opt.buffer_entries;
