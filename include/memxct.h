@@ -93,7 +93,13 @@ typedef enum {
      * entries so that many slices' inputs fit in shared memory, and (FP32) the entries of every
      * row are stored in a shared-memory-bank-aware order instead of ascending input order (same
      * sums up to fp32 rounding order).  Default 1. */
-    MEMXCT_OPT_SLICES = 8
+    MEMXCT_OPT_SLICES = 8,
+    /* P > 1 exchange: 0 = grouped ncclSend/ncclRecv all-to-allv between the SpMV and
+     * the reduction (default); 1 = fused over peer memory (FP32, P <= 16): the SpMV epilogue
+     * stores partials straight into the owners' receive buffers and the owners' pack kernel stores
+     * ray values straight into the peers' footprint buffers (CUDA IPC mappings over NVLink),
+     * synchronised by epoch/credit flags -- no separate collective on the data path. */
+    MEMXCT_OPT_EXCHANGE = 9
 } memxct_option_t;
 
 /* Create a plan for an N x N tomogram and an M x C sinogram.  Host only; no device

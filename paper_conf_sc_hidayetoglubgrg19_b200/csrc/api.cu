@@ -172,6 +172,7 @@ memxct_status_t memxct_plan_set_option(memxct_plan_t plan, memxct_option_t optio
             case MEMXCT_OPT_CG_VARIANT: range(0, 1); P.opt.cg_variant = value; break;
             case MEMXCT_OPT_VECTOR_ORDER: range(0, 1); P.opt.vector_order = value; break;
             case MEMXCT_OPT_SLICES: range(1, 8); P.opt.slices = value; break;
+            case MEMXCT_OPT_EXCHANGE: range(0, 1); P.opt.exchange = value; break;
             default: mx::fail(MEMXCT_ERR_INVALID_ARG, "unknown option");
         }
     });
@@ -191,6 +192,7 @@ memxct_status_t memxct_plan_get_option(memxct_plan_t plan, memxct_option_t optio
             case MEMXCT_OPT_CG_VARIANT: *value = P.opt.cg_variant; break;
             case MEMXCT_OPT_VECTOR_ORDER: *value = P.opt.vector_order; break;
             case MEMXCT_OPT_SLICES: *value = P.opt.slices; break;
+            case MEMXCT_OPT_EXCHANGE: *value = P.opt.exchange; break;
             default: mx::fail(MEMXCT_ERR_INVALID_ARG, "unknown option");
         }
     });

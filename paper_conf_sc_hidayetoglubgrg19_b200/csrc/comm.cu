@@ -93,6 +93,7 @@ public:
         nccl().check(nccl().CommInitRank(&comm_, n, id, r), "ncclCommInitRank");
     }
     ~NcclComm() override {
+        for (void* p : opened_) cudaIpcCloseMemHandle(p);
         if (comm_) NcclApi::get().CommDestroy(comm_);
     }
     bool capturable() const override { return true; }
@@ -121,18 +122,43 @@ public:
         a.check(a.GroupEnd(), "ncclGroupEnd");
     }
     std::vector<int64_t> allgather_host(int64_t v, cudaStream_t st) override {
+        return allgather_vec(std::vector<int64_t>{v}, st);
+    }
+    std::vector<int64_t> allgather_vec(const std::vector<int64_t>& v, cudaStream_t st) override {
+        const int64_t n = (int64_t)v.size();
         DevArr<int64_t> d;
-        d.alloc(nranks + 1);
-        MX_CUDA(cudaMemcpyAsync(d.p() + nranks, &v, 8, cudaMemcpyHostToDevice, st));
-        nccl().check(nccl().AllGather(d.p() + nranks, d.p(), 1, ncclInt64, comm_, st), "ncclAllGather");
-        std::vector<int64_t> h(nranks);
-        MX_CUDA(cudaMemcpyAsync(h.data(), d.p(), 8 * nranks, cudaMemcpyDeviceToHost, st));
+        d.alloc(n * (nranks + 1));
+        int64_t* mine = d.p() + n * nranks;
+        if (n > 0) MX_CUDA(cudaMemcpyAsync(mine, v.data(), 8 * n, cudaMemcpyHostToDevice, st));
+        nccl().check(nccl().AllGather(mine, d.p(), (size_t)n, ncclInt64, comm_, st), "ncclAllGather");
+        std::vector<int64_t> h(n * nranks);
+        if (n > 0) MX_CUDA(cudaMemcpyAsync(h.data(), d.p(), 8 * n * nranks, cudaMemcpyDeviceToHost, st));
         MX_CUDA(cudaStreamSynchronize(st));
         return h;
+    }
+    std::vector<void*> map_peers(void* local, cudaStream_t st) override {
+        cudaIpcMemHandle_t h;
+        MX_CUDA(cudaIpcGetMemHandle(&h, local));
+        static_assert(sizeof(h) % 8 == 0, "IPC handle size");
+        std::vector<int64_t> words(sizeof(h) / 8);
+        std::memcpy(words.data(), &h, sizeof(h));
+        const auto all = allgather_vec(words, st);
+        std::vector<void*> out(nranks, nullptr);
+        for (int q = 0; q < nranks; ++q) {
+            if (q == rank) { out[q] = local; continue; }
+            cudaIpcMemHandle_t hq;
+            std::memcpy(&hq, all.data() + q * words.size(), sizeof(hq));
+            void* p = nullptr;
+            MX_CUDA(cudaIpcOpenMemHandle(&p, hq, cudaIpcMemLazyEnablePeerAccess));
+            opened_.push_back(p);
+            out[q] = p;
+        }
+        return out;
     }
 
 private:
     ncclComm_t comm_ = nullptr;
+    std::vector<void*> opened_;
 };
 
 }  // namespace
@@ -232,6 +258,24 @@ public:
         g_->barrier();
         std::vector<int64_t> out(nranks);
         for (int q = 0; q < nranks; ++q) out[q] = g_->posts[q].value;
+        g_->barrier();
+        return out;
+    }
+
+    std::vector<int64_t> allgather_vec(const std::vector<int64_t>& v, cudaStream_t st) override {
+        g_->posts[rank].vec = &v;
+        g_->barrier();
+        std::vector<int64_t> out;
+        for (int q = 0; q < nranks; ++q) out.insert(out.end(), g_->posts[q].vec->begin(), g_->posts[q].vec->end());
+        g_->barrier();
+        return out;
+    }
+
+    std::vector<void*> map_peers(void* local, cudaStream_t st) override {
+        g_->posts[rank].buf = local;  // same device, same process: plain pointers
+        g_->barrier();
+        std::vector<void*> out(nranks);
+        for (int q = 0; q < nranks; ++q) out[q] = g_->posts[q].buf;
         g_->barrier();
         return out;
     }

@@ -35,6 +35,12 @@ public:
                            const int64_t* rcount, const int64_t* rdispl, DType t, cudaStream_t st) = 0;
     // gather one int64 per rank on the host (build-time bookkeeping)
     virtual std::vector<int64_t> allgather_host(int64_t v, cudaStream_t st) = 0;
+    // gather a vector of n int64 per rank: out[q * n + i] (build-time)
+    virtual std::vector<int64_t> allgather_vec(const std::vector<int64_t>& v, cudaStream_t st) = 0;
+    // Peer memory: every rank passes a cudaMalloc'ed device buffer; returns each rank's buffer as
+    // a pointer this rank's kernels can load/store (NVLink peer mapping via CUDA IPC for NCCL
+    // ranks, the plain pointer for virtual ranks).  Collective.  Throws if peers are unreachable.
+    virtual std::vector<void*> map_peers(void* local, cudaStream_t st) = 0;
 };
 
 std::unique_ptr<Comm> make_nccl_comm(int rank, int nranks, const void* unique_id);
@@ -54,6 +60,7 @@ struct LocalGroup {
         const int64_t* scount = nullptr;
         void* buf = nullptr;
         int64_t value = 0;
+        const std::vector<int64_t>* vec = nullptr;
     };
     std::vector<Post> posts;
     void barrier();

@@ -213,6 +213,7 @@ void build_exchange(Plan& P, cudaStream_t st) {
     X.y_fp.alloc(P.esize * std::max<int64_t>(P.nfp, 1));
     X.recv_buf.alloc(P.esize * std::max<int64_t>(X.nrecv, 1));
     MX_CUDA(cudaStreamSynchronize(st));
+    if (P.opt.exchange == 1) peer_setup(P, st);  // fused peer-memory exchange (peer.cu)
 }
 
 template <class T>
@@ -379,13 +380,21 @@ void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStrea
     *us_back = 1e3 * b / reps;
 }
 
+void reduce_partials(Plan& P, const float* recv, float* y, cudaStream_t st) {
+    const int64_t nown = P.s1 - P.s0;
+    reduce_kernel<float><<<nblocks(nown), kT, 0, st>>>(recv, P.ex.red_ptr.p(), P.ex.red_pos.p(), nown, y);
+    MX_LAUNCHED();
+}
+
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st) {
-    if (P.esize == 4) forward_t<float>(P, (const float*)x, (float*)y, st);
+    if (P.ex.peer) peer_forward(P, (const float*)x, (float*)y, st);
+    else if (P.esize == 4) forward_t<float>(P, (const float*)x, (float*)y, st);
     else forward_t<double>(P, (const double*)x, (double*)y, st);
 }
 
 void apply_back(Plan& P, const void* y, void* x, cudaStream_t st) {
-    if (P.esize == 4) back_t<float>(P, (const float*)y, (float*)x, st);
+    if (P.ex.peer) peer_back(P, (const float*)y, (float*)x, st);
+    else if (P.esize == 4) back_t<float>(P, (const float*)y, (float*)x, st);
     else back_t<double>(P, (const double*)y, (double*)x, st);
 }
 

@@ -1,0 +1,180 @@
+// peer.cu -- fused compute + exchange over peer memory (the "overlapped
+// interactions" of P:744-756 and the C step of A = R C A_p), EXCHANGE = 1.
+//
+// Instead of SpMV -> all-to-allv (NCCL) -> reduce, each rank maps its peers' receive buffers,
+// footprint buffers and flag arrays into its address space (CUDA IPC over NVLink for NCCL ranks,
+// plain pointers for virtual ranks) and:
+//   forward  the SpMV epilogue stores every footprint row's partial directly into its owner's
+//            receive buffer and publishes an epoch flag (spmv.cu: remote_epilogue); the owner
+//            waits for every peer's flag and reduces (R) in fixed peer order;
+//   back     the owner's pack kernel stores its ray values directly into every interacting
+//            rank's footprint buffer (R^T and C^T in one kernel) and publishes a flag; each rank
+//            waits for all owners, then runs A_p^T.
+// Credit flags make buffer reuse safe for any call sequence: a rank writes into a peer's buffer
+// only after that peer has finished consuming the previous contents.  All waits are one-thread
+// kernels (a spinning CTA never blocks a co-resident rank's kernels), with a time-out that traps
+// instead of hanging.
+#include "plan.h"
+
+namespace mx {
+
+namespace {
+
+constexpr int kT = 256;
+
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// wait until flags[base + q] >= flags[target_index] for every q < P
+__global__ void wait_kernel(const unsigned long long* flags, int P, int base, int target_index) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const unsigned long long target = ld_acquire_sys(flags + target_index);
+    const long long t0 = clock64();
+    for (int q = 0; q < P; ++q) {
+        while (ld_acquire_sys(flags + base + q) < target) {
+            __nanosleep(64);
+            if (clock64() - t0 > 40000000000LL) __trap();  // ~20 s: a peer is gone -- fail, don't hang
+        }
+    }
+}
+
+// peer_flags[q][slot] = flags[value_index] for every q (credit: "done with what you sent me")
+struct SignalArgs {
+    unsigned long long* flag[kMaxPeers];
+};
+__global__ void signal_kernel(SignalArgs sa, int P, int slot, const unsigned long long* flags, int value_index) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const unsigned long long v = flags[value_index];
+    __threadfence_system();
+    for (int q = 0; q < P; ++q) st_release(sa.flag[q] + slot, v);
+}
+
+// R^T + C^T: value j (recv order, peer g = the range containing j) goes to g's footprint buffer
+__global__ void pack_remote_kernel(const float* __restrict__ y, const int32_t* __restrict__ idx, int64_t n,
+                                   PeerArgs pa) {
+    __shared__ bool am_last;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+        int g = 0;
+        while (g + 1 < pa.P && j >= pa.bound[g + 1]) ++g;
+        pa.dst[g][pa.off[g] + j] = y[idx[j]];
+    }
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
+    __syncthreads();
+    if (!am_last || threadIdx.x != 0) return;
+    __threadfence_system();
+    const unsigned long long e = pa.my_flags[pa.epoch_index] + 1;
+    pa.my_flags[pa.epoch_index] = e;
+    for (int g = 0; g < pa.P; ++g) st_release(pa.flag[g] + pa.slot + pa.me, e);
+    *pa.ticket = 0u;
+}
+
+unsigned nblocks(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 4 * 148)); }
+
+SignalArgs signal_args(const Plan& P) {
+    SignalArgs sa{};
+    for (int q = 0; q < P.nranks; ++q) sa.flag[q] = static_cast<unsigned long long*>(P.ex.peer_flags[q]);
+    return sa;
+}
+
+}  // namespace
+
+void peer_setup(Plan& P, cudaStream_t st) {
+    Exchange& X = P.ex;
+    const int np = P.nranks;
+    if (np > kMaxPeers) fail(MEMXCT_ERR_UNSUPPORTED, "fused peer exchange supports up to 16 ranks");
+    if (P.esize != 4) fail(MEMXCT_ERR_UNSUPPORTED, "fused peer exchange is FP32 only");
+    Comm& C = *P.comm;
+    X.flags.alloc(4 * np + 2);
+    MX_CUDA(cudaMemsetAsync(X.flags.p(), 0, 8 * (4 * np + 2), st));
+    X.tickets.alloc(4);
+    MX_CUDA(cudaMemsetAsync(X.tickets.p(), 0, 16, st));
+    MX_CUDA(cudaStreamSynchronize(st));
+    // where my rows land in every owner's receive buffer, and my values in every peer's footprint
+    std::vector<int64_t> rd(X.rdispl.begin(), X.rdispl.end()), sd(X.sdispl.begin(), X.sdispl.end());
+    const auto all_rd = C.allgather_vec(rd, st);  // [q][np + 1]
+    const auto all_sd = C.allgather_vec(sd, st);
+    X.fwd_off.assign(np, 0);
+    X.back_off.assign(np, 0);
+    for (int h = 0; h < np; ++h) X.fwd_off[h] = all_rd[h * (np + 1) + P.rank] - X.sdispl[h];
+    for (int g = 0; g < np; ++g) X.back_off[g] = all_sd[g * (np + 1) + P.rank] - X.rdispl[g];
+    X.peer_recv = C.map_peers(X.recv_buf.get(), st);
+    X.peer_yfp = C.map_peers(X.y_fp.get(), st);
+    X.peer_flags = C.map_peers(X.flags.p(), st);
+    X.peer = true;
+}
+
+void peer_forward(Plan& P, const float* x, float* y, cudaStream_t st) {
+    Exchange& X = P.ex;
+    const int np = P.nranks;
+    unsigned long long* fl = X.flags.p();
+    // 1. owners have consumed my previous partials (forward credits >= my epoch)
+    wait_kernel<<<1, 32, 0, st>>>(fl, np, 2 * np, 4 * np);
+    MX_LAUNCHED();
+    // 2. A_p with the partials stored straight into the owners' receive buffers (C), flags out
+    PeerArgs pa;
+    pa.P = np;
+    pa.me = P.rank;
+    for (int h = 0; h <= np; ++h) pa.bound[h] = X.sdispl[h];
+    for (int h = 0; h < np; ++h) {
+        pa.dst[h] = static_cast<float*>(X.peer_recv[h]);
+        pa.off[h] = X.fwd_off[h];
+        pa.flag[h] = static_cast<unsigned long long*>(X.peer_flags[h]);
+    }
+    pa.my_flags = fl;
+    pa.ticket = X.tickets.p();
+    pa.slot = 0;
+    pa.epoch_index = 4 * np;
+    spmv_f32_remote(P.fwd, x, pa, st);
+    // 3. every peer's partials for my rays have arrived
+    wait_kernel<<<1, 32, 0, st>>>(fl, np, 0, 4 * np);
+    MX_LAUNCHED();
+    // 4. R
+    reduce_partials(P, X.recv_buf.as<float>(), y, st);
+    // 5. credits: my receive buffer may be overwritten again
+    signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 2 * np + P.rank, fl, 4 * np);
+    MX_LAUNCHED();
+}
+
+void peer_back(Plan& P, const float* y, float* x, cudaStream_t st) {
+    Exchange& X = P.ex;
+    const int np = P.nranks;
+    unsigned long long* fl = X.flags.p();
+    // 1. every peer has finished reading my previous values from its footprint buffer
+    wait_kernel<<<1, 32, 0, st>>>(fl, np, 3 * np, 4 * np + 1);
+    MX_LAUNCHED();
+    // 2. R^T + C^T: owned ray values straight into the peers' footprint buffers, flags out
+    PeerArgs pa;
+    pa.P = np;
+    pa.me = P.rank;
+    for (int g = 0; g <= np; ++g) pa.bound[g] = X.rdispl[g];
+    for (int g = 0; g < np; ++g) {
+        pa.dst[g] = static_cast<float*>(X.peer_yfp[g]);
+        pa.off[g] = X.back_off[g];
+        pa.flag[g] = static_cast<unsigned long long*>(X.peer_flags[g]);
+    }
+    pa.my_flags = fl;
+    pa.ticket = X.tickets.p() + 1;
+    pa.slot = np;
+    pa.epoch_index = 4 * np + 1;
+    pack_remote_kernel<<<nblocks(X.nrecv), kT, 0, st>>>(y, X.recv_idx.p(), X.nrecv, pa);
+    MX_LAUNCHED();
+    // 3. every owner's values for my footprint have arrived
+    wait_kernel<<<1, 32, 0, st>>>(fl, np, np, 4 * np + 1);
+    MX_LAUNCHED();
+    // 4. A_p^T
+    spmv_f32(P.back, X.y_fp.as<float>(), x, nullptr, nullptr, nullptr, st);
+    // 5. credits: my footprint buffer may be overwritten again
+    signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 3 * np + P.rank, fl, 4 * np + 1);
+    MX_LAUNCHED();
+}
+
+}  // namespace mx

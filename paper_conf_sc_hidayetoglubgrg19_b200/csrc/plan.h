@@ -64,12 +64,27 @@ struct Options {
     int64_t cg_variant = 0;
     int64_t vector_order = 0;  // 0 natural, 1 plan
     int64_t slices = 1;        // slices per batched call the stage buffer is sized for
+    int64_t exchange = 0;      // P > 1: 0 = transport collectives (NCCL), 1 = fused peer memory
 };
 
 // host-side angle tables on the device (reading R1)
 struct Geometry {
     const double* cos_t = nullptr;
     const double* sin_t = nullptr;
+};
+
+// Arguments of the fused SpMV + exchange epilogue and of the peer-memory pack (P > 1)
+constexpr int kMaxPeers = 16;
+struct PeerArgs {
+    int32_t P = 0, me = 0;
+    int64_t bound[kMaxPeers + 1] = {};           // row ranges per destination rank
+    float* dst[kMaxPeers] = {};                  // destination buffer of rank h (peer pointer)
+    int64_t off[kMaxPeers] = {};                 // element offset: dst[h][off[h] + row]
+    unsigned long long* flag[kMaxPeers] = {};    // flag array of rank h (peer pointer)
+    unsigned long long* my_flags = nullptr;      // this rank's flag array
+    unsigned int* ticket = nullptr;              // last-CTA counter
+    int32_t slot = 0;                            // arrival slot base in the peers' flag arrays
+    int32_t epoch_index = 0;                     // this rank's epoch counter in my_flags
 };
 
 // sparse all-to-allv plan of this rank (P > 1)
@@ -84,6 +99,14 @@ struct Exchange {
     DevBuf y_fp, recv_buf;     // footprint partials, receive / pack buffer
     DevBuf y_fp_b, recv_b;     // the same for batched (multi-slice) calls
     int32_t batch_cap = 0;
+    // fused peer-memory exchange (EXCHANGE = 1): peers' buffers and flags mapped into this rank
+    bool peer = false;
+    DevArr<unsigned long long> flags;  // [4P + 2]: arrivals fwd | arrivals back | credits fwd |
+                                       // credits back | my fwd epoch | my back epoch
+    DevArr<unsigned int> tickets;      // last-CTA counters of the fused kernels
+    std::vector<void*> peer_recv, peer_yfp, peer_flags;
+    std::vector<int64_t> fwd_off;      // owner h: my partial of footprint row i goes to recv_h[fwd_off[h] + i]
+    std::vector<int64_t> back_off;     // peer g: my value j (recv order) goes to yfp_g[back_off[g] + j]
     int64_t device_bytes() const {
         return (int64_t)(recv_idx.buf.bytes() + red_ptr.buf.bytes() + red_pos.buf.bytes() + y_fp.bytes() +
                          recv_buf.bytes() + y_fp_b.bytes() + recv_b.bytes());
@@ -184,6 +207,11 @@ void build_exchange(Plan& P, cudaStream_t st);
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
 void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);
 void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
+void reduce_partials(Plan& P, const float* recv, float* y, cudaStream_t st);
+// peer.cu: fused SpMV + exchange over peer memory (EXCHANGE = 1)
+void peer_setup(Plan& P, cudaStream_t st);
+void peer_forward(Plan& P, const float* x, float* y, cudaStream_t st);
+void peer_back(Plan& P, const float* y, float* x, cudaStream_t st);
 // K slices, slice-major [K][local_len] fp32 vectors
 void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t st);
 void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st);
@@ -194,6 +222,7 @@ void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, doubl
               unsigned int* ticket, cudaStream_t st);
 void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
               unsigned int* ticket, bool canonical, cudaStream_t st);
+void spmv_f32_remote(const Layout& L, const float* x, const PeerArgs& pa, cudaStream_t st);
 // K in {1, 2, 4, 8} slices at once: x[s*ldx + i], y[s*ldy + r]
 void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int64_t ldy, cudaStream_t st);
 int spmm_max_slices(const Layout& L);

@@ -142,9 +142,37 @@ __device__ void finish_dot_canonical(const SpmvArgs& a, const double* rows_val, 
 
 constexpr int kMaxThreads = 1024;
 
-template <bool kNatOut, bool kDot>
+__device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// Fused exchange epilogue (P > 1): every footprint row's partial is stored
+// straight into its owner's receive buffer (peer memory over NVLink), then the last CTA bumps
+// this rank's forward epoch and publishes it to every owner's arrival flag (release, system
+// scope).  Replaces the separate all-to-allv of C in A = R C A_p.
+__device__ void remote_epilogue(const PeerArgs& pa, int64_t row, bool valid, float acc) {
+    __shared__ bool am_last;
+    if (valid) {
+        int h = 0;
+        while (h + 1 < pa.P && row >= pa.bound[h + 1]) ++h;
+        pa.dst[h][pa.off[h] + row] = acc;
+    }
+    __threadfence_system();
+    __syncthreads();
+    if (threadIdx.x == 0) am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
+    __syncthreads();
+    if (!am_last || threadIdx.x != 0) return;
+    __threadfence_system();
+    const unsigned long long e = pa.my_flags[pa.epoch_index] + 1;
+    pa.my_flags[pa.epoch_index] = e;
+    for (int h = 0; h < pa.P; ++h) st_release_sys(pa.flag[h] + pa.slot + pa.me, e);
+    *pa.ticket = 0u;
+}
+
+// kEpi: 0 = plain output, 1 = fused dot (last-CTA tree), 2 = fused exchange (remote_epilogue)
+template <bool kNatOut, int kEpi>
 __global__ void __launch_bounds__(kMaxThreads, 1)
-spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) {
+spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, PeerArgs pa) {
     extern __shared__ __align__(16) float sbuf[];
     const int64_t p = blockIdx.x;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -193,8 +221,12 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) 
     }
     const int64_t row = p * a.R + threadIdx.x;
     const bool valid = row < a.nrows;
+    if (kEpi == 2) {
+        remote_epilogue(pa, row, valid, acc);
+        return;
+    }
     if (valid) y[kNatOut ? a.out_idx[row] : row] = acc;
-    if (kDot) finish_dot_tree<kMaxThreads>(a, valid ? (double)acc * (double)acc : 0.0);
+    if (kEpi == 1) finish_dot_tree<kMaxThreads>(a, valid ? (double)acc * (double)acc : 0.0);
 }
 
 // MIXED precision: fp64 stage buffer, fp64 input/output, one fp64 fma chain per row in ascending
@@ -440,9 +472,17 @@ void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, doubl
     const SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
     const size_t smem = sizeof(float) * (size_t)L.B;
     const bool nat = L.out_idx.p() != nullptr, dot = dot_out != nullptr;
-    auto kern = nat ? (dot ? spmv_f32_kernel<true, true> : spmv_f32_kernel<true, false>)
-                    : (dot ? spmv_f32_kernel<false, true> : spmv_f32_kernel<false, false>);
-    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, y);
+    auto kern = nat ? (dot ? spmv_f32_kernel<true, 1> : spmv_f32_kernel<true, 0>)
+                    : (dot ? spmv_f32_kernel<false, 1> : spmv_f32_kernel<false, 0>);
+    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, y, PeerArgs{});
+    MX_LAUNCHED();
+}
+
+void spmv_f32_remote(const Layout& L, const float* x, const PeerArgs& pa, cudaStream_t st) {
+    if (L.nparts == 0) fail(MEMXCT_ERR_UNSUPPORTED, "internal: empty A_p with the fused exchange");
+    const SpmvArgs a = make_args(L, nullptr, nullptr, nullptr);
+    const size_t smem = sizeof(float) * (size_t)L.B;
+    spmv_f32_kernel<false, 2><<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, nullptr, pa);
     MX_LAUNCHED();
 }
 
@@ -465,10 +505,11 @@ void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, dou
 void spmv_init() {
     static bool done = false;
     if (done) return;
-    set_smem(spmv_f32_kernel<true, true>);
-    set_smem(spmv_f32_kernel<true, false>);
-    set_smem(spmv_f32_kernel<false, true>);
-    set_smem(spmv_f32_kernel<false, false>);
+    set_smem(spmv_f32_kernel<true, 1>);
+    set_smem(spmv_f32_kernel<true, 0>);
+    set_smem(spmv_f32_kernel<false, 1>);
+    set_smem(spmv_f32_kernel<false, 0>);
+    set_smem(spmv_f32_kernel<false, 2>);
     set_smem(spmv_f64_kernel<true, 0>);
     set_smem(spmv_f64_kernel<true, 1>);
     set_smem(spmv_f64_kernel<true, 2>);
