@@ -212,7 +212,12 @@ public:
         const size_t es = dtype_size(t);
         g_->posts[rank].buf = buf;
         g_->barrier();
-        DevBuf tmp(es * (size_t)std::max<int64_t>(count, 1) * nranks);
+        // grow-only scratch: a cudaFree here would synchronise the whole device, i.e. wait for
+        // the other virtual ranks' kernels -- which, with the fused peer exchange, may be waiting
+        // for this rank's next kernels (deadlock)
+        const size_t need = es * (size_t)std::max<int64_t>(count, 1) * nranks;
+        if (scratch_.bytes() < need) scratch_.alloc(std::max(need, (size_t)4096));
+        DevBuf& tmp = scratch_;
         for (int q = 0; q < nranks; ++q)
             if (count > 0)
                 MX_CUDA(cudaMemcpyAsync(static_cast<char*>(tmp.get()) + q * count * es, g_->posts[q].buf, count * es,
@@ -282,6 +287,7 @@ public:
 
 private:
     std::shared_ptr<LocalGroup> g_;
+    DevBuf scratch_;
 };
 
 }  // namespace
