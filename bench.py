@@ -263,6 +263,37 @@ def bench_multislice(args, plan1, y1, n, m, c, stream):
     return out
 
 
+def bench_peer_exchange(args, n, m, c, y, local, stream, world):
+    """N > 1: the same CG with EXCHANGE = 1 (SpMV epilogue / pack kernel store straight into the
+    peers' buffers over NVLink, NEXT-2), reported beside the NCCL-exchange headline.  Failures are
+    reported, not fatal (the peer path is new on multi-GPU hardware)."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, bootstrap_unique_id
+    try:
+        uid = bootstrap_unique_id(dist.get_rank())
+        plan = MemXCT(n, m, c, rank=dist.get_rank(), nranks=world, unique_id=uid, device=local,
+                      vector_order="plan", exchange="peer").build()
+        x = torch.empty(plan.local_size(0), dtype=torch.float32, device=y.device)
+        for _ in range(max(1, args.warmup)):
+            plan.cg(y, args.iters, x=x, stream=stream)
+        dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            plan.cg(y, args.iters, x=x, stream=stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=y.device)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        plan.close()
+        return {"value": args.iters * args.steps / (float(t.item()) * 1e-3), "unit": "CG iter/s",
+                "ms_per_step": float(t.item()) / args.steps}
+    except Exception as e:  # noqa: BLE001
+        return {"error": str(e)[:300]}
+
+
 def run_ours(args, rank, world):
     import torch
     import torch.distributed as dist
@@ -369,6 +400,10 @@ def run_ours(args, rank, world):
         exch_t = {"fwd_us": float(et[0]), "back_us": float(et[1]),
                   "per_cg_iter_us": float(et[0] + et[1]), "how": "max over ranks, CUDA events, 20 reps"}
 
+    peer = None
+    if world > 1:
+        peer = bench_peer_exchange(args, n, m, c, y, local, stream, world)
+
     multislice = None
     if args.slices > 1 and world == 1:
         multislice = bench_multislice(args, plan, y, n, m, c, stream)
@@ -422,6 +457,8 @@ def run_ours(args, rank, world):
         line["exchange"] = {**plan.exchange_info(), **exch_t}
     if multislice is not None:
         line["multislice"] = multislice
+    if peer is not None:
+        line["fused_peer_exchange"] = peer
     if not args.no_cpu_baseline and world == 1:
         line["cpu_baseline"] = cpu_baseline(cfg, st["nnz"])
     print(json.dumps(line), flush=True)

@@ -144,15 +144,25 @@ public:
         std::memcpy(words.data(), &h, sizeof(h));
         const auto all = allgather_vec(words, st);
         std::vector<void*> out(nranks, nullptr);
-        for (int q = 0; q < nranks; ++q) {
+        std::string err;
+        for (int q = 0; q < nranks && err.empty(); ++q) {
             if (q == rank) { out[q] = local; continue; }
             cudaIpcMemHandle_t hq;
             std::memcpy(&hq, all.data() + q * words.size(), sizeof(hq));
             void* p = nullptr;
-            MX_CUDA(cudaIpcOpenMemHandle(&p, hq, cudaIpcMemLazyEnablePeerAccess));
+            const cudaError_t e = cudaIpcOpenMemHandle(&p, hq, cudaIpcMemLazyEnablePeerAccess);
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                err = std::string("cudaIpcOpenMemHandle(peer ") + std::to_string(q) + "): " + cudaGetErrorString(e);
+                break;
+            }
             opened_.push_back(p);
             out[q] = p;
         }
+        // agree on success before anyone goes on (a one-sided failure would hang the others)
+        const auto ok = allgather_host(err.empty() ? 1 : 0, st);
+        for (int64_t v : ok)
+            if (!v) fail(MEMXCT_ERR_UNSUPPORTED, err.empty() ? "peer mapping failed on another rank" : err);
         return out;
     }
 
