@@ -1,0 +1,98 @@
+"""Cases of the fused peer-memory exchange on virtual ranks, run in a child process by
+tests/test_gpu_peer_exchange.py.
+
+Virtual ranks share ONE device, so any device-wide synchronisation issued by one rank's thread
+(cudaFree from a garbage-collected plan, an allocator trim, ...) waits for the other ranks'
+spinning flag waits while those ranks wait for it: a deadlock that cannot happen with one
+process per GPU (a rank's own waits only depend on kernels its peers have already queued).  The
+cases therefore run in a fresh process with the garbage collector off and pre-allocated tensors,
+and a failure (the wait kernels trap after ~20 s instead of hanging) cannot poison the main test
+process's CUDA context.
+"""
+import gc
+import os
+import sys
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, HERE)
+sys.path.insert(0, os.path.dirname(HERE))
+
+
+def rel_l2(a, b):
+    return float(np.linalg.norm(np.asarray(a) - np.asarray(b)) / np.linalg.norm(np.asarray(b)))
+
+
+def case_projections(nranks, n, m, c):
+    import torch
+
+    import oracle
+    from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
+    from test_gpu_multirank import build_group, gather, run_ranks, scatter
+    g0, coll = build_group(n, m, c, nranks)
+    g1, peer = build_group(n, m, c, nranks, exchange="peer")
+    x = inputs.uniform(n * n, 1)
+    y = inputs.uniform(m * c, 2)
+    res = {}
+    for name, plans in (("coll", coll), ("peer", peer)):
+        xs, ys = scatter(plans, x, 0, np.float32), scatter(plans, y, 1, np.float32)
+        xs2 = [v * 2 for v in xs]
+        ys3 = [v * 3 for v in ys]
+        outs = [[torch.empty(p.local_size(1), device="cuda") for _ in range(3)] +
+                [torch.empty(p.local_size(0), device="cuda") for _ in range(3)] for p in plans]
+        torch.cuda.synchronize()
+
+        def body(r, plans=plans, xs=xs, ys=ys, xs2=xs2, ys3=ys3, outs=outs):
+            p, o = plans[r], outs[r]
+            p.forward(xs[r], o[0])
+            p.forward(xs2[r], o[1])
+            p.back(ys[r], o[3])
+            p.back(ys3[r], o[4])
+            p.forward(xs[r], o[2])
+            p.back(ys[r], o[5])
+            return o
+        res[name] = run_ranks(nranks, body)
+    for r in range(nranks):
+        for k in range(6):
+            assert torch.equal(res["coll"][r][k], res["peer"][r][k]), (r, k)
+    rows, cols, vals = oracle.trace_all(n, m, c)
+    yf = gather(peer, [o[0] for o in res["peer"]], 1, m * c)
+    assert rel_l2(yf, oracle.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)) <= 1e-5
+    xb = gather(peer, [o[3] for o in res["peer"]], 0, n * n)
+    assert rel_l2(xb, oracle.spmv_coo(cols, rows, vals, y.astype(np.float64), n * n)) <= 1e-5
+
+
+def case_cg(nranks, n, m, c):
+    import torch
+
+    import oracle
+    from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
+    from test_gpu_multirank import build_group, gather, run_ranks, scatter
+    g0, coll = build_group(n, m, c, nranks)
+    g1, peer = build_group(n, m, c, nranks, exchange="peer")
+    rows, cols, vals = oracle.trace_all(n, m, c)
+    xt = inputs.shepp_logan(n)
+    y32 = oracle.spmv_coo(rows, cols, vals, xt, m * c).astype(np.float32)
+    out = {}
+    for name, plans in (("coll", coll), ("peer", peer)):
+        ys = scatter(plans, y32, 1, np.float32)
+        xs = [torch.empty(p.local_size(0), device="cuda") for p in plans]
+        torch.cuda.synchronize()
+        out[name] = run_ranks(nranks, lambda r, plans=plans, ys=ys, xs=xs: plans[r].cg(ys[r], 30, x=xs[r]))
+    for a, b in zip(out["coll"], out["peer"]):
+        assert torch.equal(a, b)
+    xr = gather(peer, out["peer"], 0, n * n)
+    x_orc = oracle.cgls(rows, cols, vals, y32.astype(np.float64), m * c, n * n, 30)[0]
+    assert rel_l2(xr, xt) <= 1.1 * rel_l2(x_orc, xt)
+
+
+if __name__ == "__main__":
+    import torch
+    gc.disable()
+    torch.cuda.init()
+    case, nranks, n, m, c = sys.argv[1], *map(int, sys.argv[2:6])
+    {"projections": case_projections, "cg": case_cg}[case](nranks, n, m, c)
+    torch.cuda.synchronize()
+    print("CASE OK", case, nranks, n, m, c, flush=True)
+    os._exit(0)  # skip teardown frees while nothing else runs; the process ends here
