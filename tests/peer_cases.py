@@ -12,12 +12,52 @@ process's CUDA context.
 import gc
 import os
 import sys
+import threading
 
 import numpy as np
+
+# Concurrent streams of one process share a few hardware queues (CUDA_DEVICE_MAX_CONNECTIONS,
+# default 8); two virtual ranks whose streams land on the same queue serialise, and a rank's
+# flag wait would then block the very kernel it waits for.  Give every stream its own queue and
+# create the ranks' streams once.
+os.environ["CUDA_DEVICE_MAX_CONNECTIONS"] = "32"
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, HERE)
 sys.path.insert(0, os.path.dirname(HERE))
+
+_STREAMS = {}
+
+
+def run_ranks(nranks, fn):
+    import torch
+    for r in range(nranks):
+        _STREAMS.setdefault(r, torch.cuda.Stream())
+    out, err = [None] * nranks, [None] * nranks
+
+    def body(r):
+        try:
+            with torch.cuda.stream(_STREAMS[r]):
+                out[r] = fn(r)
+                _STREAMS[r].synchronize()
+        except BaseException as e:  # noqa: BLE001
+            err[r] = e
+    ts = [threading.Thread(target=body, args=(r,)) for r in range(nranks)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(timeout=600)
+    for e in err:
+        if e is not None:
+            raise e
+    return out
+
+
+def build_group(n, m, c, nranks, **kw):
+    from paper_conf_sc_hidayetoglubgrg19_b200 import LocalGroup, MemXCT
+    g = LocalGroup(nranks)
+    plans = run_ranks(nranks, lambda r: MemXCT(n, m, c, group=g, rank=r, vector_order="plan", **kw).build())
+    return g, plans
 
 
 def rel_l2(a, b):
@@ -29,9 +69,12 @@ def case_projections(nranks, n, m, c):
 
     import oracle
     from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
-    from test_gpu_multirank import build_group, gather, run_ranks, scatter
+    from test_gpu_multirank import gather, scatter
+    import time
+    t0 = time.time()
     g0, coll = build_group(n, m, c, nranks)
     g1, peer = build_group(n, m, c, nranks, exchange="peer")
+    print(f"built {time.time() - t0:.2f}s", flush=True)
     x = inputs.uniform(n * n, 1)
     y = inputs.uniform(m * c, 2)
     res = {}
@@ -52,7 +95,10 @@ def case_projections(nranks, n, m, c):
             p.forward(xs[r], o[2])
             p.back(ys[r], o[5])
             return o
-        res[name] = run_ranks(nranks, body)
+        try:
+            res[name] = run_ranks(nranks, body)
+        finally:
+            print(f"{name} done {time.time() - t0:.2f}s", flush=True)
     for r in range(nranks):
         for k in range(6):
             assert torch.equal(res["coll"][r][k], res["peer"][r][k]), (r, k)
@@ -68,7 +114,7 @@ def case_cg(nranks, n, m, c):
 
     import oracle
     from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
-    from test_gpu_multirank import build_group, gather, run_ranks, scatter
+    from test_gpu_multirank import gather, scatter
     g0, coll = build_group(n, m, c, nranks)
     g1, peer = build_group(n, m, c, nranks, exchange="peer")
     rows, cols, vals = oracle.trace_all(n, m, c)
