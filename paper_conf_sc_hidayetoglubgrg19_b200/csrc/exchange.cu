@@ -380,6 +380,13 @@ void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStrea
     *us_back = 1e3 * b / reps;
 }
 
+void preload_exchange_kernels() {
+    cudaFuncAttributes fa;
+    MX_CUDA(cudaFuncGetAttributes(&fa, reduce_kernel<float>));
+    MX_CUDA(cudaFuncGetAttributes(&fa, reduce_kernel<double>));
+    MX_CUDA(cudaFuncGetAttributes(&fa, pack_kernel<float>));
+}
+
 void reduce_partials(Plan& P, const float* recv, float* y, cudaStream_t st) {
     const int64_t nown = P.s1 - P.s0;
     reduce_kernel<float><<<nblocks(nown), kT, 0, st>>>(recv, P.ex.red_ptr.p(), P.ex.red_pos.p(), nown, y);

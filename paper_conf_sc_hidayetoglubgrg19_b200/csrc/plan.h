@@ -208,6 +208,7 @@ void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
 void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);
 void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 void reduce_partials(Plan& P, const float* recv, float* y, cudaStream_t st);
+void preload_exchange_kernels();
 // peer.cu: fused SpMV + exchange over peer memory (EXCHANGE = 1)
 void peer_setup(Plan& P, cudaStream_t st);
 void peer_forward(Plan& P, const float* x, float* y, cudaStream_t st);

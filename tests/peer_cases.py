@@ -21,6 +21,7 @@ import numpy as np
 # flag wait would then block the very kernel it waits for.  Give every stream its own queue and
 # create the ranks' streams once.
 os.environ["CUDA_DEVICE_MAX_CONNECTIONS"] = "32"
+os.environ["CUDA_MODULE_LOADING"] = "EAGER"  # no kernel loading (and its device waits) mid-run
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, HERE)
@@ -39,7 +40,6 @@ def run_ranks(nranks, fn):
         try:
             with torch.cuda.stream(_STREAMS[r]):
                 out[r] = fn(r)
-                _STREAMS[r].synchronize()
         except BaseException as e:  # noqa: BLE001
             err[r] = e
     ts = [threading.Thread(target=body, args=(r,)) for r in range(nranks)]
@@ -47,6 +47,8 @@ def run_ranks(nranks, fn):
         t.start()
     for t in ts:
         t.join(timeout=600)
+    for r in range(nranks):  # synchronise only after every rank has queued all of its work
+        _STREAMS[r].synchronize()
     for e in err:
         if e is not None:
             raise e
