@@ -321,8 +321,11 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
             else P.comm = mx::make_nccl_comm(P.rank, P.nranks, P.unique_id.data());
         }
         resolve_tuning(P);
+        // CG dots fused into the SpMV epilogue (per-CTA tree + last-CTA sum, deterministic):
+        // default since the jagged kernel (3.874 vs 3.882 ms per cfg3 iteration, one kernel
+        // fewer per SpMV); MEMXCT_FUSED_DOT=0 restores the separate dot kernels
         const char* fd = std::getenv("MEMXCT_FUSED_DOT");
-        P.fused_dot = fd && fd[0] == '1';
+        P.fused_dot = !(fd && fd[0] == '0');
         mx::build_matrices(P, st);
         MX_CUDA(cudaStreamSynchronize(st));
         P.built = true;

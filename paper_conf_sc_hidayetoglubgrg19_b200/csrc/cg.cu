@@ -178,12 +178,13 @@ unsigned vec_blocks(int64_t n) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(kVecBlocks, ceil_div(n, kVT)));
 }
 
-// Projection of K slices followed by the per-slice dot of the output.  Canonical mode (K = 1,
-// P = 1) fuses the dot into the SpMV epilogue (per-partition fma chains, reading R16).
-// Otherwise a separate small dot kernel is used: measured on B200, the fused last-CTA epilogue
-// slowed the 2 ms SpMV by ~0.5 ms (profiles/r01a_launches.md), while the separate pass over the
-// 4-6 MB vector costs a few us.  P > 1: the projection includes the exchange (A = R C A_p) and
-// the local dots are allreduced.
+// Projection of K slices followed by the per-slice dot of the output.  At K = 1, P = 1 the dot
+// is fused into the SpMV epilogue: canonical mode as per-partition fma chains (reading R16),
+// otherwise as a per-CTA tree + last-CTA sum in partition order (deterministic).  (With the
+// first, uniform-width kernel that epilogue cost 0.5 ms per 2 ms SpMV, profiles/r01a_launches.md;
+// with the jagged kernel it is free, so it is the default; MEMXCT_FUSED_DOT=0 selects the
+// separate dot kernel.)  Batched and P > 1: separate dot kernels; P > 1 allreduces them (the
+// projection then includes the exchange, A = R C A_p).
 template <class T>
 void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, int64_t dot_stride,
             cudaStream_t st) {

@@ -136,7 +136,7 @@ struct Plan {
     bool built = false;
     int32_t rank = 0, nranks = 1, device = -1;
     int32_t tile_tomo = 0, tile_sino = 0;
-    bool fused_dot = false;  // MEMXCT_FUSED_DOT=1: fuse CG dots into the SpMV epilogue (tuning)
+    bool fused_dot = true;   // CG dots in the SpMV epilogue (MEMXCT_FUSED_DOT=0: separate kernels)
     int32_t part_rows = 0, buffer_entries = 0;  // resolved tuning (build)
 
     // domain decomposition: this rank owns Hilbert pixels [t0, t1) and rays [s0, s1)
