@@ -51,6 +51,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--spmv-reps", type=int, default=20)
     ap.add_argument("--slices", type=int, default=4, help="multi-slice batch measured beside the headline (1 = off)")
+    ap.add_argument("--distributed", action="store_true",
+                    help="run the decomposed path (NCCL communicator, exchange, allreduce) even at N = 1")
     return ap.parse_args()
 
 
@@ -310,8 +312,9 @@ def run_ours(args, rank, world):
         kw["part_rows"] = args.part_rows
     if args.buffer:
         kw["buffer_entries"] = args.buffer
+    dist_mode = world > 1 or args.distributed
     t0 = time.perf_counter()
-    if world > 1:
+    if dist_mode:
         # domain decomposition over the ranks (A = R C A_p), NCCL exchange
         from paper_conf_sc_hidayetoglubgrg19_b200 import bootstrap_unique_id
         uid = bootstrap_unique_id(rank)
@@ -327,7 +330,7 @@ def run_ours(args, rank, world):
     # synthetic slice: phantom sinogram from our own forward projection (values do not change
     # the access pattern; the parity tests pin the values against the oracle)
     ph = inputs.shepp_logan(n).astype(np.float32)
-    if world > 1:
+    if dist_mode:
         ph = np.ascontiguousarray(ph[plan.local_indices(0)])
     x_ph = torch.from_numpy(ph).to(dev)
     y = plan.forward(x_ph)
@@ -341,7 +344,7 @@ def run_ours(args, rank, world):
     clocks = Clocks(local)
     clocks.start()
     time.sleep(0.3)
-    if world > 1:
+    if dist_mode:
         dist.barrier()
     torch.cuda.synchronize()
     k0 = kernel_launch_count()
@@ -372,7 +375,7 @@ def run_ours(args, rank, world):
     clk = clocks.stop()
 
     t = torch.tensor([ms], dtype=torch.float64, device=dev)
-    if world > 1:
+    if dist_mode:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_max = float(t.item())
 
@@ -381,19 +384,19 @@ def run_ours(args, rank, world):
     y_host.copy_(y.cpu())
     x_host = torch.empty(plan.local_size(0), dtype=torch.float32, pin_memory=True)
     plan.cg_host_ptr(y_host.data_ptr(), x_host.data_ptr(), args.iters, stream=stream)  # warm
-    if world > 1:
+    if dist_mode:
         dist.barrier()
     te0 = time.perf_counter()
     for _ in range(args.steps):
         plan.cg_host_ptr(y_host.data_ptr(), x_host.data_ptr(), args.iters, stream=stream)
     te = time.perf_counter() - te0
     te_t = torch.tensor([te], dtype=torch.float64, device=dev)
-    if world > 1:
+    if dist_mode:
         dist.all_reduce(te_t, op=dist.ReduceOp.MAX)
     te = float(te_t.item())
 
     exch_t = None
-    if world > 1:
+    if dist_mode:
         exch_t = plan.exchange_time(20, stream=stream)
         et = torch.tensor([exch_t["fwd_us"], exch_t["back_us"]], dtype=torch.float64, device=dev)
         dist.all_reduce(et, op=dist.ReduceOp.MAX)
@@ -401,11 +404,11 @@ def run_ours(args, rank, world):
                   "per_cg_iter_us": float(et[0] + et[1]), "how": "max over ranks, CUDA events, 20 reps"}
 
     peer = None
-    if world > 1:
+    if dist_mode:
         peer = bench_peer_exchange(args, n, m, c, y, local, stream, world)
 
     multislice = None
-    if args.slices > 1 and world == 1:
+    if args.slices > 1 and not dist_mode:
         multislice = bench_multislice(args, plan, y, n, m, c, stream)
 
     if rank != 0:
@@ -424,16 +427,16 @@ def run_ours(args, rank, world):
     line = {
         "metric": "CG iter/s", "value": value, "unit": "CG iter/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
-        "higher_is_better": True, "scaling": "strong" if world > 1 else "weak", "vs_baseline": None,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
         "dtype": "f32",
         "data": "synthetic",
         "config": {"workload": workload_name(cfg, args.iters),
                    "l2": "no flush: the matrix stream per SpMV (%.1f GB) exceeds the 126 MB L2" %
-                         ((st["stored_slots"] * 3) / 2 / 1e9),
+                         (6 * st["stored_slots"] / 2 / 1e9),
                    "part_rows": plan.get_option("part_rows"),
                    "buffer_entries": plan.get_option("buffer_entries"),
                    "parallelism": (f"domain decomposition over {world} GPUs (A = R C A_p, NCCL all-to-allv)"
-                                   if world > 1 else "single GPU")},
+                                   if dist_mode else "single GPU")},
         "spmv": {"fwd_ms": tf * 1e3, "back_ms": tb * 1e3,
                  "fwd_gflops": 2 * fi["nnz"] / tf / 1e9, "back_gflops": 2 * bi["nnz"] / tb / 1e9,
                  "fwd_gbs": fb / tf / 1e9, "back_gbs": bb / tb / 1e9,
@@ -453,7 +456,7 @@ def run_ours(args, rank, world):
         "build_s": build_s,
         "device_bytes": st["device_bytes"],
     }
-    if world > 1:
+    if dist_mode:
         line["exchange"] = {**plan.exchange_info(), **exch_t}
     if multislice is not None:
         line["multislice"] = multislice
@@ -468,7 +471,11 @@ def main():
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    if world > 1:
+    if world == 1 and args.distributed and args.impl == "ours":
+        for k, v in (("MASTER_ADDR", "127.0.0.1"), ("MASTER_PORT", "29533"), ("RANK", "0"),
+                     ("WORLD_SIZE", "1"), ("LOCAL_RANK", "0")):
+            os.environ.setdefault(k, v)
+    if world > 1 or (args.distributed and args.impl == "ours"):
         import torch.distributed as dist
         if args.impl == "ours":
             import torch
@@ -482,7 +489,7 @@ def main():
         else:
             run_ours(args, rank, world)
     finally:
-        if world > 1:
+        if world > 1 or (args.distributed and args.impl == "ours"):
             import torch.distributed as dist
             dist.destroy_process_group()
 

@@ -113,7 +113,9 @@ memxct_status_t memxct_plan_get_option(memxct_plan_t plan, memxct_option_t optio
 
 /* Multi-GPU (P > 1, A = R C A_p): rank in [0, nranks), a 128-byte ncclUniqueId
  * produced by rank 0 and broadcast by the caller, and the CUDA device of this rank.  Before
- * build.  nranks == 1 is accepted and means single GPU. */
+ * build.  With nranks == 1: a NULL id means the plain single-GPU plan; a non-NULL id runs the
+ * decomposed path (footprint, exchange maps, NCCL send/recv and allreduce) on a one-rank
+ * communicator -- same results, used to exercise the multi-GPU code on one device. */
 memxct_status_t memxct_plan_set_comm(memxct_plan_t plan, int32_t rank, int32_t nranks,
                                      const void* nccl_unique_id, int32_t cuda_device);
 

@@ -204,12 +204,13 @@ memxct_status_t memxct_plan_set_comm(memxct_plan_t plan, int32_t rank, int32_t n
         mx::Plan& P = plan_of(plan);
         if (P.built) mx::fail(MEMXCT_ERR_STATE, "set_comm must precede memxct_build");
         if (nranks < 1 || rank < 0 || rank >= nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank / nranks");
-        if (nranks > 1) {
-            need(nccl_unique_id, "nccl_unique_id");
+        if (nranks > 1) need(nccl_unique_id, "nccl_unique_id");
+        P.unique_id.clear();
+        if (nccl_unique_id)
             P.unique_id.assign((const uint8_t*)nccl_unique_id, (const uint8_t*)nccl_unique_id + 128);
-        }
         P.rank = rank;
         P.nranks = nranks;
+        P.dist = nccl_unique_id != nullptr;
         P.device = cuda_device;
         P.local_group.reset();
     });
@@ -242,6 +243,7 @@ memxct_status_t memxct_plan_set_comm_local(memxct_plan_t plan, memxct_group_t gr
         if (rank < 0 || rank >= group->g->nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank");
         P.rank = rank;
         P.nranks = group->g->nranks;
+        P.dist = true;
         P.local_group = group->g;
     });
 }
@@ -294,8 +296,8 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
         if (P.built) mx::fail(MEMXCT_ERR_STATE, "plan already built");
         if (P.opt.canonical && P.opt.precision != 1)
             mx::fail(MEMXCT_ERR_INVALID_ARG, "CANONICAL requires PRECISION = MIXED");
-        if (P.opt.vector_order == 0 && P.nranks > 1)
-            mx::fail(MEMXCT_ERR_INVALID_ARG, "natural vector order requires P = 1");
+        if (P.opt.vector_order == 0 && P.dist)
+            mx::fail(MEMXCT_ERR_INVALID_ARG, "natural vector order requires the undecomposed plan");
         int ndev = 0;
         if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
             cudaGetLastError();
@@ -315,7 +317,7 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
         mx::build_hilbert(P.n, P.n, P.tile_tomo, P.tomo_nat_of_h.p(), P.tomo_h_of_nat.p(), &P.tomo_tile_off, st);
         mx::build_hilbert(P.m, P.c, P.tile_sino, P.sino_nat_of_h.p(), P.sino_h_of_nat.p(), &P.sino_tile_off, st);
         P.esize = P.opt.precision == 1 ? 8 : 4;
-        if (P.nranks > 1) {
+        if (P.dist) {
             if (P.opt.canonical) mx::fail(MEMXCT_ERR_UNSUPPORTED, "CANONICAL mode is single-GPU only");
             if (P.local_group) P.comm = mx::make_local_comm(P.local_group, P.rank);
             else P.comm = mx::make_nccl_comm(P.rank, P.nranks, P.unique_id.data());

@@ -188,8 +188,8 @@ unsigned vec_blocks(int64_t n) {
 template <class T>
 void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, int64_t dot_stride,
             cudaStream_t st) {
-    const bool fused = dot_out && K == 1 && P.nranks == 1 && (P.opt.canonical != 0 || P.fused_dot);
-    if (P.nranks == 1 && K == 1) {
+    const bool fused = dot_out && K == 1 && !P.dist && (P.opt.canonical != 0 || P.fused_dot);
+    if (!P.dist && K == 1) {
         const Layout& L = forward ? P.fwd : P.back;
         double* part = forward ? P.part_fwd.p() : P.part_back.p();
         if constexpr (sizeof(T) == 4)
@@ -212,13 +212,13 @@ void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, 
         dot_kernel<T><<<dim3(vec_blocks(n), K), kVT, 0, st>>>(out, n, dot_out, dot_stride, P.part_vec.p(),
                                                               P.tickets.p() + 64);
         MX_LAUNCHED();
-        if (P.nranks > 1)
+        if (P.dist)
             for (int s = 0; s < K; ++s) P.comm->allreduce_sum(dot_out + s * dot_stride, 1, DType::F64, st);
     }
 }
 
 void allreduce_slices(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) {
-    if (P.nranks > 1)
+    if (P.dist)
         for (int s = 0; s < K; ++s) P.comm->allreduce_sum(v + s * stride, 1, DType::F64, st);
 }
 
@@ -295,7 +295,7 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, int32_t K, cudaStrea
         P.scal.alloc(nd);
         MX_CUDA(cudaMemsetAsync(P.scal.p(), 0, 8 * nd, st));
     }
-    if (P.nranks > 1 && !P.comm->capturable()) {  // virtual ranks: eager launches
+    if (P.dist && !P.comm->capturable()) {  // virtual ranks: eager launches
         cg_enqueue_any(P, y, x, iters, K, st);
         return;
     }

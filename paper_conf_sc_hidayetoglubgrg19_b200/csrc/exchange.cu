@@ -97,7 +97,7 @@ std::vector<int64_t> tile_sums(const int32_t* w, const std::vector<int64_t>& til
 // a3: tomogram and sinogram ranges of this rank
 void decompose(Plan& P, const Geometry& G, cudaStream_t st) {
     const int64_t npix = (int64_t)P.n * P.n, nrays = (int64_t)P.m * P.c;
-    if (P.nranks == 1) {
+    if (!P.dist) {
         P.t0 = 0; P.t1 = npix; P.s0 = 0; P.s1 = nrays;
         P.tomo_bounds = {0, npix};
         P.sino_bounds = {0, nrays};
@@ -134,7 +134,7 @@ void decompose(Plan& P, const Geometry& G, cudaStream_t st) {
 // footprint rays of the local tomogram subdomain (all rays at P = 1) and their row lengths
 int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStream_t st) {
     const int64_t nrays = (int64_t)P.m * P.c;
-    if (P.nranks == 1) {
+    if (!P.dist) {
         fp_len.alloc(nrays);
         trace_count(P, G, nullptr, 0, nrays, 0, 0, false, fp_len.p(), st);
         P.fp_rays.reset();
@@ -166,7 +166,7 @@ int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStrea
 
 // a6: exchange maps (P > 1)
 void build_exchange(Plan& P, cudaStream_t st) {
-    if (P.nranks == 1) return;
+    if (!P.dist) return;
     Comm& C = *P.comm;
     Exchange& X = P.ex;
     const int np = P.nranks;
@@ -218,7 +218,7 @@ void build_exchange(Plan& P, cudaStream_t st) {
 
 template <class T>
 static void forward_t(Plan& P, const T* x, T* y, cudaStream_t st) {
-    if (P.nranks == 1) {
+    if (!P.dist) {
         spmv_any(P, P.fwd, x, y, st);
         return;
     }
@@ -235,7 +235,7 @@ static void forward_t(Plan& P, const T* x, T* y, cudaStream_t st) {
 
 template <class T>
 static void back_t(Plan& P, const T* y, T* x, cudaStream_t st) {
-    if (P.nranks == 1) {
+    if (!P.dist) {
         spmv_any(P, P.back, y, x, st);
         return;
     }
@@ -278,7 +278,7 @@ void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t 
         const int k = group_size(P, K - s0);
         const float* xs = x + s0 * nx;
         float* ys = y + s0 * ny;
-        if (P.nranks == 1) {
+        if (!P.dist) {
             spmm_f32(P.fwd, k, xs, nx, ys, ny, st);
         } else {
             ensure_batch_buffers(P, k);
@@ -304,7 +304,7 @@ void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st)
         const int k = group_size(P, K - s0);
         const float* ys = y + s0 * ny;
         float* xs = x + s0 * nx;
-        if (P.nranks == 1) {
+        if (!P.dist) {
             spmm_f32(P.back, k, ys, ny, xs, nx, st);
         } else {
             ensure_batch_buffers(P, k);
@@ -331,7 +331,7 @@ void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st)
 // of the north star (one forward + one back exchange per CG iteration).
 void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st) {
     *us_fwd = *us_back = 0.0;
-    if (P.nranks == 1 || reps < 1) return;
+    if (!P.dist || reps < 1) return;
     Exchange& X = P.ex;
     const DType t = P.esize == 4 ? DType::F32 : DType::F64;
     const int64_t nown = P.s1 - P.s0;

@@ -703,7 +703,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
     // rows of A_p = footprint rays (every ray at P = 1) and their lengths
     DevArr<int32_t> fp_len;
     const int64_t nrows = P.nfp = footprint(P, G, fp_len, st);
-    const int32_t* hray = P.nranks == 1 ? nullptr : P.fp_rays.p();
+    const int32_t* hray = !P.dist ? nullptr : P.fp_rays.p();
     const bool natural = (P.opt.vector_order == 0);  // P = 1 only
     const int32_t R = P.part_rows;
     const int32_t B = P.opt.precision == 1 ? P.buffer_entries / 2 : P.buffer_entries;

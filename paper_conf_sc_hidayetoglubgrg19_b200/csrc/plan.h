@@ -135,6 +135,9 @@ struct Plan {
     Options opt;
     bool built = false;
     int32_t rank = 0, nranks = 1, device = -1;
+    // decomposed path (A = R C A_p with a communicator): set by set_comm / set_comm_local, also
+    // at nranks = 1 (a one-rank communicator runs every exchange step against itself)
+    bool dist = false;
     int32_t tile_tomo = 0, tile_sino = 0;
     bool fused_dot = true;   // CG dots in the SpMV epilogue (MEMXCT_FUSED_DOT=0: separate kernels)
     int32_t part_rows = 0, buffer_entries = 0;  // resolved tuning (build)

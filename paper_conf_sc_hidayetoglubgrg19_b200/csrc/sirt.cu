@@ -94,7 +94,7 @@ void sirt_t(Plan& P, const T* y, T* x, int32_t iters, double* res2_dev, cudaStre
         MX_LAUNCHED();
         sum_parts_kernel<<<1, 32, 0, st>>>(S.part.p(), (int)g, res2_dev + k);       // ||y - A x_k||^2
         MX_LAUNCHED();
-        if (P.nranks > 1) P.comm->allreduce_sum(res2_dev + k, 1, DType::F64, st);
+        if (P.dist) P.comm->allreduce_sum(res2_dev + k, 1, DType::F64, st);
         if (k == iters) break;
         apply_back(P, S.r.get(), S.s.get(), st);                                    // A^T R (y - A x_k)
         update_kernel<T><<<nb(nx), kT, 0, st>>>(x, S.s.as<T>(), S.cinv.as<T>(), nx);

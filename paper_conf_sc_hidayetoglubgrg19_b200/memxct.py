@@ -198,7 +198,7 @@ class MemXCT:
         self.nranks = group.nranks if group is not None else int(nranks)
         if group is not None:
             _check(lib().memxct_plan_set_comm_local(self._h, group._h, int(rank)), "memxct_plan_set_comm_local")
-        elif nranks > 1 or device is not None:
+        elif nranks > 1 or device is not None or unique_id is not None:
             uid = None if unique_id is None else ctypes.create_string_buffer(unique_id, 128)
             _check(lib().memxct_plan_set_comm(self._h, rank, nranks, uid,
                                               -1 if device is None else int(device)),

@@ -63,7 +63,7 @@ def gather(plans, parts, domain, size):
     return out
 
 
-@pytest.mark.parametrize("nranks", [2, 3, 4])
+@pytest.mark.parametrize("nranks", [1, 2, 3, 4])
 @pytest.mark.parametrize("geom", [(64, 90, 64), (256, 360, 256)])
 def test_decomposition_and_fp32_projections(orc, coo_cache, nranks, geom):
     n, m, c = geom
@@ -132,3 +132,43 @@ def test_fp32_cg_multirank_recovers_phantom(orc, coo_cache):
     x_orc = orc.cgls(rows, cols, vals, y32.astype(np.float64), m * c, n * n, 30)[0]
     assert rel_l2(xr, xt) <= 1.1 * rel_l2(x_orc, xt)
     assert np.all(np.diff(res[0][1]) <= 1e-6 * res[0][1][0])
+
+
+@pytest.mark.parametrize("exchange", ["collective", "peer"])
+def test_one_rank_nccl_communicator(orc, coo_cache, exchange):
+    """The decomposed path on a real one-rank NCCL communicator (memxct_get_unique_id + set_comm
+    with nranks = 1): NCCL loading, communicator init, grouped send/recv to self, allreduce,
+    allgather, CUDA IPC peer mapping and the graph-captured CG run exactly as on a multi-GPU
+    node.  Projections are bit-identical to the plain plan in plan order (one partial per ray:
+    the reduction adds it to zero); CG differs only in the dot summation order."""
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, get_unique_id
+    n, m, c = 256, 360, 256
+    dist = MemXCT(n, m, c, rank=0, nranks=1, unique_id=get_unique_id(), device=0,
+                  vector_order="plan", exchange=exchange).build()
+    plain = MemXCT(n, m, c, vector_order="plan").build()
+    for d in (0, 1):
+        assert np.array_equal(dist.local_indices(d), plain.local_indices(d))
+    info = dist.exchange_info()
+    assert info["sent"] == info["received"] and info["peers"] <= 1
+    rows, cols, vals = coo_cache(n, m, c)
+    xt = inputs.shepp_logan(n)
+    x = torch.from_numpy(xt[plain.local_indices(0)].astype(np.float32)).cuda()
+    y = torch.from_numpy(inputs.uniform(m * c, 5)[plain.local_indices(1)].astype(np.float32)).cuda()
+    for _ in range(2):  # repeated calls exercise the peer path's credit flags
+        assert torch.equal(dist.forward(x), plain.forward(x))
+        assert torch.equal(dist.back(y), plain.back(y))
+    y32 = orc.spmv_coo(rows, cols, vals, xt, m * c).astype(np.float32)
+    ys = torch.from_numpy(y32[plain.local_indices(1)]).cuda()
+    xd, rd = dist.cg(ys, 30, residuals=True)
+    xp, rp = plain.cg(ys, 30, residuals=True)
+    xd2 = dist.cg(ys, 30)  # graph replay
+    assert torch.equal(xd, xd2)
+    assert rel_l2(xd.cpu().numpy(), xp.cpu().numpy()) <= 1e-3
+    xr = np.zeros(n * n)
+    xr[plain.local_indices(0)] = xd.cpu().numpy()
+    x_orc = orc.cgls(rows, cols, vals, y32.astype(np.float64), m * c, n * n, 30)[0]
+    assert rel_l2(xr, xt) <= 1.1 * rel_l2(x_orc, xt)
+    t = dist.exchange_time(5)
+    assert t["fwd_us"] > 0 and t["back_us"] > 0
+    dist.close()
+    plain.close()

@@ -30,7 +30,7 @@ def run_case(*args):
     assert r.returncode == 0 and "CASE OK" in r.stdout, (r.stdout[-2000:], r.stderr[-4000:])
 
 
-@pytest.mark.parametrize("nranks", [2, 3, 4])
+@pytest.mark.parametrize("nranks", [1, 2, 3, 4])
 @pytest.mark.parametrize("geom", [(64, 90, 64), (256, 360, 256)])
 def test_peer_exchange_bit_identical_to_collective(nranks, geom):
     run_case("projections", nranks, *geom)
