@@ -398,10 +398,14 @@ def run_ours(args, rank, world):
     exch_t = None
     if dist_mode:
         exch_t = plan.exchange_time(20, stream=stream)
-        et = torch.tensor([exch_t["fwd_us"], exch_t["back_us"]], dtype=torch.float64, device=dev)
+        sp_t = plan.spmv_time(20, stream=stream)
+        et = torch.tensor([exch_t["fwd_us"], exch_t["back_us"], sp_t["fwd_us"], sp_t["back_us"]],
+                          dtype=torch.float64, device=dev)
         dist.all_reduce(et, op=dist.ReduceOp.MAX)
         exch_t = {"fwd_us": float(et[0]), "back_us": float(et[1]),
-                  "per_cg_iter_us": float(et[0] + et[1]), "how": "max over ranks, CUDA events, 20 reps"}
+                  "per_cg_iter_us": float(et[0] + et[1]),
+                  "local_spmv_fwd_us": float(et[2]), "local_spmv_back_us": float(et[3]),
+                  "how": "max over ranks, CUDA events, 20 reps; local_spmv = A_p / A_p^T kernels alone"}
 
     peer = None
     if dist_mode:

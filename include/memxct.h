@@ -69,11 +69,13 @@ typedef enum {
     MEMXCT_OPT_TILE_TOMO = 0,
     MEMXCT_OPT_TILE_SINO = 1,
     /* Rows per partition (one CTA per partition; one 32-row slice per warp).
-     * Multiple of 32 in [32, 1024], or 0 = auto (default): the largest of 1024/512/256/128 that
-     * leaves >= 1 partition per SM in the smaller direction (1024 at configs 3-5, 256 at cfg2). */
+     * Multiple of 32 in [32, 1024] used for both directions, or 0 = auto (default), chosen per
+     * direction: the largest multiple of 32 in [128, 1024] whose partition count spreads over the
+     * SMs with <= 3 % wave-quantisation loss (layout.cu: resolve_tuning).  get_option returns
+     * the forward value after build; memxct_layout_info reports both. */
     MEMXCT_OPT_PART_ROWS = 2,
     /* Stage-buffer capacity in fp32 entries (16-bit local addressing).
-     * 256 <= value <= 57344 (224 KB), or 0 = auto (default): 36 * PART_ROWS.  MIXED mode stages
+     * 256 <= value <= 57344 (224 KB), or 0 = auto (default, per direction): 36 * R.  MIXED mode stages
      * value/2 fp64 entries in the same bytes. */
     MEMXCT_OPT_BUFFER_ENTRIES = 3,
     /* 0 = FP32 (fp32 vectors, fp32 FMA; the paper's precision), 1 = MIXED (fp32 A, fp64
@@ -193,6 +195,13 @@ memxct_status_t memxct_sirt(memxct_plan_t plan, const void* y_sino, void* x_tomo
 memxct_status_t memxct_exchange_time(memxct_plan_t plan, int32_t reps, double* us_forward,
                                      double* us_back, void* cuda_stream);
 
+/* Local, not collective: device time, in microseconds, of this rank's forward SpMV (A_p, or A
+ * at P = 1) and back SpMV (A_p^T / A^T) kernels alone, without exchange, averaged over `reps`
+ * back-to-back launches per direction (CUDA events on `cuda_stream`; zero-valued scratch inputs,
+ * the access pattern does not depend on values).  Synchronous.  reps < 0: INVALID_ARG. */
+memxct_status_t memxct_spmv_time(memxct_plan_t plan, int32_t reps, double* us_forward,
+                                 double* us_back, void* cuda_stream);
+
 /* Multi-slice variants (the paper reuses the memoized matrices for every
  * slice): `slices` independent slices with the same geometry, vectors slice-major
  * (x[s * local_size(0) + i], y[s * local_size(1) + r]), FP32 only.  The slices are processed in
@@ -223,10 +232,13 @@ memxct_status_t memxct_stats(memxct_plan_t plan, int64_t* nnz, int64_t* stored_s
                              int64_t* map_entries, int64_t* device_bytes);
 
 /* Per-direction layout sizes (dir 0 = A / forward, 1 = A^T / back): partitions, total stages,
- * stored slots, map entries, rows, nonzeros.  Any pointer may be NULL. */
+ * stored slots, map entries, rows, nonzeros, rows per partition (CTA) and stage-buffer entries
+ * (fp64 entries in MIXED mode).  The automatic tuning picks R and B per direction.  Any pointer
+ * may be NULL. */
 memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* parts,
                                    int64_t* stages, int64_t* slots, int64_t* map_entries,
-                                   int64_t* rows, int64_t* nnz);
+                                   int64_t* rows, int64_t* nnz, int64_t* part_rows,
+                                   int64_t* buffer_entries);
 
 /* Copy the layout of partitions [p0, p1) of direction `dir` to host arrays (introspection for
  * tests; the layout is documented in DESIGN.md section 5):

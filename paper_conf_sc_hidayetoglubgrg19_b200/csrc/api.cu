@@ -81,39 +81,6 @@ void run_forward(mx::Plan& P, const void* x, void* y, cudaStream_t st) { mx::app
 
 void run_back(mx::Plan& P, const void* y, void* x, cudaStream_t st) { mx::apply_back(P, y, x, st); }
 
-// Default tuning (measured B200 sweep, profiles/r01_sweep.md): the largest partition (CTA) size
-// in {1024, 512, 256, 128} rows that still gives >= 2 CTAs per SM in the smaller direction, and
-// a stage buffer of 36 fp32 entries per row (144 KB at R = 1024): ~147 KB of shared memory per SM
-// at the register-limited residency of 1024/R CTAs per SM.
-void resolve_tuning(mx::Plan& P) {
-    int dev = 0, sms = 148;
-    MX_CUDA(cudaGetDevice(&dev));
-    MX_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-    const int64_t rows = std::min<int64_t>((int64_t)P.n * P.n, (int64_t)P.m * P.c) / P.nranks;
-    int32_t R = (int32_t)P.opt.part_rows;
-    if (R == 0) {
-        // largest partition still giving every SM a CTA in the smaller direction (cfg2 sweep,
-        // profiles/r01_sweep_cfg2.md: R = 256 / 512 beat 128 by 25 %)
-        R = 128;
-        for (int32_t cand : {1024, 512, 256}) {
-            if (mx::ceil_div(rows, cand) >= (int64_t)sms) { R = cand; break; }
-        }
-    }
-    int32_t B = (int32_t)P.opt.buffer_entries;
-    if (B == 0) {
-        int32_t k = 1;
-        while (k < P.opt.slices) k *= 2;  // batched calls stage k slices per buffer entry
-        // single slice: 36 entries per row (sweep r01_sweep.md); k slices: 192 KB of k-wide
-        // entries per CTA at R = 1024 (sweep r01_sweep_spmm.md: 4 slices, B = 12288 best; 200 KB
-        // pushes the shared-memory carveout to 228 KB and the L1 left for the gathers drops to
-        // 28 KB: 26 % slower)
-        B = (k == 1) ? std::min<int32_t>(57344, 36 * R) : std::min<int32_t>(49152, 144 * R) / k;
-        B = std::max<int32_t>(256, B - B % 256);
-    }
-    P.part_rows = R;
-    P.buffer_entries = B;
-}
-
 void ensure_host_staging(mx::Plan& P) {
     if (!P.h_in.get()) {
         const int64_t mx_len = std::max(P.local_len(0), P.local_len(1));
@@ -322,7 +289,6 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
             if (P.local_group) P.comm = mx::make_local_comm(P.local_group, P.rank);
             else P.comm = mx::make_nccl_comm(P.rank, P.nranks, P.unique_id.data());
         }
-        resolve_tuning(P);
         // CG dots fused into the SpMV epilogue (per-CTA tree + last-CTA sum, deterministic):
         // default since the jagged kernel (3.874 vs 3.882 ms per cfg3 iteration, one kernel
         // fewer per SpMV); MEMXCT_FUSED_DOT=0 restores the separate dot kernels
@@ -453,6 +419,17 @@ memxct_status_t memxct_exchange_time(memxct_plan_t plan, int32_t reps, double* u
     });
 }
 
+memxct_status_t memxct_spmv_time(memxct_plan_t plan, int32_t reps, double* us_forward, double* us_back,
+                                 void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(us_forward, "us_forward");
+        need(us_back, "us_back");
+        if (reps < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "reps < 0");
+        mx::time_spmv(P, reps, us_forward, us_back, stream_of(cuda_stream));
+    });
+}
+
 memxct_status_t memxct_forward_batch(memxct_plan_t plan, int32_t slices, const void* x_tomo, void* y_sino,
                                      void* cuda_stream) {
     return guarded([&] {
@@ -504,7 +481,8 @@ memxct_status_t memxct_stats(memxct_plan_t plan, int64_t* nnz, int64_t* stored_s
 }
 
 memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* parts, int64_t* stages,
-                                   int64_t* slots, int64_t* map_entries, int64_t* rows, int64_t* nnz) {
+                                   int64_t* slots, int64_t* map_entries, int64_t* rows, int64_t* nnz,
+                                   int64_t* part_rows, int64_t* buffer_entries) {
     return guarded([&] {
         mx::Plan& P = built_plan(plan);
         if (dir != 0 && dir != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "dir must be 0 or 1");
@@ -515,6 +493,8 @@ memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* par
         if (map_entries) *map_entries = L.nmap;
         if (rows) *rows = L.nrows;
         if (nnz) *nnz = L.nnz;
+        if (part_rows) *part_rows = L.R;
+        if (buffer_entries) *buffer_entries = L.B;
     });
 }
 

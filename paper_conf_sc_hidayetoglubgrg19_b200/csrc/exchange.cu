@@ -380,6 +380,42 @@ void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStrea
     *us_back = 1e3 * b / reps;
 }
 
+// Local (non-collective) device time of the A_p and A_p^T kernels alone -- the compute share of
+// an iteration, next to time_exchange's communication share.  Zero inputs (the access pattern
+// does not depend on values), `reps` back-to-back launches per direction, CUDA events on `st`.
+void time_spmv(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st) {
+    *us_fwd = *us_back = 0.0;
+    if (reps < 1) return;
+    const int64_t ntomo = std::max<int64_t>(P.t1 - P.t0, 1);
+    const int64_t nsino = std::max<int64_t>(P.dist ? P.nfp : P.s1 - P.s0, 1);
+    DevBuf xt(P.esize * ntomo), ys(P.esize * nsino);
+    MX_CUDA(cudaMemsetAsync(xt.get(), 0, P.esize * ntomo, st));
+    MX_CUDA(cudaMemsetAsync(ys.get(), 0, P.esize * nsino, st));
+    auto run = [&](bool fwd) {
+        const Layout& L = fwd ? P.fwd : P.back;
+        void* in = fwd ? xt.get() : ys.get();
+        void* out = fwd ? ys.get() : xt.get();
+        if (P.esize == 4) spmv_any(P, L, static_cast<const float*>(in), static_cast<float*>(out), st);
+        else spmv_any(P, L, static_cast<const double*>(in), static_cast<double*>(out), st);
+    };
+    run(true);
+    run(false);  // warm-up
+    cudaEvent_t e[3];
+    for (auto& ev : e) MX_CUDA(cudaEventCreate(&ev));
+    MX_CUDA(cudaEventRecord(e[0], st));
+    for (int i = 0; i < reps; ++i) run(true);
+    MX_CUDA(cudaEventRecord(e[1], st));
+    for (int i = 0; i < reps; ++i) run(false);
+    MX_CUDA(cudaEventRecord(e[2], st));
+    MX_CUDA(cudaEventSynchronize(e[2]));
+    float a = 0.f, b = 0.f;
+    MX_CUDA(cudaEventElapsedTime(&a, e[0], e[1]));
+    MX_CUDA(cudaEventElapsedTime(&b, e[1], e[2]));
+    for (auto& ev : e) cudaEventDestroy(ev);
+    *us_fwd = 1e3 * a / reps;
+    *us_back = 1e3 * b / reps;
+}
+
 void preload_exchange_kernels() {
     cudaFuncAttributes fa;
     MX_CUDA(cudaFuncGetAttributes(&fa, reduce_kernel<float>));

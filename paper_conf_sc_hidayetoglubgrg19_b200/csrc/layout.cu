@@ -572,6 +572,46 @@ struct Builder {
 };
 
 // budget of chunk entries: what is free after the finished layouts of both directions
+// Default tuning of one direction with `rows` output rows on this rank (B200 sweeps:
+// profiles/r01_sweep.md, r01_sweep_cfg2.md, r01_sweep_spmm.md, r01_virtual_scaling.md).
+//  * R (rows per partition = threads per CTA, a multiple of 32): 1024 (32 warps, one CTA per SM;
+//    Hilbert-aligned partitions, the best input reuse) whenever that gives >= 0.8 CTAs per SM --
+//    ~120 streaming SMs already saturate HBM (virtual-rank sweep: cfg3 A^T at P = 8, 128 CTAs,
+//    is as fast as any balanced split).  Smaller problems would leave most SMs idle: then R is
+//    the largest multiple of 32 in [128, 1024] whose parts spread over the SMs with
+//    w / ceil(w) >= 0.97, w = parts / SMs (else the most balanced one); cfg2: 640 / 448, 4.5 %
+//    more CG iter/s than 256.
+//  * B (stage buffer entries): 36 fp32 entries per row for one slice (144 KB at R = 1024); for
+//    k-slice plans 192 KB of k-wide entries (a 200 KB buffer leaves 28 KB of L1 for the gathers).
+void resolve_tuning(const Plan& P, int64_t rows, int32_t* R_out, int32_t* B_out) {
+    int dev = 0, sms = 148;
+    MX_CUDA(cudaGetDevice(&dev));
+    MX_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    int32_t R = (int32_t)P.opt.part_rows;
+    if (R == 0 && 5 * ceil_div(std::max<int64_t>(rows, 1), (int64_t)1024) >= 4 * (int64_t)sms) R = 1024;
+    if (R == 0) {
+        rows = std::max<int64_t>(rows, 1);
+        double best = -1.0;
+        int32_t best_r = 128;
+        for (int32_t cand = 1024; cand >= 128; cand -= 32) {
+            const double w = (double)ceil_div(rows, (int64_t)cand) / sms;
+            const double eff = w / std::ceil(w);
+            if (eff >= 0.97) { best_r = cand; break; }
+            if (eff > best + 1e-12) { best = eff; best_r = cand; }
+        }
+        R = best_r;
+    }
+    int32_t B = (int32_t)P.opt.buffer_entries;
+    if (B == 0) {
+        int32_t k = 1;
+        while (k < P.opt.slices) k *= 2;  // batched calls stage k slices per buffer entry
+        B = (k == 1) ? std::min<int32_t>(57344, 36 * R) : std::min<int32_t>(49152, 144 * R) / k;
+        B = std::max<int32_t>(256, B - B % 256);
+    }
+    *R_out = R;
+    *B_out = B;
+}
+
 int64_t chunk_budget(int64_t nnz_both_dirs_remaining) {
     size_t fr = 0, tot = 0;
     MX_CUDA(cudaMemGetInfo(&fr, &tot));
@@ -705,8 +745,15 @@ void build_matrices(Plan& P, cudaStream_t st) {
     const int64_t nrows = P.nfp = footprint(P, G, fp_len, st);
     const int32_t* hray = !P.dist ? nullptr : P.fp_rays.p();
     const bool natural = (P.opt.vector_order == 0);  // P = 1 only
-    const int32_t R = P.part_rows;
-    const int32_t B = P.opt.precision == 1 ? P.buffer_entries / 2 : P.buffer_entries;
+    int32_t R, B, Rb, Bb;
+    resolve_tuning(P, nrows, &R, &B);  // A_p: rows = footprint rays
+    resolve_tuning(P, npix, &Rb, &Bb);  // A_p^T: rows = local pixels
+    P.part_rows = R;
+    P.buffer_entries = B;
+    if (P.opt.precision == 1) {  // fp64 stage buffer: half the entries
+        B /= 2;
+        Bb /= 2;
+    }
 
     const auto fwd_part_nnz = partition_sums(fp_len.p(), nrows, R, st);
     int64_t nnz = 0;
@@ -754,7 +801,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
     pix_cnt.alloc(std::max<int64_t>(npix, 1));
     MX_CUDA(cudaMemsetAsync(pix_cnt.p(), 0, 4 * std::max<int64_t>(npix, 1), st));
     trace_hist(P, G, hray, 0, nrows, P.t0, P.t1, true, pix_cnt.p(), st);
-    const auto back_part_nnz = partition_sums(pix_cnt.p(), npix, R, st);
+    const auto back_part_nnz = partition_sums(pix_cnt.p(), npix, Rb, st);
     pix_cnt.reset();
     Generator gen_back = [&](int64_t ra, int64_t rb, Entries& E, cudaStream_t s) {
         const int64_t lo = P.t0 + ra, hi = P.t0 + rb;
@@ -792,7 +839,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
         }
         MX_CUDA(cudaStreamSynchronize(s));
     };
-    build_direction(P.back, npix, nrows, back_part_nnz, R, B, gen_back, natural ? P.sino_nat_of_h.p() : nullptr,
+    build_direction(P.back, npix, nrows, back_part_nnz, Rb, Bb, gen_back, natural ? P.sino_nat_of_h.p() : nullptr,
                     natural ? P.tomo_nat_of_h.p() : nullptr, chunk_budget(nnz), bank, st);
 
     // a6: exchange maps of the sparse all-to-allv (P > 1)

@@ -140,7 +140,7 @@ struct Plan {
     bool dist = false;
     int32_t tile_tomo = 0, tile_sino = 0;
     bool fused_dot = true;   // CG dots in the SpMV epilogue (MEMXCT_FUSED_DOT=0: separate kernels)
-    int32_t part_rows = 0, buffer_entries = 0;  // resolved tuning (build)
+    int32_t part_rows = 0, buffer_entries = 0;  // resolved tuning of A_p (A_p^T: back.R / back.B)
 
     // domain decomposition: this rank owns Hilbert pixels [t0, t1) and rays [s0, s1)
     std::unique_ptr<Comm> comm;
@@ -210,6 +210,7 @@ void build_exchange(Plan& P, cudaStream_t st);
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
 void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);
 void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
+void time_spmv(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 void reduce_partials(Plan& P, const float* recv, float* y, cudaStream_t st);
 void preload_exchange_kernels();
 // peer.cu: fused SpMV + exchange over peer memory (EXCHANGE = 1)

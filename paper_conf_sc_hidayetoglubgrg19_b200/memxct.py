@@ -32,7 +32,7 @@ SYMBOLS = [
     "memxct_local_group_create", "memxct_local_group_destroy", "memxct_plan_set_comm_local",
     "memxct_partition_ranges", "memxct_domain_ranges", "memxct_exchange_info",
     "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
-    "memxct_sirt",
+    "memxct_sirt", "memxct_spmv_time",
 ]
 
 
@@ -71,7 +71,7 @@ def lib():
             "memxct_back_host": [vp, vp, vp, vp],
             "memxct_cg_host": [vp, vp, vp, i32, vp, vp],
             "memxct_stats": [vp, P64, P64, P64, P64],
-            "memxct_layout_info": [vp, i32, P64, P64, P64, P64, P64, P64],
+            "memxct_layout_info": [vp, i32, P64, P64, P64, P64, P64, P64, P64, P64],
             "memxct_layout_export": [vp, i32, i64, i64, vp, vp, vp, vp, vp, vp, vp, P64, P64, P64],
             "memxct_plan_destroy": [vp],
             "memxct_local_group_create": [i32, ctypes.POINTER(vp)],
@@ -86,6 +86,8 @@ def lib():
             "memxct_sirt": [vp, vp, vp, i32, vp, vp],
             "memxct_exchange_time": [vp, i32, ctypes.POINTER(ctypes.c_double),
                                      ctypes.POINTER(ctypes.c_double), vp],
+            "memxct_spmv_time": [vp, i32, ctypes.POINTER(ctypes.c_double),
+                                 ctypes.POINTER(ctypes.c_double), vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -273,11 +275,19 @@ class MemXCT:
                                           _stream(stream)), "memxct_exchange_time")
         return {"fwd_us": f.value, "back_us": b.value}
 
+    def spmv_time(self, reps: int = 20, stream=None) -> dict:
+        """Local: device microseconds of this rank's A_p / A_p^T kernels alone (no exchange)."""
+        f, b = ctypes.c_double(), ctypes.c_double()
+        _check(lib().memxct_spmv_time(self._h, int(reps), ctypes.byref(f), ctypes.byref(b),
+                                      _stream(stream)), "memxct_spmv_time")
+        return {"fwd_us": f.value, "back_us": b.value}
+
     def layout_info(self, direction: int) -> dict:
-        v = [ctypes.c_int64() for _ in range(6)]
+        v = [ctypes.c_int64() for _ in range(8)]
         _check(lib().memxct_layout_info(self._h, direction, *[ctypes.byref(x) for x in v]),
                "memxct_layout_info")
-        return dict(zip(["parts", "stages", "slots", "map_entries", "rows", "nnz"], [x.value for x in v]))
+        return dict(zip(["parts", "stages", "slots", "map_entries", "rows", "nnz", "part_rows", "buffer_entries"],
+                        [x.value for x in v]))
 
     def layout_export(self, direction: int, p0: int = 0, p1: int = None) -> dict:
         if p1 is None:

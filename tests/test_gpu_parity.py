@@ -78,7 +78,7 @@ def _pattern_keys(plan, direction, npix, R, B):
 
 
 @pytest.mark.parametrize("n,m,c", GEOMS + [(256, 360, 256)])
-@pytest.mark.parametrize("part_rows,buf", [(512, 12288), (128, 700)])
+@pytest.mark.parametrize("part_rows,buf", [(512, 12288), (128, 700), (448, 8192)])
 def test_sparsity_pattern_and_values_exact(orc, coo_cache, n, m, c, part_rows, buf):
     if (n, m, c) == (256, 360, 256) and part_rows == 128:
         pytest.skip("covered by the default tuning at this size")
