@@ -142,6 +142,27 @@ __device__ void finish_dot_canonical(const SpmvArgs& a, const double* rows_val, 
 
 constexpr int kMaxThreads = 1024;
 
+// Stage gather buf[i] = x[map[i]]: U entries per thread in flight -- all U map loads
+// first, then the U dependent input loads (mostly L2 hits) -- so a stage costs ~cnt / (U * bd)
+// L2 round trips instead of cnt / bd (the unbatched loop spent ~24 % of the cfg3 kernel's warp
+// time here, profiles/r01b: while an SM gathers it streams nothing from HBM).
+template <int U, class T>
+__device__ __forceinline__ void stage_gather(T* __restrict__ buf, const T* __restrict__ x,
+                                             const int32_t* __restrict__ mp, int cnt) {
+    const int bd = blockDim.x;
+    for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+        int32_t j[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) j[u] = (i0 + u * bd < cnt) ? __ldg(mp + i0 + u * bd) : -1;
+        T v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = (j[u] >= 0) ? __ldg(x + j[u]) : T(0);
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if (i0 + u * bd < cnt) buf[i0 + u * bd] = v[u];
+    }
+}
+
 __device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned long long v) {
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -186,7 +207,7 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();  // previous stage fully consumed
-        for (int i = threadIdx.x; i < cnt; i += blockDim.x) sbuf[i] = __ldg(x + __ldg(mp + i));
+        stage_gather<8>(sbuf, x, mp, cnt);
         __syncthreads();
         const int64_t blk = g * a.SPP + warp;
         const int64_t base = a.slot_off[blk];
@@ -248,7 +269,7 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();
-        for (int i = threadIdx.x; i < cnt; i += blockDim.x) dbuf[i] = __ldg(x + __ldg(mp + i));
+        stage_gather<4>(dbuf, x, mp, cnt);
         __syncthreads();
         const int64_t blk = g * a.SPP + warp;
         const int64_t base = a.slot_off[blk];
@@ -384,18 +405,29 @@ spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __r
         const int cnt = (int)min((int64_t)a.B, D - st * a.B);
         const int32_t* __restrict__ mp = a.map + m0 + st * a.B;
         if (g != g0) __syncthreads();
-        for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
-            const int64_t col = __ldg(mp + i);
-            float v[K];
+        constexpr int U = K >= 8 ? 1 : 8 / K;  // 8 input loads in flight per thread (stage_gather)
+        const int bd = blockDim.x;
+        for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+            int64_t col[U];
 #pragma unroll
-            for (int s = 0; s < K; ++s) v[s] = __ldg(x + s * ldx + col);
-            if constexpr (K == 2) {
-                reinterpret_cast<float2*>(kbuf)[i] = make_float2(v[0], v[1]);
-            } else if constexpr (K == 4) {
-                reinterpret_cast<float4*>(kbuf)[i] = make_float4(v[0], v[1], v[2], v[3]);
-            } else {
-                reinterpret_cast<float4*>(kbuf)[2 * i] = make_float4(v[0], v[1], v[2], v[3]);
-                reinterpret_cast<float4*>(kbuf)[2 * i + 1] = make_float4(v[4], v[5], v[6], v[7]);
+            for (int u = 0; u < U; ++u) col[u] = (i0 + u * bd < cnt) ? (int64_t)__ldg(mp + i0 + u * bd) : -1;
+            float v[U][K];
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+#pragma unroll
+                for (int s = 0; s < K; ++s) v[u][s] = col[u] >= 0 ? __ldg(x + s * ldx + col[u]) : 0.f;
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int i = i0 + u * bd;
+                if (i >= cnt) continue;
+                if constexpr (K == 2) {
+                    reinterpret_cast<float2*>(kbuf)[i] = make_float2(v[u][0], v[u][1]);
+                } else if constexpr (K == 4) {
+                    reinterpret_cast<float4*>(kbuf)[i] = make_float4(v[u][0], v[u][1], v[u][2], v[u][3]);
+                } else {
+                    reinterpret_cast<float4*>(kbuf)[2 * i] = make_float4(v[u][0], v[u][1], v[u][2], v[u][3]);
+                    reinterpret_cast<float4*>(kbuf)[2 * i + 1] = make_float4(v[u][4], v[u][5], v[u][6], v[u][7]);
+                }
             }
         }
         __syncthreads();
