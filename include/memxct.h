@@ -249,12 +249,14 @@ memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* par
  *   ind         uint16[...]      local buffer index of each slot
  *   val         float[...]       value of each slot (0 for padding)
  *   lane_chunks uint16[(n_slot_off-1)*32]  8-slot chunks of each lane of each block
+ *   part_row0   int64[p1-p0+1]   first row of each partition (R rows each, or equal-work
+ *                                partitions of <= R rows under the automatic tuning)
  * Pass NULL for all arrays to query sizes through the int64 out-parameters. */
 memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0, int64_t p1,
                                      int64_t* stage_base, int64_t* map_off, int32_t* map,
                                      int64_t* slot_off, uint16_t* ind, float* val,
-                                     uint16_t* lane_chunks, int64_t* n_map, int64_t* n_slot_off,
-                                     int64_t* n_slots);
+                                     uint16_t* lane_chunks, int64_t* part_row0, int64_t* n_map,
+                                     int64_t* n_slot_off, int64_t* n_slots);
 
 /* Destroy a plan and free everything it owns.  NULL-safe. */
 memxct_status_t memxct_plan_destroy(memxct_plan_t plan);

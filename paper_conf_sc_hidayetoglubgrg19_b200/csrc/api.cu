@@ -500,8 +500,8 @@ memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* par
 
 memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0, int64_t p1,
                                      int64_t* stage_base, int64_t* map_off, int32_t* map, int64_t* slot_off,
-                                     uint16_t* ind, float* val, uint16_t* lane_chunks, int64_t* n_map,
-                                     int64_t* n_slot_off, int64_t* n_slots) {
+                                     uint16_t* ind, float* val, uint16_t* lane_chunks, int64_t* part_row0,
+                                     int64_t* n_map, int64_t* n_slot_off, int64_t* n_slots) {
     return guarded([&] {
         mx::Plan& P = built_plan(plan);
         if (dir != 0 && dir != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "dir must be 0 or 1");
@@ -525,6 +525,7 @@ memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0
         if (slot_off) MX_CUDA(cudaMemcpy(slot_off, L.slot_off.p() + b0, 8 * (b1 - b0 + 1), cudaMemcpyDeviceToHost));
         if (ind && so[1] > so[0]) MX_CUDA(cudaMemcpy(ind, L.ind.p() + so[0], 2 * (so[1] - so[0]), cudaMemcpyDeviceToHost));
         if (val && so[1] > so[0]) MX_CUDA(cudaMemcpy(val, L.val.p() + so[0], 4 * (so[1] - so[0]), cudaMemcpyDeviceToHost));
+        if (part_row0) MX_CUDA(cudaMemcpy(part_row0, L.prow0.p() + p0, 8 * (p1 - p0 + 1), cudaMemcpyDeviceToHost));
         if (lane_chunks && b1 > b0)
             MX_CUDA(cudaMemcpy(lane_chunks, L.lane_chunks.p() + b0 * 32, 2 * 32 * (b1 - b0), cudaMemcpyDeviceToHost));
     });

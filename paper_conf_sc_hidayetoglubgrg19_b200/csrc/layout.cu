@@ -27,7 +27,9 @@
 #include <cub/device/device_scan.cuh>
 #include <cub/device/device_segmented_sort.cuh>
 
+#include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <functional>
 #include <vector>
 
@@ -64,10 +66,10 @@ __global__ void row_ptr_kernel(const uint32_t* __restrict__ row_ids, int64_t nnz
 
 // mark the input of every entry of partitions [pa, ...) in the sub-chunk bitmap
 __global__ void mark_kernel(const uint32_t* __restrict__ row_ids, const uint32_t* __restrict__ cols,
-                            int64_t e0, int64_t e1, int32_t R, int64_t pa, int64_t words,
+                            int64_t e0, int64_t e1, const int32_t* __restrict__ row_part, int64_t pa, int64_t words,
                             uint32_t* __restrict__ bitmap) {
     for (int64_t e = e0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e1; e += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t p = row_ids[e] / R - pa;
+        const int64_t p = row_part[row_ids[e]] - pa;
         const uint32_t c = cols[e];
         atomicOr(bitmap + p * words + (c >> 5), 1u << (c & 31));
     }
@@ -97,11 +99,11 @@ prefix_kernel(const uint32_t* __restrict__ bitmap, int64_t words, int64_t pa,
 }
 
 __global__ void rank_kernel(const uint32_t* __restrict__ row_ids, const uint32_t* __restrict__ cols,
-                            int64_t e0, int64_t e1, int32_t R, int64_t pa, int64_t words,
+                            int64_t e0, int64_t e1, const int32_t* __restrict__ row_part, int64_t pa, int64_t words,
                             const uint32_t* __restrict__ bitmap, const uint32_t* __restrict__ word_prefix,
                             uint32_t* __restrict__ rank) {
     for (int64_t e = e0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e1; e += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t p = row_ids[e] / R - pa;
+        const int64_t p = row_part[row_ids[e]] - pa;
         const uint32_t c = cols[e];
         const int64_t w = p * words + (c >> 5);
         rank[e] = word_prefix[w] + (uint32_t)__popc(bitmap[w] & ((1u << (c & 31)) - 1u));
@@ -138,12 +140,13 @@ __global__ void stage_part_kernel(const int64_t* __restrict__ stage_base, int64_
 
 // per (chunk row, local stage): start of the stage's run inside the row and its length
 __global__ void runs_kernel(const int64_t* __restrict__ row_ptr, const uint32_t* __restrict__ rank,
-                            const int64_t* __restrict__ nst, int64_t ra, int64_t nr, int32_t R, int32_t B,
-                            int32_t maxS, int32_t* __restrict__ run_start, int32_t* __restrict__ run_len) {
+                            const int64_t* __restrict__ nst, int64_t ra, int64_t nr,
+                            const int32_t* __restrict__ row_part, int32_t B, int32_t maxS,
+                            int32_t* __restrict__ run_start, int32_t* __restrict__ run_len) {
     MX_LOOP(i, nr * maxS) {
         const int64_t r = i / maxS;
         const int32_t s = (int32_t)(i % maxS);
-        const int64_t S = nst[(ra + r) / R];
+        const int64_t S = nst[row_part[ra + r]];
         if (s >= S) { run_start[i] = 0; run_len[i] = 0; continue; }
         const int64_t b = row_ptr[r], e = row_ptr[r + 1];
         auto lower = [&](uint64_t key) {
@@ -164,8 +167,8 @@ __global__ void runs_kernel(const int64_t* __restrict__ row_ptr, const uint32_t*
 // block stores only the chunks lanes actually have (jagged SELL, plan.h)
 __global__ void width_kernel(const int32_t* __restrict__ stage_part, const int64_t* __restrict__ cs_base,
                              const int32_t* __restrict__ run_len, int64_t nblk, int32_t SPP, int64_t pa,
-                             int64_t ra, int64_t nrows, int32_t R, int32_t maxS, int64_t* __restrict__ blk_slots,
-                             uint16_t* __restrict__ lane_chunks) {
+                             int64_t ra, const int64_t* __restrict__ prow0, int32_t maxS,
+                             int64_t* __restrict__ blk_slots, uint16_t* __restrict__ lane_chunks) {
     const int lane = threadIdx.x & 31;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x / 32);
     for (int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / 32; wi < nblk; wi += warps) {
@@ -173,8 +176,8 @@ __global__ void width_kernel(const int32_t* __restrict__ stage_part, const int64
         const int32_t w = (int32_t)(wi % SPP);
         const int64_t pl = stage_part[g];
         const int64_t s = g - cs_base[pl];
-        const int64_t row = (pa + pl) * R + (int64_t)w * 32 + lane;
-        const int32_t len = (row < nrows) ? run_len[(row - ra) * maxS + s] : 0;
+        const int64_t row = prow0[pa + pl] + (int64_t)w * 32 + lane;
+        const int32_t len = (row < prow0[pa + pl + 1]) ? run_len[(row - ra) * maxS + s] : 0;
         const int32_t nch = (len + kVec - 1) / kVec;
         lane_chunks[wi * 32 + lane] = (uint16_t)nch;
         const int32_t tot = __reduce_add_sync(0xffffffffu, nch);
@@ -320,13 +323,15 @@ __global__ void scatter_kernel(const uint32_t* __restrict__ row_ids, const float
                                const uint32_t* __restrict__ rank, const int64_t* __restrict__ row_ptr,
                                const int32_t* __restrict__ run_start, const int64_t* __restrict__ stage_base,
                                const int64_t* __restrict__ slot_off, const uint16_t* __restrict__ lane_chunks,
-                               const int32_t* __restrict__ jnew, int64_t nnz, int64_t ra, int32_t R, int32_t SPP,
+                               const int32_t* __restrict__ jnew, int64_t nnz, int64_t ra,
+                               const int32_t* __restrict__ row_part, const int64_t* __restrict__ prow0, int32_t SPP,
                                int32_t B, int32_t maxS, uint16_t* __restrict__ ind, float* __restrict__ val) {
     MX_LOOP(e, nnz) {
         const int64_t row = row_ids[e];
         const int64_t r = row - ra;
-        const int64_t p = row / R;
-        const int32_t wl = (int32_t)((row % R) >> 5), lane = (int32_t)(row & 31);
+        const int64_t p = row_part[row];
+        const int64_t lr = row - prow0[p];  // row inside its partition: warp lr / 32, lane lr % 32
+        const int32_t wl = (int32_t)(lr >> 5), lane = (int32_t)(lr & 31);
         const uint32_t rk = rank[e];
         const int32_t s = (int32_t)(rk / (uint32_t)B);
         const uint32_t local = rk % (uint32_t)B;
@@ -355,15 +360,10 @@ __global__ void gather_u32_f32(const uint32_t* __restrict__ perm, const uint32_t
 
 __global__ void offset_u32_kernel(uint32_t* v, int64_t n, uint32_t add) { MX_LOOP(i, n) v[i] += add; }
 
-// per partition of R rows: sum of 32-bit per-row counts
-__global__ void part_sum_kernel(const int32_t* __restrict__ cnt, int64_t nrows, int32_t R, int64_t np,
-                                int64_t* __restrict__ out) {
-    MX_LOOP(p, np) {
-        int64_t s = 0;
-        const int64_t r1 = min(nrows, (p + 1) * (int64_t)R);
-        for (int64_t r = p * R; r < r1; ++r) s += cnt[r];
-        out[p] = s;
-    }
+// row_part[r] = partition of row r
+__global__ void row_part_kernel(const int64_t* __restrict__ prow0, int64_t np, int32_t* __restrict__ row_part) {
+    MX_LOOP(p, np)
+    for (int64_t r = prow0[p]; r < prow0[p + 1]; ++r) row_part[r] = (int32_t)p;
 }
 
 template <class T> T read_scalar(const T* dptr, cudaStream_t st) {
@@ -427,6 +427,11 @@ void stable_sort_by_key(const uint32_t* keys_in, uint32_t* keys_out, uint32_t* p
 // ---- chunked layout builder ------------------------------------------------------------------
 namespace {
 
+struct Partitions {         // host: partition p = rows [row0[p], row0[p+1]), nnz[p] nonzeros
+    std::vector<int64_t> row0, nnz;
+    bool balanced = false;
+};
+
 struct Entries {            // one chunk of a direction, sorted by (row, input)
     DevArr<uint32_t> row;   // absolute row ids
     DevArr<uint32_t> col;   // input index (plan order, local to the rank)
@@ -441,6 +446,9 @@ struct Builder {
     int64_t nrows, ncols;
     int32_t R, B, SPP;
     const int32_t* in_translate;
+    const int32_t* row_part;        // device: partition of every row
+    const int64_t* prow0;           // device: first row of every partition (nparts + 1)
+    std::vector<int64_t> h_prow0;   // host copy
     int64_t words;
     int64_t bitmap_parts;   // partitions per bitmap sub-chunk
     int32_t bank_classes;   // 0 = ascending local index in every run; else bank-aware order
@@ -456,11 +464,11 @@ struct Builder {
         wprefix.alloc(q * words);
         for (int64_t qa = pa; qa < pb; qa += q) {
             const int64_t qb = std::min(pb, qa + q);
-            const int64_t e0 = h_row_ptr[std::min<int64_t>(qa * R, nrows) - ra];
-            const int64_t e1 = h_row_ptr[std::min<int64_t>(qb * R, nrows) - ra];
+            const int64_t e0 = h_row_ptr[h_prow0[qa] - ra];
+            const int64_t e1 = h_row_ptr[h_prow0[qb] - ra];
             MX_CUDA(cudaMemsetAsync(bitmap.p(), 0, 4 * (qb - qa) * words, st));
             if (e1 > e0) {
-                mark_kernel<<<blocks_for(e1 - e0), kThreads, 0, st>>>(E.row.p(), E.col.p(), e0, e1, R, qa, words,
+                mark_kernel<<<blocks_for(e1 - e0), kThreads, 0, st>>>(E.row.p(), E.col.p(), e0, e1, row_part, qa, words,
                                                                       bitmap.p());
                 MX_LAUNCHED();
             }
@@ -468,7 +476,7 @@ struct Builder {
                                                                         distinct.p());
             MX_LAUNCHED();
             if (e1 > e0) {
-                rank_kernel<<<blocks_for(e1 - e0), kThreads, 0, st>>>(E.row.p(), E.col.p(), e0, e1, R, qa, words,
+                rank_kernel<<<blocks_for(e1 - e0), kThreads, 0, st>>>(E.row.p(), E.col.p(), e0, e1, row_part, qa, words,
                                                                       bitmap.p(), wprefix.p(), rank.p());
                 MX_LAUNCHED();
             }
@@ -482,7 +490,7 @@ struct Builder {
     }
 
     void process(const Entries& E, int64_t pa, int64_t pb, int pass, cudaStream_t st) {
-        const int64_t ra = pa * R, rb = std::min<int64_t>(pb * R, nrows), nr = rb - ra, np = pb - pa;
+        const int64_t ra = h_prow0[pa], rb = h_prow0[pb], nr = rb - ra, np = pb - pa;
         DevArr<int64_t> row_ptr;
         row_ptr.alloc(nr + 1);
         row_ptr_kernel<<<blocks_for(nr + 1), kThreads, 0, st>>>(E.row.p(), E.n, ra, nr, row_ptr.p());
@@ -508,8 +516,8 @@ struct Builder {
         run_start.alloc(std::max<int64_t>(nr * maxS, 1));
         run_len.alloc(std::max<int64_t>(nr * maxS, 1));
         if (nr > 0) {
-            runs_kernel<<<blocks_for(nr * maxS), kThreads, 0, st>>>(row_ptr.p(), rank.p(), nst.p(), ra, nr, R, B,
-                                                                    (int32_t)maxS, run_start.p(), run_len.p());
+            runs_kernel<<<blocks_for(nr * maxS), kThreads, 0, st>>>(row_ptr.p(), rank.p(), nst.p(), ra, nr, row_part,
+                                                                    B, (int32_t)maxS, run_start.p(), run_len.p());
             MX_LAUNCHED();
         }
         stage_part.alloc(std::max<int64_t>(ns, 1));
@@ -525,7 +533,7 @@ struct Builder {
         else { lanes.alloc(std::max<int64_t>(nblk * 32, 1)); lane_out = lanes.p(); }
         if (nblk > 0) {
             width_kernel<<<blocks_for(nblk * 32), kThreads, 0, st>>>(stage_part.p(), cs.p(), run_len.p(), nblk, SPP,
-                                                                     pa, ra, nrows, R, (int32_t)maxS, blk_slots.p(),
+                                                                     pa, ra, prow0, (int32_t)maxS, blk_slots.p(),
                                                                      lane_out);
             MX_LAUNCHED();
         }
@@ -563,8 +571,8 @@ struct Builder {
         if (E.n > 0) {
             scatter_kernel<<<blocks_for(E.n), kThreads, 0, st>>>(E.row.p(), E.val.p(), rank.p(), row_ptr.p(),
                                                                  run_start.p(), L.stage_base.p(), L.slot_off.p(),
-                                                                 L.lane_chunks.p(), jnew.p(), E.n, ra, R, SPP, B,
-                                                                 (int32_t)maxS, L.ind.p(), L.val.p());
+                                                                 L.lane_chunks.p(), jnew.p(), E.n, ra, row_part, prow0,
+                                                                 SPP, B, (int32_t)maxS, L.ind.p(), L.val.p());
             MX_LAUNCHED();
         }
         MX_CUDA(cudaStreamSynchronize(st));
@@ -622,7 +630,7 @@ int64_t chunk_budget(int64_t nnz_both_dirs_remaining) {
     return std::max<int64_t>(1 << 24, std::min<int64_t>(cap, (int64_t)(avail / 48.0)));
 }
 
-void build_direction(Layout& L, int64_t nrows, int64_t ncols, const std::vector<int64_t>& part_nnz, int32_t R,
+void build_direction(Layout& L, int64_t nrows, int64_t ncols, const Partitions& parts, int32_t R,
                      int32_t B, const Generator& gen, const int32_t* in_translate, const int32_t* out_translate,
                      int64_t budget, int32_t bank_classes, cudaStream_t st) {
     L = Layout{};
@@ -631,10 +639,20 @@ void build_direction(Layout& L, int64_t nrows, int64_t ncols, const std::vector<
     L.R = R;
     L.SPP = R / 32;
     L.B = B;
-    L.nparts = ceil_div(nrows, R);
+    L.nparts = (int64_t)parts.row0.size() - 1;
+    L.balanced = parts.balanced;
     L.bank_ordered = bank_classes > 0;
     const int64_t nparts = L.nparts;
-    Builder b{L, nrows, ncols, R, B, R / 32, in_translate};
+    const std::vector<int64_t>& part_nnz = parts.nnz;
+    L.prow0.alloc(nparts + 1);
+    MX_CUDA(cudaMemcpyAsync(L.prow0.p(), parts.row0.data(), 8 * (nparts + 1), cudaMemcpyHostToDevice, st));
+    DevArr<int32_t> row_part;
+    row_part.alloc(std::max<int64_t>(nrows, 1));
+    if (nparts > 0) {
+        row_part_kernel<<<blocks_for(nparts), kThreads, 0, st>>>(L.prow0.p(), nparts, row_part.p());
+        MX_LAUNCHED();
+    }
+    Builder b{L, nrows, ncols, R, B, R / 32, in_translate, row_part.p(), L.prow0.p(), parts.row0};
     b.bank_classes = bank_classes;
     b.words = std::max<int64_t>(1, ceil_div(ncols, 32));
     b.bitmap_parts = std::max<int64_t>(1, ((int64_t)2 << 30) / (b.words * 8));
@@ -658,7 +676,7 @@ void build_direction(Layout& L, int64_t nrows, int64_t ncols, const std::vector<
     // pass 1: sizes
     for (auto& c : chunks) {
         Entries E;
-        gen(c.first * R, std::min<int64_t>(c.second * R, nrows), E, st);
+        gen(parts.row0[c.first], parts.row0[c.second], E, st);
         b.process(E, c.first, c.second, 1, st);
         if (chunks.size() == 1) keep = std::move(E);
     }
@@ -695,7 +713,7 @@ void build_direction(Layout& L, int64_t nrows, int64_t ncols, const std::vector<
             b.process(keep, c.first, c.second, 2, st);
         } else {
             Entries E;
-            gen(c.first * R, std::min<int64_t>(c.second * R, nrows), E, st);
+            gen(parts.row0[c.first], parts.row0[c.second], E, st);
             b.process(E, c.first, c.second, 2, st);
         }
     }
@@ -706,15 +724,57 @@ void build_direction(Layout& L, int64_t nrows, int64_t ncols, const std::vector<
     MX_CUDA(cudaStreamSynchronize(st));
 }
 
-std::vector<int64_t> partition_sums(const int32_t* cnt, int64_t nrows, int32_t R, cudaStream_t st) {
-    const int64_t np = ceil_div(nrows, R);
-    DevArr<int64_t> out;
-    out.alloc(std::max<int64_t>(np, 1));
-    if (np > 0) {
-        part_sum_kernel<<<blocks_for(np), kThreads, 0, st>>>(cnt, nrows, R, np, out.p());
-        MX_LAUNCHED();
+// Partitions of one direction from its per-row nonzero counts.  Fixed: R rows each (reading R10,
+// the paper's blocks of consecutive Hilbert rows).  Balanced (automatic tuning): still <= R
+// consecutive Hilbert rows each, but cut at equal shares of the work (nonzeros + kRowCost per
+// row) into a multiple of the SM count, so no SM is left with a heavier last partition -- the
+// tail that left a third of the SMs idle in the single-wave A_p^T of a P = 8 rank
+// (profiles/r01_virtual_scaling_cfg3.log).  Boundaries are clamped so every partition keeps
+// 1..R rows.
+Partitions make_partitions(const int32_t* cnt, int64_t nrows, int32_t R, bool balanced, cudaStream_t st) {
+    constexpr int64_t kRowCost = 8;
+    Partitions out;
+    out.balanced = balanced;
+    const auto h = to_host(cnt, nrows, st);
+    std::vector<int64_t> w(nrows + 1, 0);
+    for (int64_t r = 0; r < nrows; ++r) w[r + 1] = w[r] + h[r] + kRowCost;
+    const int64_t np0 = ceil_div(nrows, (int64_t)R);
+    int64_t np = np0;
+    int dev = 0, sms = 148;
+    MX_CUDA(cudaGetDevice(&dev));
+    MX_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    // MEMXCT_BALANCE: 0 = never, 1 = only when the launch has few waves (default), 2 = always
+    int mode = 1;
+    if (const char* e = std::getenv("MEMXCT_BALANCE")) mode = atoi(e);
+    if (mode == 1 && np0 >= 4 * (int64_t)sms) balanced = false;  // many waves: the scheduler evens out
+    if (mode == 0) balanced = false;
+    if (balanced && nrows > 0) {
+        if (2 * np0 >= sms) np = ceil_div(np0, (int64_t)sms) * sms;
+        np = std::min<int64_t>(np, nrows);
+    } else {
+        out.balanced = false;
     }
-    return to_host(out.p(), np, st);
+    out.row0.assign(np + 1, 0);
+    for (int64_t j = 1; j < np; ++j) {
+        int64_t b;
+        if (out.balanced) {
+            const double target = (double)w[nrows] * (double)j / (double)np;
+            b = std::lower_bound(w.begin(), w.end(), (int64_t)std::llround(target)) - w.begin();
+            b = (b + 16) / 32 * 32;  // whole warps where the clamps allow
+            const int64_t prev = out.row0[j - 1];
+            const int64_t lo = std::max<int64_t>(prev + 1, nrows - (np - j) * (int64_t)R);
+            const int64_t hi = std::min<int64_t>(prev + R, nrows - (np - j));
+            b = std::min(std::max(b, lo), hi);
+        } else {
+            b = std::min<int64_t>(j * (int64_t)R, nrows);
+        }
+        out.row0[j] = b;
+    }
+    out.row0[np] = nrows;
+    out.nnz.assign(np, 0);
+    for (int64_t p = 0; p < np; ++p)
+        for (int64_t r = out.row0[p]; r < out.row0[p + 1]; ++r) out.nnz[p] += h[r];
+    return out;
 }
 
 }  // namespace
@@ -755,9 +815,12 @@ void build_matrices(Plan& P, cudaStream_t st) {
         Bb /= 2;
     }
 
-    const auto fwd_part_nnz = partition_sums(fp_len.p(), nrows, R, st);
+    // equal-work partitions only under the automatic tuning (PART_ROWS given: the user's fixed
+    // blocks; CANONICAL: the oracle's fixed R-row dot chunks)
+    const bool balance = P.opt.part_rows == 0 && !P.opt.canonical;
+    const Partitions fwd_parts = make_partitions(fp_len.p(), nrows, R, balance, st);
     int64_t nnz = 0;
-    for (int64_t v : fwd_part_nnz) nnz += v;
+    for (int64_t v : fwd_parts.nnz) nnz += v;
     const int64_t budget = chunk_budget(2 * nnz);
     // bank-aware run order for FP32 plans tuned for batched calls (16 B entries: 8 lanes per
     // shared-memory phase; 8 B: 16); canonical order (ascending) otherwise
@@ -792,7 +855,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
         }
         MX_CUDA(cudaStreamSynchronize(s));
     };
-    build_direction(P.fwd, nrows, npix, fwd_part_nnz, R, B, gen_fwd, natural ? P.tomo_nat_of_h.p() : nullptr,
+    build_direction(P.fwd, nrows, npix, fwd_parts, R, B, gen_fwd, natural ? P.tomo_nat_of_h.p() : nullptr,
                     natural ? P.sino_nat_of_h.p() : nullptr, budget, bank, st);
 
     // ---- A_p^T: rows = local pixels; every footprint ray re-traced with the chunk's pixel range,
@@ -801,7 +864,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
     pix_cnt.alloc(std::max<int64_t>(npix, 1));
     MX_CUDA(cudaMemsetAsync(pix_cnt.p(), 0, 4 * std::max<int64_t>(npix, 1), st));
     trace_hist(P, G, hray, 0, nrows, P.t0, P.t1, true, pix_cnt.p(), st);
-    const auto back_part_nnz = partition_sums(pix_cnt.p(), npix, Rb, st);
+    const Partitions back_parts = make_partitions(pix_cnt.p(), npix, Rb, balance, st);
     pix_cnt.reset();
     Generator gen_back = [&](int64_t ra, int64_t rb, Entries& E, cudaStream_t s) {
         const int64_t lo = P.t0 + ra, hi = P.t0 + rb;
@@ -839,7 +902,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
         }
         MX_CUDA(cudaStreamSynchronize(s));
     };
-    build_direction(P.back, npix, nrows, back_part_nnz, Rb, Bb, gen_back, natural ? P.sino_nat_of_h.p() : nullptr,
+    build_direction(P.back, npix, nrows, back_parts, Rb, Bb, gen_back, natural ? P.sino_nat_of_h.p() : nullptr,
                     natural ? P.tomo_nat_of_h.p() : nullptr, chunk_budget(nnz), bank, st);
 
     // a6: exchange maps of the sparse all-to-allv (P > 1)

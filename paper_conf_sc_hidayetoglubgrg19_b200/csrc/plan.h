@@ -37,6 +37,8 @@ struct Layout {
     int32_t R = 0, SPP = 0, B = 0;
     int32_t max_stages = 0;
     bool bank_ordered = false;   // runs in bank-aware order instead of ascending local index
+    bool balanced = false;       // partitions cut for equal work (else fixed R rows each)
+    DevArr<int64_t> prow0;       // nparts + 1: first row of each partition (<= R rows each)
     DevArr<int64_t> stage_base;  // nparts + 1
     DevArr<int64_t> map_off;     // nparts + 1
     DevArr<int32_t> map;         // nmap
@@ -46,7 +48,7 @@ struct Layout {
     DevArr<uint16_t> lane_chunks;  // nstages * SPP * 32
     DevArr<int32_t> out_idx;     // nrows, optional: output position of each row (natural order)
     int64_t device_bytes() const {
-        return (int64_t)(stage_base.buf.bytes() + map_off.buf.bytes() + map.buf.bytes() +
+        return (int64_t)(prow0.buf.bytes() + stage_base.buf.bytes() + map_off.buf.bytes() + map.buf.bytes() +
                          slot_off.buf.bytes() + ind.buf.bytes() + val.buf.bytes() +
                          lane_chunks.buf.bytes() + out_idx.buf.bytes());
     }

@@ -76,6 +76,7 @@ struct SpmvArgs {
     const float* val;
     const uint16_t* lane_chunks;
     const int32_t* out_idx;
+    const int64_t* prow0;  // first row of each partition (nparts + 1)
     int64_t nrows;
     int64_t nparts;
     int32_t R, SPP, B;
@@ -240,8 +241,8 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
             pref += na;
         }
     }
-    const int64_t row = p * a.R + threadIdx.x;
-    const bool valid = row < a.nrows;
+    const int64_t row = a.prow0[p] + threadIdx.x;
+    const bool valid = row < a.prow0[p + 1];
     if (kEpi == 2) {
         remote_epilogue(pa, row, valid, acc);
         return;
@@ -302,15 +303,15 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
             pref += na;
         }
     }
-    const int64_t row = p * a.R + threadIdx.x;
-    const bool valid = row < a.nrows;
+    const int64_t row = a.prow0[p] + threadIdx.x;
+    const bool valid = row < a.prow0[p + 1];
     if (valid) y[kNatOut ? a.out_idx[row] : row] = acc;
     if (kDotMode == 1) finish_dot_tree<kMaxThreads>(a, valid ? acc * acc : 0.0);
     if (kDotMode == 2) {
         __syncthreads();  // the stage buffer is free: reuse it for this partition's row values
         dbuf[threadIdx.x] = valid ? acc : 0.0;
         __syncthreads();
-        const int64_t nvalid = min((int64_t)a.R, a.nrows - p * a.R);
+        const int64_t nvalid = a.prow0[p + 1] - a.prow0[p];
         finish_dot_canonical(a, dbuf, (int)nvalid);
     }
 }
@@ -335,6 +336,7 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.val = L.val.p();
     a.lane_chunks = L.lane_chunks.p();
     a.out_idx = L.out_idx.p();
+    a.prow0 = L.prow0.p();
     a.nrows = L.nrows;
     a.nparts = L.nparts;
     a.R = L.R;
@@ -459,8 +461,8 @@ spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __r
             pref += na;
         }
     }
-    const int64_t row = p * a.R + threadIdx.x;
-    if (row < a.nrows) {
+    const int64_t row = a.prow0[p] + threadIdx.x;
+    if (row < a.prow0[p + 1]) {
         const int64_t o = kNatOut ? a.out_idx[row] : row;
 #pragma unroll
         for (int s = 0; s < K; ++s) y[s * ldy + o] = acc[s];

@@ -72,7 +72,7 @@ def lib():
             "memxct_cg_host": [vp, vp, vp, i32, vp, vp],
             "memxct_stats": [vp, P64, P64, P64, P64],
             "memxct_layout_info": [vp, i32, P64, P64, P64, P64, P64, P64, P64, P64],
-            "memxct_layout_export": [vp, i32, i64, i64, vp, vp, vp, vp, vp, vp, vp, P64, P64, P64],
+            "memxct_layout_export": [vp, i32, i64, i64, vp, vp, vp, vp, vp, vp, vp, vp, P64, P64, P64],
             "memxct_plan_destroy": [vp],
             "memxct_local_group_create": [i32, ctypes.POINTER(vp)],
             "memxct_local_group_destroy": [vp],
@@ -294,17 +294,19 @@ class MemXCT:
             p1 = self.layout_info(direction)["parts"]
         nm, nso, ns = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
         z = ctypes.c_void_p()
-        _check(lib().memxct_layout_export(self._h, direction, p0, p1, z, z, z, z, z, z, z,
+        _check(lib().memxct_layout_export(self._h, direction, p0, p1, z, z, z, z, z, z, z, z,
                                           ctypes.byref(nm), ctypes.byref(nso), ctypes.byref(ns)),
                "memxct_layout_export")
         out = {"stage_base": np.empty(p1 - p0 + 1, np.int64), "map_off": np.empty(p1 - p0 + 1, np.int64),
                "map": np.empty(nm.value, np.int32), "slot_off": np.empty(nso.value, np.int64),
                "ind": np.empty(ns.value, np.uint16), "val": np.empty(ns.value, np.float32),
-               "lane_chunks": np.empty(32 * (nso.value - 1), np.uint16)}
+               "lane_chunks": np.empty(32 * (nso.value - 1), np.uint16),
+               "prow0": np.empty(p1 - p0 + 1, np.int64)}
         P = lambda a: a.ctypes.data_as(ctypes.c_void_p)
         _check(lib().memxct_layout_export(self._h, direction, p0, p1, P(out["stage_base"]),
                                           P(out["map_off"]), P(out["map"]), P(out["slot_off"]),
-                                          P(out["ind"]), P(out["val"]), P(out["lane_chunks"]), ctypes.byref(nm),
+                                          P(out["ind"]), P(out["val"]), P(out["lane_chunks"]), P(out["prow0"]),
+                                          ctypes.byref(nm),
                                           ctypes.byref(nso), ctypes.byref(ns)),
                "memxct_layout_export")
         return out

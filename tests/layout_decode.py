@@ -48,7 +48,13 @@ def decode(ex, R, B, p0=0):
     w = b % SPP
     part = np.searchsorted(sb, g, side="right") - 1
     s = g - sb[part]
-    row = (part + p0) * R + w * 32 + lane
+    if "prow0" in ex:  # partitions of <= R rows (equal-work cuts under the automatic tuning)
+        pr = ex["prow0"]
+        assert np.all(np.diff(pr) >= 1) and np.all(np.diff(pr) <= R)
+        row = pr[part] + w * 32 + lane
+        assert np.all(row < pr[part + 1]), "slots in a lane beyond its partition's rows"
+    else:
+        row = (part + p0) * R + w * 32 + lane
     cnt_stage = np.minimum(B, (mo[part + 1] - mo[part]) - s * B)
     assert np.all(ind < np.maximum(cnt_stage, 1))
     map_pos = (mo[part] - mo[0]) + s * B + ind

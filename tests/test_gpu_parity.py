@@ -98,6 +98,24 @@ def test_sparsity_pattern_and_values_exact(orc, coo_cache, n, m, c, part_rows, b
         assert np.all(np.diff(ex["map_off"]) >= 0)
 
 
+@pytest.mark.parametrize("n,m,c", [(256, 360, 256), (96, 120, 96)])
+def test_balanced_partitions_pattern_exact(orc, coo_cache, n, m, c):
+    """Automatic tuning: equal-work partitions of <= R rows (layout.cu: make_partitions); the
+    decoded pattern and values are still exactly the oracle's, partitions cover the rows."""
+    plan = make_plan(n, m, c)
+    rows, cols, vals = coo_cache(n, m, c)
+    npix = n * n
+    okey = rows.astype(np.int64) * npix + cols
+    oo = np.argsort(okey)
+    okey, oval = okey[oo], vals[oo].astype(np.float32)
+    for direction in (0, 1):
+        li = plan.layout_info(direction)
+        key, val, ex = _pattern_keys(plan, direction, npix, li["part_rows"], li["buffer_entries"])
+        assert ex["prow0"][0] == 0 and ex["prow0"][-1] == li["rows"]
+        assert np.array_equal(key, okey), direction
+        assert np.array_equal(val, oval), direction
+
+
 def _vectors(n, m, c):
     x_ph = inputs.shepp_logan(n)
     rng = np.random.default_rng(11)
