@@ -134,6 +134,19 @@ memxct_status_t memxct_local_group_create(int32_t nranks, memxct_group_t* out);
 memxct_status_t memxct_local_group_destroy(memxct_group_t group);
 memxct_status_t memxct_plan_set_comm_local(memxct_plan_t plan, memxct_group_t group, int32_t rank);
 
+/* Shard probe: build on this device only rank `rank`'s part of a `nranks`-way decomposition
+ * -- the same tile ranges (R12), footprint rays, A_p, A_p^T and exchange counts /
+ * maps that rank would build inside a real P-rank job, with no peers and no communicator (the
+ * build's collective steps are replaced by tracing every ray locally).  It answers "what does
+ * one of P GPUs hold and how fast are its kernels" for decompositions whose other ranks do not
+ * fit or do not exist (config 5's 11293^2 slice, ~43 GB of A_p per rank at P = 8).  Before
+ * build.  After build: memxct_footprint_*, memxct_spmv_time, memxct_exchange_info / _counts,
+ * memxct_domain_ranges, memxct_local_size / _indices, memxct_stats and memxct_layout_info work;
+ * the whole operators (forward, back, cg, sirt, batched and host variants, exchange_time) return
+ * MEMXCT_ERR_UNSUPPORTED, as does EXCHANGE = 1 at build. */
+memxct_status_t memxct_plan_set_shard(memxct_plan_t plan, int32_t rank, int32_t nranks,
+                                      int32_t cuda_device);
+
 /* Domain decomposition helper (host only, reading R12): split `count` tiles with
  * nonnegative `weights` (nonzeros per tile, in Hilbert order) into `parts` contiguous ranges
  * with about equal weight; bounds[0..parts] (host) receives the range boundaries, every range
@@ -151,6 +164,25 @@ memxct_status_t memxct_domain_ranges(memxct_plan_t plan, int32_t domain, int64_t
 memxct_status_t memxct_exchange_info(memxct_plan_t plan, int64_t* footprint_rays,
                                      int64_t* sent_entries, int64_t* received_entries,
                                      int32_t* peers);
+
+/* After build, decomposed plans only (set_comm with an id, set_comm_local, set_shard; else
+ * INVALID_ARG): send_counts[q] / recv_counts[q] (host, nranks int64 each, nullable) = partial-sinogram
+ * entries this rank sends to / receives from rank q per forward exchange (q = rank: its own slice). */
+memxct_status_t memxct_exchange_counts(memxct_plan_t plan, int64_t* send_counts, int64_t* recv_counts);
+
+/* The local operator A_p of P:758-761 alone, decomposed plans only.  Rows of A_p are this rank's
+ * footprint rays: every ray with a segment in its pixels, in Hilbert order (owner, Hilbert).
+ * memxct_footprint_rays writes their natural indices (host, footprint_rays int64, see
+ * memxct_exchange_info).  memxct_footprint_forward: y_footprint[i] = sum over LOCAL pixels p of
+ * A[ray_i, p] x_local[p] (x_local in plan order, local_size(0) entries; y_footprint:
+ * footprint_rays entries) -- the partial projection before exchange and reduction.
+ * memxct_footprint_back: x_local = A_p^T y_footprint.  Device pointers, dtype per PRECISION,
+ * stream-ordered, outputs overwritten. */
+memxct_status_t memxct_footprint_rays(memxct_plan_t plan, int64_t* natural_ray);
+memxct_status_t memxct_footprint_forward(memxct_plan_t plan, const void* x_local, void* y_footprint,
+                                         void* cuda_stream);
+memxct_status_t memxct_footprint_back(memxct_plan_t plan, const void* y_footprint, void* x_local,
+                                      void* cuda_stream);
 
 /* Preprocessing: Hilbert ordering and domain decomposition, Siddon tracing of A on
  * the device, order-preserving transposition to A^T, partitioning and the multi-stage buffered

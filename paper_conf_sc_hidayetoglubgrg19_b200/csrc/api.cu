@@ -71,6 +71,21 @@ mx::Plan& built_plan(memxct_plan_t plan) {
     return P;
 }
 
+// a plan whose forward/back operators are whole: not a shard probe (which has no peers to
+// exchange partials with)
+mx::Plan& full_plan(memxct_plan_t plan) {
+    mx::Plan& P = built_plan(plan);
+    if (P.shard) mx::fail(MEMXCT_ERR_UNSUPPORTED, "a shard probe has no peers: use the memxct_footprint_* calls");
+    return P;
+}
+
+// a decomposed plan (P >= 1 ranks: NCCL, virtual ranks or a shard probe)
+mx::Plan& decomposed_plan(memxct_plan_t plan) {
+    mx::Plan& P = built_plan(plan);
+    if (!P.dist) mx::fail(MEMXCT_ERR_INVALID_ARG, "the plan is not decomposed (no set_comm / set_shard)");
+    return P;
+}
+
 cudaStream_t stream_of(void* s) { return reinterpret_cast<cudaStream_t>(s); }
 
 void need(const void* p, const char* what) {
@@ -178,8 +193,24 @@ memxct_status_t memxct_plan_set_comm(memxct_plan_t plan, int32_t rank, int32_t n
         P.rank = rank;
         P.nranks = nranks;
         P.dist = nccl_unique_id != nullptr;
+        P.shard = false;
         P.device = cuda_device;
         P.local_group.reset();
+    });
+}
+
+memxct_status_t memxct_plan_set_shard(memxct_plan_t plan, int32_t rank, int32_t nranks, int32_t cuda_device) {
+    return guarded([&] {
+        mx::Plan& P = plan_of(plan);
+        if (P.built) mx::fail(MEMXCT_ERR_STATE, "set_shard must precede memxct_build");
+        if (nranks < 1 || rank < 0 || rank >= nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank / nranks");
+        P.unique_id.clear();
+        P.local_group.reset();
+        P.rank = rank;
+        P.nranks = nranks;
+        P.dist = true;
+        P.shard = true;
+        P.device = cuda_device;
     });
 }
 
@@ -211,6 +242,7 @@ memxct_status_t memxct_plan_set_comm_local(memxct_plan_t plan, memxct_group_t gr
         P.rank = rank;
         P.nranks = group->g->nranks;
         P.dist = true;
+        P.shard = false;
         P.local_group = group->g;
     });
 }
@@ -286,7 +318,9 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
         P.esize = P.opt.precision == 1 ? 8 : 4;
         if (P.dist) {
             if (P.opt.canonical) mx::fail(MEMXCT_ERR_UNSUPPORTED, "CANONICAL mode is single-GPU only");
-            if (P.local_group) P.comm = mx::make_local_comm(P.local_group, P.rank);
+            if (P.shard && P.opt.exchange == 1) mx::fail(MEMXCT_ERR_UNSUPPORTED, "a shard probe has no peers to map");
+            if (P.shard) P.comm.reset();
+            else if (P.local_group) P.comm = mx::make_local_comm(P.local_group, P.rank);
             else P.comm = mx::make_nccl_comm(P.rank, P.nranks, P.unique_id.data());
         }
         // CG dots fused into the SpMV epilogue (per-CTA tree + last-CTA sum, deterministic):
@@ -324,7 +358,7 @@ memxct_status_t memxct_local_indices(memxct_plan_t plan, int32_t domain, int64_t
 
 memxct_status_t memxct_forward(memxct_plan_t plan, const void* x_tomo, void* y_sino, void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_tomo, "x_tomo");
         need(y_sino, "y_sino");
         run_forward(P, x_tomo, y_sino, stream_of(cuda_stream));
@@ -333,7 +367,7 @@ memxct_status_t memxct_forward(memxct_plan_t plan, const void* x_tomo, void* y_s
 
 memxct_status_t memxct_back(memxct_plan_t plan, const void* y_sino, void* x_tomo, void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_tomo, "x_tomo");
         need(y_sino, "y_sino");
         run_back(P, y_sino, x_tomo, stream_of(cuda_stream));
@@ -343,7 +377,7 @@ memxct_status_t memxct_back(memxct_plan_t plan, const void* y_sino, void* x_tomo
 memxct_status_t memxct_cg(memxct_plan_t plan, const void* y_sino, void* x_tomo, int32_t iters,
                           double* residual_norms, void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_tomo, "x_tomo");
         need(y_sino, "y_sino");
         if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
@@ -355,7 +389,7 @@ memxct_status_t memxct_cg(memxct_plan_t plan, const void* y_sino, void* x_tomo, 
 
 memxct_status_t memxct_forward_host(memxct_plan_t plan, const void* x_host, void* y_host, void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_host, "x_host");
         need(y_host, "y_host");
         ensure_host_staging(P);
@@ -369,7 +403,7 @@ memxct_status_t memxct_forward_host(memxct_plan_t plan, const void* x_host, void
 
 memxct_status_t memxct_back_host(memxct_plan_t plan, const void* y_host, void* x_host, void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_host, "x_host");
         need(y_host, "y_host");
         ensure_host_staging(P);
@@ -384,7 +418,7 @@ memxct_status_t memxct_back_host(memxct_plan_t plan, const void* y_host, void* x
 memxct_status_t memxct_cg_host(memxct_plan_t plan, const void* y_host, void* x_host, int32_t iters,
                                double* residual_norms, void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_host, "x_host");
         need(y_host, "y_host");
         if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
@@ -401,7 +435,7 @@ memxct_status_t memxct_cg_host(memxct_plan_t plan, const void* y_host, void* x_h
 memxct_status_t memxct_sirt(memxct_plan_t plan, const void* y_sino, void* x_tomo, int32_t iters,
                             double* residual_norms, void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_tomo, "x_tomo");
         need(y_sino, "y_sino");
         if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
@@ -412,7 +446,7 @@ memxct_status_t memxct_sirt(memxct_plan_t plan, const void* y_sino, void* x_tomo
 memxct_status_t memxct_exchange_time(memxct_plan_t plan, int32_t reps, double* us_forward, double* us_back,
                                      void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(us_forward, "us_forward");
         need(us_back, "us_back");
         mx::time_exchange(P, reps, us_forward, us_back, stream_of(cuda_stream));
@@ -433,7 +467,7 @@ memxct_status_t memxct_spmv_time(memxct_plan_t plan, int32_t reps, double* us_fo
 memxct_status_t memxct_forward_batch(memxct_plan_t plan, int32_t slices, const void* x_tomo, void* y_sino,
                                      void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_tomo, "x_tomo");
         need(y_sino, "y_sino");
         if (slices < 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "slices < 1");
@@ -445,7 +479,7 @@ memxct_status_t memxct_forward_batch(memxct_plan_t plan, int32_t slices, const v
 memxct_status_t memxct_back_batch(memxct_plan_t plan, int32_t slices, const void* y_sino, void* x_tomo,
                                   void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_tomo, "x_tomo");
         need(y_sino, "y_sino");
         if (slices < 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "slices < 1");
@@ -457,7 +491,7 @@ memxct_status_t memxct_back_batch(memxct_plan_t plan, int32_t slices, const void
 memxct_status_t memxct_cg_batch(memxct_plan_t plan, int32_t slices, const void* y_sino, void* x_tomo,
                                 int32_t iters, double* residual_norms, void* cuda_stream) {
     return guarded([&] {
-        mx::Plan& P = built_plan(plan);
+        mx::Plan& P = full_plan(plan);
         need(x_tomo, "x_tomo");
         need(y_sino, "y_sino");
         if (iters < 0) mx::fail(MEMXCT_ERR_INVALID_ARG, "iters < 0");
@@ -466,6 +500,52 @@ memxct_status_t memxct_cg_batch(memxct_plan_t plan, int32_t slices, const void* 
         cudaStream_t st = stream_of(cuda_stream);
         mx::cg_run(P, y_sino, x_tomo, iters, slices, st);
         if (residual_norms) mx::cg_fetch_norms(P, iters, slices, residual_norms, st);
+    });
+}
+
+memxct_status_t memxct_footprint_rays(memxct_plan_t plan, int64_t* natural_ray) {
+    return guarded([&] {
+        mx::Plan& P = decomposed_plan(plan);
+        need(natural_ray, "natural_ray");
+        std::vector<int32_t> h(P.nfp);
+        if (P.nfp > 0) {
+            MX_CUDA(cudaMemcpy(h.data(), P.fp_rays.p(), 4 * P.nfp, cudaMemcpyDeviceToHost));
+            std::vector<int32_t> perm((size_t)P.m * P.c);
+            MX_CUDA(cudaMemcpy(perm.data(), P.sino_nat_of_h.p(), 4 * perm.size(), cudaMemcpyDeviceToHost));
+            for (int64_t i = 0; i < P.nfp; ++i) natural_ray[i] = perm[h[i]];
+        }
+    });
+}
+
+memxct_status_t memxct_footprint_forward(memxct_plan_t plan, const void* x_local, void* y_footprint,
+                                         void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = decomposed_plan(plan);
+        need(x_local, "x_local");
+        need(y_footprint, "y_footprint");
+        if (P.esize == 4) mx::spmv_any(P, P.fwd, (const float*)x_local, (float*)y_footprint, stream_of(cuda_stream));
+        else mx::spmv_any(P, P.fwd, (const double*)x_local, (double*)y_footprint, stream_of(cuda_stream));
+    });
+}
+
+memxct_status_t memxct_footprint_back(memxct_plan_t plan, const void* y_footprint, void* x_local,
+                                      void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = decomposed_plan(plan);
+        need(x_local, "x_local");
+        need(y_footprint, "y_footprint");
+        if (P.esize == 4) mx::spmv_any(P, P.back, (const float*)y_footprint, (float*)x_local, stream_of(cuda_stream));
+        else mx::spmv_any(P, P.back, (const double*)y_footprint, (double*)x_local, stream_of(cuda_stream));
+    });
+}
+
+memxct_status_t memxct_exchange_counts(memxct_plan_t plan, int64_t* send_counts, int64_t* recv_counts) {
+    return guarded([&] {
+        mx::Plan& P = decomposed_plan(plan);
+        for (int q = 0; q < P.nranks; ++q) {
+            if (send_counts) send_counts[q] = P.ex.scount[q];
+            if (recv_counts) recv_counts[q] = P.ex.rcount[q];
+        }
     });
 }
 

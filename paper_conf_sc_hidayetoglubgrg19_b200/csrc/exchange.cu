@@ -103,14 +103,15 @@ void decompose(Plan& P, const Geometry& G, cudaStream_t st) {
         P.sino_bounds = {0, nrays};
         return;
     }
-    Comm& C = *P.comm;
     // per-pixel nonzeros (column counts of A): each rank traces 1/P of the rays, then allreduce
+    // (a shard probe has no peers: it traces every ray itself, the same counts)
     DevArr<int32_t> hist;
     hist.alloc(npix);
     MX_CUDA(cudaMemsetAsync(hist.p(), 0, 4 * npix, st));
-    const int64_t ra = nrays * P.rank / P.nranks, rb = nrays * (P.rank + 1) / P.nranks;
+    const int64_t ra = P.shard ? 0 : nrays * P.rank / P.nranks;
+    const int64_t rb = P.shard ? nrays : nrays * (P.rank + 1) / P.nranks;
     trace_hist(P, G, nullptr, ra, rb - ra, 0, 0, false, hist.p(), st);
-    C.allreduce_sum(hist.p(), npix, DType::I32, st);
+    if (!P.shard) P.comm->allreduce_sum(hist.p(), npix, DType::I32, st);
     const auto tw = tile_sums(hist.p(), P.tomo_tile_off, st);
     hist.reset();
     // per-ray nonzeros (row lengths of A)
@@ -164,10 +165,39 @@ int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStrea
     return nfp;
 }
 
+// a6, receive side of a shard probe (no peers to ask): rank q's footprint slice bound for this
+// owner is, in Hilbert order, every owned ray with a segment in q's pixel range [tomo_bounds[q],
+// tomo_bounds[q+1]) -- exactly the rays q's own footprint pass selects.  Re-tracing the owned rays
+// once per rank gives the counts (rcount) and owned-local indices (recv_idx) that the allgather and
+// all-to-allv of build_exchange deliver on a real P-rank build.
+void shard_receive_maps(Plan& P, const Geometry& G, cudaStream_t st) {
+    Exchange& X = P.ex;
+    const int np = P.nranks;
+    const int64_t nown = P.s1 - P.s0;
+    X.rcount.assign(np, 0);
+    std::vector<int32_t> idx;
+    std::vector<int32_t> len(std::max<int64_t>(nown, 1));
+    DevArr<int32_t> dlen;
+    dlen.alloc(std::max<int64_t>(nown, 1));
+    for (int q = 0; q < np; ++q) {
+        if (nown > 0) {
+            trace_count(P, G, nullptr, P.s0, nown, P.tomo_bounds[q], P.tomo_bounds[q + 1], true, dlen.p(), st);
+            MX_CUDA(cudaMemcpyAsync(len.data(), dlen.p(), 4 * nown, cudaMemcpyDeviceToHost, st));
+            MX_CUDA(cudaStreamSynchronize(st));
+        }
+        const size_t before = idx.size();
+        for (int64_t i = 0; i < nown; ++i)
+            if (len[i] > 0) idx.push_back((int32_t)i);
+        X.rcount[q] = (int64_t)(idx.size() - before);
+    }
+    X.recv_idx.alloc(std::max<int64_t>((int64_t)idx.size(), 1));
+    if (!idx.empty())
+        MX_CUDA(cudaMemcpy(X.recv_idx.p(), idx.data(), 4 * idx.size(), cudaMemcpyHostToDevice));
+}
+
 // a6: exchange maps (P > 1)
 void build_exchange(Plan& P, cudaStream_t st) {
     if (!P.dist) return;
-    Comm& C = *P.comm;
     Exchange& X = P.ex;
     const int np = P.nranks;
     std::vector<int32_t> fp(P.nfp);
@@ -178,10 +208,12 @@ void build_exchange(Plan& P, cudaStream_t st) {
     X.sdispl[np] = P.nfp;
     X.scount.assign(np, 0);
     for (int h = 0; h < np; ++h) X.scount[h] = X.sdispl[h + 1] - X.sdispl[h];
-    X.rcount.assign(np, 0);
-    for (int h = 0; h < np; ++h) {
-        const auto v = C.allgather_host(X.scount[h], st);  // v[q] = what rank q sends to owner h
-        if (h == P.rank) X.rcount = v;
+    if (!P.shard) {  // a shard probe has its rcount from shard_receive_maps
+        X.rcount.assign(np, 0);
+        for (int h = 0; h < np; ++h) {
+            const auto v = P.comm->allgather_host(X.scount[h], st);  // v[q] = what rank q sends to owner h
+            if (h == P.rank) X.rcount = v;
+        }
     }
     X.rdispl.assign(np + 1, 0);
     for (int q = 0; q < np; ++q) X.rdispl[q + 1] = X.rdispl[q] + X.rcount[q];
@@ -190,13 +222,15 @@ void build_exchange(Plan& P, cudaStream_t st) {
     std::vector<int32_t> idx(std::max<int64_t>(P.nfp, 1));
     for (int h = 0; h < np; ++h)
         for (int64_t i = X.sdispl[h]; i < X.sdispl[h + 1]; ++i) idx[i] = (int32_t)(fp[i] - P.sino_bounds[h]);
-    DevArr<int32_t> send_idx;
-    send_idx.alloc(std::max<int64_t>(P.nfp, 1));
-    MX_CUDA(cudaMemcpy(send_idx.p(), idx.data(), 4 * P.nfp, cudaMemcpyHostToDevice));
-    X.recv_idx.alloc(std::max<int64_t>(X.nrecv, 1));
-    C.alltoallv(send_idx.p(), X.scount.data(), X.sdispl.data(), X.recv_idx.p(), X.rcount.data(), X.rdispl.data(),
-                DType::I32, st);
-    MX_CUDA(cudaStreamSynchronize(st));
+    if (!P.shard) {  // ... and its recv_idx
+        DevArr<int32_t> send_idx;
+        send_idx.alloc(std::max<int64_t>(P.nfp, 1));
+        MX_CUDA(cudaMemcpy(send_idx.p(), idx.data(), 4 * P.nfp, cudaMemcpyHostToDevice));
+        X.recv_idx.alloc(std::max<int64_t>(X.nrecv, 1));
+        P.comm->alltoallv(send_idx.p(), X.scount.data(), X.sdispl.data(), X.recv_idx.p(), X.rcount.data(),
+                          X.rdispl.data(), DType::I32, st);
+        MX_CUDA(cudaStreamSynchronize(st));
+    }
     // reduction map R: for every owned ray, its received partials in peer order (stable sort)
     const int64_t nown = P.s1 - P.s0;
     DevArr<uint32_t> keys_out, perm;

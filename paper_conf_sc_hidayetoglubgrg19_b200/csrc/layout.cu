@@ -906,6 +906,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
                     natural ? P.tomo_nat_of_h.p() : nullptr, chunk_budget(nnz), bank, st);
 
     // a6: exchange maps of the sparse all-to-allv (P > 1)
+    if (P.shard) shard_receive_maps(P, G, st);
     build_exchange(P, st);
 }
 

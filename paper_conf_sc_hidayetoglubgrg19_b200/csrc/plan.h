@@ -140,6 +140,10 @@ struct Plan {
     // decomposed path (A = R C A_p with a communicator): set by set_comm / set_comm_local, also
     // at nranks = 1 (a one-rank communicator runs every exchange step against itself)
     bool dist = false;
+    // shard probe (memxct_plan_set_shard): this device builds rank `rank`'s A_p, A_p^T and
+    // exchange maps of a P-way decomposition alone, with no peers and no communicator; the
+    // collective steps of the build are replaced by local re-tracing (exchange.cu)
+    bool shard = false;
     int32_t tile_tomo = 0, tile_sino = 0;
     bool fused_dot = true;   // CG dots in the SpMV epilogue (MEMXCT_FUSED_DOT=0: separate kernels)
     int32_t part_rows = 0, buffer_entries = 0;  // resolved tuning of A_p (A_p^T: back.R / back.B)
@@ -208,6 +212,7 @@ void row_ptr_from_sorted(const uint32_t* row_ids, int64_t nnz, int64_t nrows, in
 std::vector<int64_t> partition_ranges(const std::vector<int64_t>& w, int32_t parts);
 void decompose(Plan& P, const Geometry& G, cudaStream_t st);
 int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStream_t st);
+void shard_receive_maps(Plan& P, const Geometry& G, cudaStream_t st);
 void build_exchange(Plan& P, cudaStream_t st);
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
 void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);

@@ -32,7 +32,8 @@ SYMBOLS = [
     "memxct_local_group_create", "memxct_local_group_destroy", "memxct_plan_set_comm_local",
     "memxct_partition_ranges", "memxct_domain_ranges", "memxct_exchange_info",
     "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
-    "memxct_sirt", "memxct_spmv_time",
+    "memxct_sirt", "memxct_spmv_time", "memxct_plan_set_shard", "memxct_exchange_counts",
+    "memxct_footprint_rays", "memxct_footprint_forward", "memxct_footprint_back",
 ]
 
 
@@ -88,6 +89,11 @@ def lib():
                                      ctypes.POINTER(ctypes.c_double), vp],
             "memxct_spmv_time": [vp, i32, ctypes.POINTER(ctypes.c_double),
                                  ctypes.POINTER(ctypes.c_double), vp],
+            "memxct_plan_set_shard": [vp, i32, i32, i32],
+            "memxct_exchange_counts": [vp, vp, vp],
+            "memxct_footprint_rays": [vp, vp],
+            "memxct_footprint_forward": [vp, vp, vp, vp],
+            "memxct_footprint_back": [vp, vp, vp, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -181,7 +187,7 @@ class MemXCT:
                  buffer_entries: int = None, tile_tomo: int = None, tile_sino: int = None,
                  cg_variant: int = 0, rank: int = 0, nranks: int = 1, unique_id: bytes = None,
                  device: int = None, group: "LocalGroup" = None, slices: int = None,
-                 exchange: str = None):
+                 exchange: str = None, shard: bool = False):
         self.n, self.m, self.c = int(n), int(projections), int(channels)
         self._h = ctypes.c_void_p()
         _check(lib().memxct_plan_create(self.n, self.m, self.c, ctypes.byref(self._h)),
@@ -198,7 +204,10 @@ class MemXCT:
         self._group = group  # keep the virtual-rank group alive as long as the plan
         self.rank = int(rank)
         self.nranks = group.nranks if group is not None else int(nranks)
-        if group is not None:
+        if shard:
+            _check(lib().memxct_plan_set_shard(self._h, self.rank, int(nranks), -1 if device is None else int(device)),
+                   "memxct_plan_set_shard")
+        elif group is not None:
             _check(lib().memxct_plan_set_comm_local(self._h, group._h, int(rank)), "memxct_plan_set_comm_local")
         elif nranks > 1 or device is not None or unique_id is not None:
             uid = None if unique_id is None else ctypes.create_string_buffer(unique_id, 128)
@@ -267,6 +276,46 @@ class MemXCT:
         _check(lib().memxct_exchange_info(self._h, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c),
                                           ctypes.byref(d)), "memxct_exchange_info")
         return {"footprint_rays": a.value, "sent": b.value, "received": c.value, "peers": d.value}
+
+    def exchange_counts(self) -> dict:
+        """Entries sent to / received from every rank per forward exchange (decomposed plans)."""
+        sc = np.empty(self.nranks, np.int64)
+        rc = np.empty(self.nranks, np.int64)
+        _check(lib().memxct_exchange_counts(self._h, sc.ctypes.data_as(ctypes.c_void_p),
+                                            rc.ctypes.data_as(ctypes.c_void_p)), "memxct_exchange_counts")
+        return {"send": sc, "recv": rc}
+
+    def footprint_rays(self) -> np.ndarray:
+        """Natural indices of this rank's footprint rays (rows of A_p), in A_p row order."""
+        out = np.empty(self.exchange_info()["footprint_rays"], np.int64)
+        _check(lib().memxct_footprint_rays(self._h, out.ctypes.data_as(ctypes.c_void_p)), "memxct_footprint_rays")
+        return out
+
+    def footprint_forward(self, x_local, y_fp=None, stream=None):
+        """Partial projection y_fp = A_p x_local (before exchange and reduction)."""
+        import torch
+        self._vec(x_local, 0, "x_local")
+        nfp = self.exchange_info()["footprint_rays"]
+        if y_fp is None:
+            y_fp = torch.empty(nfp, dtype=self.dtype, device=x_local.device)
+        if y_fp.numel() != nfp or y_fp.dtype != self.dtype or not y_fp.is_contiguous():
+            raise ValueError(f"y_fp must be a contiguous {self.dtype} tensor of {nfp} elements")
+        _check(lib().memxct_footprint_forward(self._h, _ptr(x_local), _ptr(y_fp), _stream(stream)),
+               "memxct_footprint_forward")
+        return y_fp
+
+    def footprint_back(self, y_fp, x_local=None, stream=None):
+        """Partial backprojection x_local = A_p^T y_fp."""
+        import torch
+        nfp = self.exchange_info()["footprint_rays"]
+        if y_fp.numel() != nfp or y_fp.dtype != self.dtype or not y_fp.is_contiguous() or not y_fp.is_cuda:
+            raise ValueError(f"y_fp must be a contiguous CUDA {self.dtype} tensor of {nfp} elements")
+        if x_local is None:
+            x_local = torch.empty(self.local_size(0), dtype=self.dtype, device=y_fp.device)
+        self._vec(x_local, 0, "x_local")
+        _check(lib().memxct_footprint_back(self._h, _ptr(y_fp), _ptr(x_local), _stream(stream)),
+               "memxct_footprint_back")
+        return x_local
 
     def exchange_time(self, reps: int = 20, stream=None) -> dict:
         """Collective: device microseconds of one forward and one back exchange (P > 1)."""
