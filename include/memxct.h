@@ -101,7 +101,18 @@ typedef enum {
      * stores partials straight into the owners' receive buffers and the owners' pack kernel stores
      * ray values straight into the peers' footprint buffers (CUDA IPC mappings over NVLink),
      * synchronised by epoch/credit flags -- no separate collective on the data path. */
-    MEMXCT_OPT_EXCHANGE = 9
+    MEMXCT_OPT_EXCHANGE = 9,
+    /* Row grouping of the forward SpMV's partitions (A_p rows = rays).  -1 = the paper's: a
+     * partition is PART_ROWS consecutive rays in Hilbert order (a square of about
+     * sqrt(R) x sqrt(R) projections x channels).  a > 0 (power of two <= PART_ROWS / 32): rays are
+     * grouped into blocks of `a` consecutive projections x PART_ROWS / a consecutive channels
+     * (projection-major, channel-minor inside a block) before being cut into partitions, which
+     * raises the stage-buffer reuse when consecutive projections are many pixels apart (few
+     * projections, wide detector: config 5).  0 = auto (default): blocks with a = the power of
+     * two nearest sqrt(R / (L pi / M)), L = side of the local tomogram, when that a is <= sqrt(R)/4,
+     * else -1.  Vector layouts and results are unchanged: each row still sums its entries in
+     * ascending Hilbert input order (FP32 outputs bit-identical).  CANONICAL forces -1. */
+    MEMXCT_OPT_RAY_BLOCK = 10
 } memxct_option_t;
 
 /* Create a plan for an N x N tomogram and an M x C sinogram.  Host only; no device

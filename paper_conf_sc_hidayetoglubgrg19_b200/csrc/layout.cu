@@ -779,6 +779,53 @@ Partitions make_partitions(const int32_t* cnt, int64_t nrows, int32_t R, bool ba
 
 }  // namespace
 
+// ---- forward row grouping (MEMXCT_OPT_RAY_BLOCK) ----------------------------------------------
+// Key of footprint row i: (block of `a` projections x `w` channels, then projection, channel).
+__global__ void ray_block_key_kernel(const int32_t* __restrict__ hray, const int32_t* __restrict__ sino_nat_of_h,
+                                     int64_t nrows, int32_t c, int32_t a, int32_t w, uint64_t* __restrict__ key) {
+    MX_LOOP(i, nrows) {
+        const int32_t h = hray ? hray[i] : (int32_t)i;
+        const int32_t nat = sino_nat_of_h[h];
+        const int32_t m = nat / c, k = nat % c;
+        const uint64_t blk = (uint64_t)(m / a) * (uint64_t)((c + w - 1) / w) + (uint64_t)(k / w);
+        key[i] = (blk << 32) | (uint64_t)((int64_t)(m % a) * c + k);
+    }
+}
+
+// Blocked row j = footprint row perm[j]: its Hilbert ray, its length, and where its output goes
+// (natural ray index, footprint position, or Hilbert index -- the plan's output order).
+__global__ void ray_block_gather_kernel(const uint32_t* __restrict__ perm, const int32_t* __restrict__ hray,
+                                        const int32_t* __restrict__ len, const int32_t* __restrict__ sino_nat_of_h,
+                                        int64_t nrows, int mode, int32_t* __restrict__ hray_b,
+                                        int32_t* __restrict__ len_b, int32_t* __restrict__ out_b) {
+    MX_LOOP(j, nrows) {
+        const uint32_t i = perm[j];
+        const int32_t h = hray ? hray[i] : (int32_t)i;
+        hray_b[j] = h;
+        len_b[j] = len[i];
+        out_b[j] = mode == 0 ? sino_nat_of_h[h] : mode == 1 ? (int32_t)i : h;
+    }
+}
+
+// MEMXCT_OPT_RAY_BLOCK resolved: projections per forward row block, or -1 (Hilbert rows).
+// A partition of R rays that spans `a` projections and R/a channels touches about the fewest
+// distinct pixels when the angular fan of the block across the local tomogram (side L, angle step
+// pi/M, so (a-1) L pi/M pixels of drift) is comparable to its width R/a: a* = sqrt(R / (L pi / M)).
+// The paper's Hilbert rows form ~sqrt(R) x sqrt(R) squares, which is that optimum when L pi/M ~ 1
+// (configs 1-4: 2.1-2.7); blocks are used only when a* is >= 4x smaller (config 5: L pi/M ~ 35-99).
+int32_t resolve_ray_block(const Plan& P, int64_t local_pixels, int32_t R) {
+    if (P.opt.canonical || P.opt.ray_block < 0) return -1;
+    int32_t a = (int32_t)P.opt.ray_block;
+    if (a == 0) {
+        const double drift = std::sqrt((double)std::max<int64_t>(local_pixels, 1)) * M_PI / (double)P.m;
+        const double astar = std::sqrt((double)R / std::max(drift, 1e-9));
+        if (astar > std::sqrt((double)R) / 4.0) return -1;
+        a = 1;
+        while (a * 2 <= R / 32 && std::fabs(std::log2(a * 2.0) - std::log2(astar)) < std::fabs(std::log2((double)a) - std::log2(astar))) a *= 2;
+    }
+    return std::min<int32_t>(a, std::max(1, R / 32));
+}
+
 void build_matrices(Plan& P, cudaStream_t st) {
     // angle tables (reading R1), the same expression as the paper's geometry in DESIGN.md
     std::vector<double> hc(P.m), hs(P.m);
@@ -815,10 +862,46 @@ void build_matrices(Plan& P, cudaStream_t st) {
         Bb /= 2;
     }
 
+    // forward rows grouped into projection x channel blocks (MEMXCT_OPT_RAY_BLOCK), or the
+    // footprint's Hilbert order; the A_p^T build below keeps the footprint order for its columns
+    P.ray_block = resolve_ray_block(P, npix, R);
+    DevArr<int32_t> hray_b, len_b, out_b;
+    const int32_t* fwd_hray = hray;
+    const int32_t* fwd_len = fp_len.p();
+    const int32_t* fwd_out = natural ? P.sino_nat_of_h.p() : nullptr;
+    if (P.ray_block > 0 && nrows > 1) {
+        const int32_t a = P.ray_block, w = std::max(1, R / a);
+        DevArr<uint64_t> key, key_s;
+        DevArr<uint32_t> idx, perm;
+        key.alloc(nrows);
+        key_s.alloc(nrows);
+        idx.alloc(nrows);
+        perm.alloc(nrows);
+        ray_block_key_kernel<<<blocks_for(nrows), kThreads, 0, st>>>(hray, P.sino_nat_of_h.p(), nrows, P.c, a, w, key.p());
+        MX_LAUNCHED();
+        iota_kernel<uint32_t><<<blocks_for(nrows), kThreads, 0, st>>>(idx.p(), nrows);
+        MX_LAUNCHED();
+        size_t tb = 0;
+        MX_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, key.p(), key_s.p(), idx.p(), perm.p(), (int)nrows, 0, 64, st));
+        DevBuf tmp(tb);
+        MX_CUDA(cub::DeviceRadixSort::SortPairs(tmp.get(), tb, key.p(), key_s.p(), idx.p(), perm.p(), (int)nrows, 0, 64, st));
+        MX_LAUNCHED();
+        hray_b.alloc(nrows);
+        len_b.alloc(nrows);
+        out_b.alloc(nrows);
+        const int mode = natural ? 0 : (P.dist ? 1 : 2);
+        ray_block_gather_kernel<<<blocks_for(nrows), kThreads, 0, st>>>(perm.p(), hray, fp_len.p(), P.sino_nat_of_h.p(),
+                                                                        nrows, mode, hray_b.p(), len_b.p(), out_b.p());
+        MX_LAUNCHED();
+        fwd_hray = hray_b.p();
+        fwd_len = len_b.p();
+        fwd_out = out_b.p();
+    }
+
     // equal-work partitions only under the automatic tuning (PART_ROWS given: the user's fixed
     // blocks; CANONICAL: the oracle's fixed R-row dot chunks)
     const bool balance = P.opt.part_rows == 0 && !P.opt.canonical;
-    const Partitions fwd_parts = make_partitions(fp_len.p(), nrows, R, balance, st);
+    const Partitions fwd_parts = make_partitions(fwd_len, nrows, R, balance, st);
     int64_t nnz = 0;
     for (int64_t v : fwd_parts.nnz) nnz += v;
     const int64_t budget = chunk_budget(2 * nnz);
@@ -832,7 +915,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
         DevArr<int64_t> len64, rp;
         len64.alloc(nr + 1);
         rp.alloc(nr + 1);
-        widen_i32_to_i64(fp_len.p() + ra, len64.p(), nr, s);
+        widen_i32_to_i64(fwd_len + ra, len64.p(), nr, s);
         MX_CUDA(cudaMemsetAsync(len64.p() + nr, 0, 8, s));
         exclusive_scan_i64(len64.p(), rp.p(), nr + 1, s);
         E.n = read_scalar(rp.p() + nr, s);
@@ -841,7 +924,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
         col.alloc(std::max<int64_t>(E.n, 1));
         val.alloc(std::max<int64_t>(E.n, 1));
         E.row.alloc(std::max<int64_t>(E.n, 1));
-        trace_emit(P, G, hray, ra, nr, P.t0, P.t1, rp.p(), col.p(), val.p(), E.row.p(), s);
+        trace_emit(P, G, fwd_hray, ra, nr, P.t0, P.t1, rp.p(), col.p(), val.p(), E.row.p(), s);
         E.col.alloc(std::max<int64_t>(E.n, 1));
         E.val.alloc(std::max<int64_t>(E.n, 1));
         if (E.n > 0) {
@@ -856,7 +939,10 @@ void build_matrices(Plan& P, cudaStream_t st) {
         MX_CUDA(cudaStreamSynchronize(s));
     };
     build_direction(P.fwd, nrows, npix, fwd_parts, R, B, gen_fwd, natural ? P.tomo_nat_of_h.p() : nullptr,
-                    natural ? P.sino_nat_of_h.p() : nullptr, budget, bank, st);
+                    fwd_out, budget, bank, st);
+    hray_b.reset();
+    len_b.reset();
+    out_b.reset();
 
     // ---- A_p^T: rows = local pixels; every footprint ray re-traced with the chunk's pixel range,
     // then the order-preserving (stable) sort by pixel -------------------------------------------

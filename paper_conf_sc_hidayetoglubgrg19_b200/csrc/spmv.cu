@@ -172,12 +172,12 @@ __device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned l
 // straight into its owner's receive buffer (peer memory over NVLink), then the last CTA bumps
 // this rank's forward epoch and publishes it to every owner's arrival flag (release, system
 // scope).  Replaces the separate all-to-allv of C in A = R C A_p.
-__device__ void remote_epilogue(const PeerArgs& pa, int64_t row, bool valid, float acc) {
+__device__ void remote_epilogue(const PeerArgs& pa, int64_t o, bool valid, float acc) {
     __shared__ bool am_last;
-    if (valid) {
+    if (valid) {  // o = footprint position of the row
         int h = 0;
-        while (h + 1 < pa.P && row >= pa.bound[h + 1]) ++h;
-        pa.dst[h][pa.off[h] + row] = acc;
+        while (h + 1 < pa.P && o >= pa.bound[h + 1]) ++h;
+        pa.dst[h][pa.off[h] + o] = acc;
     }
     __threadfence_system();
     __syncthreads();
@@ -243,11 +243,12 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
     }
     const int64_t row = a.prow0[p] + threadIdx.x;
     const bool valid = row < a.prow0[p + 1];
+    const int64_t o = (kNatOut && valid) ? (int64_t)a.out_idx[row] : row;
     if (kEpi == 2) {
-        remote_epilogue(pa, row, valid, acc);
+        remote_epilogue(pa, o, valid, acc);
         return;
     }
-    if (valid) y[kNatOut ? a.out_idx[row] : row] = acc;
+    if (valid) y[o] = acc;
     if (kEpi == 1) finish_dot_tree<kMaxThreads>(a, valid ? (double)acc * (double)acc : 0.0);
 }
 
@@ -516,7 +517,8 @@ void spmv_f32_remote(const Layout& L, const float* x, const PeerArgs& pa, cudaSt
     if (L.nparts == 0) fail(MEMXCT_ERR_UNSUPPORTED, "internal: empty A_p with the fused exchange");
     const SpmvArgs a = make_args(L, nullptr, nullptr, nullptr);
     const size_t smem = sizeof(float) * (size_t)L.B;
-    spmv_f32_kernel<false, 2><<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, nullptr, pa);
+    auto kern = L.out_idx.p() ? spmv_f32_kernel<true, 2> : spmv_f32_kernel<false, 2>;  // blocked rows
+    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, nullptr, pa);
     MX_LAUNCHED();
 }
 
@@ -544,6 +546,7 @@ void spmv_init() {
     set_smem(spmv_f32_kernel<false, 1>);
     set_smem(spmv_f32_kernel<false, 0>);
     set_smem(spmv_f32_kernel<false, 2>);
+    set_smem(spmv_f32_kernel<true, 2>);
     set_smem(spmv_f64_kernel<true, 0>);
     set_smem(spmv_f64_kernel<true, 1>);
     set_smem(spmv_f64_kernel<true, 2>);

@@ -19,7 +19,8 @@ STATUS = {0: "MEMXCT_OK", 1: "MEMXCT_ERR_INVALID_ARG", 2: "MEMXCT_ERR_STATE",
           3: "MEMXCT_ERR_OUT_OF_MEMORY", 4: "MEMXCT_ERR_CUDA", 5: "MEMXCT_ERR_NCCL",
           6: "MEMXCT_ERR_UNSUPPORTED"}
 OPT = {"tile_tomo": 0, "tile_sino": 1, "part_rows": 2, "buffer_entries": 3, "precision": 4,
-       "canonical": 5, "cg_variant": 6, "vector_order": 7, "slices": 8, "exchange": 9}
+       "canonical": 5, "cg_variant": 6, "vector_order": 7, "slices": 8, "exchange": 9,
+       "ray_block": 10}
 
 #: every symbol include/memxct.h declares (checked by tests/test_abi.py)
 SYMBOLS = [
@@ -187,7 +188,7 @@ class MemXCT:
                  buffer_entries: int = None, tile_tomo: int = None, tile_sino: int = None,
                  cg_variant: int = 0, rank: int = 0, nranks: int = 1, unique_id: bytes = None,
                  device: int = None, group: "LocalGroup" = None, slices: int = None,
-                 exchange: str = None, shard: bool = False):
+                 exchange: str = None, shard: bool = False, ray_block: int = None):
         self.n, self.m, self.c = int(n), int(projections), int(channels)
         self._h = ctypes.c_void_p()
         _check(lib().memxct_plan_create(self.n, self.m, self.c, ctypes.byref(self._h)),
@@ -196,7 +197,7 @@ class MemXCT:
         opts = {"precision": {"fp32": 0, "mixed": 1}[precision], "canonical": int(bool(canonical)),
                 "vector_order": {"natural": 0, "plan": 1}[vector_order], "cg_variant": cg_variant,
                 "part_rows": part_rows, "buffer_entries": buffer_entries, "tile_tomo": tile_tomo,
-                "tile_sino": tile_sino, "slices": slices,
+                "tile_sino": tile_sino, "slices": slices, "ray_block": ray_block,
                 "exchange": None if exchange is None else {"collective": 0, "peer": 1}[exchange]}
         for k, v in opts.items():
             if v is not None:

@@ -66,7 +66,7 @@ def rel_l2(a, b):
     return float(np.linalg.norm(np.asarray(a) - np.asarray(b)) / np.linalg.norm(np.asarray(b)))
 
 
-def case_projections(nranks, n, m, c):
+def case_projections(nranks, n, m, c, ray_block=None):
     import torch
 
     import oracle
@@ -75,7 +75,7 @@ def case_projections(nranks, n, m, c):
     import time
     t0 = time.time()
     g0, coll = build_group(n, m, c, nranks)
-    g1, peer = build_group(n, m, c, nranks, exchange="peer")
+    g1, peer = build_group(n, m, c, nranks, exchange="peer", ray_block=ray_block)
     print(f"built {time.time() - t0:.2f}s", flush=True)
     x = inputs.uniform(n * n, 1)
     y = inputs.uniform(m * c, 2)
@@ -140,7 +140,8 @@ if __name__ == "__main__":
     gc.disable()
     torch.cuda.init()
     case, nranks, n, m, c = sys.argv[1], *map(int, sys.argv[2:6])
-    {"projections": case_projections, "cg": case_cg}[case](nranks, n, m, c)
+    extra = [int(v) for v in sys.argv[6:]]  # projections: RAY_BLOCK of the peer group
+    {"projections": case_projections, "cg": case_cg}[case](nranks, n, m, c, *extra)
     torch.cuda.synchronize()
     print("CASE OK", case, nranks, n, m, c, flush=True)
     os._exit(0)  # skip teardown frees while nothing else runs; the process ends here

@@ -38,3 +38,11 @@ def test_peer_exchange_bit_identical_to_collective(nranks, geom):
 
 def test_peer_exchange_cg():
     run_case("cg", 4, 256, 360, 256)
+
+
+@pytest.mark.parametrize("ray_block", [2, 8])
+def test_peer_exchange_blocked_rows(ray_block):
+    """Forward rows grouped in projection blocks (RAY_BLOCK): the fused epilogue stores each
+    partial at its footprint position, so outputs stay bit-identical to the collective path on
+    Hilbert rows."""
+    run_case("projections", 3, 256, 360, 256, ray_block)
