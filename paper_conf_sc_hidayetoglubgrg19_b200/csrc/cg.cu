@@ -21,7 +21,11 @@ namespace mx {
 namespace {
 
 constexpr int kVT = 256;
-constexpr int kVecBlocks = 296;  // 2 x 148 SMs
+// Vector steps are HBM streams of a few MB: 8 CTAs x 256 threads per SM and 4 independent
+// elements per thread per pass keep ~10 MB of loads in flight (296 CTAs with one element per
+// pass ran at ~1 TB/s: 32 us for the 30 MB of the x/r update at cfg3).
+constexpr int kVecBlocks = 8 * 148;
+constexpr int kU = 4;
 
 // scalar slots of slice s: gam[s*n1 + k], del[...], res2[...]; stop flags per slice
 struct Scal {
@@ -67,15 +71,32 @@ __device__ void vec_dot_finish(double mine, double* part, double* out, unsigned 
     __syncthreads();
     if (!am_last) return;
     __threadfence();
+    // fixed-order parallel sum of the per-block partials: thread t adds blocks t, t + kVT, ...
+    double t = 0.0;
+    for (unsigned i = threadIdx.x; i < gridDim.x; i += kVT) t += ((volatile double*)part)[i];
+    for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+    __syncthreads();
+    if (lane == 0) red[warp] = t;
+    __syncthreads();
     if (threadIdx.x == 0) {
-        double t = 0.0;
-        for (unsigned i = 0; i < gridDim.x; ++i) t += ((volatile double*)part)[i];
-        *out = t;
+        double tot = 0.0;
+        for (int w = 0; w < kVT / 32; ++w) tot += red[w];
+        *out = tot;
         *ticket = 0u;
     }
 }
 
 #define MX_GRID_LOOP(i, n) for (int64_t i = (int64_t)blockIdx.x * kVT + threadIdx.x; i < (n); i += (int64_t)gridDim.x * kVT)
+// kU elements per thread per pass, strided by the grid so every warp access stays coalesced:
+// body(i) for i = i0 + u * stride, u < kU, i < n (loads of the kU elements are independent)
+#define MX_GRID_LOOP_U(i, n, body)                                                                \
+    for (int64_t i##0 = (int64_t)blockIdx.x * kVT + threadIdx.x, i##s = (int64_t)gridDim.x * kVT; \
+         i##0 < (n); i##0 += kU * i##s) {                                                          \
+        _Pragma("unroll") for (int u_ = 0; u_ < kU; ++u_) {                                        \
+            const int64_t i = i##0 + u_ * i##s;                                                    \
+            if (i < (n)) { body }                                                                  \
+        }                                                                                          \
+    }
 
 // r = y ; x = 0 ; res2[0] = <r, r> ; stop = 0
 template <class T>
@@ -85,12 +106,8 @@ cg_init_kernel(const T* __restrict__ y, T* __restrict__ r, int64_t nr, T* __rest
     const int s = blockIdx.y;
     y += s * nr; r += s * nr; x += s * nx;
     double acc = 0.0;
-    MX_GRID_LOOP(i, nr) {
-        const T v = y[i];
-        r[i] = v;
-        acc += (double)v * (double)v;
-    }
-    MX_GRID_LOOP(i, nx) x[i] = T(0);
+    MX_GRID_LOOP_U(i, nr, const T v = y[i]; r[i] = v; acc += (double)v * (double)v;)
+    MX_GRID_LOOP_U(i, nx, x[i] = T(0);)
     if (blockIdx.x == 0 && threadIdx.x == 0) { sc.stop[s] = 0; sc.stop_at[s] = 0x7fffffff; }
     vec_dot_finish(acc, part, sc.res2 + (int64_t)s * sc.n1, ticket);
 }
@@ -98,7 +115,7 @@ cg_init_kernel(const T* __restrict__ y, T* __restrict__ r, int64_t nr, T* __rest
 template <class T>
 __global__ void __launch_bounds__(kVT) copy_kernel(const T* __restrict__ a, T* __restrict__ b, int64_t n) {
     a += blockIdx.y * n; b += blockIdx.y * n;
-    MX_GRID_LOOP(i, n) b[i] = a[i];
+    MX_GRID_LOOP_U(i, n, b[i] = a[i];)
 }
 
 __device__ __forceinline__ float upd(float a, double s, float b) { return (float)__fma_rn(s, (double)a, (double)b); }
@@ -119,14 +136,10 @@ cg_update_xr_kernel(T* __restrict__ x, const T* __restrict__ p, int64_t nx, T* _
         return;
     }
     const double alpha = __ddiv_rn(g, d);
-    MX_GRID_LOOP(i, nx) x[i] = upd(p[i], alpha, x[i]);
+    MX_GRID_LOOP_U(i, nx, x[i] = upd(p[i], alpha, x[i]);)
     if (kUpdateR) {
         double acc = 0.0;
-        MX_GRID_LOOP(i, nr) {
-            const T v = upd(q[i], -alpha, r[i]);
-            r[i] = v;
-            acc += (double)v * (double)v;
-        }
+        MX_GRID_LOOP_U(i, nr, const T v = upd(q[i], -alpha, r[i]); r[i] = v; acc += (double)v * (double)v;)
         vec_dot_finish(acc, part, sc.res2 + o + k, ticket);
     }
 }
@@ -140,11 +153,7 @@ cg_explicit_r_kernel(const T* __restrict__ y, const T* __restrict__ ax, T* __res
     if (sc.stop[s]) return;
     y += s * nr; ax += s * nr; r += s * nr;
     double acc = 0.0;
-    MX_GRID_LOOP(i, nr) {
-        const T v = y[i] - ax[i];
-        r[i] = v;
-        acc += (double)v * (double)v;
-    }
+    MX_GRID_LOOP_U(i, nr, const T v = y[i] - ax[i]; r[i] = v; acc += (double)v * (double)v;)
     vec_dot_finish(acc, part, sc.res2 + (int64_t)s * sc.n1 + k, ticket);
 }
 
@@ -157,7 +166,7 @@ cg_update_p_kernel(T* __restrict__ p, const T* __restrict__ sv, int64_t nx, Scal
     const int64_t o = (int64_t)s * sc.n1;
     p += s * nx; sv += s * nx;
     const double beta = __ddiv_rn(sc.gam[o + k], sc.gam[o + k - 1]);
-    MX_GRID_LOOP(i, nx) p[i] = upd(p[i], beta, sv[i]);
+    MX_GRID_LOOP_U(i, nx, p[i] = upd(p[i], beta, sv[i]);)
 }
 
 // <v, v> in fp64 over a fixed grid (deterministic: fixed element->thread map, fixed tree);
@@ -167,15 +176,12 @@ __global__ void __launch_bounds__(kVT)
 dot_kernel(const T* __restrict__ v, int64_t n, double* out, int64_t stride, double* part, unsigned int* ticket) {
     v += blockIdx.y * n;
     double acc = 0.0;
-    MX_GRID_LOOP(i, n) {
-        const double e = (double)v[i];
-        acc += e * e;
-    }
+    MX_GRID_LOOP_U(i, n, const double e = (double)v[i]; acc += e * e;)
     vec_dot_finish(acc, part, out + blockIdx.y * stride, ticket);
 }
 
 unsigned vec_blocks(int64_t n) {
-    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(kVecBlocks, ceil_div(n, kVT)));
+    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(kVecBlocks, ceil_div(n, (int64_t)kVT * kU)));
 }
 
 // Projection of K slices followed by the per-slice dot of the output.  At K = 1, P = 1 the dot
