@@ -112,7 +112,16 @@ typedef enum {
      * two nearest sqrt(R / (L pi / M)), L = side of the local tomogram, when that a is <= sqrt(R)/4,
      * else -1.  Vector layouts and results are unchanged: each row still sums its entries in
      * ascending Hilbert input order (FP32 outputs bit-identical).  CANONICAL forces -1. */
-    MEMXCT_OPT_RAY_BLOCK = 10
+    MEMXCT_OPT_RAY_BLOCK = 10,
+    /* Stage order of the forward SpMV (A_p): -1 = the paper's (reading R10): a partition's
+     * distinct input pixels sorted by Hilbert index and cut into stages of BUFFER_ENTRIES.
+     * 1 = slab order: sorted by (band of 16 pixels across the direction of the partition's rays,
+     * then Hilbert index), so every stage is a band that all of the partition's rays cross and all
+     * warps have work in every stage.  Same map entries and bytes; each
+     * row sums the same products in another order (FP32 results equal up to rounding).  0 = auto
+     * (default): slab order together with projection blocks (RAY_BLOCK > 0), else -1.
+     * CANONICAL forces -1. */
+    MEMXCT_OPT_STAGE_ORDER = 11
 } memxct_option_t;
 
 /* Create a plan for an N x N tomogram and an M x C sinogram.  Host only; no device
@@ -300,6 +309,13 @@ memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0
                                      int64_t* slot_off, uint16_t* ind, float* val,
                                      uint16_t* lane_chunks, int64_t* part_row0, int64_t* n_map,
                                      int64_t* n_slot_off, int64_t* n_slots);
+
+/* Output position of every layout row (dir 0: rows of A / A_p, dir 1: rows of A^T / A_p^T), host
+ * array of layout_info rows int64: the index the row's result is written to in the call's output
+ * vector -- natural (VECTOR_ORDER = 0), plan / Hilbert order (1) or footprint position (A_p of a
+ * decomposed plan).  Identity unless the rows were regrouped (RAY_BLOCK) or the plan writes
+ * natural order. */
+memxct_status_t memxct_layout_rows(memxct_plan_t plan, int32_t dir, int64_t* out_index);
 
 /* Destroy a plan and free everything it owns.  NULL-safe. */
 memxct_status_t memxct_plan_destroy(memxct_plan_t plan);

@@ -160,6 +160,10 @@ memxct_status_t memxct_plan_set_option(memxct_plan_t plan, memxct_option_t optio
                 if (value > 0 && (value & (value - 1))) mx::fail(MEMXCT_ERR_INVALID_ARG, "RAY_BLOCK must be -1, 0 or a power of two");
                 P.opt.ray_block = value;
                 break;
+            case MEMXCT_OPT_STAGE_ORDER:
+                range(-1, 1);
+                P.opt.stage_order = value;
+                break;
             default: mx::fail(MEMXCT_ERR_INVALID_ARG, "unknown option");
         }
     });
@@ -181,6 +185,7 @@ memxct_status_t memxct_plan_get_option(memxct_plan_t plan, memxct_option_t optio
             case MEMXCT_OPT_SLICES: *value = P.opt.slices; break;
             case MEMXCT_OPT_EXCHANGE: *value = P.opt.exchange; break;
             case MEMXCT_OPT_RAY_BLOCK: *value = P.built ? P.ray_block : P.opt.ray_block; break;
+            case MEMXCT_OPT_STAGE_ORDER: *value = P.built ? P.stage_order : P.opt.stage_order; break;
             default: mx::fail(MEMXCT_ERR_INVALID_ARG, "unknown option");
         }
     });
@@ -614,6 +619,22 @@ memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0
         if (part_row0) MX_CUDA(cudaMemcpy(part_row0, L.prow0.p() + p0, 8 * (p1 - p0 + 1), cudaMemcpyDeviceToHost));
         if (lane_chunks && b1 > b0)
             MX_CUDA(cudaMemcpy(lane_chunks, L.lane_chunks.p() + b0 * 32, 2 * 32 * (b1 - b0), cudaMemcpyDeviceToHost));
+    });
+}
+
+memxct_status_t memxct_layout_rows(memxct_plan_t plan, int32_t dir, int64_t* out_index) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(out_index, "out_index");
+        if (dir != 0 && dir != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "dir must be 0 or 1");
+        const mx::Layout& L = dir == 0 ? P.fwd : P.back;
+        if (L.out_idx.p()) {
+            std::vector<int32_t> h(L.nrows);
+            if (L.nrows > 0) MX_CUDA(cudaMemcpy(h.data(), L.out_idx.p(), 4 * L.nrows, cudaMemcpyDeviceToHost));
+            for (int64_t r = 0; r < L.nrows; ++r) out_index[r] = h[r];
+        } else {
+            for (int64_t r = 0; r < L.nrows; ++r) out_index[r] = r;
+        }
     });
 }
 

@@ -111,18 +111,23 @@ __global__ void rank_kernel(const uint32_t* __restrict__ row_ids, const uint32_t
 }
 
 // map[map_off[p] + rank] = translated input of every set bit of partition p's bitmap
+// (slab stage order: the bitmap is over the partition's class order col' = K_c[col]; inv holds
+// the C inverse orders [C][ncols] and part_class the class of every partition)
 __global__ void map_kernel(const uint32_t* __restrict__ bitmap, const uint32_t* __restrict__ word_prefix,
                            int64_t words, int64_t nsub, int64_t pa, const int64_t* __restrict__ map_off,
-                           const int32_t* __restrict__ translate, int32_t* __restrict__ map) {
+                           const int32_t* __restrict__ translate, const int32_t* __restrict__ inv,
+                           const int32_t* __restrict__ part_class, int64_t ncols, int32_t* __restrict__ map) {
     MX_LOOP(i, nsub * words) {
         uint32_t b = bitmap[i];
         if (!b) continue;
         const int64_t p = i / words, w = i % words;
         int64_t r = map_off[pa + p] + word_prefix[i];
+        const int32_t* iv = inv ? inv + (int64_t)part_class[pa + p] * ncols : nullptr;
         while (b) {
             const int bit = __ffs(b) - 1;
             b &= b - 1;
-            const int64_t col = w * 32 + bit;
+            int64_t col = w * 32 + bit;
+            if (iv) col = iv[col];
             map[r++] = translate ? translate[col] : (int32_t)col;
         }
     }
@@ -452,6 +457,8 @@ struct Builder {
     int64_t words;
     int64_t bitmap_parts;   // partitions per bitmap sub-chunk
     int32_t bank_classes;   // 0 = ascending local index in every run; else bank-aware order
+    const int32_t* col_inv = nullptr;     // slab stage order: [C][ncols] col' -> col (else null)
+    const int32_t* part_class = nullptr;  // slab stage order: class of every partition
     DevArr<int64_t> distinct, nst, slots_p;
     std::vector<int64_t> h_stage_base, h_part_slot;
 
@@ -483,7 +490,8 @@ struct Builder {
             if (write_map) {
                 map_kernel<<<blocks_for((qb - qa) * words), kThreads, 0, st>>>(bitmap.p(), wprefix.p(), words,
                                                                                 qb - qa, qa, L.map_off.p(),
-                                                                                in_translate, L.map.p());
+                                                                                in_translate, col_inv, part_class,
+                                                                                ncols, L.map.p());
                 MX_LAUNCHED();
             }
         }
@@ -632,7 +640,8 @@ int64_t chunk_budget(int64_t nnz_both_dirs_remaining) {
 
 void build_direction(Layout& L, int64_t nrows, int64_t ncols, const Partitions& parts, int32_t R,
                      int32_t B, const Generator& gen, const int32_t* in_translate, const int32_t* out_translate,
-                     int64_t budget, int32_t bank_classes, cudaStream_t st) {
+                     int64_t budget, int32_t bank_classes, cudaStream_t st, const int32_t* col_inv = nullptr,
+                     const int32_t* part_class = nullptr) {
     L = Layout{};
     L.nrows = nrows;
     L.ncols = ncols;
@@ -654,6 +663,8 @@ void build_direction(Layout& L, int64_t nrows, int64_t ncols, const Partitions& 
     }
     Builder b{L, nrows, ncols, R, B, R / 32, in_translate, row_part.p(), L.prow0.p(), parts.row0};
     b.bank_classes = bank_classes;
+    b.col_inv = col_inv;
+    b.part_class = part_class;
     b.words = std::max<int64_t>(1, ceil_div(ncols, 32));
     b.bitmap_parts = std::max<int64_t>(1, ((int64_t)2 << 30) / (b.words * 8));
     b.distinct.alloc(nparts + 1);
@@ -779,6 +790,65 @@ Partitions make_partitions(const int32_t* cnt, int64_t nrows, int32_t R, bool ba
 
 }  // namespace
 
+// ---- slab stage order of the forward partitions (MEMXCT_OPT_STAGE_ORDER) ----------------------
+// The paper cuts a partition's distinct inputs, sorted by Hilbert index, into stages (R10).  A
+// stage is then a compact patch of pixels that only some of the partition's rays cross, so per
+// stage only some warps (32 rays each) have work and the CTA waits at the stage barrier for the
+// busiest (profiles/r01_layout_efficiency.log: 34-43 % barrier efficiency on config 5).  In slab
+// order the inputs are sorted by (slab across the rays, Hilbert index): slab = floor(along /
+// kSlabThick) with along = the pixel centre's coordinate along the direction (-sin phi, cos phi)
+// of the partition's rays, so every stage is a band that every ray of the partition crosses.
+// Directions are quantised to kSlabClasses classes phi_c = (c + 1/2) pi / C; partition p uses the
+// class of its middle ray.  K_c (col -> col') and its inverse are permutations of the local
+// pixels, built once per class.
+constexpr int32_t kSlabClasses = 16;
+constexpr double kSlabThick = 16.0;
+
+__global__ void slab_key_kernel(const int32_t* __restrict__ tomo_nat_of_h, int64_t t0, int64_t npix, int32_t n,
+                                double cphi, double sphi, uint64_t* __restrict__ key) {
+    MX_LOOP(col, npix) {
+        const int32_t nat = tomo_nat_of_h[t0 + col];
+        const double u = (double)(nat % n) + 0.5 - 0.5 * n, v = (double)(nat / n) + 0.5 - 0.5 * n;
+        const double along = -u * sphi + v * cphi;                 // |along| <= n / sqrt(2)
+        const int64_t slab = (int64_t)floor(along / kSlabThick) + (int64_t)(n / kSlabThick) + 2;
+        key[col] = ((uint64_t)slab << 32) | (uint64_t)col;       // (slab, Hilbert)
+    }
+}
+
+__global__ void invert_kernel(const uint32_t* __restrict__ inv, int64_t n, int32_t* __restrict__ inv_out,
+                              int32_t* __restrict__ fwd_out) {
+    MX_LOOP(j, n) {
+        inv_out[j] = (int32_t)inv[j];
+        fwd_out[inv[j]] = (int32_t)j;
+    }
+}
+
+// class of every forward partition: direction of its middle ray
+__global__ void part_class_kernel(const int64_t* __restrict__ row0, int64_t np, const int32_t* __restrict__ hray,
+                                  const int32_t* __restrict__ sino_nat_of_h, int32_t c_chan, int32_t m_proj,
+                                  int32_t* __restrict__ part_class) {
+    MX_LOOP(p, np) {
+        const int64_t mid = (row0[p] + row0[p + 1]) / 2;
+        const int32_t h = hray ? hray[mid] : (int32_t)mid;
+        const int64_t m = sino_nat_of_h[h] / c_chan;
+        const int64_t cl = m * kSlabClasses / m_proj;
+        part_class[p] = (int32_t)(cl < kSlabClasses - 1 ? cl : kSlabClasses - 1);
+    }
+}
+
+__global__ void row_class_kernel(const int64_t* __restrict__ row0, int64_t np, const int32_t* __restrict__ part_class,
+                                 int32_t* __restrict__ row_class) {
+    MX_LOOP(p, np)
+    for (int64_t r = row0[p]; r < row0[p + 1]; ++r) row_class[r] = part_class[p];
+}
+
+// entry columns of a generated chunk -> their partition class order
+__global__ void apply_class_order_kernel(const uint32_t* __restrict__ rows, int64_t n,
+                                         const int32_t* __restrict__ row_class, const int32_t* __restrict__ kfwd,
+                                         int64_t ncols, uint32_t* __restrict__ cols) {
+    MX_LOOP(e, n) cols[e] = (uint32_t)kfwd[(int64_t)row_class[rows[e]] * ncols + cols[e]];
+}
+
 // ---- forward row grouping (MEMXCT_OPT_RAY_BLOCK) ----------------------------------------------
 // Key of footprint row i: (block of `a` projections x `w` channels, then projection, channel).
 __global__ void ray_block_key_kernel(const int32_t* __restrict__ hray, const int32_t* __restrict__ sino_nat_of_h,
@@ -902,6 +972,49 @@ void build_matrices(Plan& P, cudaStream_t st) {
     // blocks; CANONICAL: the oracle's fixed R-row dot chunks)
     const bool balance = P.opt.part_rows == 0 && !P.opt.canonical;
     const Partitions fwd_parts = make_partitions(fwd_len, nrows, R, balance, st);
+
+    // slab stage order (MEMXCT_OPT_STAGE_ORDER): per-class column orders, class of every partition
+    // and row; auto = with projection blocks (the geometries whose Hilbert stages are sparse)
+    P.stage_order = (P.opt.canonical || P.opt.stage_order < 0) ? -1
+                    : P.opt.stage_order > 0 ? 1 : (P.ray_block > 0 ? 1 : -1);
+    DevArr<int32_t> kfwd, kinv, part_class, row_class;
+    const int64_t fnp = (int64_t)fwd_parts.row0.size() - 1;
+    if (P.stage_order == 1 && npix > 0 && nrows > 0) {
+        kfwd.alloc((int64_t)kSlabClasses * npix);
+        kinv.alloc((int64_t)kSlabClasses * npix);
+        DevArr<uint64_t> key, key_s;
+        DevArr<uint32_t> idx, inv;
+        key.alloc(npix);
+        key_s.alloc(npix);
+        idx.alloc(npix);
+        inv.alloc(npix);
+        size_t tb = 0;
+        MX_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, key.p(), key_s.p(), idx.p(), inv.p(), (int)npix, 0, 64, st));
+        DevBuf tmp(tb);
+        for (int32_t cl = 0; cl < kSlabClasses; ++cl) {
+            const double phi = (cl + 0.5) * M_PI / kSlabClasses;
+            slab_key_kernel<<<blocks_for(npix), kThreads, 0, st>>>(P.tomo_nat_of_h.p(), P.t0, npix, P.n, std::cos(phi),
+                                                                   std::sin(phi), key.p());
+            MX_LAUNCHED();
+            iota_kernel<uint32_t><<<blocks_for(npix), kThreads, 0, st>>>(idx.p(), npix);
+            MX_LAUNCHED();
+            MX_CUDA(cub::DeviceRadixSort::SortPairs(tmp.get(), tb, key.p(), key_s.p(), idx.p(), inv.p(), (int)npix, 0, 64, st));
+            MX_LAUNCHED();
+            invert_kernel<<<blocks_for(npix), kThreads, 0, st>>>(inv.p(), npix, kinv.p() + cl * npix, kfwd.p() + cl * npix);
+            MX_LAUNCHED();
+        }
+        DevArr<int64_t> row0;
+        row0.alloc(fnp + 1);
+        MX_CUDA(cudaMemcpyAsync(row0.p(), fwd_parts.row0.data(), 8 * (fnp + 1), cudaMemcpyHostToDevice, st));
+        part_class.alloc(std::max<int64_t>(fnp, 1));
+        row_class.alloc(nrows);
+        part_class_kernel<<<blocks_for(fnp), kThreads, 0, st>>>(row0.p(), fnp, fwd_hray, P.sino_nat_of_h.p(), P.c, P.m,
+                                                                part_class.p());
+        MX_LAUNCHED();
+        row_class_kernel<<<blocks_for(fnp), kThreads, 0, st>>>(row0.p(), fnp, part_class.p(), row_class.p());
+        MX_LAUNCHED();
+        MX_CUDA(cudaStreamSynchronize(st));
+    }
     int64_t nnz = 0;
     for (int64_t v : fwd_parts.nnz) nnz += v;
     const int64_t budget = chunk_budget(2 * nnz);
@@ -925,6 +1038,11 @@ void build_matrices(Plan& P, cudaStream_t st) {
         val.alloc(std::max<int64_t>(E.n, 1));
         E.row.alloc(std::max<int64_t>(E.n, 1));
         trace_emit(P, G, fwd_hray, ra, nr, P.t0, P.t1, rp.p(), col.p(), val.p(), E.row.p(), s);
+        if (kfwd.p() && E.n > 0) {  // slab stage order: sort each row by its partition's class order
+            apply_class_order_kernel<<<blocks_for(E.n), kThreads, 0, s>>>(E.row.p(), E.n, row_class.p(), kfwd.p(),
+                                                                          npix, col.p());
+            MX_LAUNCHED();
+        }
         E.col.alloc(std::max<int64_t>(E.n, 1));
         E.val.alloc(std::max<int64_t>(E.n, 1));
         if (E.n > 0) {
@@ -939,7 +1057,11 @@ void build_matrices(Plan& P, cudaStream_t st) {
         MX_CUDA(cudaStreamSynchronize(s));
     };
     build_direction(P.fwd, nrows, npix, fwd_parts, R, B, gen_fwd, natural ? P.tomo_nat_of_h.p() : nullptr,
-                    fwd_out, budget, bank, st);
+                    fwd_out, budget, bank, st, kinv.p(), part_class.p());
+    kfwd.reset();
+    kinv.reset();
+    part_class.reset();
+    row_class.reset();
     hray_b.reset();
     len_b.reset();
     out_b.reset();

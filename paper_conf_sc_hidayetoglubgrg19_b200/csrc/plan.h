@@ -68,6 +68,7 @@ struct Options {
     int64_t slices = 1;        // slices per batched call the stage buffer is sized for
     int64_t exchange = 0;      // P > 1: 0 = transport collectives (NCCL), 1 = fused peer memory
     int64_t ray_block = 0;     // forward partitions: -1 Hilbert rows, a > 0 blocks of a projections, 0 auto
+    int64_t stage_order = 0;   // forward stages: -1 Hilbert (paper), 1 slabs across the rays, 0 auto
 };
 
 // host-side angle tables on the device (reading R1)
@@ -149,6 +150,7 @@ struct Plan {
     bool fused_dot = true;   // CG dots in the SpMV epilogue (MEMXCT_FUSED_DOT=0: separate kernels)
     int32_t part_rows = 0, buffer_entries = 0;  // resolved tuning of A_p (A_p^T: back.R / back.B)
     int32_t ray_block = -1;                     // resolved MEMXCT_OPT_RAY_BLOCK (-1: Hilbert rows)
+    int32_t stage_order = -1;                   // resolved MEMXCT_OPT_STAGE_ORDER (-1 Hilbert, 1 slab)
 
     // domain decomposition: this rank owns Hilbert pixels [t0, t1) and rays [s0, s1)
     std::unique_ptr<Comm> comm;

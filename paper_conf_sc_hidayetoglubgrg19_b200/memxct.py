@@ -20,7 +20,7 @@ STATUS = {0: "MEMXCT_OK", 1: "MEMXCT_ERR_INVALID_ARG", 2: "MEMXCT_ERR_STATE",
           6: "MEMXCT_ERR_UNSUPPORTED"}
 OPT = {"tile_tomo": 0, "tile_sino": 1, "part_rows": 2, "buffer_entries": 3, "precision": 4,
        "canonical": 5, "cg_variant": 6, "vector_order": 7, "slices": 8, "exchange": 9,
-       "ray_block": 10}
+       "ray_block": 10, "stage_order": 11}
 
 #: every symbol include/memxct.h declares (checked by tests/test_abi.py)
 SYMBOLS = [
@@ -34,7 +34,7 @@ SYMBOLS = [
     "memxct_partition_ranges", "memxct_domain_ranges", "memxct_exchange_info",
     "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
     "memxct_sirt", "memxct_spmv_time", "memxct_plan_set_shard", "memxct_exchange_counts",
-    "memxct_footprint_rays", "memxct_footprint_forward", "memxct_footprint_back",
+    "memxct_footprint_rays", "memxct_footprint_forward", "memxct_footprint_back", "memxct_layout_rows",
 ]
 
 
@@ -95,6 +95,7 @@ def lib():
             "memxct_footprint_rays": [vp, vp],
             "memxct_footprint_forward": [vp, vp, vp, vp],
             "memxct_footprint_back": [vp, vp, vp, vp],
+            "memxct_layout_rows": [vp, i32, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -188,7 +189,8 @@ class MemXCT:
                  buffer_entries: int = None, tile_tomo: int = None, tile_sino: int = None,
                  cg_variant: int = 0, rank: int = 0, nranks: int = 1, unique_id: bytes = None,
                  device: int = None, group: "LocalGroup" = None, slices: int = None,
-                 exchange: str = None, shard: bool = False, ray_block: int = None):
+                 exchange: str = None, shard: bool = False, ray_block: int = None,
+                 stage_order: int = None):
         self.n, self.m, self.c = int(n), int(projections), int(channels)
         self._h = ctypes.c_void_p()
         _check(lib().memxct_plan_create(self.n, self.m, self.c, ctypes.byref(self._h)),
@@ -197,7 +199,7 @@ class MemXCT:
         opts = {"precision": {"fp32": 0, "mixed": 1}[precision], "canonical": int(bool(canonical)),
                 "vector_order": {"natural": 0, "plan": 1}[vector_order], "cg_variant": cg_variant,
                 "part_rows": part_rows, "buffer_entries": buffer_entries, "tile_tomo": tile_tomo,
-                "tile_sino": tile_sino, "slices": slices, "ray_block": ray_block,
+                "tile_sino": tile_sino, "slices": slices, "ray_block": ray_block, "stage_order": stage_order,
                 "exchange": None if exchange is None else {"collective": 0, "peer": 1}[exchange]}
         for k, v in opts.items():
             if v is not None:
@@ -338,6 +340,12 @@ class MemXCT:
                "memxct_layout_info")
         return dict(zip(["parts", "stages", "slots", "map_entries", "rows", "nnz", "part_rows", "buffer_entries"],
                         [x.value for x in v]))
+
+    def layout_rows(self, direction: int) -> np.ndarray:
+        """Output position of every layout row (memxct_layout_rows)."""
+        out = np.empty(self.layout_info(direction)["rows"], np.int64)
+        _check(lib().memxct_layout_rows(self._h, direction, out.ctypes.data_as(ctypes.c_void_p)), "memxct_layout_rows")
+        return out
 
     def layout_export(self, direction: int, p0: int = 0, p1: int = None) -> dict:
         if p1 is None:

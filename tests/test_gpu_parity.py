@@ -68,7 +68,9 @@ def _pattern_keys(plan, direction, npix, R, B):
     d = decode(ex, R, B)
     check_structure(d)
     e = real_entries(d)
-    row_nat = plan.local_indices(1 if direction == 0 else 0)[e["row"]]
+    out = plan.layout_rows(direction)[e["row"]]          # regrouped rows (RAY_BLOCK) write elsewhere
+    natural = plan.get_option("vector_order") == 0
+    row_nat = out if natural else plan.local_indices(1 if direction == 0 else 0)[out]
     if direction == 0:
         key = row_nat * npix + e["col"]
     else:
@@ -96,6 +98,34 @@ def test_sparsity_pattern_and_values_exact(orc, coo_cache, n, m, c, part_rows, b
         assert np.array_equal(val, oval), direction          # fp32 RN of the fp64 length
         # every stage holds at most B distinct inputs, and maps are sorted (Hilbert order)
         assert np.all(np.diff(ex["map_off"]) >= 0)
+
+
+@pytest.mark.parametrize("n,m,c", [(64, 90, 64), (40, 24, 36), (256, 360, 256)])
+@pytest.mark.parametrize("ray_block,stage_order,order", [(4, 1, "natural"), (2, -1, "plan"), (-1, 1, "plan"),
+                                                         (8, 1, "plan")])
+def test_regrouped_rows_and_slab_stages_pattern_exact(orc, coo_cache, n, m, c, ray_block, stage_order, order):
+    """Projection-block rows (RAY_BLOCK) and slab stages (STAGE_ORDER): the decoded pattern and
+    values are still exactly the oracle's; stage maps hold <= B inputs and runs ascend by local
+    index (check_structure)."""
+    plan = make_plan(n, m, c, ray_block=ray_block, stage_order=stage_order, vector_order=order)
+    assert plan.get_option("stage_order") == stage_order
+    rows, cols, vals = coo_cache(n, m, c)
+    npix = n * n
+    okey = rows.astype(np.int64) * npix + cols
+    oo = np.argsort(okey)
+    okey, oval = okey[oo], vals[oo].astype(np.float32)
+    for direction in (0, 1):
+        li = plan.layout_info(direction)
+        key, val, ex = _pattern_keys(plan, direction, npix, li["part_rows"], li["buffer_entries"])
+        assert np.array_equal(key, okey), direction
+        assert np.array_equal(val, oval), direction
+    x = inputs.uniform(n * n, 5)
+    xi = x if order == "natural" else x[plan.local_indices(0)]
+    y = plan.forward(torch.from_numpy(np.ascontiguousarray(xi)).cuda()).cpu().numpy()
+    y_orc = orc.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)
+    if order == "plan":
+        y_orc = y_orc[plan.local_indices(1)]
+    assert rel_l2(y, y_orc) <= 1e-5
 
 
 @pytest.mark.parametrize("n,m,c", [(256, 360, 256), (96, 120, 96)])

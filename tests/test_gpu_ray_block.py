@@ -44,7 +44,7 @@ def test_blocked_rows_bit_identical(orc, coo_cache, geom, order):
         yo[ref.local_indices(1)] = y_ref.cpu().numpy()
     assert rel_l2(yo, y_orc) <= 1e-5
     for a in (1, 2, 4, 8):
-        p = MemXCT(n, m, c, vector_order=order, ray_block=a).build()
+        p = MemXCT(n, m, c, vector_order=order, ray_block=a, stage_order=-1).build()
         assert p.get_option("ray_block") == min(a, p.layout_info(0)["part_rows"] // 32)
         assert p.layout_info(0)["nnz"] == ref.layout_info(0)["nnz"]
         assert torch.equal(p.forward(xt), y_ref), a
@@ -64,15 +64,19 @@ def test_blocked_rows_batched_and_mixed():
     n, m, c = 64, 90, 64
     x = inputs.uniform(n * n, 41)
     ref = MemXCT(n, m, c, ray_block=-1, slices=4).build()
-    blk = MemXCT(n, m, c, ray_block=4, slices=4).build()
+    blk = MemXCT(n, m, c, ray_block=4, slices=4).build()        # slab stages (auto with blocks)
+    assert blk.get_option("stage_order") == 1
     X = torch.from_numpy(np.stack([x, 2 * x, x[::-1].copy()])).cuda()
     assert rel_l2(blk.forward_batch(X).cpu().numpy(), ref.forward_batch(X).cpu().numpy()) <= 1e-6
     mref = MemXCT(n, m, c, ray_block=-1, precision="mixed").build()
-    mblk = MemXCT(n, m, c, ray_block=4, precision="mixed").build()
+    mblk = MemXCT(n, m, c, ray_block=4, precision="mixed", stage_order=-1).build()
     xd = torch.from_numpy(x.astype(np.float64)).cuda()
     assert torch.equal(mblk.forward(xd), mref.forward(xd))   # one fp64 chain per row, same order
     can = MemXCT(n, m, c, ray_block=4, precision="mixed", canonical=True).build()
     assert can.get_option("ray_block") == -1                    # canonical keeps the Hilbert rows
+    assert can.get_option("stage_order") == -1                  # ... and the Hilbert stages
+    slab = MemXCT(n, m, c, ray_block=4, precision="mixed").build()
+    assert rel_l2(slab.forward(xd).cpu().numpy(), mref.forward(xd).cpu().numpy()) <= 1e-14
 
 
 def test_auto_rule():
@@ -90,7 +94,7 @@ def test_blocked_rows_virtual_ranks_and_shard(nranks):
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
     n, m, c = 256, 360, 256
     g0, ref = build_group(n, m, c, nranks, ray_block=-1)
-    g1, blk = build_group(n, m, c, nranks, ray_block=4)
+    g1, blk = build_group(n, m, c, nranks, ray_block=4, stage_order=-1)
     x = inputs.uniform(n * n, 51)
     xs = scatter(ref, x, 0, np.float32)
     y0 = run_ranks(nranks, lambda r: ref[r].forward(xs[r]))
@@ -98,7 +102,27 @@ def test_blocked_rows_virtual_ranks_and_shard(nranks):
     for a, b in zip(y0, y1):
         assert torch.equal(a, b)
     for r in range(nranks):
-        sp = MemXCT(n, m, c, rank=r, nranks=nranks, shard=True, vector_order="plan", ray_block=4).build()
+        sp = MemXCT(n, m, c, rank=r, nranks=nranks, shard=True, vector_order="plan", ray_block=4,
+                    stage_order=-1).build()
         assert torch.equal(sp.footprint_forward(xs[r]), ref[r].footprint_forward(xs[r]))
         sp.close()
     assert rel_l2(gather(blk, y1, 1, m * c), gather(ref, y0, 1, m * c)) == 0.0
+
+
+def test_slab_stages_virtual_ranks_peer_and_shard():
+    """Slab stages (STAGE_ORDER = 1) on the decomposed path: same sums up to fp32 rounding order,
+    in the collective and the shard builds alike (identical layouts, bit-identical A_p)."""
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
+    n, m, c, nranks = 256, 360, 256, 3
+    g0, ref = build_group(n, m, c, nranks, ray_block=-1)
+    g1, slab = build_group(n, m, c, nranks, ray_block=4, stage_order=1)
+    x = inputs.uniform(n * n, 61)
+    xs = scatter(ref, x, 0, np.float32)
+    y0 = gather(ref, run_ranks(nranks, lambda r: ref[r].forward(xs[r])), 1, m * c)
+    y1 = gather(slab, run_ranks(nranks, lambda r: slab[r].forward(xs[r])), 1, m * c)
+    assert rel_l2(y1, y0) <= 1e-6
+    for r in range(nranks):
+        sp = MemXCT(n, m, c, rank=r, nranks=nranks, shard=True, vector_order="plan", ray_block=4,
+                    stage_order=1).build()
+        assert torch.equal(sp.footprint_forward(xs[r]), slab[r].footprint_forward(xs[r]))
+        sp.close()
