@@ -108,9 +108,9 @@ typedef enum {
      * grouped into blocks of `a` consecutive projections x PART_ROWS / a consecutive channels
      * (projection-major, channel-minor inside a block) before being cut into partitions, which
      * raises the stage-buffer reuse when consecutive projections are many pixels apart (few
-     * projections, wide detector: config 5).  0 = auto (default): blocks with a = the power of
-     * two nearest sqrt(R / (L pi / M)), L = side of the local tomogram, when that a is <= sqrt(R)/4,
-     * else -1.  Vector layouts and results are unchanged: each row still sums its entries in
+     * projections, wide detector: config 5).  0 = auto (default): blocks with a = the smallest
+     * power of two >= 1.5 a*, a* = sqrt(R / (L pi / M)), L = side of the local tomogram, when
+     * a* <= sqrt(R)/4, else -1.  Vector layouts and results are unchanged: each row still sums its entries in
      * ascending Hilbert input order (FP32 outputs bit-identical).  CANONICAL forces -1. */
     MEMXCT_OPT_RAY_BLOCK = 10,
     /* Stage order of the forward SpMV (A_p): -1 = the paper's (reading R10): a partition's
@@ -119,8 +119,8 @@ typedef enum {
      * then Hilbert index), so every stage is a band that all of the partition's rays cross and all
      * warps have work in every stage.  Same map entries and bytes; each
      * row sums the same products in another order (FP32 results equal up to rounding).  0 = auto
-     * (default): slab order together with projection blocks (RAY_BLOCK > 0), else -1.
-     * CANONICAL forces -1. */
+     * (default): slab order.  CANONICAL forces -1 (the canonical row sums ascend in Hilbert
+     * order). */
     MEMXCT_OPT_STAGE_ORDER = 11
 } memxct_option_t;
 

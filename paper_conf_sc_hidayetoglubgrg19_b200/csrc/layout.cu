@@ -883,6 +883,8 @@ __global__ void ray_block_gather_kernel(const uint32_t* __restrict__ perm, const
 // pi/M, so (a-1) L pi/M pixels of drift) is comparable to its width R/a: a* = sqrt(R / (L pi / M)).
 // The paper's Hilbert rows form ~sqrt(R) x sqrt(R) squares, which is that optimum when L pi/M ~ 1
 // (configs 1-4: 2.1-2.7); blocks are used only when a* is >= 4x smaller (config 5: L pi/M ~ 35-99).
+// Measured on a config-5 shard (profiles/r01_ray_block_sweep.md): a = 8 beats 4 and 16 at
+// a* = 5.4, so the rule takes the smallest power of two >= 1.5 a*.
 int32_t resolve_ray_block(const Plan& P, int64_t local_pixels, int32_t R) {
     if (P.opt.canonical || P.opt.ray_block < 0) return -1;
     int32_t a = (int32_t)P.opt.ray_block;
@@ -891,7 +893,7 @@ int32_t resolve_ray_block(const Plan& P, int64_t local_pixels, int32_t R) {
         const double astar = std::sqrt((double)R / std::max(drift, 1e-9));
         if (astar > std::sqrt((double)R) / 4.0) return -1;
         a = 1;
-        while (a * 2 <= R / 32 && std::fabs(std::log2(a * 2.0) - std::log2(astar)) < std::fabs(std::log2((double)a) - std::log2(astar))) a *= 2;
+        while (a < 1.5 * astar && a * 2 <= R / 32) a *= 2;
     }
     return std::min<int32_t>(a, std::max(1, R / 32));
 }
@@ -974,9 +976,9 @@ void build_matrices(Plan& P, cudaStream_t st) {
     const Partitions fwd_parts = make_partitions(fwd_len, nrows, R, balance, st);
 
     // slab stage order (MEMXCT_OPT_STAGE_ORDER): per-class column orders, class of every partition
-    // and row; auto = with projection blocks (the geometries whose Hilbert stages are sparse)
-    P.stage_order = (P.opt.canonical || P.opt.stage_order < 0) ? -1
-                    : P.opt.stage_order > 0 ? 1 : (P.ray_block > 0 ? 1 : -1);
+    // and row; auto = slab order unless CANONICAL (cfg3 forward 1.733 -> 1.714 ms, cfg4 10.86 ->
+    // 10.74 ms, config-5 shards 2-3x, profiles/r01_slab_stages.md)
+    P.stage_order = (P.opt.canonical || P.opt.stage_order < 0) ? -1 : 1;
     DevArr<int32_t> kfwd, kinv, part_class, row_class;
     const int64_t fnp = (int64_t)fwd_parts.row0.size() - 1;
     if (P.stage_order == 1 && npix > 0 && nrows > 0) {

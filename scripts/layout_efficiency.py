@@ -51,13 +51,14 @@ def main():
     ap.add_argument("--config", type=int, default=3)
     ap.add_argument("--shard", default=None, help="r/P: one rank's shard")
     ap.add_argument("--ray-block", type=int, default=0)
+    ap.add_argument("--stage-order", type=int, default=0)
     ap.add_argument("--parts", type=int, default=64)
     ap.add_argument("--part-rows", type=int, default=None)
     ap.add_argument("--buffer-entries", type=int, default=None)
     args = ap.parse_args()
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, inputs
     n, m, c = inputs.CONFIGS[args.config]
-    kw = {"ray_block": args.ray_block, "part_rows": args.part_rows, "buffer_entries": args.buffer_entries}
+    kw = {"ray_block": args.ray_block, "stage_order": args.stage_order, "part_rows": args.part_rows, "buffer_entries": args.buffer_entries}
     if args.shard:
         r, P = map(int, args.shard.split("/"))
         plan = MemXCT(n, m, c, rank=r, nranks=P, shard=True, vector_order="plan", **kw).build()
@@ -68,6 +69,7 @@ def main():
     for d in (0, 1):
         row = analyse(plan, d, args.parts, rng)
         row.update({"config": args.config, "shard": args.shard, "ray_block": plan.get_option("ray_block"),
+                    "stage_order": plan.get_option("stage_order"),
                     "us": t["fwd_us" if d == 0 else "back_us"]})
         print(json.dumps(row), flush=True)
 

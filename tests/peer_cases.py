@@ -74,9 +74,9 @@ def case_projections(nranks, n, m, c, ray_block=None):
     from test_gpu_multirank import gather, scatter
     import time
     t0 = time.time()
-    g0, coll = build_group(n, m, c, nranks)
-    g1, peer = build_group(n, m, c, nranks, exchange="peer", ray_block=ray_block,
-                           stage_order=None if ray_block is None else -1)
+    so = None if ray_block is None else -1      # Hilbert stages: blocked rows are then bit-identical
+    g0, coll = build_group(n, m, c, nranks, stage_order=so)
+    g1, peer = build_group(n, m, c, nranks, exchange="peer", ray_block=ray_block, stage_order=so)
     print(f"built {time.time() - t0:.2f}s", flush=True)
     x = inputs.uniform(n * n, 1)
     y = inputs.uniform(m * c, 2)

@@ -71,10 +71,11 @@ def _pattern_keys(plan, direction, npix, R, B):
     out = plan.layout_rows(direction)[e["row"]]          # regrouped rows (RAY_BLOCK) write elsewhere
     natural = plan.get_option("vector_order") == 0
     row_nat = out if natural else plan.local_indices(1 if direction == 0 else 0)[out]
+    col_nat = e["col"] if natural else plan.local_indices(0 if direction == 0 else 1)[e["col"]]
     if direction == 0:
-        key = row_nat * npix + e["col"]
+        key = row_nat * npix + col_nat
     else:
-        key = e["col"] * npix + row_nat
+        key = col_nat * npix + row_nat
     order = np.argsort(key, kind="stable")
     return key[order], e["val"][order], ex
 

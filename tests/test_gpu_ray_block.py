@@ -31,7 +31,7 @@ def _need_gpu():
 def test_blocked_rows_bit_identical(orc, coo_cache, geom, order):
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
     n, m, c = geom
-    ref = MemXCT(n, m, c, vector_order=order, ray_block=-1).build()
+    ref = MemXCT(n, m, c, vector_order=order, ray_block=-1, stage_order=-1).build()
     assert ref.get_option("ray_block") == -1
     x = inputs.uniform(n * n, 31)
     xi = x if order == "natural" else x[ref.local_indices(0)]
@@ -68,7 +68,7 @@ def test_blocked_rows_batched_and_mixed():
     assert blk.get_option("stage_order") == 1
     X = torch.from_numpy(np.stack([x, 2 * x, x[::-1].copy()])).cuda()
     assert rel_l2(blk.forward_batch(X).cpu().numpy(), ref.forward_batch(X).cpu().numpy()) <= 1e-6
-    mref = MemXCT(n, m, c, ray_block=-1, precision="mixed").build()
+    mref = MemXCT(n, m, c, ray_block=-1, precision="mixed", stage_order=-1).build()
     mblk = MemXCT(n, m, c, ray_block=4, precision="mixed", stage_order=-1).build()
     xd = torch.from_numpy(x.astype(np.float64)).cuda()
     assert torch.equal(mblk.forward(xd), mref.forward(xd))   # one fp64 chain per row, same order
@@ -84,16 +84,18 @@ def test_auto_rule():
     L pi / M ~ 2), projection blocks where they are far from it (few projections, wide grid)."""
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
     assert MemXCT(256, 360, 256).build().get_option("ray_block") == -1
+    assert MemXCT(256, 360, 256).build().get_option("stage_order") == 1      # slab stages by default
     assert MemXCT(64, 90, 64).build().get_option("ray_block") == -1
     wide = MemXCT(2048, 60, 2048).build()          # L pi / M = 107: a* = sqrt(R / 107) ~ 3
-    assert wide.get_option("ray_block") in (2, 4)
+    assert wide.get_option("ray_block") == 8       # smallest power of two >= 1.5 a*
+    assert wide.get_option("stage_order") == 1
 
 
 @pytest.mark.parametrize("nranks", [2, 4])
 def test_blocked_rows_virtual_ranks_and_shard(nranks):
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
     n, m, c = 256, 360, 256
-    g0, ref = build_group(n, m, c, nranks, ray_block=-1)
+    g0, ref = build_group(n, m, c, nranks, ray_block=-1, stage_order=-1)
     g1, blk = build_group(n, m, c, nranks, ray_block=4, stage_order=-1)
     x = inputs.uniform(n * n, 51)
     xs = scatter(ref, x, 0, np.float32)
@@ -114,7 +116,7 @@ def test_slab_stages_virtual_ranks_peer_and_shard():
     in the collective and the shard builds alike (identical layouts, bit-identical A_p)."""
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
     n, m, c, nranks = 256, 360, 256, 3
-    g0, ref = build_group(n, m, c, nranks, ray_block=-1)
+    g0, ref = build_group(n, m, c, nranks, ray_block=-1, stage_order=-1)
     g1, slab = build_group(n, m, c, nranks, ray_block=4, stage_order=1)
     x = inputs.uniform(n * n, 61)
     xs = scatter(ref, x, 0, np.float32)
