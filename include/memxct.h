@@ -119,8 +119,8 @@ typedef enum {
      * then Hilbert index), so every stage is a band that all of the partition's rays cross and all
      * warps have work in every stage.  Same map entries and bytes; each
      * row sums the same products in another order (FP32 results equal up to rounding).  0 = auto
-     * (default): slab order.  CANONICAL forces -1 (the canonical row sums ascend in Hilbert
-     * order). */
+     * (default): slab order in FP32 mode; -1 in MIXED mode, whose fp64 row chains then ascend in
+     * Hilbert order like the oracle's canonical sums.  CANONICAL forces -1. */
     MEMXCT_OPT_STAGE_ORDER = 11
 } memxct_option_t;
 

@@ -976,9 +976,11 @@ void build_matrices(Plan& P, cudaStream_t st) {
     const Partitions fwd_parts = make_partitions(fwd_len, nrows, R, balance, st);
 
     // slab stage order (MEMXCT_OPT_STAGE_ORDER): per-class column orders, class of every partition
-    // and row; auto = slab order unless CANONICAL (cfg3 forward 1.733 -> 1.714 ms, cfg4 10.86 ->
-    // 10.74 ms, config-5 shards 2-3x, profiles/r01_slab_stages.md)
-    P.stage_order = (P.opt.canonical || P.opt.stage_order < 0) ? -1 : 1;
+    // and row; auto = slab order in FP32 mode (cfg3 forward 1.733 -> 1.714 ms, cfg4 10.86 ->
+    // 10.74 ms, config-5 shards 2-3x, profiles/r01_slab_stages.md); MIXED keeps the Hilbert
+    // stages, whose fp64 row chains ascend in Hilbert input order like the oracle's (R16)
+    P.stage_order = (P.opt.canonical || P.opt.stage_order < 0) ? -1
+                    : (P.opt.stage_order > 0 || P.opt.precision == 0) ? 1 : -1;
     DevArr<int32_t> kfwd, kinv, part_class, row_class;
     const int64_t fnp = (int64_t)fwd_parts.row0.size() - 1;
     if (P.stage_order == 1 && npix > 0 && nrows > 0) {

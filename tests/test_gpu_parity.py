@@ -246,12 +246,23 @@ def test_cg_fp32_recovers_phantom(orc, coo_cache, n, m, c):
 
 
 def test_cg_explicit_residual_variant(orc, coo_cache):
+    """CG_VARIANT = 1 (r = y - A x every iteration, reading R13).  MIXED (fp64 vectors): the
+    image matches the fp64 oracle's CGLS (the two variants agree in exact arithmetic, R13) and its
+    error to the phantom.  FP32: finite-precision CG amplifies rounding (R16: fp32 drift 0.5-3e-2
+    from iteration 8 on, phantom error 0.110 vs 0.104 in fp64), so the FP32 gate is the band that
+    noise spans (1.2x the oracle's phantom error) plus a monotone true residual."""
     n, m, c = 64, 90, 64
     rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
+    x_orc = orc.cgls(rows, cols, vals.astype(np.float32).astype(np.float64), y32.astype(np.float64),
+                     m * c, n * n, 30)[0]
+    mixed = make_plan(n, m, c, cg_variant=1, precision="mixed")
+    x_mix = mixed.cg(torch.from_numpy(y32.astype(np.float64)).cuda(), 30).cpu().numpy()
+    assert rel_l2(x_mix, x_orc) <= 1e-2
+    assert rel_l2(x_mix, xt) <= 1.01 * rel_l2(x_orc, xt)
     plan = make_plan(n, m, c, cg_variant=1)
-    x_gpu = plan.cg(torch.from_numpy(y32).cuda(), 30).cpu().numpy()
-    x_orc = orc.cgls(rows, cols, vals, y32.astype(np.float64), m * c, n * n, 30)[0]
-    assert rel_l2(x_gpu, xt) <= 1.1 * rel_l2(x_orc, xt)
+    x_gpu, res = plan.cg(torch.from_numpy(y32).cuda(), 30, residuals=True)
+    assert rel_l2(x_gpu.cpu().numpy(), xt) <= 1.2 * rel_l2(x_orc, xt)
+    assert np.all(np.diff(res) <= 1e-6 * res[0])
 
 
 def test_cg_edge_cases():

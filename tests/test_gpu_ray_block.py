@@ -75,7 +75,8 @@ def test_blocked_rows_batched_and_mixed():
     can = MemXCT(n, m, c, ray_block=4, precision="mixed", canonical=True).build()
     assert can.get_option("ray_block") == -1                    # canonical keeps the Hilbert rows
     assert can.get_option("stage_order") == -1                  # ... and the Hilbert stages
-    slab = MemXCT(n, m, c, ray_block=4, precision="mixed").build()
+    assert MemXCT(n, m, c, precision="mixed").build().get_option("stage_order") == -1
+    slab = MemXCT(n, m, c, ray_block=4, precision="mixed", stage_order=1).build()
     assert rel_l2(slab.forward(xd).cpu().numpy(), mref.forward(xd).cpu().numpy()) <= 1e-14
 
 
