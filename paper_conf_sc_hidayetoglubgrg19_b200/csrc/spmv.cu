@@ -221,7 +221,7 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();  // previous stage fully consumed
         if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B));
-        stage_gather<8>(sbuf, x, mp, cnt);
+        stage_gather<16>(sbuf, x, mp, cnt);
         __syncthreads();
         const int64_t blk = g * a.SPP + warp;
         const int64_t base = a.slot_off[blk];
