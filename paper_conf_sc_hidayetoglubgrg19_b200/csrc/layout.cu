@@ -851,15 +851,35 @@ __global__ void apply_class_order_kernel(const uint32_t* __restrict__ rows, int6
 
 // ---- forward row grouping (MEMXCT_OPT_RAY_BLOCK) ----------------------------------------------
 // Key of footprint row i: (block of `a` projections x `w` channels, then projection, channel).
+// Channels are counted from shift[m] = the channel of the local tomogram's centre at projection m
+// (0 for a whole tomogram centred on the rotation axis): rays of one block with equal offsets
+// k - shift[m] are tangent to one circle around that centre and cross each other inside the
+// local region, so the block's strips overlap there (a block with fixed channels crosses on the
+// line through the rotation axis, which a rank's region need not contain).
 __global__ void ray_block_key_kernel(const int32_t* __restrict__ hray, const int32_t* __restrict__ sino_nat_of_h,
-                                     int64_t nrows, int32_t c, int32_t a, int32_t w, uint64_t* __restrict__ key) {
+                                     int64_t nrows, int32_t c, int32_t a, int32_t w,
+                                     const int32_t* __restrict__ shift, uint64_t* __restrict__ key) {
     MX_LOOP(i, nrows) {
         const int32_t h = hray ? hray[i] : (int32_t)i;
         const int32_t nat = sino_nat_of_h[h];
         const int32_t m = nat / c, k = nat % c;
-        const uint64_t blk = (uint64_t)(m / a) * (uint64_t)((c + w - 1) / w) + (uint64_t)(k / w);
+        const int64_t ks = (int64_t)k - shift[m] + 2 * (int64_t)c;  // >= 0
+        const uint64_t blk = (uint64_t)(m / a) * (uint64_t)((4 * (int64_t)c + w - 1) / w) + (uint64_t)(ks / w);
         key[i] = (blk << 32) | (uint64_t)((int64_t)(m % a) * c + k);
     }
+}
+
+// centroid of the local pixels (integer sums: exact, so the layout is deterministic)
+__global__ void centroid_kernel(const int32_t* __restrict__ tomo_nat_of_h, int64_t t0, int64_t npix, int32_t n,
+                                unsigned long long* __restrict__ sums) {
+    unsigned long long si = 0, sj = 0;
+    MX_LOOP(q, npix) {
+        const int32_t nat = tomo_nat_of_h[t0 + q];
+        si += (unsigned long long)(nat / n);
+        sj += (unsigned long long)(nat % n);
+    }
+    atomicAdd(sums, si);
+    atomicAdd(sums + 1, sj);
 }
 
 // Blocked row j = footprint row perm[j]: its Hilbert ray, its length, and where its output goes
@@ -883,8 +903,9 @@ __global__ void ray_block_gather_kernel(const uint32_t* __restrict__ perm, const
 // pi/M, so (a-1) L pi/M pixels of drift) is comparable to its width R/a: a* = sqrt(R / (L pi / M)).
 // The paper's Hilbert rows form ~sqrt(R) x sqrt(R) squares, which is that optimum when L pi/M ~ 1
 // (configs 1-4: 2.1-2.7); blocks are used only when a* is >= 4x smaller (config 5: L pi/M ~ 35-99).
-// Measured on a config-5 shard (profiles/r01_ray_block_sweep.md): a = 8 beats 4 and 16 at
-// a* = 5.4, so the rule takes the smallest power of two >= 1.5 a*.
+// Measured (profiles/r01_ray_block_sweep.md): whole tomograms 2048^2 / 60 and 4096^2 / 180
+// (a* = 3.1, 3.8) are fastest at a = 8, i.e. the smallest power of two >= 1.5 a*; a config-5
+// shard (a* = 5.4, blocks sheared onto its region, ray_block_key_kernel) at a = 16, i.e. >= 3 a*.
 int32_t resolve_ray_block(const Plan& P, int64_t local_pixels, int32_t R) {
     if (P.opt.canonical || P.opt.ray_block < 0) return -1;
     int32_t a = (int32_t)P.opt.ray_block;
@@ -892,8 +913,9 @@ int32_t resolve_ray_block(const Plan& P, int64_t local_pixels, int32_t R) {
         const double drift = std::sqrt((double)std::max<int64_t>(local_pixels, 1)) * M_PI / (double)P.m;
         const double astar = std::sqrt((double)R / std::max(drift, 1e-9));
         if (astar > std::sqrt((double)R) / 4.0) return -1;
+        const double f = P.dist ? 3.0 : 1.5;
         a = 1;
-        while (a < 1.5 * astar && a * 2 <= R / 32) a *= 2;
+        while (a < f * astar && a * 2 <= R / 32) a *= 2;
     }
     return std::min<int32_t>(a, std::max(1, R / 32));
 }
@@ -949,7 +971,26 @@ void build_matrices(Plan& P, cudaStream_t st) {
         key_s.alloc(nrows);
         idx.alloc(nrows);
         perm.alloc(nrows);
-        ray_block_key_kernel<<<blocks_for(nrows), kThreads, 0, st>>>(hray, P.sino_nat_of_h.p(), nrows, P.c, a, w, key.p());
+        // channel of the local tomogram's centre per projection (all 0 for the whole tomogram)
+        std::vector<int32_t> h_shift(P.m, 0);
+        if (P.dist && npix > 0) {
+            DevArr<unsigned long long> sums;
+            sums.alloc(2);
+            MX_CUDA(cudaMemsetAsync(sums.p(), 0, 16, st));
+            centroid_kernel<<<blocks_for(npix), kThreads, 0, st>>>(P.tomo_nat_of_h.p(), P.t0, npix, P.n, sums.p());
+            MX_LAUNCHED();
+            const auto hs = to_host(sums.p(), 2, st);
+            const double cy = (double)hs[0] / npix + 0.5 - 0.5 * P.n, cx = (double)hs[1] / npix + 0.5 - 0.5 * P.n;
+            for (int32_t mm = 0; mm < P.m; ++mm) {
+                const double th = (double)mm * M_PI / (double)P.m;
+                h_shift[mm] = (int32_t)std::lround(cx * std::cos(th) + cy * std::sin(th));
+            }
+        }
+        DevArr<int32_t> shift;
+        shift.alloc(P.m);
+        MX_CUDA(cudaMemcpyAsync(shift.p(), h_shift.data(), 4 * P.m, cudaMemcpyHostToDevice, st));
+        ray_block_key_kernel<<<blocks_for(nrows), kThreads, 0, st>>>(hray, P.sino_nat_of_h.p(), nrows, P.c, a, w,
+                                                                     shift.p(), key.p());
         MX_LAUNCHED();
         iota_kernel<uint32_t><<<blocks_for(nrows), kThreads, 0, st>>>(idx.p(), nrows);
         MX_LAUNCHED();
