@@ -256,6 +256,16 @@ memxct_status_t memxct_exchange_time(memxct_plan_t plan, int32_t reps, double* u
 memxct_status_t memxct_spmv_time(memxct_plan_t plan, int32_t reps, double* us_forward,
                                  double* us_back, void* cuda_stream);
 
+/* Plan-independent probe of the roofline denominator: the achievable HBM read bandwidth of the
+ * current device, in GB/s (1e9 B/s).  Allocates `bytes` (rounded down to 16 B; >= 16) of
+ * device scratch, zeroes it, and streams it `reps` times (>= 1) with the SpMV's own 16 B
+ * read-only, L1-bypassing, L2-evict-first load, grid-stride interleaved over all SMs, for three
+ * launch shapes; writes the best average (CUDA events on `cuda_stream`).  Synchronous.  The
+ * driver's MEASURED_PEAKS.json figure is a read+write copy, which a read-only stream (the
+ * SpMV's matrix) may exceed; this gives the read-only ceiling beside it.  Errors: INVALID_ARG
+ * (sizes, NULL gbs), OUT_OF_MEMORY, CUDA. */
+memxct_status_t memxct_read_ceiling(int64_t bytes, int32_t reps, double* gbs, void* cuda_stream);
+
 /* Multi-slice variants (the paper reuses the memoized matrices for every
  * slice): `slices` independent slices with the same geometry, vectors slice-major
  * (x[s * local_size(0) + i], y[s * local_size(1) + r]), FP32 only.  The slices are processed in

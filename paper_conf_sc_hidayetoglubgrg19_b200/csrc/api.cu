@@ -475,6 +475,13 @@ memxct_status_t memxct_spmv_time(memxct_plan_t plan, int32_t reps, double* us_fo
     });
 }
 
+memxct_status_t memxct_read_ceiling(int64_t bytes, int32_t reps, double* gbs, void* cuda_stream) {
+    return guarded([&] {
+        need(gbs, "gbs");
+        *gbs = mx::read_ceiling_gbs(bytes, reps, stream_of(cuda_stream));
+    });
+}
+
 memxct_status_t memxct_forward_batch(memxct_plan_t plan, int32_t slices, const void* x_tomo, void* y_sino,
                                      void* cuda_stream) {
     return guarded([&] {

@@ -587,6 +587,32 @@ struct Builder {
     }
 };
 
+// Launch order of the partitions (MEMXCT_PART_ORDER: 0 = partition order (default), 1 = heaviest
+// first).  A CTA's time is ~ its streamed bytes (6 B per slot, 8 B per map entry, 4 B per row)
+// plus a gather round trip per stage; longest-processing-time order leaves the lightest
+// partitions for the last, partly filled wave.  Measured on one B200 (profiles/r01h_order_ab.jsonl):
+// cfg3 back -1.6 %, forward +1.1 %, cfg2 and cfg4 +0.5-1 % -- within a wave-tail effect of ~1 %,
+// so partition (Hilbert) order stays the default.
+void set_part_order(Layout& L, const std::vector<int64_t>& row0, const std::vector<int64_t>& part_slot,
+                    const std::vector<int64_t>& stage_base, cudaStream_t st) {
+    int mode = 0;
+    if (const char* e = std::getenv("MEMXCT_PART_ORDER")) mode = atoi(e);
+    const int64_t np = L.nparts;
+    if (mode == 0 || np < 2) return;
+    constexpr int64_t kStageCost = 16384;  // bytes of streaming time per stage barrier + gather
+    const auto moff = to_host(L.map_off.p(), np + 1, st);
+    std::vector<int64_t> work(np);
+    for (int64_t p = 0; p < np; ++p)
+        work[p] = 6 * (part_slot[p + 1] - part_slot[p]) + 8 * (moff[p + 1] - moff[p]) +
+                  4 * (row0[p + 1] - row0[p]) + kStageCost * (stage_base[p + 1] - stage_base[p]);
+    std::vector<int32_t> ord(np);
+    for (int64_t p = 0; p < np; ++p) ord[p] = (int32_t)p;
+    std::stable_sort(ord.begin(), ord.end(), [&](int32_t u, int32_t v) { return work[u] > work[v]; });
+    L.part_order.alloc(np);
+    MX_CUDA(cudaMemcpyAsync(L.part_order.p(), ord.data(), 4 * np, cudaMemcpyHostToDevice, st));
+    MX_CUDA(cudaStreamSynchronize(st));  // ord is a host temporary
+}
+
 // budget of chunk entries: what is free after the finished layouts of both directions
 // Default tuning of one direction with `rows` output rows on this rank (B200 sweeps:
 // profiles/r01_sweep.md, r01_sweep_cfg2.md, r01_sweep_spmm.md, r01_virtual_scaling.md).
@@ -732,6 +758,7 @@ void build_direction(Layout& L, int64_t nrows, int64_t ncols, const Partitions& 
         L.out_idx.alloc(std::max<int64_t>(nrows, 1));
         MX_CUDA(cudaMemcpyAsync(L.out_idx.p(), out_translate, 4 * nrows, cudaMemcpyDeviceToDevice, st));
     }
+    set_part_order(L, parts.row0, b.h_part_slot, b.h_stage_base, st);
     MX_CUDA(cudaStreamSynchronize(st));
 }
 

@@ -47,10 +47,11 @@ struct Layout {
     DevArr<float> val;           // nslots
     DevArr<uint16_t> lane_chunks;  // nstages * SPP * 32
     DevArr<int32_t> out_idx;     // nrows, optional: output position of each row (natural order)
+    DevArr<int32_t> part_order;  // nparts, optional: partition run by CTA b (heaviest first)
     int64_t device_bytes() const {
         return (int64_t)(prow0.buf.bytes() + stage_base.buf.bytes() + map_off.buf.bytes() + map.buf.bytes() +
                          slot_off.buf.bytes() + ind.buf.bytes() + val.buf.bytes() +
-                         lane_chunks.buf.bytes() + out_idx.buf.bytes());
+                         lane_chunks.buf.bytes() + out_idx.buf.bytes() + part_order.buf.bytes());
     }
 };
 
@@ -222,6 +223,7 @@ void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
 void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);
 void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 void time_spmv(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
+double read_ceiling_gbs(int64_t bytes, int reps, cudaStream_t st);  // memxct_read_ceiling
 void reduce_partials(Plan& P, const float* recv, float* y, cudaStream_t st);
 void preload_exchange_kernels();
 // peer.cu: fused SpMV + exchange over peer memory (EXCHANGE = 1)

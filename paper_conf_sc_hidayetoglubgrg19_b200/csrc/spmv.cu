@@ -77,6 +77,7 @@ struct SpmvArgs {
     const uint16_t* lane_chunks;
     const int32_t* out_idx;
     const int64_t* prow0;  // first row of each partition (nparts + 1)
+    const int32_t* order;  // nullable: partition of CTA b (launch order, heaviest first)
     int64_t nrows;
     int64_t nparts;
     int32_t R, SPP, B;
@@ -84,6 +85,15 @@ struct SpmvArgs {
     double* dot_out;
     unsigned int* ticket;
 };
+
+// Partition processed by this CTA.  Partitions differ in work (forward: rays near the detector
+// edge are short chords), so they are launched heaviest first (longest-processing-time order):
+// the last wave then holds the lightest partitions and the tail in which few SMs stream is short.
+// Per-partition results (rows, dot partials) are indexed by partition, so the order changes no
+// result.
+__device__ __forceinline__ int64_t part_of_cta(const SpmvArgs& a) {
+    return a.order ? (int64_t)__ldg(a.order + blockIdx.x) : (int64_t)blockIdx.x;
+}
 
 // deterministic last-CTA reduction of the per-CTA partials, in partition order
 template <int kThreads>
@@ -98,7 +108,7 @@ __device__ void finish_dot_tree(const SpmvArgs& a, double mine) {
     if (threadIdx.x == 0) {
         double s = 0.0;
         for (int w = 0; w < nw; ++w) s += red[w];
-        a.dot_part[blockIdx.x] = s;
+        a.dot_part[part_of_cta(a)] = s;
         __threadfence();
         const unsigned t = atomicAdd(a.ticket, 1u);
         am_last = (t == (unsigned)(a.nparts - 1));
@@ -127,7 +137,7 @@ __device__ void finish_dot_canonical(const SpmvArgs& a, const double* rows_val, 
     if (threadIdx.x == 0) {
         double part = 0.0;
         for (int i = 0; i < nvalid; ++i) part = __fma_rn(rows_val[i], rows_val[i], part);
-        a.dot_part[blockIdx.x] = part;
+        a.dot_part[part_of_cta(a)] = part;
         __threadfence();
         const unsigned t = atomicAdd(a.ticket, 1u);
         am_last = (t == (unsigned)(a.nparts - 1));
@@ -208,7 +218,7 @@ template <bool kNatOut, int kEpi>
 __global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, PeerArgs pa) {
     extern __shared__ __align__(16) float sbuf[];
-    const int64_t p = blockIdx.x;
+    const int64_t p = part_of_cta(a);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
     const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
@@ -272,7 +282,7 @@ template <bool kNatOut, int kDotMode>  // kDotMode: 0 none, 1 tree, 2 canonical 
 __global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y) {
     extern __shared__ __align__(16) double dbuf[];
-    const int64_t p = blockIdx.x;
+    const int64_t p = part_of_cta(a);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
     const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
@@ -352,6 +362,7 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.lane_chunks = L.lane_chunks.p();
     a.out_idx = L.out_idx.p();
     a.prow0 = L.prow0.p();
+    a.order = L.part_order.p();
     a.nrows = L.nrows;
     a.nparts = L.nparts;
     a.R = L.R;
@@ -408,7 +419,7 @@ template <int K, bool kNatOut>
 __global__ void __launch_bounds__(kMaxThreads, 1)
 spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __restrict__ y, int64_t ldy) {
     extern __shared__ __align__(16) float kbuf[];  // [B][K]
-    const int64_t p = blockIdx.x;
+    const int64_t p = part_of_cta(a);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
     const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
@@ -551,6 +562,30 @@ void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, dou
     MX_LAUNCHED();
 }
 
+// ---- read-bandwidth ceiling (memxct_read_ceiling) -------------------------------------------
+// The SpMV's roofline denominator in MEASURED_PEAKS.json is a read+write copy; the matrix stream
+// is read-only.  This probe streams a buffer with the SpMV's own load (16 B ld.global.nc,
+// L1::no_allocate, L2 evict_first), grid-stride interleaved so that all SMs read neighbouring
+// addresses, U loads in flight per thread: the achievable read bandwidth of this GPU.
+template <int U>
+__global__ void __launch_bounds__(1024) read_probe_kernel(const uint4* __restrict__ a, int64_t n16,
+                                                          unsigned* __restrict__ sink) {
+    const uint64_t pol = evict_first_policy();
+    const int64_t T = (int64_t)gridDim.x * blockDim.x;
+    unsigned acc = 0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += (int64_t)U * T) {
+        uint4 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t j = i + (int64_t)u * T;
+            v[u] = j < n16 ? ld_stream_u4(a + j, pol) : make_uint4(0u, 0u, 0u, 0u);
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) acc ^= v[u].x ^ v[u].y ^ v[u].z ^ v[u].w;
+    }
+    if (acc == 0x9e3779b9u) sink[0] = acc;  // keeps the loads live; never true for a zero buffer
+}
+
 // Raise the dynamic shared-memory limit of every SpMV instantiation once (outside any stream
 // capture): stage buffers go up to 227 KB per CTA.
 void spmv_init() {
@@ -575,6 +610,43 @@ void spmv_init() {
     set_smem(spmm_f32_kernel<8, true>);
     set_smem(spmm_f32_kernel<8, false>);
     done = true;
+}
+
+double read_ceiling_gbs(int64_t bytes, int reps, cudaStream_t st) {
+    const int64_t n16 = bytes / 16;
+    if (n16 < 1 || reps < 1) fail(MEMXCT_ERR_INVALID_ARG, "read ceiling: bytes >= 16 and reps >= 1");
+    int dev = 0, sms = 148;
+    MX_CUDA(cudaGetDevice(&dev));
+    MX_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    DevArr<uint4> buf;
+    DevArr<unsigned> sink;
+    buf.alloc(n16);
+    sink.alloc(1);
+    MX_CUDA(cudaMemsetAsync(buf.p(), 0, 16 * (size_t)n16, st));
+    cudaEvent_t e0, e1;
+    MX_CUDA(cudaEventCreate(&e0));
+    MX_CUDA(cudaEventCreate(&e1));
+    double best = 0.0;
+    // shapes: one 1024-thread CTA per SM with 16 or 8 loads in flight per thread, 8 x 256 per SM
+    const int grids[3] = {sms, sms, 8 * sms}, threads[3] = {1024, 1024, 256}, us[3] = {16, 8, 16};
+    for (int k = 0; k < 3; ++k) {
+        auto launch = [&] {
+            if (us[k] == 16) read_probe_kernel<16><<<grids[k], threads[k], 0, st>>>(buf.p(), n16, sink.p());
+            else read_probe_kernel<8><<<grids[k], threads[k], 0, st>>>(buf.p(), n16, sink.p());
+            MX_LAUNCHED();
+        };
+        launch();  // warm-up
+        MX_CUDA(cudaEventRecord(e0, st));
+        for (int r = 0; r < reps; ++r) launch();
+        MX_CUDA(cudaEventRecord(e1, st));
+        MX_CUDA(cudaEventSynchronize(e1));
+        float ms = 0.f;
+        MX_CUDA(cudaEventElapsedTime(&ms, e0, e1));
+        best = std::max(best, 16.0 * (double)n16 * reps / (1e6 * ms));
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    return best;
 }
 
 }  // namespace mx

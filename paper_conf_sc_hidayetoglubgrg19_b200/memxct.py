@@ -35,7 +35,16 @@ SYMBOLS = [
     "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
     "memxct_sirt", "memxct_spmv_time", "memxct_plan_set_shard", "memxct_exchange_counts",
     "memxct_footprint_rays", "memxct_footprint_forward", "memxct_footprint_back", "memxct_layout_rows",
+    "memxct_read_ceiling",
 ]
+
+
+def read_ceiling(nbytes: int = 11_600_000_000, reps: int = 10, stream=None) -> float:
+    """memxct_read_ceiling: achievable HBM read bandwidth of the current device, GB/s."""
+    g = ctypes.c_double()
+    _check(lib().memxct_read_ceiling(int(nbytes), int(reps), ctypes.byref(g), _stream(stream)),
+           "memxct_read_ceiling")
+    return g.value
 
 
 class MemXCTError(RuntimeError):
@@ -96,6 +105,7 @@ def lib():
             "memxct_footprint_forward": [vp, vp, vp, vp],
             "memxct_footprint_back": [vp, vp, vp, vp],
             "memxct_layout_rows": [vp, i32, vp],
+            "memxct_read_ceiling": [i64, i32, ctypes.POINTER(ctypes.c_double), vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)

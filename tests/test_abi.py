@@ -95,3 +95,10 @@ def test_no_cpu_fallback_without_gpu(L):
     assert L.memxct_build(h, None) == 4                        # MEMXCT_ERR_CUDA: no device
     assert b"no CPU fallback" in L.memxct_last_error() or b"CUDA" in L.memxct_last_error()
     L.memxct_plan_destroy(h)
+
+
+def test_read_ceiling_validates_arguments(L):
+    g = ctypes.c_double()
+    assert L.memxct_read_ceiling(8, 1, ctypes.byref(g), None) == 1     # < 16 bytes
+    assert L.memxct_read_ceiling(1 << 20, 0, ctypes.byref(g), None) == 1  # reps < 1
+    assert L.memxct_read_ceiling(1 << 20, 1, None, None) == 1          # NULL output

@@ -379,3 +379,29 @@ def test_batched_cg_bit_identical_to_single(orc, coo_cache):
         assert torch.equal(X[s], xs1), s
         assert np.array_equal(R[s], r1)
     assert torch.all(X[3] == 0)   # the zero sinogram stops at once
+
+
+@pytest.mark.parametrize("n,m,c,prec", [(256, 360, 256, "fp32"), (64, 90, 64, "mixed"), (33, 17, 33, "fp32")])
+def test_partition_launch_order_changes_no_result(monkeypatch, n, m, c, prec):
+    """MEMXCT_PART_ORDER: partitions launched heaviest first or in partition order (default).
+    Rows and the fused CG dot partials are indexed by partition, so projections and CG iterates
+    are bit-identical either way (the dot's last-CTA sum runs in partition order)."""
+    dt = np.float32 if prec == "fp32" else np.float64
+    x = torch.from_numpy(inputs.uniform(n * n, 11).astype(dt)).cuda()
+    y = torch.from_numpy(inputs.uniform(m * c, 12).astype(dt)).cuda()
+    out = []
+    for order in ("0", "1"):
+        monkeypatch.setenv("MEMXCT_PART_ORDER", order)
+        plan = make_plan(n, m, c, precision=prec)
+        xc, res = plan.cg(y, 12, residuals=True)
+        out.append((plan.forward(x).cpu().numpy(), plan.back(y).cpu().numpy(), xc.cpu().numpy(), res))
+    for a, b in zip(*out):
+        assert np.array_equal(a, b)
+
+
+def test_read_ceiling_probe():
+    """memxct_read_ceiling: a read-only stream of a buffer far larger than L2 runs at an HBM rate
+    (B200 nominal 8 TB/s; well above 1 TB/s, below 10 TB/s)."""
+    from paper_conf_sc_hidayetoglubgrg19_b200.memxct import read_ceiling
+    g = read_ceiling(2_000_000_000, 3)
+    assert 1000.0 < g < 10000.0, g
