@@ -47,6 +47,19 @@ def main():
     out["iter_ms"] = (out[f"cg{ks[1]}_ms"] - out[f"cg{ks[0]}_ms"]) / (ks[1] - ks[0])
     t = plan.spmv_time(20)
     out["spmv_pair_ms"] = (t["fwd_us"] + t["back_us"]) / 1e3
+    # the same two kernels alternating on real vectors (forward into q, back into s), as in CG
+    q, s_ = torch.empty_like(y), torch.empty_like(x)
+    for _ in range(3):
+        plan.forward(x, q)
+        plan.back(y, s_)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(20):
+        plan.forward(x, q)
+        plan.back(y, s_)
+    e1.record()
+    torch.cuda.synchronize()
+    out["alternating_pair_ms"] = e0.elapsed_time(e1) / 20
     out["overhead_us"] = 1e3 * (out["iter_ms"] - out["spmv_pair_ms"])
     out["overhead_frac"] = out["overhead_us"] / 1e3 / out["iter_ms"]
     print(json.dumps(out), flush=True)
