@@ -109,8 +109,8 @@ typedef enum {
      * (projection-major, channel-minor inside a block) before being cut into partitions, which
      * raises the stage-buffer reuse when consecutive projections are many pixels apart (few
      * projections, wide detector: config 5).  0 = auto (default): blocks with a = the smallest
-     * power of two >= f a*, a* = sqrt(R / (L pi / M)), L = side of the local tomogram, f = 1.5
-     * for a whole tomogram and 3 for a rank's region (measured), when a* <= sqrt(R)/4, else -1.
+     * power of two >= 2 a*, a* = sqrt(R / (L pi / M)), L = side of the local tomogram (measured
+     * optimum for whole tomograms and for rank regions), when a* <= sqrt(R)/4, else -1.
      * A rank's blocks count channels from the channel of its region's centre at each projection,
      * so a block's rays cross inside the region.  Vector layouts and results are unchanged: each row still sums its entries in
      * ascending Hilbert input order (FP32 outputs bit-identical).  CANONICAL forces -1. */

@@ -184,6 +184,17 @@ unsigned vec_blocks(int64_t n) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(kVecBlocks, ceil_div(n, (int64_t)kVT * kU)));
 }
 
+// CG dots at P > 1: one fp64 per slice summed over the ranks -- over peer memory with the fused
+// exchange (peer_allreduce, rank order), else by the transport's allreduce (NCCL / virtual ranks).
+void allreduce_slices(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) {
+    if (!P.dist) return;
+    if (P.ex.peer) {
+        peer_allreduce(P, v, K, stride, st);
+        return;
+    }
+    for (int s = 0; s < K; ++s) P.comm->allreduce_sum(v + s * stride, 1, DType::F64, st);
+}
+
 // Projection of K slices followed by the per-slice dot of the output.  At K = 1, P = 1 the dot
 // is fused into the SpMV epilogue: canonical mode as per-partition fma chains (reading R16),
 // otherwise as a per-CTA tree + last-CTA sum in partition order (deterministic).  (With the
@@ -218,14 +229,8 @@ void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, 
         dot_kernel<T><<<dim3(vec_blocks(n), K), kVT, 0, st>>>(out, n, dot_out, dot_stride, P.part_vec.p(),
                                                               P.tickets.p() + 64);
         MX_LAUNCHED();
-        if (P.dist)
-            for (int s = 0; s < K; ++s) P.comm->allreduce_sum(dot_out + s * dot_stride, 1, DType::F64, st);
+        if (P.dist) allreduce_slices(P, dot_out, K, dot_stride, st);
     }
-}
-
-void allreduce_slices(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) {
-    if (P.dist)
-        for (int s = 0; s < K; ++s) P.comm->allreduce_sum(v + s * stride, 1, DType::F64, st);
 }
 
 template <class T>
@@ -242,7 +247,6 @@ void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, int K, cudaStream_t st
     const unsigned gb = vec_blocks(std::max(nx, nr));
     cg_init_kernel<T><<<dim3(gb, K), kVT, 0, st>>>(y, r, nr, x, nx, sc, vpart, tick);
     MX_LAUNCHED();
-    allreduce_slices(P, sc.res2, K, sc.n1, st);
     op_dir<T>(P, false, K, r, s, sc.gam, sc.n1, st);                    // s = A^T r, gamma_0
     copy_kernel<T><<<dim3(vec_blocks(nx), K), kVT, 0, st>>>(s, p, nx);  // p = s
     MX_LAUNCHED();
@@ -259,11 +263,15 @@ void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, int K, cudaStream_t st
             cg_update_xr_kernel<T, true><<<dim3(gb, K), kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k, vpart, tick);
             MX_LAUNCHED();
         }
-        allreduce_slices(P, sc.res2 + k, K, sc.n1, st);
         op_dir<T>(P, false, K, r, s, sc.gam + k, sc.n1, st);            // s = A^T r, gamma_k
         cg_update_p_kernel<T><<<dim3(vec_blocks(nx), K), kVT, 0, st>>>(p, s, nx, sc, k);
         MX_LAUNCHED();
     }
+    // ||r_k||^2 only reports (no step depends on it): the local partials of every iteration are
+    // summed over the ranks once, after the loop -- one collective per slice per solve instead of
+    // one per iteration.  Iterations that did not run are ignored by cg_fetch_norms.
+    if (P.dist)
+        for (int sl = 0; sl < K; ++sl) P.comm->allreduce_sum(sc.res2 + (int64_t)sl * sc.n1, iters + 1, DType::F64, st);
 }
 
 void cg_enqueue_any(Plan& P, const void* y, void* x, int32_t iters, int K, cudaStream_t st) {

@@ -931,8 +931,10 @@ __global__ void ray_block_gather_kernel(const uint32_t* __restrict__ perm, const
 // The paper's Hilbert rows form ~sqrt(R) x sqrt(R) squares, which is that optimum when L pi/M ~ 1
 // (configs 1-4: 2.1-2.7); blocks are used only when a* is >= 4x smaller (config 5: L pi/M ~ 35-99).
 // Measured (profiles/r01_ray_block_sweep.md): whole tomograms 2048^2 / 60 and 4096^2 / 180
-// (a* = 3.1, 3.8) are fastest at a = 8, i.e. the smallest power of two >= 1.5 a*; a config-5
-// shard (a* = 5.4, blocks sheared onto its region, ray_block_key_kernel) at a = 16, i.e. >= 3 a*.
+// (a* = 3.1, 3.8) are fastest at a = 8, config-5 shards (a* = 5.35, blocks sheared onto the
+// rank's region, ray_block_key_kernel) at a = 16 (8.0 ms vs 8.6 at a = 8 and 8.8 at a = 32):
+// the smallest power of two >= 2 a* in all three.  (The earlier factor 3 for decomposed plans
+// gave a = 32 at a* = 5.35: profiles/r01h_shard_cfg5_p8.jsonl.)
 int32_t resolve_ray_block(const Plan& P, int64_t local_pixels, int32_t R) {
     if (P.opt.canonical || P.opt.ray_block < 0) return -1;
     int32_t a = (int32_t)P.opt.ray_block;
@@ -940,9 +942,8 @@ int32_t resolve_ray_block(const Plan& P, int64_t local_pixels, int32_t R) {
         const double drift = std::sqrt((double)std::max<int64_t>(local_pixels, 1)) * M_PI / (double)P.m;
         const double astar = std::sqrt((double)R / std::max(drift, 1e-9));
         if (astar > std::sqrt((double)R) / 4.0) return -1;
-        const double f = P.dist ? 3.0 : 1.5;
         a = 1;
-        while (a < f * astar && a * 2 <= R / 32) a *= 2;
+        while (a < 2.0 * astar && a * 2 <= R / 32) a *= 2;
     }
     return std::min<int32_t>(a, std::max(1, R / 32));
 }

@@ -92,6 +92,49 @@ __global__ void pack_remote_kernel(const float* __restrict__ y, const int32_t* _
     *pa.ticket = 0u;
 }
 
+// CG dot products over peer memory (EXCHANGE = 1): the B200-native form of the two fp64
+// allreduces per CG iteration, which on NVSwitch cost a collective launch each
+// (~10-20 us) against a per-rank SpMV pair of ~0.5 ms at P = 8 (config 3).  One thread: bump my
+// epoch e; store my K values into every rank's slot [e & 1][me] (peer stores over NVLink), fence,
+// publish e to every rank's arrival flag [me]; wait until every rank's flag in my array reaches e;
+// sum the P slots in rank order (rank 0's value first: the same fp64 additions on every rank, and
+// the same as the virtual-rank transport's sum).  Two parity slots suffice: a rank can write epoch
+// e + 2 into slot e & 1 only after it has seen every rank's epoch e + 1 arrival, which each rank
+// publishes after it has read its epoch-e slots.
+struct DotArgs {
+    double* dst[kMaxPeers];              // rank q's value array (peer pointer)
+    unsigned long long* flag[kMaxPeers];  // rank q's flag array (peer pointer)
+    const double* mine;                  // my value array
+    unsigned long long* my_flags;        // my flag array: [P arrivals | epoch]
+};
+__global__ void peer_allreduce_kernel(DotArgs da, int P, int me, double* v, int K, int64_t stride, int notrap) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    const unsigned long long e = da.my_flags[P] + 1;
+    da.my_flags[P] = e;
+    const int par = (int)(e & 1ull);
+    for (int q = 0; q < P; ++q)
+        for (int s = 0; s < K; ++s) da.dst[q][((int64_t)par * P + me) * kMaxDotSlices + s] = v[s * stride];
+    __threadfence_system();
+    for (int q = 0; q < P; ++q) st_release(da.flag[q] + me, e);
+    const long long t0 = clock64();
+    for (int q = 0; q < P; ++q) {
+        while (ld_acquire_sys(da.my_flags + q) < e) {
+            __nanosleep(32);
+            if (clock64() - t0 > 40000000000LL) {
+                printf("memxct peer dot timeout: rank %d waits for rank %d epoch %llu\n", me, q, e);
+                if (notrap) return;
+                __trap();
+            }
+        }
+    }
+    for (int s = 0; s < K; ++s) {
+        const volatile double* m = da.mine + (int64_t)par * P * kMaxDotSlices + s;
+        double acc = m[0];
+        for (int q = 1; q < P; ++q) acc += m[(int64_t)q * kMaxDotSlices];
+        v[s * stride] = acc;
+    }
+}
+
 unsigned nblocks(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 4 * 148)); }
 
 SignalArgs signal_args(const Plan& P) {
@@ -112,6 +155,7 @@ void peer_setup(Plan& P, cudaStream_t st) {
         MX_CUDA(cudaFuncGetAttributes(&fa, wait_kernel));
         MX_CUDA(cudaFuncGetAttributes(&fa, signal_kernel));
         MX_CUDA(cudaFuncGetAttributes(&fa, pack_remote_kernel));
+        MX_CUDA(cudaFuncGetAttributes(&fa, peer_allreduce_kernel));
         preload_exchange_kernels();
     }
     if (np > kMaxPeers) fail(MEMXCT_ERR_UNSUPPORTED, "fused peer exchange supports up to 16 ranks");
@@ -133,6 +177,12 @@ void peer_setup(Plan& P, cudaStream_t st) {
     X.peer_recv = C.map_peers(X.recv_buf.get(), st);
     X.peer_yfp = C.map_peers(X.y_fp.get(), st);
     X.peer_flags = C.map_peers(X.flags.p(), st);
+    X.dotx.alloc(2 * (int64_t)np * kMaxDotSlices);
+    X.dflags.alloc(np + 1);
+    MX_CUDA(cudaMemsetAsync(X.dflags.p(), 0, 8 * (np + 1), st));
+    MX_CUDA(cudaStreamSynchronize(st));
+    X.peer_dotx = C.map_peers(X.dotx.p(), st);
+    X.peer_dflags = C.map_peers(X.dflags.p(), st);
     X.peer = true;
 }
 
@@ -198,6 +248,21 @@ void peer_back(Plan& P, const float* y, float* x, cudaStream_t st) {
     spmv_f32(P.back, X.y_fp.as<float>(), x, nullptr, nullptr, nullptr, st);
     // 5. credits: my footprint buffer may be overwritten again
     signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 3 * np + P.rank, fl, 4 * np + 1);
+    MX_LAUNCHED();
+}
+
+void peer_allreduce(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) {
+    if (K < 1) return;
+    if (K > kMaxDotSlices) fail(MEMXCT_ERR_INVALID_ARG, "peer dot: more than 64 slices");
+    Exchange& X = P.ex;
+    DotArgs da{};
+    for (int q = 0; q < P.nranks; ++q) {
+        da.dst[q] = static_cast<double*>(X.peer_dotx[q]);
+        da.flag[q] = static_cast<unsigned long long*>(X.peer_dflags[q]);
+    }
+    da.mine = X.dotx.p();
+    da.my_flags = X.dflags.p();
+    peer_allreduce_kernel<<<1, 32, 0, st>>>(da, P.nranks, P.rank, v, K, stride, notrap_env());
     MX_LAUNCHED();
 }
 

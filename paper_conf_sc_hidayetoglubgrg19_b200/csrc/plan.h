@@ -80,6 +80,7 @@ struct Geometry {
 
 // Arguments of the fused SpMV + exchange epilogue and of the peer-memory pack (P > 1)
 constexpr int kMaxPeers = 16;
+constexpr int kMaxDotSlices = 64;  // slices per CG call (cg_run's K bound)
 struct PeerArgs {
     int32_t P = 0, me = 0;
     int64_t bound[kMaxPeers + 1] = {};           // row ranges per destination rank
@@ -112,6 +113,11 @@ struct Exchange {
     std::vector<void*> peer_recv, peer_yfp, peer_flags;
     std::vector<int64_t> fwd_off;      // owner h: my partial of footprint row i goes to recv_h[fwd_off[h] + i]
     std::vector<int64_t> back_off;     // peer g: my value j (recv order) goes to yfp_g[back_off[g] + j]
+    // CG dots over peer memory (peer_allreduce): values [2 parities][P][kMaxDotSlices] and flags
+    // [P arrivals | my epoch], mapped into every rank
+    DevArr<double> dotx;
+    DevArr<unsigned long long> dflags;
+    std::vector<void*> peer_dotx, peer_dflags;
     int64_t device_bytes() const {
         return (int64_t)(recv_idx.buf.bytes() + red_ptr.buf.bytes() + red_pos.buf.bytes() + y_fp.bytes() +
                          recv_buf.bytes() + y_fp_b.bytes() + recv_b.bytes());
@@ -230,6 +236,8 @@ void preload_exchange_kernels();
 void peer_setup(Plan& P, cudaStream_t st);
 void peer_forward(Plan& P, const float* x, float* y, cudaStream_t st);
 void peer_back(Plan& P, const float* y, float* x, cudaStream_t st);
+// v[s * stride] (s < K) summed over ranks in rank order, in place, over peer memory
+void peer_allreduce(Plan& P, double* v, int K, int64_t stride, cudaStream_t st);
 // K slices, slice-major [K][local_len] fp32 vectors
 void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t st);
 void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st);

@@ -405,3 +405,26 @@ def test_read_ceiling_probe():
     from paper_conf_sc_hidayetoglubgrg19_b200.memxct import read_ceiling
     g = read_ceiling(2_000_000_000, 3)
     assert 1000.0 < g < 10000.0, g
+
+
+@pytest.mark.slow
+def test_cfg3_cg_properties_full_size():
+    """The bench's workload and launch configuration (cfg3, 30 FP32 CGLS iterations through
+    memxct_cg): properties that hold at any size.  On the consistent system
+    y = A x_true the CGLS residual ||r_k|| and the error ||x_k - x_true|| are non-increasing
+    (up to fp32 noise), the recursive residual tracks the true ||y - A x_30||, and 30 iterations
+    reduce the error to the phantom well below its start (configs 1-2: 0.10-0.12, C.4)."""
+    n, m, c = inputs.CONFIGS[3]
+    plan = make_plan(n, m, c)
+    xt = torch.from_numpy(inputs.shepp_logan(n).astype(np.float32)).cuda()
+    y = plan.forward(xt)
+    errs = []
+    for k in (5, 10, 20, 30):
+        xk = plan.cg(y, k)
+        errs.append(float(torch.linalg.vector_norm((xk - xt).double()) / torch.linalg.vector_norm(xt.double())))
+    x30, res = plan.cg(y, 30, residuals=True)
+    assert np.all(np.diff(res) <= 1e-6 * res[0])
+    assert all(b <= a * (1 + 1e-4) for a, b in zip(errs, errs[1:])), errs
+    assert errs[-1] < 0.12, errs
+    true_res = float(torch.linalg.vector_norm((y - plan.forward(x30)).double()))
+    assert abs(true_res - res[-1]) <= 1e-3 * res[0], (true_res, res[-1], res[0])

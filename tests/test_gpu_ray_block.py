@@ -88,7 +88,7 @@ def test_auto_rule():
     assert MemXCT(256, 360, 256).build().get_option("stage_order") == 1      # slab stages by default
     assert MemXCT(64, 90, 64).build().get_option("ray_block") == -1
     wide = MemXCT(2048, 60, 2048).build()          # L pi / M = 107: a* = sqrt(R / 107) ~ 3
-    assert wide.get_option("ray_block") == 8       # smallest power of two >= 1.5 a*
+    assert wide.get_option("ray_block") == 8       # smallest power of two >= 2 a*
     assert wide.get_option("stage_order") == 1
 
 

@@ -139,6 +139,7 @@ def test_cfg5_shard_sampled_rows(orc):
     hr_s = orc.hilbert_rank(m, c, sp.get_option("tile_sino") or 32)
     assert np.array_equal(sp.local_indices(1), local_hilbert_range(hr_s, sb[r], sb[r + 1]))
     del hr_s
+    assert sp.get_option("ray_block") == 16        # 2 a* = 10.7 (a* = sqrt(1024 / (4100 pi / 360)))
     info = sp.layout_info(0)
     assert 0.9 < info["nnz"] * nranks / (1.1953 * m * c * n) < 1.1      # about 1/P of nnz(A)
     fp = sp.footprint_rays()
