@@ -21,7 +21,7 @@ __device__ __forceinline__ uint4 ld_stream(const void* p, uint64_t pol) {
 
 // contiguous chunk per CTA (like a partition), U independent 16 B loads per thread per step
 template <int U>
-__global__ void read_kernel(const uint4* __restrict__ a, int64_t n16, int64_t per_cta, unsigned* out) {
+__global__ void __launch_bounds__(1024) read_kernel(const uint4* __restrict__ a, int64_t n16, int64_t per_cta, unsigned* out) {
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
     const int64_t b0 = (int64_t)blockIdx.x * per_cta;
@@ -42,7 +42,7 @@ __global__ void read_kernel(const uint4* __restrict__ a, int64_t n16, int64_t pe
 
 // grid-stride interleaved: at any moment all CTAs read neighbouring addresses
 template <int U>
-__global__ void read_interleaved(const uint4* __restrict__ a, int64_t n16, unsigned* out) {
+__global__ void __launch_bounds__(1024) read_interleaved(const uint4* __restrict__ a, int64_t n16, unsigned* out) {
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
     const int64_t T = (int64_t)gridDim.x * blockDim.x;
@@ -58,6 +58,53 @@ __global__ void read_interleaved(const uint4* __restrict__ a, int64_t n16, unsig
         for (int u = 0; u < U; ++u) acc ^= v[u].x ^ v[u].y ^ v[u].z ^ v[u].w;
     }
     if (acc == 0x12345678u) out[0] = acc;
+}
+
+// SpMV-shaped streams: one CTA of 32 warps per "partition", every warp streams `nch` chunks,
+// each chunk = 512 B of a 2-byte array (ind) + 1 KB of a 4-byte array (val), 4 chunks unrolled.
+// mode 0: warp-private contiguous blocks (the SpMV's SELL layout: warp w's chunks back to back);
+// mode 1: chunks of the CTA's 32 warps interleaved (chunk c of warp w at c * 32 + w).
+template <int MODE>
+__global__ void __launch_bounds__(1024) spmv_shape_kernel(const uint4* __restrict__ ind, const uint4* __restrict__ val,
+                                                          int nch, unsigned* out) {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t cta0 = (int64_t)blockIdx.x * 32 * nch;  // chunk index base of this CTA
+    unsigned acc = 0;
+#pragma unroll 4
+    for (int c = 0; c < nch; ++c) {
+        const int64_t ch = MODE == 0 ? cta0 + (int64_t)warp * nch + c : cta0 + (int64_t)c * 32 + warp;
+        const uint4 a = ld_stream(ind + ch * 32 + lane, pol);
+        const uint4 b = ld_stream(val + ch * 64 + lane, pol);
+        const uint4 d = ld_stream(val + ch * 64 + 32 + lane, pol);
+        acc ^= a.x ^ b.y ^ d.z ^ a.w ^ b.x ^ d.w;
+    }
+    if (acc == 0x12345678u) out[0] = acc;
+}
+
+template <int MODE>
+void run_shape(const uint4* a, int64_t n16, int ctas, unsigned* out, int reps) {
+    // split the buffer: ind third, val two thirds
+    const int64_t chunks = n16 / 96;  // 96 x 16 B = 1.5 KB per chunk
+    const int nch = (int)(chunks / ((int64_t)ctas * 32));
+    const uint4* ind = a;
+    const uint4* val = a + (int64_t)ctas * 32 * nch * 32;
+    const double bytes = (double)ctas * 32 * nch * 1536.0;
+    cudaEvent_t e0, e1;
+    CK(cudaEventCreate(&e0));
+    CK(cudaEventCreate(&e1));
+    for (int w = 0; w < 2; ++w) spmv_shape_kernel<MODE><<<ctas, 1024>>>(ind, val, nch, out);
+    CK(cudaEventRecord(e0));
+    for (int r = 0; r < reps; ++r) spmv_shape_kernel<MODE><<<ctas, 1024>>>(ind, val, nch, out);
+    CK(cudaEventRecord(e1));
+    CK(cudaEventSynchronize(e1));
+    CK(cudaGetLastError());
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, e0, e1));
+    ms /= reps;
+    printf("{\"mode\": \"spmv_shape_%s\", \"ctas\": %d, \"chunks_per_warp\": %d, \"ms\": %.4f, \"GBs\": %.1f}\n",
+           MODE == 0 ? "warp_private" : "cta_interleaved", ctas, nch, ms, bytes / (ms * 1e6));
 }
 
 template <int U>
@@ -124,5 +171,11 @@ int main(int argc, char** argv) {
     run_il<8>(a, n16, 8 * sms, 256, out, reps, bytes);
     run_il<16>(a, n16, 8 * sms, 256, out, reps, bytes);
     run_il<4>(a, n16, 4 * sms, 512, out, reps, bytes);
+    run_shape<0>(a, n16, 1500, out, reps);
+    run_shape<1>(a, n16, 1500, out, reps);
+    run_shape<0>(a, n16, 148, out, reps);
+    run_shape<1>(a, n16, 148, out, reps);
+    run_shape<0>(a, n16, 4440, out, reps);
+    run_shape<1>(a, n16, 4440, out, reps);
     return 0;
 }
