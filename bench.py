@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--spmv-reps", type=int, default=20)
     ap.add_argument("--slices", type=int, default=4, help="multi-slice batch measured beside the headline (1 = off)")
+    ap.add_argument("--variant", default=None, choices=["peer", "dense"], help=argparse.SUPPRESS)
     ap.add_argument("--distributed", action="store_true",
                     help="run the decomposed path (NCCL communicator, exchange, allreduce) even at N = 1")
     return ap.parse_args()
@@ -265,35 +266,69 @@ def bench_multislice(args, plan1, y1, n, m, c, stream):
     return out
 
 
-def bench_peer_exchange(args, n, m, c, y, local, stream, world):
-    """N > 1: the same CG with EXCHANGE = 1 (SpMV epilogue / pack kernel store straight into the
-    peers' buffers over NVLink, NEXT-2), reported beside the NCCL-exchange headline.  Failures are
-    reported, not fatal (the peer path is new on multi-GPU hardware)."""
+def variant_child(args):
+    """Child process of bench_exchange_variant: one rank of the same job on its own NCCL
+    communicator (a fresh rendezvous), the CG with exchange `args.variant`; rank 0 prints one
+    JSON line."""
     import torch
     import torch.distributed as dist
-    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, bootstrap_unique_id
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, bootstrap_unique_id, inputs
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(local)
+    dist.init_process_group("nccl")
+    rank, world = dist.get_rank(), dist.get_world_size()
+    n, m, c = inputs.CONFIGS[args.config]
+    uid = bootstrap_unique_id(rank)
+    plan = MemXCT(n, m, c, rank=rank, nranks=world, unique_id=uid, device=local,
+                  vector_order="plan", exchange=args.variant).build()
+    ph = np.ascontiguousarray(inputs.shepp_logan(n).astype(np.float32)[plan.local_indices(0)])
+    stream = torch.cuda.current_stream()
+    y = plan.forward(torch.from_numpy(ph).cuda())
+    x = torch.empty(plan.local_size(0), dtype=torch.float32, device=y.device)
+    for _ in range(max(1, args.warmup)):
+        plan.cg(y, args.iters, x=x, stream=stream)
+    dist.barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        plan.cg(y, args.iters, x=x, stream=stream)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ex = plan.exchange_time(20, stream=stream) if args.variant == "dense" else {"fwd_us": 0.0, "back_us": 0.0}
+    t = torch.tensor([e0.elapsed_time(e1), ex["fwd_us"], ex["back_us"]], dtype=torch.float64, device=y.device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    out = {"value": args.iters * args.steps / (float(t[0]) * 1e-3), "unit": "CG iter/s",
+           "ms_per_step": float(t[0]) / args.steps}
+    if args.variant == "dense":
+        out["exchange_us_per_cg_iter"] = float(t[1] + t[2])
+    plan.close()
+    dist.destroy_process_group()
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+
+
+def bench_exchange_variant(args, rank, world, kind):
+    """N > 1: the same CG with another exchange, reported beside the NCCL all-to-allv headline:
+    "peer" = EXCHANGE 1 (SpMV epilogue / pack kernel store straight into the peers' buffers over
+    NVLink, CG dots over peer memory, NEXT-2); "dense" = EXCHANGE 2 (reduce-scatter / allgather of
+    the whole partial sinogram, SURVEY 8(e)'s comparison).  Every rank runs it in a child process
+    with its own rendezvous, so a failure there (a peer-flag wait traps after ~20 s instead of
+    hanging) is reported without taking down the headline's process."""
+    env = dict(os.environ)
+    env["MASTER_PORT"] = str(int(os.environ.get("MASTER_PORT", "29500")) + (17 if kind == "peer" else 23))
+    cmd = [sys.executable, os.path.abspath(__file__), "--variant", kind, "--config", str(args.config),
+           "--iters", str(args.iters), "--steps", str(args.steps), "--warmup", str(args.warmup)]
     try:
-        uid = bootstrap_unique_id(dist.get_rank())
-        plan = MemXCT(n, m, c, rank=dist.get_rank(), nranks=world, unique_id=uid, device=local,
-                      vector_order="plan", exchange="peer").build()
-        x = torch.empty(plan.local_size(0), dtype=torch.float32, device=y.device)
-        for _ in range(max(1, args.warmup)):
-            plan.cg(y, args.iters, x=x, stream=stream)
-        dist.barrier()
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(args.steps):
-            plan.cg(y, args.iters, x=x, stream=stream)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=y.device)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        plan.close()
-        return {"value": args.iters * args.steps / (float(t.item()) * 1e-3), "unit": "CG iter/s",
-                "ms_per_step": float(t.item()) / args.steps}
-    except Exception as e:  # noqa: BLE001
-        return {"error": str(e)[:300]}
+        r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=900)
+    except subprocess.TimeoutExpired:
+        return {"error": "timed out after 900 s"}
+    if rank != 0:
+        return None
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    if r.returncode != 0 or not lines:
+        return {"error": f"exit {r.returncode}: " + (r.stderr.strip().splitlines() or [""])[-1][:300]}
+    return json.loads(lines[-1])
 
 
 def run_ours(args, rank, world):
@@ -407,9 +442,12 @@ def run_ours(args, rank, world):
                   "local_spmv_fwd_us": float(et[2]), "local_spmv_back_us": float(et[3]),
                   "how": "max over ranks, CUDA events, 20 reps; local_spmv = A_p / A_p^T kernels alone"}
 
-    peer = None
+    peer = dense = None
     if dist_mode:
-        peer = bench_peer_exchange(args, n, m, c, y, local, stream, world)
+        dist.barrier()
+        peer = bench_exchange_variant(args, rank, world, "peer")
+        dense = bench_exchange_variant(args, rank, world, "dense")
+        dist.barrier()
 
     multislice = None
     if args.slices > 1 and not dist_mode:
@@ -472,6 +510,8 @@ def run_ours(args, rank, world):
         line["multislice"] = multislice
     if peer is not None:
         line["fused_peer_exchange"] = peer
+    if dense is not None:
+        line["dense_exchange"] = dense
     if not args.no_cpu_baseline and world == 1:
         line["cpu_baseline"] = cpu_baseline(cfg, st["nnz"])
     print(json.dumps(line), flush=True)
@@ -479,6 +519,9 @@ def run_ours(args, rank, world):
 
 def main():
     args = parse()
+    if args.variant:
+        variant_child(args)
+        return
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     if world == 1 and args.distributed and args.impl == "ours":

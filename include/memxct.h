@@ -100,7 +100,11 @@ typedef enum {
      * the reduction (default); 1 = fused over peer memory (FP32, P <= 16): the SpMV epilogue
      * stores partials straight into the owners' receive buffers and the owners' pack kernel stores
      * ray values straight into the peers' footprint buffers (CUDA IPC mappings over NVLink),
-     * synchronised by epoch/credit flags -- no separate collective on the data path. */
+     * synchronised by epoch/credit flags -- no separate collective on the data path; the CG dots
+     * go over peer memory too.  2 = dense collectives (the comparison of SURVEY 8(e)): forward
+     * partials scattered into a zeroed P x max-owned-range sinogram and ncclReduceScatter, back
+     * ncclAllGather of the owned values and a gather of the footprint rays -- more bytes moved
+     * (the whole sinogram instead of the ~0.4 M C interacting rays), no per-peer bookkeeping. */
     MEMXCT_OPT_EXCHANGE = 9,
     /* Row grouping of the forward SpMV's partitions (A_p rows = rays).  -1 = the paper's: a
      * partition is PART_ROWS consecutive rays in Hilbert order (a square of about

@@ -154,7 +154,7 @@ memxct_status_t memxct_plan_set_option(memxct_plan_t plan, memxct_option_t optio
             case MEMXCT_OPT_CG_VARIANT: range(0, 1); P.opt.cg_variant = value; break;
             case MEMXCT_OPT_VECTOR_ORDER: range(0, 1); P.opt.vector_order = value; break;
             case MEMXCT_OPT_SLICES: range(1, 8); P.opt.slices = value; break;
-            case MEMXCT_OPT_EXCHANGE: range(0, 1); P.opt.exchange = value; break;
+            case MEMXCT_OPT_EXCHANGE: range(0, 2); P.opt.exchange = value; break;
             case MEMXCT_OPT_RAY_BLOCK:
                 range(-1, 32);
                 if (value > 0 && (value & (value - 1))) mx::fail(MEMXCT_ERR_INVALID_ARG, "RAY_BLOCK must be -1, 0 or a power of two");

@@ -200,12 +200,15 @@ void allreduce_slices(Plan& P, double* v, int K, int64_t stride, cudaStream_t st
 // otherwise as a per-CTA tree + last-CTA sum in partition order (deterministic).  (With the
 // first, uniform-width kernel that epilogue cost 0.5 ms per 2 ms SpMV, profiles/r01a_launches.md;
 // with the jagged kernel it is free, so it is the default; MEMXCT_FUSED_DOT=0 selects the
-// separate dot kernel.)  Batched and P > 1: separate dot kernels; P > 1 allreduces them (the
-// projection then includes the exchange, A = R C A_p).
+// separate dot kernel.)  P > 1 (the projection includes the exchange, A = R C A_p): the local
+// dot is fused into the last kernel of the projection -- the reduction R forward, A_p^T back --
+// and summed over the ranks.  Batched: separate dot kernels.
 template <class T>
 void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, int64_t dot_stride,
             cudaStream_t st) {
-    const bool fused = dot_out && K == 1 && !P.dist && (P.opt.canonical != 0 || P.fused_dot);
+    // P > 1: the rank's local dot is fused into the reduction R (forward) or into A_p^T's
+    // epilogue (back) for every exchange, then summed over the ranks (allreduce_slices)
+    const bool fused = dot_out && K == 1 && (P.dist || P.opt.canonical != 0 || P.fused_dot);
     if (!P.dist && K == 1) {
         const Layout& L = forward ? P.fwd : P.back;
         double* part = forward ? P.part_fwd.p() : P.part_back.p();
@@ -214,8 +217,8 @@ void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, 
         else
             spmv_f64(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), P.opt.canonical != 0, st);
     } else if (K == 1) {
-        if (forward) apply_forward(P, in, out, st);
-        else apply_back(P, in, out, st);
+        if (forward) apply_forward(P, in, out, st, fused ? dot_out : nullptr);
+        else apply_back(P, in, out, st, fused ? dot_out : nullptr);
     } else {
         if constexpr (sizeof(T) == 4) {
             if (forward) apply_forward_batch(P, K, in, out, st);
@@ -229,8 +232,8 @@ void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, 
         dot_kernel<T><<<dim3(vec_blocks(n), K), kVT, 0, st>>>(out, n, dot_out, dot_stride, P.part_vec.p(),
                                                               P.tickets.p() + 64);
         MX_LAUNCHED();
-        if (P.dist) allreduce_slices(P, dot_out, K, dot_stride, st);
     }
+    if (dot_out && P.dist) allreduce_slices(P, dot_out, K, dot_stride, st);
 }
 
 template <class T>

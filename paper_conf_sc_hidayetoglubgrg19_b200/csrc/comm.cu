@@ -27,6 +27,7 @@ struct NcclApi {
     decltype(&ncclCommDestroy) CommDestroy = nullptr;
     decltype(&ncclAllReduce) AllReduce = nullptr;
     decltype(&ncclAllGather) AllGather = nullptr;
+    decltype(&ncclReduceScatter) ReduceScatter = nullptr;
     decltype(&ncclSend) Send = nullptr;
     decltype(&ncclRecv) Recv = nullptr;
     decltype(&ncclGroupStart) GroupStart = nullptr;
@@ -51,6 +52,7 @@ struct NcclApi {
         MX_SYM(CommDestroy, "ncclCommDestroy");
         MX_SYM(AllReduce, "ncclAllReduce");
         MX_SYM(AllGather, "ncclAllGather");
+        MX_SYM(ReduceScatter, "ncclReduceScatter");
         MX_SYM(Send, "ncclSend");
         MX_SYM(Recv, "ncclRecv");
         MX_SYM(GroupStart, "ncclGroupStart");
@@ -58,7 +60,7 @@ struct NcclApi {
         MX_SYM(GetErrorString, "ncclGetErrorString");
 #undef MX_SYM
         if (!a.GetUniqueId || !a.CommInitRank || !a.AllReduce || !a.Send || !a.Recv || !a.GroupStart ||
-            !a.GroupEnd || !a.AllGather || !a.CommDestroy)
+            !a.GroupEnd || !a.AllGather || !a.ReduceScatter || !a.CommDestroy)
             a.error = "libnccl.so.2 lacks required symbols";
         return a;
     }
@@ -100,6 +102,15 @@ public:
     void allreduce_sum(void* buf, int64_t count, DType t, cudaStream_t st) override {
         if (count == 0) return;
         nccl().check(nccl().AllReduce(buf, buf, (size_t)count, nccl_type(t), ncclSum, comm_, st), "ncclAllReduce");
+    }
+    void reduce_scatter_sum(const void* send, void* recv, int64_t count, DType t, cudaStream_t st) override {
+        if (count == 0) return;
+        nccl().check(nccl().ReduceScatter(send, recv, (size_t)count, nccl_type(t), ncclSum, comm_, st),
+                     "ncclReduceScatter");
+    }
+    void allgather(const void* send, void* recv, int64_t count, DType t, cudaStream_t st) override {
+        if (count == 0) return;
+        nccl().check(nccl().AllGather(send, recv, (size_t)count, nccl_type(t), comm_, st), "ncclAllGather");
     }
     void alltoallv(const void* send, const int64_t* scount, const int64_t* sdispl, void* recv,
                    const int64_t* rcount, const int64_t* rdispl, DType t, cudaStream_t st) override {
@@ -245,6 +256,45 @@ public:
             MX_LAUNCHED();
         }
         MX_CUDA(cudaStreamSynchronize(st));
+    }
+
+    void reduce_scatter_sum(const void* send, void* recv, int64_t count, DType t, cudaStream_t st) override {
+        MX_CUDA(cudaStreamSynchronize(st));
+        const size_t es = dtype_size(t);
+        g_->posts[rank].send = send;
+        g_->barrier();
+        const size_t need = es * (size_t)std::max<int64_t>(count, 1) * nranks;
+        if (scratch_.bytes() < need) scratch_.alloc(std::max(need, (size_t)4096));
+        for (int q = 0; q < nranks; ++q)
+            if (count > 0)
+                MX_CUDA(cudaMemcpyAsync(static_cast<char*>(scratch_.get()) + q * count * es,
+                                        static_cast<const char*>(g_->posts[q].send) + rank * count * es, count * es,
+                                        cudaMemcpyDeviceToDevice, st));
+        MX_CUDA(cudaStreamSynchronize(st));
+        g_->barrier();  // every rank has read its block of every send buffer
+        if (count > 0) {
+            const unsigned blocks = (unsigned)std::min<int64_t>(1024, ceil_div(count, 256));
+            switch (t) {
+                case DType::F32: sum_ranks_kernel<<<blocks, 256, 0, st>>>(scratch_.as<float>(), nranks, count, (float*)recv); break;
+                case DType::F64: sum_ranks_kernel<<<blocks, 256, 0, st>>>(scratch_.as<double>(), nranks, count, (double*)recv); break;
+                default: fail(MEMXCT_ERR_UNSUPPORTED, "internal: integer reduce-scatter");
+            }
+            MX_LAUNCHED();
+        }
+        MX_CUDA(cudaStreamSynchronize(st));
+    }
+
+    void allgather(const void* send, void* recv, int64_t count, DType t, cudaStream_t st) override {
+        MX_CUDA(cudaStreamSynchronize(st));
+        const size_t es = dtype_size(t);
+        g_->posts[rank].send = send;
+        g_->barrier();
+        for (int q = 0; q < nranks; ++q)
+            if (count > 0)
+                MX_CUDA(cudaMemcpyAsync(static_cast<char*>(recv) + q * count * es, g_->posts[q].send, count * es,
+                                        cudaMemcpyDeviceToDevice, st));
+        MX_CUDA(cudaStreamSynchronize(st));
+        g_->barrier();
     }
 
     void alltoallv(const void* send, const int64_t* scount, const int64_t* sdispl, void* recv,

@@ -33,6 +33,11 @@ public:
     // receive `rcount[q]` elements into recv + rdispl[q] (host count/displacement arrays).
     virtual void alltoallv(const void* send, const int64_t* scount, const int64_t* sdispl, void* recv,
                            const int64_t* rcount, const int64_t* rdispl, DType t, cudaStream_t st) = 0;
+    // dense collectives (EXCHANGE = 2, the comparison of SURVEY 8(e)): every rank's `send` holds
+    // nranks blocks of `count` elements; rank g receives the elementwise sum over ranks of block g
+    virtual void reduce_scatter_sum(const void* send, void* recv, int64_t count, DType t, cudaStream_t st) = 0;
+    // every rank contributes `count` elements; recv = the nranks contributions in rank order
+    virtual void allgather(const void* send, void* recv, int64_t count, DType t, cudaStream_t st) = 0;
     // gather one int64 per rank on the host (build-time bookkeeping)
     virtual std::vector<int64_t> allgather_host(int64_t v, cudaStream_t st) = 0;
     // gather a vector of n int64 per rank: out[q * n + i] (build-time)

@@ -45,20 +45,86 @@ constexpr int kT = 256;
 
 unsigned nblocks(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 1 << 20)); }
 
+// R: owned ray i = its received partials added in peer order (reduction-map CSR ptr / pos;
+// ptr == nullptr: y[i] = recv[i], the dense exchange's owned block).  Optionally the CG dot
+// <y, y> of the owned rays: per-CTA fixed tree, the last CTA (ticket) adds the CTA partials in
+// CTA order -- deterministic, and the same sums for every exchange (same grid, same values).
+// pa.fold (fused exchange on NCCL ranks, peer.cu): thread 0 of every CTA first waits for every
+// peer's arrival flag, and the last CTA returns the credits (receive buffer consumed).
 template <class T>
-__global__ void reduce_kernel(const T* __restrict__ recv, const int64_t* __restrict__ ptr,
-                              const int32_t* __restrict__ pos, int64_t nown, T* __restrict__ y) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nown; i += (int64_t)gridDim.x * blockDim.x) {
-        T acc = T(0);
-        for (int64_t k = ptr[i]; k < ptr[i + 1]; ++k) acc += recv[pos[k]];  // peer order
-        y[i] = acc;
+__global__ void __launch_bounds__(kT)
+reduce_dot_kernel(const T* __restrict__ recv, const int64_t* __restrict__ ptr, const int32_t* __restrict__ pos,
+                  int64_t nown, T* __restrict__ y, double* part, double* dot_out, unsigned int* ticket, PeerArgs pa) {
+    __shared__ double red[kT / 32];
+    __shared__ bool am_last;
+    if (pa.fold) {
+        if (threadIdx.x == 0)
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.notrap);
+        __syncthreads();
     }
+    double d = 0.0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nown; i += (int64_t)gridDim.x * blockDim.x) {
+        T acc;
+        if (ptr) {
+            acc = T(0);
+            for (int64_t k = ptr[i]; k < ptr[i + 1]; ++k) acc += recv[pos[k]];  // peer order
+        } else {
+            acc = recv[i];
+        }
+        y[i] = acc;
+        d += (double)acc * (double)acc;
+    }
+    if (!dot_out && !pa.fold) return;
+    if (dot_out) {
+        for (int o = 16; o; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+        if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = d;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (dot_out) {
+            double t = 0.0;
+            for (int w = 0; w < kT / 32; ++w) t += red[w];
+            part[blockIdx.x] = t;
+        }
+        __threadfence();
+        am_last = (atomicAdd(ticket, 1u) == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!am_last) return;
+    __threadfence();
+    if (dot_out) {  // the last CTA adds the CTA partials: strided per thread, then the fixed tree
+        double t = 0.0;
+        for (unsigned b = threadIdx.x; b < gridDim.x; b += blockDim.x) t += ((volatile double*)part)[b];
+        for (int o = 16; o; o >>= 1) t += __shfl_xor_sync(0xffffffffu, t, o);
+        __syncthreads();
+        if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = t;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double tot = 0.0;
+            for (int w = 0; w < kT / 32; ++w) tot += red[w];
+            *dot_out = tot;
+        }
+    }
+    if (threadIdx.x != 0) return;
+    if (pa.fold) {
+        __threadfence_system();
+        const unsigned long long e = pa.my_flags[pa.epoch_index];
+        for (int q = 0; q < pa.P; ++q) st_release_sys(pa.flag[q] + pa.slot + pa.me, e);
+    }
+    *ticket = 0u;
 }
 
 template <class T>
 __global__ void pack_kernel(const T* __restrict__ y, const int32_t* __restrict__ idx, int64_t n, T* __restrict__ out) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         out[i] = y[idx[i]];
+}
+
+template <class T>
+__global__ void scatter_dense_kernel(const T* __restrict__ yfp, const int32_t* __restrict__ pos, int64_t n,
+                                     T* __restrict__ dense) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        dense[pos[i]] = yfp[i];
 }
 
 __global__ void flag_kernel(const int32_t* __restrict__ len, int64_t n, int32_t* __restrict__ flag) {
@@ -246,43 +312,112 @@ void build_exchange(Plan& P, cudaStream_t st) {
         MX_CUDA(cudaMemcpyAsync(X.red_pos.p(), perm.p(), 4 * X.nrecv, cudaMemcpyDeviceToDevice, st));
     X.y_fp.alloc(P.esize * std::max<int64_t>(P.nfp, 1));
     X.recv_buf.alloc(P.esize * std::max<int64_t>(X.nrecv, 1));
+    X.tickets.alloc(8);
+    MX_CUDA(cudaMemsetAsync(X.tickets.p(), 0, 32, st));
+    X.dot_part.alloc(std::max<int64_t>({P.back.nparts, (int64_t)nblocks(nown), 4 * 148}));
+    if (P.opt.exchange == 2) {  // dense collectives: footprint row i -> [owner][owned-local index]
+        X.maxown = 0;
+        for (int h = 0; h < np; ++h) X.maxown = std::max(X.maxown, P.sino_bounds[h + 1] - P.sino_bounds[h]);
+        if ((int64_t)np * X.maxown >= INT32_MAX) fail(MEMXCT_ERR_UNSUPPORTED, "dense exchange: sinogram too large");
+        std::vector<int32_t> dpos(std::max<int64_t>(P.nfp, 1));
+        for (int h = 0; h < np; ++h)
+            for (int64_t i = X.sdispl[h]; i < X.sdispl[h + 1]; ++i) dpos[i] = (int32_t)(h * X.maxown + idx[i]);
+        X.dense_pos.alloc(std::max<int64_t>(P.nfp, 1));
+        MX_CUDA(cudaMemcpy(X.dense_pos.p(), dpos.data(), 4 * std::max<int64_t>(P.nfp, 1), cudaMemcpyHostToDevice));
+        X.dense_buf.alloc(P.esize * std::max<int64_t>(np * X.maxown, 1));
+        X.dense_own.alloc(P.esize * std::max<int64_t>(X.maxown, 1));
+        X.dense = true;
+    }
     MX_CUDA(cudaStreamSynchronize(st));
     if (P.opt.exchange == 1) peer_setup(P, st);  // fused peer-memory exchange (peer.cu)
 }
 
 template <class T>
-static void forward_t(Plan& P, const T* x, T* y, cudaStream_t st) {
+void launch_reduce_dot(Plan& P, const T* recv, bool csr, T* y, double* dot_out, const PeerArgs& pa, cudaStream_t st) {
+    Exchange& X = P.ex;
+    const int64_t nown = P.s1 - P.s0;
+    reduce_dot_kernel<T><<<nblocks(nown), kT, 0, st>>>(recv, csr ? X.red_ptr.p() : nullptr, X.red_pos.p(), nown, y,
+                                                       X.dot_part.p(), dot_out, X.tickets.p() + 2, pa);
+    MX_LAUNCHED();
+}
+
+// Forward communication: footprint partials `yfp` (nfp) -> owned ray values `yown` (nown).
+// Sparse (default): C = all-to-allv of the per-owner slices into `rb` (nrecv), R = per owned ray
+// the received partials added in peer order.  Dense (EXCHANGE = 2): the partials scattered into a
+// zeroed [P][maxown] sinogram, reduce-scatter (rank g receives block g summed over the ranks).
+template <class T>
+static void exchange_fwd(Plan& P, const T* yfp, T* rb, T* yown, cudaStream_t st, double* dot_out = nullptr) {
+    Exchange& X = P.ex;
+    const DType t = sizeof(T) == 4 ? DType::F32 : DType::F64;
+    const int64_t nown = P.s1 - P.s0;
+    if (X.dense) {
+        T* d = X.dense_buf.as<T>();
+        MX_CUDA(cudaMemsetAsync(d, 0, sizeof(T) * (size_t)(P.nranks * X.maxown), st));
+        if (P.nfp > 0) {
+            scatter_dense_kernel<T><<<nblocks(P.nfp), kT, 0, st>>>(yfp, X.dense_pos.p(), P.nfp, d);
+            MX_LAUNCHED();
+        }
+        P.comm->reduce_scatter_sum(d, X.dense_own.get(), X.maxown, t, st);
+        launch_reduce_dot<T>(P, X.dense_own.as<T>(), false, yown, dot_out, PeerArgs{}, st);  // copy (+ dot)
+        return;
+    }
+    P.comm->alltoallv(yfp, X.scount.data(), X.sdispl.data(), rb, X.rcount.data(), X.rdispl.data(), t, st);  // C
+    launch_reduce_dot<T>(P, rb, true, yown, dot_out, PeerArgs{}, st);                                      // R
+}
+
+// Back communication: owned ray values `yown` -> every footprint ray's value in `yfp`.  Sparse:
+// R^T = pack of the owned values each peer needs (recv order) into `rb`, C^T = the reverse
+// all-to-allv straight into the footprint slices.  Dense: allgather of the owned values into the
+// [P][maxown] sinogram, gather of the footprint rays.
+template <class T>
+static void exchange_back(Plan& P, const T* yown, T* rb, T* yfp, cudaStream_t st) {
+    Exchange& X = P.ex;
+    const DType t = sizeof(T) == 4 ? DType::F32 : DType::F64;
+    if (X.dense) {
+        const int64_t nown = P.s1 - P.s0;
+        if (nown > 0)
+            MX_CUDA(cudaMemcpyAsync(X.dense_own.get(), yown, sizeof(T) * nown, cudaMemcpyDeviceToDevice, st));
+        P.comm->allgather(X.dense_own.get(), X.dense_buf.get(), X.maxown, t, st);
+        if (P.nfp > 0) {
+            pack_kernel<T><<<nblocks(P.nfp), kT, 0, st>>>(X.dense_buf.as<T>(), X.dense_pos.p(), P.nfp, yfp);
+            MX_LAUNCHED();
+        }
+        return;
+    }
+    if (X.nrecv > 0) {
+        pack_kernel<T><<<nblocks(X.nrecv), kT, 0, st>>>(yown, X.recv_idx.p(), X.nrecv, rb);  // R^T
+        MX_LAUNCHED();
+    }
+    P.comm->alltoallv(rb, X.rcount.data(), X.rdispl.data(), yfp, X.scount.data(), X.sdispl.data(), t, st);  // C^T
+}
+
+// P > 1 with dot_out: the CG dot of the rank's output part is fused into the reduction
+// (forward) or into A_p^T's epilogue (back, per-partition tree + last-CTA sum); the caller sums
+// it over the ranks.
+template <class T>
+static void forward_t(Plan& P, const T* x, T* y, double* dot_out, cudaStream_t st) {
     if (!P.dist) {
         spmv_any(P, P.fwd, x, y, st);
         return;
     }
     Exchange& X = P.ex;
     T* yfp = X.y_fp.as<T>();
-    T* rb = X.recv_buf.as<T>();
     spmv_any(P, P.fwd, x, yfp, st);                                         // A_p
-    P.comm->alltoallv(yfp, X.scount.data(), X.sdispl.data(), rb, X.rcount.data(), X.rdispl.data(),
-                      sizeof(T) == 4 ? DType::F32 : DType::F64, st);        // C
-    const int64_t nown = P.s1 - P.s0;
-    reduce_kernel<T><<<nblocks(nown), kT, 0, st>>>(rb, X.red_ptr.p(), X.red_pos.p(), nown, y);  // R
-    MX_LAUNCHED();
+    exchange_fwd<T>(P, yfp, X.recv_buf.as<T>(), y, st, dot_out);            // R C
 }
 
 template <class T>
-static void back_t(Plan& P, const T* y, T* x, cudaStream_t st) {
+static void back_t(Plan& P, const T* y, T* x, double* dot_out, cudaStream_t st) {
     if (!P.dist) {
         spmv_any(P, P.back, y, x, st);
         return;
     }
     Exchange& X = P.ex;
     T* yfp = X.y_fp.as<T>();
-    T* rb = X.recv_buf.as<T>();
-    if (X.nrecv > 0) {
-        pack_kernel<T><<<nblocks(X.nrecv), kT, 0, st>>>(y, X.recv_idx.p(), X.nrecv, rb);   // R^T
-        MX_LAUNCHED();
-    }
-    P.comm->alltoallv(rb, X.rcount.data(), X.rdispl.data(), yfp, X.scount.data(), X.sdispl.data(),
-                      sizeof(T) == 4 ? DType::F32 : DType::F64, st);        // C^T
-    spmv_any(P, P.back, yfp, x, st);                                        // A_p^T
+    exchange_back<T>(P, y, X.recv_buf.as<T>(), yfp, st);                    // C^T R^T
+    double* part = dot_out ? X.dot_part.p() : nullptr;                      // A_p^T
+    if constexpr (sizeof(T) == 4) spmv_f32(P.back, yfp, x, part, dot_out, X.tickets.p() + 4, st);
+    else spmv_f64(P.back, yfp, x, part, dot_out, X.tickets.p() + 4, false, st);
 }
 
 // ---- K slices at once (slice-major vectors): one matrix stream per group of <= 8 slices -----
@@ -320,13 +455,8 @@ void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t 
             float* yfp = X.y_fp_b.as<float>();
             float* rb = X.recv_b.as<float>();
             spmm_f32(P.fwd, k, xs, nx, yfp, P.nfp, st);                       // A_p, k slices
-            for (int s = 0; s < k; ++s) {
-                P.comm->alltoallv(yfp + s * P.nfp, X.scount.data(), X.sdispl.data(), rb + s * X.nrecv,
-                                  X.rcount.data(), X.rdispl.data(), DType::F32, st);          // C
-                reduce_kernel<float><<<nblocks(ny), kT, 0, st>>>(rb + s * X.nrecv, X.red_ptr.p(), X.red_pos.p(),
-                                                                 ny, ys + s * ny);            // R
-                MX_LAUNCHED();
-            }
+            for (int s = 0; s < k; ++s)
+                exchange_fwd<float>(P, yfp + s * P.nfp, rb + s * X.nrecv, ys + s * ny, st);  // R C
         }
         s0 += k;
     }
@@ -345,15 +475,8 @@ void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st)
             Exchange& X = P.ex;
             float* yfp = X.y_fp_b.as<float>();
             float* rb = X.recv_b.as<float>();
-            for (int s = 0; s < k; ++s) {
-                if (X.nrecv > 0) {
-                    pack_kernel<float><<<nblocks(X.nrecv), kT, 0, st>>>(ys + s * ny, X.recv_idx.p(), X.nrecv,
-                                                                        rb + s * X.nrecv);  // R^T
-                    MX_LAUNCHED();
-                }
-                P.comm->alltoallv(rb + s * X.nrecv, X.rcount.data(), X.rdispl.data(), yfp + s * P.nfp,
-                                  X.scount.data(), X.sdispl.data(), DType::F32, st);        // C^T
-            }
+            for (int s = 0; s < k; ++s)
+                exchange_back<float>(P, ys + s * ny, rb + s * X.nrecv, yfp + s * P.nfp, st);  // C^T R^T
             spmm_f32(P.back, k, yfp, P.nfp, xs, nx, st);                      // A_p^T, k slices
         }
         s0 += k;
@@ -367,7 +490,6 @@ void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStrea
     *us_fwd = *us_back = 0.0;
     if (!P.dist || reps < 1) return;
     Exchange& X = P.ex;
-    const DType t = P.esize == 4 ? DType::F32 : DType::F64;
     const int64_t nown = P.s1 - P.s0;
     DevBuf own(P.esize * std::max<int64_t>(nown, 1));
     MX_CUDA(cudaMemsetAsync(own.get(), 0, P.esize * std::max<int64_t>(nown, 1), st));
@@ -375,28 +497,12 @@ void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStrea
     cudaEvent_t e[3];
     for (auto& ev : e) MX_CUDA(cudaEventCreate(&ev));
     auto fwd = [&] {
-        P.comm->alltoallv(X.y_fp.get(), X.scount.data(), X.sdispl.data(), X.recv_buf.get(), X.rcount.data(),
-                          X.rdispl.data(), t, st);
-        if (P.esize == 4)
-            reduce_kernel<float><<<nblocks(nown), kT, 0, st>>>(X.recv_buf.as<float>(), X.red_ptr.p(), X.red_pos.p(),
-                                                               nown, own.as<float>());
-        else
-            reduce_kernel<double><<<nblocks(nown), kT, 0, st>>>(X.recv_buf.as<double>(), X.red_ptr.p(),
-                                                                X.red_pos.p(), nown, own.as<double>());
-        MX_LAUNCHED();
+        if (P.esize == 4) exchange_fwd<float>(P, X.y_fp.as<float>(), X.recv_buf.as<float>(), own.as<float>(), st);
+        else exchange_fwd<double>(P, X.y_fp.as<double>(), X.recv_buf.as<double>(), own.as<double>(), st);
     };
     auto back = [&] {
-        if (X.nrecv > 0) {
-            if (P.esize == 4)
-                pack_kernel<float><<<nblocks(X.nrecv), kT, 0, st>>>(own.as<float>(), X.recv_idx.p(), X.nrecv,
-                                                                    X.recv_buf.as<float>());
-            else
-                pack_kernel<double><<<nblocks(X.nrecv), kT, 0, st>>>(own.as<double>(), X.recv_idx.p(), X.nrecv,
-                                                                     X.recv_buf.as<double>());
-            MX_LAUNCHED();
-        }
-        P.comm->alltoallv(X.recv_buf.get(), X.rcount.data(), X.rdispl.data(), X.y_fp.get(), X.scount.data(),
-                          X.sdispl.data(), t, st);
+        if (P.esize == 4) exchange_back<float>(P, own.as<float>(), X.recv_buf.as<float>(), X.y_fp.as<float>(), st);
+        else exchange_back<double>(P, own.as<double>(), X.recv_buf.as<double>(), X.y_fp.as<double>(), st);
     };
     fwd();
     back();  // warm-up
@@ -452,27 +558,25 @@ void time_spmv(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t 
 
 void preload_exchange_kernels() {
     cudaFuncAttributes fa;
-    MX_CUDA(cudaFuncGetAttributes(&fa, reduce_kernel<float>));
-    MX_CUDA(cudaFuncGetAttributes(&fa, reduce_kernel<double>));
+    MX_CUDA(cudaFuncGetAttributes(&fa, reduce_dot_kernel<float>));
+    MX_CUDA(cudaFuncGetAttributes(&fa, reduce_dot_kernel<double>));
     MX_CUDA(cudaFuncGetAttributes(&fa, pack_kernel<float>));
 }
 
-void reduce_partials(Plan& P, const float* recv, float* y, cudaStream_t st) {
-    const int64_t nown = P.s1 - P.s0;
-    reduce_kernel<float><<<nblocks(nown), kT, 0, st>>>(recv, P.ex.red_ptr.p(), P.ex.red_pos.p(), nown, y);
-    MX_LAUNCHED();
+void reduce_partials(Plan& P, const float* recv, float* y, double* dot_out, const PeerArgs& pa, cudaStream_t st) {
+    launch_reduce_dot<float>(P, recv, true, y, dot_out, pa, st);
 }
 
-void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st) {
-    if (P.ex.peer) peer_forward(P, (const float*)x, (float*)y, st);
-    else if (P.esize == 4) forward_t<float>(P, (const float*)x, (float*)y, st);
-    else forward_t<double>(P, (const double*)x, (double*)y, st);
+void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st, double* dot_out) {
+    if (P.ex.peer) peer_forward(P, (const float*)x, (float*)y, dot_out, st);
+    else if (P.esize == 4) forward_t<float>(P, (const float*)x, (float*)y, dot_out, st);
+    else forward_t<double>(P, (const double*)x, (double*)y, dot_out, st);
 }
 
-void apply_back(Plan& P, const void* y, void* x, cudaStream_t st) {
-    if (P.ex.peer) peer_back(P, (const float*)y, (float*)x, st);
-    else if (P.esize == 4) back_t<float>(P, (const float*)y, (float*)x, st);
-    else back_t<double>(P, (const double*)y, (double*)x, st);
+void apply_back(Plan& P, const void* y, void* x, cudaStream_t st, double* dot_out) {
+    if (P.ex.peer) peer_back(P, (const float*)y, (float*)x, dot_out, st);
+    else if (P.esize == 4) back_t<float>(P, (const float*)y, (float*)x, dot_out, st);
+    else back_t<double>(P, (const double*)y, (double*)x, dot_out, st);
 }
 
 }  // namespace mx

@@ -22,34 +22,13 @@ namespace {
 
 constexpr int kT = 256;
 
-__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
-    unsigned long long v;
-    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-
-__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) {
-    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
+__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) { st_release_sys(p, v); }
 
 // wait until flags[base + q] >= flags[target_index] for every q < P
 __global__ void wait_kernel(const unsigned long long* flags, int P, int base, int target_index, int me,
                             int notrap) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    const unsigned long long target = ld_acquire_sys(flags + target_index);
-    const long long t0 = clock64();
-    for (int q = 0; q < P; ++q) {
-        while (ld_acquire_sys(flags + base + q) < target) {
-            __nanosleep(64);
-            if (clock64() - t0 > 40000000000LL) {  // ~20 s: a peer is gone -- fail, don't hang
-                printf("memxct peer wait timeout: rank %d base %d q %d target %llu value %llu\n", me, base, q,
-                       target, ld_acquire_sys(flags + base + q));
-                for (int i = 0; i < 4 * P + 2; ++i) printf("  rank %d flag[%d] = %llu\n", me, i, flags[i]);
-                if (notrap) return;
-                __trap();
-            }
-        }
-    }
+    wait_flags(flags, base, P, ld_acquire_sys(flags + target_index), me, notrap);
 }
 
 int notrap_env() {
@@ -72,17 +51,26 @@ __global__ void signal_kernel(SignalArgs sa, int P, int slot, const unsigned lon
 }
 
 // R^T + C^T: value j (recv order, peer g = the range containing j) goes to g's footprint buffer
+// (pa.fold: thread 0 of every CTA first waits for the peers' credits -- footprint buffers
+// consumed -- reading the epoch before this CTA's ticket, i.e. before the last CTA bumps it)
 __global__ void pack_remote_kernel(const float* __restrict__ y, const int32_t* __restrict__ idx, int64_t n,
                                    PeerArgs pa) {
     __shared__ bool am_last;
+    if (pa.fold) {
+        if (threadIdx.x == 0)
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.notrap);
+        __syncthreads();
+    }
     for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
         int g = 0;
         while (g + 1 < pa.P && j >= pa.bound[g + 1]) ++g;
         pa.dst[g][pa.off[g] + j] = y[idx[j]];
     }
-    __threadfence_system();
     __syncthreads();
-    if (threadIdx.x == 0) am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
+    if (threadIdx.x == 0) {
+        __threadfence_system();
+        am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
+    }
     __syncthreads();
     if (!am_last || threadIdx.x != 0) return;
     __threadfence_system();
@@ -116,17 +104,7 @@ __global__ void peer_allreduce_kernel(DotArgs da, int P, int me, double* v, int 
         for (int s = 0; s < K; ++s) da.dst[q][((int64_t)par * P + me) * kMaxDotSlices + s] = v[s * stride];
     __threadfence_system();
     for (int q = 0; q < P; ++q) st_release(da.flag[q] + me, e);
-    const long long t0 = clock64();
-    for (int q = 0; q < P; ++q) {
-        while (ld_acquire_sys(da.my_flags + q) < e) {
-            __nanosleep(32);
-            if (clock64() - t0 > 40000000000LL) {
-                printf("memxct peer dot timeout: rank %d waits for rank %d epoch %llu\n", me, q, e);
-                if (notrap) return;
-                __trap();
-            }
-        }
-    }
+    wait_flags(da.my_flags, 0, P, e, me, notrap);
     for (int s = 0; s < K; ++s) {
         const volatile double* m = da.mine + (int64_t)par * P * kMaxDotSlices + s;
         double acc = m[0];
@@ -163,8 +141,9 @@ void peer_setup(Plan& P, cudaStream_t st) {
     Comm& C = *P.comm;
     X.flags.alloc(4 * np + 2);
     MX_CUDA(cudaMemsetAsync(X.flags.p(), 0, 8 * (4 * np + 2), st));
-    X.tickets.alloc(4);
-    MX_CUDA(cudaMemsetAsync(X.tickets.p(), 0, 16, st));
+    // folded waits only where every rank has its own GPU (see PeerArgs::fold); MEMXCT_PEER_FOLD=0/1
+    X.fold = !P.local_group;
+    if (const char* e = std::getenv("MEMXCT_PEER_FOLD")) X.fold = e[0] == '1';
     MX_CUDA(cudaStreamSynchronize(st));
     // where my rows land in every owner's receive buffer, and my values in every peer's footprint
     std::vector<int64_t> rd(X.rdispl.begin(), X.rdispl.end()), sd(X.sdispl.begin(), X.sdispl.end());
@@ -186,69 +165,100 @@ void peer_setup(Plan& P, cudaStream_t st) {
     X.peer = true;
 }
 
-void peer_forward(Plan& P, const float* x, float* y, cudaStream_t st) {
+namespace {
+PeerArgs base_args(const Plan& P) {
+    PeerArgs pa;
+    pa.P = P.nranks;
+    pa.me = P.rank;
+    pa.my_flags = P.ex.flags.p();
+    pa.fold = P.ex.fold ? 1 : 0;
+    pa.notrap = notrap_env();
+    for (int q = 0; q < P.nranks; ++q) pa.flag[q] = static_cast<unsigned long long*>(P.ex.peer_flags[q]);
+    return pa;
+}
+}  // namespace
+
+// Flags of rank g ([4P + 2]): arrivals fwd [0, P) | arrivals back [P, 2P) | credits fwd [2P, 3P) |
+// credits back [3P, 4P) | my fwd epoch 4P | my back epoch 4P + 1.
+// Forward: (1) owners have consumed my previous partials (credits fwd >= my epoch); (2) A_p
+// stores the partials into the owners' receive buffers, last CTA bumps the epoch and publishes
+// it to every owner; (3) every peer's partials for my rays have arrived; (4) R (+ dot); (5)
+// credits back to every peer.  Folded (NCCL ranks): (1) runs inside A_p's epilogue, (3) and (5)
+// inside the reduction kernel -- two kernels per forward instead of five.
+void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream_t st) {
     Exchange& X = P.ex;
     const int np = P.nranks;
     unsigned long long* fl = X.flags.p();
-    // 1. owners have consumed my previous partials (forward credits >= my epoch)
-    wait_kernel<<<1, 32, 0, st>>>(fl, np, 2 * np, 4 * np, P.rank, notrap_env());
-    MX_LAUNCHED();
-    // 2. A_p with the partials stored straight into the owners' receive buffers (C), flags out
-    PeerArgs pa;
-    pa.P = np;
-    pa.me = P.rank;
+    if (!X.fold) {
+        wait_kernel<<<1, 32, 0, st>>>(fl, np, 2 * np, 4 * np, P.rank, notrap_env());
+        MX_LAUNCHED();
+    }
+    PeerArgs pa = base_args(P);
     for (int h = 0; h <= np; ++h) pa.bound[h] = X.sdispl[h];
     for (int h = 0; h < np; ++h) {
         pa.dst[h] = static_cast<float*>(X.peer_recv[h]);
         pa.off[h] = X.fwd_off[h];
-        pa.flag[h] = static_cast<unsigned long long*>(X.peer_flags[h]);
     }
-    pa.my_flags = fl;
     pa.ticket = X.tickets.p();
     pa.slot = 0;
     pa.epoch_index = 4 * np;
+    pa.wait_base = 2 * np;
     spmv_f32_remote(P.fwd, x, pa, st);
-    // 3. every peer's partials for my rays have arrived
-    wait_kernel<<<1, 32, 0, st>>>(fl, np, 0, 4 * np, P.rank, notrap_env());
-    MX_LAUNCHED();
-    // 4. R
-    reduce_partials(P, X.recv_buf.as<float>(), y, st);
-    // 5. credits: my receive buffer may be overwritten again
-    signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 2 * np + P.rank, fl, 4 * np);
-    MX_LAUNCHED();
+    if (!X.fold) {
+        wait_kernel<<<1, 32, 0, st>>>(fl, np, 0, 4 * np, P.rank, notrap_env());
+        MX_LAUNCHED();
+    }
+    PeerArgs ra = base_args(P);
+    ra.slot = 2 * np;          // credits fwd in the senders' arrays
+    ra.epoch_index = 4 * np;
+    ra.wait_base = 0;          // arrivals fwd
+    reduce_partials(P, X.recv_buf.as<float>(), y, dot_out, ra, st);
+    if (!X.fold) {
+        signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 2 * np + P.rank, fl, 4 * np);
+        MX_LAUNCHED();
+    }
 }
 
-void peer_back(Plan& P, const float* y, float* x, cudaStream_t st) {
+// Back: (1) every peer has finished reading my previous values from its footprint buffer
+// (credits back); (2) R^T + C^T: the owned ray values stored straight into the peers' footprint
+// buffers, last CTA publishes the back epoch; (3) every owner's values for my footprint have
+// arrived; (4) A_p^T (+ dot); (5) credits to every peer.  Folded: (1) in the pack kernel's
+// prologue, (3) in A_p^T's prologue, (5) from A_p^T's last CTA.
+void peer_back(Plan& P, const float* y, float* x, double* dot_out, cudaStream_t st) {
     Exchange& X = P.ex;
     const int np = P.nranks;
     unsigned long long* fl = X.flags.p();
-    // 1. every peer has finished reading my previous values from its footprint buffer
-    wait_kernel<<<1, 32, 0, st>>>(fl, np, 3 * np, 4 * np + 1, P.rank, notrap_env());
-    MX_LAUNCHED();
-    // 2. R^T + C^T: owned ray values straight into the peers' footprint buffers, flags out
-    PeerArgs pa;
-    pa.P = np;
-    pa.me = P.rank;
+    if (!X.fold) {
+        wait_kernel<<<1, 32, 0, st>>>(fl, np, 3 * np, 4 * np + 1, P.rank, notrap_env());
+        MX_LAUNCHED();
+    }
+    PeerArgs pa = base_args(P);
     for (int g = 0; g <= np; ++g) pa.bound[g] = X.rdispl[g];
     for (int g = 0; g < np; ++g) {
         pa.dst[g] = static_cast<float*>(X.peer_yfp[g]);
         pa.off[g] = X.back_off[g];
-        pa.flag[g] = static_cast<unsigned long long*>(X.peer_flags[g]);
     }
-    pa.my_flags = fl;
     pa.ticket = X.tickets.p() + 1;
     pa.slot = np;
     pa.epoch_index = 4 * np + 1;
+    pa.wait_base = 3 * np;
     pack_remote_kernel<<<nblocks(X.nrecv), kT, 0, st>>>(y, X.recv_idx.p(), X.nrecv, pa);
     MX_LAUNCHED();
-    // 3. every owner's values for my footprint have arrived
-    wait_kernel<<<1, 32, 0, st>>>(fl, np, np, 4 * np + 1, P.rank, notrap_env());
-    MX_LAUNCHED();
-    // 4. A_p^T
-    spmv_f32(P.back, X.y_fp.as<float>(), x, nullptr, nullptr, nullptr, st);
-    // 5. credits: my footprint buffer may be overwritten again
-    signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 3 * np + P.rank, fl, 4 * np + 1);
-    MX_LAUNCHED();
+    if (!X.fold) {
+        wait_kernel<<<1, 32, 0, st>>>(fl, np, np, 4 * np + 1, P.rank, notrap_env());
+        MX_LAUNCHED();
+    }
+    PeerArgs ba = base_args(P);
+    ba.ticket = X.tickets.p() + 3;
+    ba.slot = 3 * np;          // credits back in the owners' arrays
+    ba.epoch_index = 4 * np + 1;
+    ba.wait_base = np;         // arrivals back
+    spmv_f32_peer_back(P.back, X.y_fp.as<float>(), x, dot_out ? X.dot_part.p() : nullptr, dot_out,
+                       X.tickets.p() + 4, ba, st);
+    if (!X.fold) {
+        signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 3 * np + P.rank, fl, 4 * np + 1);
+        MX_LAUNCHED();
+    }
 }
 
 void peer_allreduce(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) {

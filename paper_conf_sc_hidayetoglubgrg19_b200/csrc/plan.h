@@ -91,7 +91,47 @@ struct PeerArgs {
     unsigned int* ticket = nullptr;              // last-CTA counter
     int32_t slot = 0;                            // arrival slot base in the peers' flag arrays
     int32_t epoch_index = 0;                     // this rank's epoch counter in my_flags
+    // Folded synchronisation (NCCL ranks, one GPU each): the kernel itself waits for my_flags
+    // [wait_base, wait_base + P) to reach the epoch (thread 0 of every CTA, before the data it
+    // guards is touched) and, for the back SpMV, publishes the credits from its last CTA --
+    // instead of separate one-thread wait / signal kernels.  Off for virtual ranks: P ranks'
+    // kernels share one GPU there, and CTAs spinning on every SM could keep a peer's kernel from
+    // ever being scheduled.
+    int32_t fold = 0;
+    int32_t wait_base = 0;
+    int32_t notrap = 0;
 };
+
+#ifdef __CUDACC__
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// One thread: wait until flags[base + q] >= target for q < P; after ~20 s print and trap (a peer
+// is gone) instead of hanging, unless notrap.
+__device__ inline void wait_flags(const unsigned long long* flags, int base, int P, unsigned long long target,
+                                  int me, int notrap) {
+    const long long t0 = clock64();
+    for (int q = 0; q < P; ++q) {
+        while (ld_acquire_sys(flags + base + q) < target) {
+            __nanosleep(64);
+            if (clock64() - t0 > 40000000000LL) {
+                printf("memxct peer wait timeout: rank %d base %d q %d target %llu value %llu\n", me, base, q,
+                       target, ld_acquire_sys(flags + base + q));
+                for (int i = 0; i < 4 * P + 2; ++i) printf("  rank %d flag[%d] = %llu\n", me, i, flags[i]);
+                if (notrap) return;
+                __trap();
+            }
+        }
+    }
+}
+#endif
 
 // sparse all-to-allv plan of this rank (P > 1)
 struct Exchange {
@@ -105,11 +145,17 @@ struct Exchange {
     DevBuf y_fp, recv_buf;     // footprint partials, receive / pack buffer
     DevBuf y_fp_b, recv_b;     // the same for batched (multi-slice) calls
     int32_t batch_cap = 0;
+    // dense collectives (EXCHANGE = 2): footprint partials scattered into a zeroed [P][maxown]
+    // sinogram (rank h's owned rays, Hilbert order, padded to the largest range), reduce-scatter;
+    // back: allgather of the owned values into it, gather of the footprint
+    bool dense = false;
+    int64_t maxown = 0;
+    DevArr<int32_t> dense_pos;  // nfp: position of footprint row i in the dense sinogram
+    DevBuf dense_buf, dense_own;
     // fused peer-memory exchange (EXCHANGE = 1): peers' buffers and flags mapped into this rank
     bool peer = false;
     DevArr<unsigned long long> flags;  // [4P + 2]: arrivals fwd | arrivals back | credits fwd |
                                        // credits back | my fwd epoch | my back epoch
-    DevArr<unsigned int> tickets;      // last-CTA counters of the fused kernels
     std::vector<void*> peer_recv, peer_yfp, peer_flags;
     std::vector<int64_t> fwd_off;      // owner h: my partial of footprint row i goes to recv_h[fwd_off[h] + i]
     std::vector<int64_t> back_off;     // peer g: my value j (recv order) goes to yfp_g[back_off[g] + j]
@@ -118,9 +164,14 @@ struct Exchange {
     DevArr<double> dotx;
     DevArr<unsigned long long> dflags;
     std::vector<void*> peer_dotx, peer_dflags;
+    DevArr<double> dot_part;           // per-CTA partials of the fused reduce + dot / A_p^T dot
+    DevArr<unsigned int> tickets;      // last-CTA counters: 0 A_p remote, 1 pack, 2 reduce, 3 A_p^T
+                                       // credits, 4 A_p^T dot
+    bool fold = false;                 // folded waits / signals (NCCL ranks; PeerArgs::fold)
     int64_t device_bytes() const {
         return (int64_t)(recv_idx.buf.bytes() + red_ptr.buf.bytes() + red_pos.buf.bytes() + y_fp.bytes() +
-                         recv_buf.bytes() + y_fp_b.bytes() + recv_b.bytes());
+                         recv_buf.bytes() + y_fp_b.bytes() + recv_b.bytes() + dense_pos.buf.bytes() +
+                         dense_buf.bytes() + dense_own.bytes());
     }
 };
 
@@ -225,17 +276,20 @@ void decompose(Plan& P, const Geometry& G, cudaStream_t st);
 int64_t footprint(Plan& P, const Geometry& G, DevArr<int32_t>& fp_len, cudaStream_t st);
 void shard_receive_maps(Plan& P, const Geometry& G, cudaStream_t st);
 void build_exchange(Plan& P, cudaStream_t st);
-void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st);
-void apply_back(Plan& P, const void* y, void* x, cudaStream_t st);
+// dot_out (nullable, P > 1): the CG dot of this rank's output part, fused into the last kernel
+void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st, double* dot_out = nullptr);
+void apply_back(Plan& P, const void* y, void* x, cudaStream_t st, double* dot_out = nullptr);
 void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 void time_spmv(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 double read_ceiling_gbs(int64_t bytes, int reps, cudaStream_t st);  // memxct_read_ceiling
-void reduce_partials(Plan& P, const float* recv, float* y, cudaStream_t st);
+// R (+ CG dot; pa.fold: folded arrival wait and credits, peer.cu) on the shared reduction grid
+void reduce_partials(Plan& P, const float* recv, float* y, double* dot_out, const PeerArgs& pa, cudaStream_t st);
 void preload_exchange_kernels();
 // peer.cu: fused SpMV + exchange over peer memory (EXCHANGE = 1)
 void peer_setup(Plan& P, cudaStream_t st);
-void peer_forward(Plan& P, const float* x, float* y, cudaStream_t st);
-void peer_back(Plan& P, const float* y, float* x, cudaStream_t st);
+// dot_out (nullable): <y, y> (forward) / <x, x> (back) of this rank's part, fused into the kernels
+void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream_t st);
+void peer_back(Plan& P, const float* y, float* x, double* dot_out, cudaStream_t st);
 // v[s * stride] (s < K) summed over ranks in rank order, in place, over peer memory
 void peer_allreduce(Plan& P, double* v, int K, int64_t stride, cudaStream_t st);
 // K slices, slice-major [K][local_len] fp32 vectors
@@ -249,6 +303,10 @@ void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, doubl
 void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
               unsigned int* ticket, bool canonical, cudaStream_t st);
 void spmv_f32_remote(const Layout& L, const float* x, const PeerArgs& pa, cudaStream_t st);
+// A_p^T of the fused exchange: the footprint input was stored by the owners (peer.cu); with
+// pa.fold the kernel waits for their arrival flags and its last CTA returns the credits
+void spmv_f32_peer_back(const Layout& L, const float* x, float* y, double* dot_part, double* dot_out,
+                        unsigned int* dot_ticket, const PeerArgs& pa, cudaStream_t st);
 // K in {1, 2, 4, 8} slices at once: x[s*ldx + i], y[s*ldy + r]
 void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int64_t ldy, cudaStream_t st);
 int spmm_max_slices(const Layout& L);

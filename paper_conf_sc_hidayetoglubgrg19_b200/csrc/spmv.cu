@@ -186,24 +186,31 @@ __device__ __forceinline__ void prefetch_map_l2(const int32_t* mp, int cnt) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"((unsigned)(a1 - a0)) : "memory");
 }
 
-__device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned long long v) {
-    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-
 // Fused exchange epilogue (P > 1): every footprint row's partial is stored
 // straight into its owner's receive buffer (peer memory over NVLink), then the last CTA bumps
 // this rank's forward epoch and publishes it to every owner's arrival flag (release, system
 // scope).  Replaces the separate all-to-allv of C in A = R C A_p.
+// With pa.fold the owners' credits (receive buffers consumed) are awaited here, by thread 0 of
+// every CTA before the CTA's stores, instead of by a wait kernel ahead of the SpMV: the epoch is
+// read before this CTA's ticket, so before the last CTA bumps it.  One system-scope fence per CTA
+// (after the barrier) orders all of the CTA's remote stores before its ticket.
 __device__ void remote_epilogue(const PeerArgs& pa, int64_t o, bool valid, float acc) {
     __shared__ bool am_last;
+    if (pa.fold) {
+        if (threadIdx.x == 0)
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.notrap);
+        __syncthreads();
+    }
     if (valid) {  // o = footprint position of the row
         int h = 0;
         while (h + 1 < pa.P && o >= pa.bound[h + 1]) ++h;
         pa.dst[h][pa.off[h] + o] = acc;
     }
-    __threadfence_system();
     __syncthreads();
-    if (threadIdx.x == 0) am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
+    if (threadIdx.x == 0) {
+        __threadfence_system();
+        am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
+    }
     __syncthreads();
     if (!am_last || threadIdx.x != 0) return;
     __threadfence_system();
@@ -213,11 +220,35 @@ __device__ void remote_epilogue(const PeerArgs& pa, int64_t o, bool valid, float
     *pa.ticket = 0u;
 }
 
-// kEpi: 0 = plain output, 1 = fused dot (last-CTA tree), 2 = fused exchange (remote_epilogue)
+// A_p^T of the fused exchange with pa.fold: after every CTA has finished reading the footprint
+// input, the last CTA tells every peer that its footprint buffer may be overwritten again
+// (credits, slot pa.slot + me, value = the back epoch the owners' pack kernels published).
+__device__ void peer_back_epilogue(const PeerArgs& pa) {
+    __shared__ bool am_last;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!am_last || threadIdx.x != 0) return;
+    __threadfence_system();
+    const unsigned long long e = pa.my_flags[pa.epoch_index];
+    for (int h = 0; h < pa.P; ++h) st_release_sys(pa.flag[h] + pa.slot + pa.me, e);
+    *pa.ticket = 0u;
+}
+
+// kEpi bits: 1 = fused dot (last-CTA tree), 2 = fused exchange (remote_epilogue), 4 = A_p^T of the
+// fused exchange (folded arrival wait before the first gather, credits from the last CTA)
 template <bool kNatOut, int kEpi>
 __global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, PeerArgs pa) {
     extern __shared__ __align__(16) float sbuf[];
+    if ((kEpi & 4) && pa.fold) {  // the owners' values for this footprint have arrived
+        if (threadIdx.x == 0)
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.notrap);
+        __syncthreads();
+    }
     const int64_t p = part_of_cta(a);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
@@ -267,12 +298,13 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
     const int64_t row = a.prow0[p] + threadIdx.x;
     const bool valid = row < a.prow0[p + 1];
     const int64_t o = (kNatOut && valid) ? (int64_t)a.out_idx[row] : row;
-    if (kEpi == 2) {
+    if (kEpi & 2) {
         remote_epilogue(pa, o, valid, acc);
         return;
     }
     if (valid) y[o] = acc;
-    if (kEpi == 1) finish_dot_tree<kMaxThreads>(a, valid ? (double)acc * (double)acc : 0.0);
+    if (kEpi & 1) finish_dot_tree<kMaxThreads>(a, valid ? (double)acc * (double)acc : 0.0);
+    if ((kEpi & 4) && pa.fold) peer_back_epilogue(pa);
 }
 
 // MIXED precision: fp64 stage buffer, fp64 input/output, one fp64 fma chain per row in ascending
@@ -548,6 +580,18 @@ void spmv_f32_remote(const Layout& L, const float* x, const PeerArgs& pa, cudaSt
     MX_LAUNCHED();
 }
 
+void spmv_f32_peer_back(const Layout& L, const float* x, float* y, double* dot_part, double* dot_out,
+                        unsigned int* dot_ticket, const PeerArgs& pa, cudaStream_t st) {
+    if (L.nparts == 0) fail(MEMXCT_ERR_UNSUPPORTED, "internal: empty A_p^T with the fused exchange");
+    const SpmvArgs a = make_args(L, dot_part, dot_out, dot_ticket);
+    const size_t smem = sizeof(float) * (size_t)L.B;
+    const bool nat = L.out_idx.p() != nullptr, dot = dot_out != nullptr;
+    auto kern = nat ? (dot ? spmv_f32_kernel<true, 5> : spmv_f32_kernel<true, 4>)
+                    : (dot ? spmv_f32_kernel<false, 5> : spmv_f32_kernel<false, 4>);
+    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, y, pa);
+    MX_LAUNCHED();
+}
+
 void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
               unsigned int* ticket, bool canonical, cudaStream_t st) {
     if (L.nparts == 0) return;
@@ -597,6 +641,10 @@ void spmv_init() {
     set_smem(spmv_f32_kernel<false, 0>);
     set_smem(spmv_f32_kernel<false, 2>);
     set_smem(spmv_f32_kernel<true, 2>);
+    set_smem(spmv_f32_kernel<false, 4>);
+    set_smem(spmv_f32_kernel<true, 4>);
+    set_smem(spmv_f32_kernel<false, 5>);
+    set_smem(spmv_f32_kernel<true, 5>);
     set_smem(spmv_f64_kernel<true, 0>);
     set_smem(spmv_f64_kernel<true, 1>);
     set_smem(spmv_f64_kernel<true, 2>);

@@ -210,7 +210,7 @@ class MemXCT:
                 "vector_order": {"natural": 0, "plan": 1}[vector_order], "cg_variant": cg_variant,
                 "part_rows": part_rows, "buffer_entries": buffer_entries, "tile_tomo": tile_tomo,
                 "tile_sino": tile_sino, "slices": slices, "ray_block": ray_block, "stage_order": stage_order,
-                "exchange": None if exchange is None else {"collective": 0, "peer": 1}[exchange]}
+                "exchange": None if exchange is None else {"collective": 0, "peer": 1, "dense": 2}[exchange]}
         for k, v in opts.items():
             if v is not None:
                 self.set_option(k, v)

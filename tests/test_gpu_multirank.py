@@ -134,7 +134,7 @@ def test_fp32_cg_multirank_recovers_phantom(orc, coo_cache):
     assert np.all(np.diff(res[0][1]) <= 1e-6 * res[0][1][0])
 
 
-@pytest.mark.parametrize("exchange", ["collective", "peer"])
+@pytest.mark.parametrize("exchange", ["collective", "peer", "dense"])
 def test_one_rank_nccl_communicator(orc, coo_cache, exchange):
     """The decomposed path on a real one-rank NCCL communicator (memxct_get_unique_id + set_comm
     with nranks = 1): NCCL loading, communicator init, grouped send/recv to self, allreduce,
@@ -172,3 +172,31 @@ def test_one_rank_nccl_communicator(orc, coo_cache, exchange):
     assert t["fwd_us"] > 0 and t["back_us"] > 0
     dist.close()
     plain.close()
+
+
+@pytest.mark.parametrize("nranks", [2, 3, 4])
+@pytest.mark.parametrize("prec", ["fp32", "mixed"])
+def test_dense_exchange_bit_identical_to_sparse(nranks, prec):
+    """EXCHANGE = 2 (dense reduce-scatter / allgather of the whole partial sinogram, SURVEY 8(e)'s
+    comparison) against the sparse all-to-allv + reduction R (default).  Ranks that do not touch a
+    ray contribute exact zeros and the virtual-rank sums run in rank order, which is the reduction
+    map's peer order: projections and CG iterates are bit-identical."""
+    n, m, c = 64, 90, 64
+    dt = np.float32 if prec == "fp32" else np.float64
+    gs, sparse = build_group(n, m, c, nranks, precision=prec)
+    gd, dense = build_group(n, m, c, nranks, precision=prec, exchange="dense")
+    x = inputs.uniform(n * n, 21)
+    y = inputs.uniform(m * c, 22)
+
+    def run(plans):
+        xs, ys = scatter(plans, x, 0, dt), scatter(plans, y, 1, dt)
+        fw = run_ranks(nranks, lambda r: plans[r].forward(xs[r]))
+        bk = run_ranks(nranks, lambda r: plans[r].back(ys[r]))
+        cg = run_ranks(nranks, lambda r: plans[r].cg(ys[r], 8, residuals=True))
+        return (gather(plans, fw, 1, m * c), gather(plans, bk, 0, n * n),
+                gather(plans, [v[0] for v in cg], 0, n * n), cg[0][1])
+    for a, b in zip(run(sparse), run(dense)):
+        assert np.array_equal(a, b)
+    assert dense[0].get_option("exchange") == 2
+    ex = run_ranks(nranks, lambda r: dense[r].exchange_time(3))
+    assert all(e["fwd_us"] > 0 and e["back_us"] > 0 for e in ex)
