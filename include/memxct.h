@@ -308,6 +308,16 @@ memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* par
                                    int64_t* rows, int64_t* nnz, int64_t* part_rows,
                                    int64_t* buffer_entries);
 
+/* Device-side export of the memoized matrix of direction `dir` (0 = A_p, 1 = A_p^T) as
+ * unsorted COO, one entry per stored slot: `rows`, `cols`, `vals` are caller-owned DEVICE
+ * arrays of memxct_layout_info's `slots` entries.  Entry = (output index, input index, value) in
+ * the plan's vector order (natural indices with VECTOR_ORDER = 0); padding slots are written as
+ * (-1, -1, 0).  Stream-ordered on `cuda_stream`.  For interoperability -- e.g. handing the same
+ * matrix to a library SpMV (scripts/cusparse_compare.py) -- not part of the hot path.
+ * Errors: STATE before build, INVALID_ARG for dir or NULL arrays. */
+memxct_status_t memxct_export_coo(memxct_plan_t plan, int32_t dir, int32_t* rows, int32_t* cols,
+                                  float* vals, void* cuda_stream);
+
 /* Copy the layout of partitions [p0, p1) of direction `dir` to host arrays (introspection for
  * tests; the layout is documented in DESIGN.md section 5):
  *   stage_base  int64[p1-p0+1]   global stage index range of each partition

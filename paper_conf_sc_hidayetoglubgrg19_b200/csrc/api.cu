@@ -629,6 +629,18 @@ memxct_status_t memxct_layout_export(memxct_plan_t plan, int32_t dir, int64_t p0
     });
 }
 
+memxct_status_t memxct_export_coo(memxct_plan_t plan, int32_t dir, int32_t* rows, int32_t* cols, float* vals,
+                                  void* cuda_stream) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        if (dir != 0 && dir != 1) mx::fail(MEMXCT_ERR_INVALID_ARG, "dir must be 0 or 1");
+        need(rows, "rows");
+        need(cols, "cols");
+        need(vals, "vals");
+        mx::export_coo(dir == 0 ? P.fwd : P.back, rows, cols, vals, stream_of(cuda_stream));
+    });
+}
+
 memxct_status_t memxct_layout_rows(memxct_plan_t plan, int32_t dir, int64_t* out_index) {
     return guarded([&] {
         mx::Plan& P = built_plan(plan);

@@ -282,6 +282,7 @@ void apply_back(Plan& P, const void* y, void* x, cudaStream_t st, double* dot_ou
 void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 void time_spmv(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 double read_ceiling_gbs(int64_t bytes, int reps, cudaStream_t st);  // memxct_read_ceiling
+void export_coo(const Layout& L, int32_t* rows, int32_t* cols, float* vals, cudaStream_t st);  // memxct_export_coo
 // R (+ CG dot; pa.fold: folded arrival wait and credits, peer.cu) on the shared reduction grid
 void reduce_partials(Plan& P, const float* recv, float* y, double* dot_out, const PeerArgs& pa, cudaStream_t st);
 void preload_exchange_kernels();

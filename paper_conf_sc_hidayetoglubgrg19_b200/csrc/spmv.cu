@@ -606,6 +606,52 @@ void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, dou
     MX_LAUNCHED();
 }
 
+// ---- layout export to COO on the device (memxct_export_coo) --------------------------------
+// Walks the layout exactly as spmv_f32_kernel streams it and writes, for every stored slot, its
+// output row (through out_idx: the plan's vector order), its input index (map) and its value;
+// padding slots get row -1 and value 0.  Slot s (ind position) -> entry s, so no scan is needed.
+// For interoperability (e.g. handing the memoized matrix to a library SpMV for comparison).
+__global__ void __launch_bounds__(kMaxThreads, 1)
+export_coo_kernel(SpmvArgs a, int32_t* __restrict__ rows, int32_t* __restrict__ cols, float* __restrict__ vals) {
+    const int64_t p = blockIdx.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    const int64_t g0 = a.stage_base[p], g1 = a.stage_base[p + 1];
+    const int64_t m0 = a.map_off[p];
+    const int64_t row = a.prow0[p] + threadIdx.x;
+    const bool valid = row < a.prow0[p + 1];
+    const int32_t orow = valid ? (a.out_idx ? a.out_idx[row] : (int32_t)row) : -1;
+    for (int64_t g = g0; g < g1; ++g) {
+        const int32_t* mp = a.map + m0 + (g - g0) * a.B;
+        const int64_t blk = g * a.SPP + warp;
+        const int64_t base = a.slot_off[blk];
+        const int nch = a.lane_chunks[blk * 32 + lane];
+        const int maxc = __reduce_max_sync(0xffffffffu, nch);
+        const int minc = __reduce_min_sync(0xffffffffu, nch);
+        auto emit = [&](int64_t ipos, int64_t v0pos, int64_t v1pos) {  // slot offsets within the block
+            for (int e = 0; e < 8; ++e) {
+                const int64_t s = base + ipos * 8 + e;
+                const float v = a.val[base + (e < 4 ? v0pos * 4 + e : v1pos * 4 + e - 4)];
+                const uint16_t li = a.ind[s];
+                rows[s] = v != 0.f ? orow : -1;
+                cols[s] = v != 0.f ? mp[li] : -1;
+                vals[s] = v;
+            }
+        };
+        for (int c = 0; c < minc; ++c) emit((int64_t)c * 32 + lane, (int64_t)c * 64 + lane, (int64_t)c * 64 + 32 + lane);
+        int64_t pref = (int64_t)minc * 32;
+        for (int c = minc; c < maxc; ++c) {
+            const unsigned act = __ballot_sync(0xffffffffu, nch > c);
+            const int na = __popc(act);
+            if (nch > c) {
+                const int r = __popc(act & lt);
+                emit(pref + r, 2 * pref + r, 2 * pref + na + r);
+            }
+            pref += na;
+        }
+    }
+}
+
 // ---- read-bandwidth ceiling (memxct_read_ceiling) -------------------------------------------
 // The SpMV's roofline denominator in MEASURED_PEAKS.json is a read+write copy; the matrix stream
 // is read-only.  This probe streams a buffer with the SpMV's own load (16 B ld.global.nc,
@@ -658,6 +704,13 @@ void spmv_init() {
     set_smem(spmm_f32_kernel<8, true>);
     set_smem(spmm_f32_kernel<8, false>);
     done = true;
+}
+
+void export_coo(const Layout& L, int32_t* rows, int32_t* cols, float* vals, cudaStream_t st) {
+    if (L.nparts == 0) return;
+    const SpmvArgs a = make_args(L, nullptr, nullptr, nullptr);
+    export_coo_kernel<<<(unsigned)L.nparts, L.R, 0, st>>>(a, rows, cols, vals);
+    MX_LAUNCHED();
 }
 
 double read_ceiling_gbs(int64_t bytes, int reps, cudaStream_t st) {

@@ -35,7 +35,7 @@ SYMBOLS = [
     "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
     "memxct_sirt", "memxct_spmv_time", "memxct_plan_set_shard", "memxct_exchange_counts",
     "memxct_footprint_rays", "memxct_footprint_forward", "memxct_footprint_back", "memxct_layout_rows",
-    "memxct_read_ceiling",
+    "memxct_read_ceiling", "memxct_export_coo",
 ]
 
 
@@ -106,6 +106,7 @@ def lib():
             "memxct_footprint_back": [vp, vp, vp, vp],
             "memxct_layout_rows": [vp, i32, vp],
             "memxct_read_ceiling": [i64, i32, ctypes.POINTER(ctypes.c_double), vp],
+            "memxct_export_coo": [vp, i32, vp, vp, vp, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -350,6 +351,18 @@ class MemXCT:
                "memxct_layout_info")
         return dict(zip(["parts", "stages", "slots", "map_entries", "rows", "nnz", "part_rows", "buffer_entries"],
                         [x.value for x in v]))
+
+    def export_coo(self, direction: int, stream=None):
+        """memxct_export_coo: (rows, cols, vals) device tensors, one entry per stored slot
+        (padding = (-1, -1, 0)), in the plan's vector order."""
+        import torch
+        n = self.layout_info(direction)["slots"]
+        rows = torch.empty(n, dtype=torch.int32, device="cuda")
+        cols = torch.empty(n, dtype=torch.int32, device="cuda")
+        vals = torch.empty(n, dtype=torch.float32, device="cuda")
+        _check(lib().memxct_export_coo(self._h, int(direction), _ptr(rows), _ptr(cols), _ptr(vals), _stream(stream)),
+               "memxct_export_coo")
+        return rows, cols, vals
 
     def layout_rows(self, direction: int) -> np.ndarray:
         """Output position of every layout row (memxct_layout_rows)."""

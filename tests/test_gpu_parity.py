@@ -428,3 +428,28 @@ def test_cfg3_cg_properties_full_size():
     assert errs[-1] < 0.12, errs
     true_res = float(torch.linalg.vector_norm((y - plan.forward(x30)).double()))
     assert abs(true_res - res[-1]) <= 1e-3 * res[0], (true_res, res[-1], res[0])
+
+
+@pytest.mark.parametrize("vector_order", ["natural", "plan"])
+def test_export_coo_is_the_oracle_matrix(orc, coo_cache, vector_order):
+    """memxct_export_coo (device COO of the memoized matrices, for library interop): the real
+    entries of A and A^T are exactly the oracle's pattern with its fp32-rounded lengths, in the
+    plan's vector order; padding slots come out as (-1, -1, 0)."""
+    n, m, c = 64, 90, 64
+    plan = make_plan(n, m, c, vector_order=vector_order)
+    rows, cols, vals = coo_cache(n, m, c)
+    pix = plan.local_indices(0) if vector_order == "plan" else np.arange(n * n)
+    ray = plan.local_indices(1) if vector_order == "plan" else np.arange(m * c)
+    expect = np.sort(rows.astype(np.int64) * (n * n) + cols)
+    for d in (0, 1):
+        r, cc, v = (t.cpu().numpy() for t in plan.export_coo(d))
+        assert len(r) == plan.layout_info(d)["slots"]
+        pad = r < 0
+        assert np.all(cc[pad] == -1) and np.all(v[pad] == 0) and np.all(v[~pad] != 0)
+        r, cc, v = r[~pad].astype(np.int64), cc[~pad].astype(np.int64), v[~pad]
+        ray_i, pix_i = (ray[r], pix[cc]) if d == 0 else (ray[cc], pix[r])
+        key = ray_i * (n * n) + pix_i
+        o = np.argsort(key)
+        assert np.array_equal(key[o], expect)
+        ko = np.argsort(rows.astype(np.int64) * (n * n) + cols)
+        assert np.array_equal(v[o], vals[ko].astype(np.float32))
