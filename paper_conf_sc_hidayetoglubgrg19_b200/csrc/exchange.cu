@@ -45,6 +45,13 @@ constexpr int kT = 256;
 
 unsigned nblocks(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 1 << 20)); }
 
+std::vector<int64_t> to_host_i64(const int64_t* d, int64_t n, cudaStream_t st) {
+    std::vector<int64_t> h(n);
+    MX_CUDA(cudaMemcpyAsync(h.data(), d, 8 * n, cudaMemcpyDeviceToHost, st));
+    MX_CUDA(cudaStreamSynchronize(st));
+    return h;
+}
+
 // R: owned ray i = its received partials added in peer order (reduction-map CSR ptr / pos;
 // ptr == nullptr: y[i] = recv[i], the dense exchange's owned block).  Optionally the CG dot
 // <y, y> of the owned rays: per-CTA fixed tree, the last CTA (ticket) adds the CTA partials in
@@ -261,6 +268,47 @@ void shard_receive_maps(Plan& P, const Geometry& G, cudaStream_t st) {
         MX_CUDA(cudaMemcpy(X.recv_idx.p(), idx.data(), 4 * idx.size(), cudaMemcpyHostToDevice));
 }
 
+// Forward overlap of the sparse collective exchange (SURVEY 8(e) forward steps 1-2): the
+// partitions of A_p are launched in two groups -- first every partition with a row owned by
+// another rank, then (on a lower-priority side stream, concurrently) the partitions whose rows
+// this rank owns itself -- so the all-to-allv of the remote slices starts while the self-owned
+// rows are still being computed; the self slice is copied into the receive buffer after both.
+// Launch order within each group: the layout's (partition order unless MEMXCT_PART_ORDER).
+// MEMXCT_FWD_OVERLAP=0 disables it.
+void setup_forward_overlap(Plan& P, cudaStream_t st) {
+    Exchange& X = P.ex;
+    Layout& L = P.fwd;
+    if (const char* e = std::getenv("MEMXCT_FWD_OVERLAP"); e && e[0] == '0') return;
+    const int64_t np = L.nparts;
+    if (np == 0) return;
+    const int64_t lo = X.sdispl[P.rank], hi = X.sdispl[P.rank + 1];  // my footprint slice
+    const auto row0 = to_host_i64(L.prow0.p(), np + 1, st);
+    std::vector<int32_t> pos(std::max<int64_t>(L.nrows, 1));
+    if (L.out_idx.p() && L.nrows > 0)
+        MX_CUDA(cudaMemcpy(pos.data(), L.out_idx.p(), 4 * L.nrows, cudaMemcpyDeviceToHost));
+    else
+        for (int64_t r = 0; r < L.nrows; ++r) pos[r] = (int32_t)r;
+    std::vector<int32_t> cur(np);
+    if (L.part_order.p()) MX_CUDA(cudaMemcpy(cur.data(), L.part_order.p(), 4 * np, cudaMemcpyDeviceToHost));
+    else for (int64_t b = 0; b < np; ++b) cur[b] = (int32_t)b;
+    std::vector<int32_t> first, second;
+    for (int32_t p : cur) {
+        bool self_only = true;
+        for (int64_t r = row0[p]; r < row0[p + 1] && self_only; ++r) self_only = pos[r] >= lo && pos[r] < hi;
+        (self_only ? second : first).push_back(p);
+    }
+    if (second.empty()) return;  // nothing to overlap
+    first.insert(first.end(), second.begin(), second.end());
+    L.part_order.alloc(np);
+    MX_CUDA(cudaMemcpy(L.part_order.p(), first.data(), 4 * np, cudaMemcpyHostToDevice));
+    L.n_first = np - (int64_t)second.size();
+    int lo_prio = 0, hi_prio = 0;
+    MX_CUDA(cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio));
+    MX_CUDA(cudaStreamCreateWithPriority(&X.side, cudaStreamNonBlocking, lo_prio));
+    MX_CUDA(cudaEventCreateWithFlags(&X.ev_fork, cudaEventDisableTiming));
+    MX_CUDA(cudaEventCreateWithFlags(&X.ev_join, cudaEventDisableTiming));
+}
+
 // a6: exchange maps (P > 1)
 void build_exchange(Plan& P, cudaStream_t st) {
     if (!P.dist) return;
@@ -315,6 +363,7 @@ void build_exchange(Plan& P, cudaStream_t st) {
     X.tickets.alloc(8);
     MX_CUDA(cudaMemsetAsync(X.tickets.p(), 0, 32, st));
     X.dot_part.alloc(std::max<int64_t>({P.back.nparts, (int64_t)nblocks(nown), 4 * 148}));
+    if (P.opt.exchange == 0 && !P.shard) setup_forward_overlap(P, st);
     if (P.opt.exchange == 2) {  // dense collectives: footprint row i -> [owner][owned-local index]
         X.maxown = 0;
         for (int h = 0; h < np; ++h) X.maxown = std::max(X.maxown, P.sino_bounds[h + 1] - P.sino_bounds[h]);
@@ -402,6 +451,28 @@ static void forward_t(Plan& P, const T* x, T* y, double* dot_out, cudaStream_t s
     }
     Exchange& X = P.ex;
     T* yfp = X.y_fp.as<T>();
+    if (X.side && !X.dense) {  // overlap: remote-owned partitions, then C while the self-owned ones run
+        const Layout& L = P.fwd;
+        T* rb = X.recv_buf.as<T>();
+        const DType t = sizeof(T) == 4 ? DType::F32 : DType::F64;
+        MX_CUDA(cudaEventRecord(X.ev_fork, st));
+        if constexpr (sizeof(T) == 4) spmv_f32(L, x, yfp, nullptr, nullptr, nullptr, st, 0, L.n_first);
+        else spmv_f64(L, x, yfp, nullptr, nullptr, nullptr, false, st, 0, L.n_first);
+        MX_CUDA(cudaStreamWaitEvent(X.side, X.ev_fork, 0));
+        if constexpr (sizeof(T) == 4) spmv_f32(L, x, yfp, nullptr, nullptr, nullptr, X.side, L.n_first, L.nparts);
+        else spmv_f64(L, x, yfp, nullptr, nullptr, nullptr, false, X.side, L.n_first, L.nparts);
+        MX_CUDA(cudaEventRecord(X.ev_join, X.side));
+        const int me = P.rank;
+        std::vector<int64_t> sc(X.scount), rc(X.rcount);  // the self slice moves after the join
+        sc[me] = rc[me] = 0;
+        P.comm->alltoallv(yfp, sc.data(), X.sdispl.data(), rb, rc.data(), X.rdispl.data(), t, st);  // C (remote)
+        MX_CUDA(cudaStreamWaitEvent(st, X.ev_join, 0));
+        if (X.scount[me] > 0)
+            MX_CUDA(cudaMemcpyAsync(rb + X.rdispl[me], yfp + X.sdispl[me], sizeof(T) * X.scount[me],
+                                    cudaMemcpyDeviceToDevice, st));
+        launch_reduce_dot<T>(P, rb, true, y, dot_out, PeerArgs{}, st);      // R
+        return;
+    }
     spmv_any(P, P.fwd, x, yfp, st);                                         // A_p
     exchange_fwd<T>(P, yfp, X.recv_buf.as<T>(), y, st, dot_out);            // R C
 }

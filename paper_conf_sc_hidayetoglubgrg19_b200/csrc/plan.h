@@ -47,7 +47,9 @@ struct Layout {
     DevArr<float> val;           // nslots
     DevArr<uint16_t> lane_chunks;  // nstages * SPP * 32
     DevArr<int32_t> out_idx;     // nrows, optional: output position of each row (natural order)
-    DevArr<int32_t> part_order;  // nparts, optional: partition run by CTA b (heaviest first)
+    DevArr<int32_t> part_order;  // nparts, optional: partition run by CTA b (launch order)
+    int64_t n_first = -1;        // P > 1 forward: the first n_first CTAs hold every partition with
+                                 // rows owned by other ranks (exchange overlap), else -1
     int64_t device_bytes() const {
         return (int64_t)(prow0.buf.bytes() + stage_base.buf.bytes() + map_off.buf.bytes() + map.buf.bytes() +
                          slot_off.buf.bytes() + ind.buf.bytes() + val.buf.bytes() +
@@ -168,6 +170,14 @@ struct Exchange {
     DevArr<unsigned int> tickets;      // last-CTA counters: 0 A_p remote, 1 pack, 2 reduce, 3 A_p^T
                                        // credits, 4 A_p^T dot
     bool fold = false;                 // folded waits / signals (NCCL ranks; PeerArgs::fold)
+    // forward overlap (sparse collective exchange): side stream for the self-owned partitions
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    ~Exchange() {
+        if (ev_fork) cudaEventDestroy(ev_fork);
+        if (ev_join) cudaEventDestroy(ev_join);
+        if (side) cudaStreamDestroy(side);
+    }
     int64_t device_bytes() const {
         return (int64_t)(recv_idx.buf.bytes() + red_ptr.buf.bytes() + red_pos.buf.bytes() + y_fp.bytes() +
                          recv_buf.bytes() + y_fp_b.bytes() + recv_b.bytes() + dense_pos.buf.bytes() +
@@ -299,10 +309,12 @@ void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st)
 
 // spmv.cu
 void spmv_init();
+// [c0, c1): the CTAs (launch-order positions, Layout::part_order) to run; c1 < 0 = all.  A
+// fused dot needs the whole launch.
 void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, double* dot_out,
-              unsigned int* ticket, cudaStream_t st);
+              unsigned int* ticket, cudaStream_t st, int64_t c0 = 0, int64_t c1 = -1);
 void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
-              unsigned int* ticket, bool canonical, cudaStream_t st);
+              unsigned int* ticket, bool canonical, cudaStream_t st, int64_t c0 = 0, int64_t c1 = -1);
 void spmv_f32_remote(const Layout& L, const float* x, const PeerArgs& pa, cudaStream_t st);
 // A_p^T of the fused exchange: the footprint input was stored by the owners (peer.cu); with
 // pa.fold the kernel waits for their arrival flags and its last CTA returns the credits

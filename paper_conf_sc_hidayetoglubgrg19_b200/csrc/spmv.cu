@@ -77,7 +77,8 @@ struct SpmvArgs {
     const uint16_t* lane_chunks;
     const int32_t* out_idx;
     const int64_t* prow0;  // first row of each partition (nparts + 1)
-    const int32_t* order;  // nullable: partition of CTA b (launch order, heaviest first)
+    const int32_t* order;  // nullable: partition of CTA b (launch order)
+    int64_t cta_base;      // launch-order position of this launch's CTA 0
     int64_t nrows;
     int64_t nparts;
     int32_t R, SPP, B;
@@ -92,7 +93,8 @@ struct SpmvArgs {
 // Per-partition results (rows, dot partials) are indexed by partition, so the order changes no
 // result.
 __device__ __forceinline__ int64_t part_of_cta(const SpmvArgs& a) {
-    return a.order ? (int64_t)__ldg(a.order + blockIdx.x) : (int64_t)blockIdx.x;
+    const int64_t b = a.cta_base + blockIdx.x;
+    return a.order ? (int64_t)__ldg(a.order + b) : b;
 }
 
 // deterministic last-CTA reduction of the per-CTA partials, in partition order
@@ -395,6 +397,7 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.out_idx = L.out_idx.p();
     a.prow0 = L.prow0.p();
     a.order = L.part_order.p();
+    a.cta_base = 0;
     a.nrows = L.nrows;
     a.nparts = L.nparts;
     a.R = L.R;
@@ -560,14 +563,17 @@ void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int
 }
 
 void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, double* dot_out,
-              unsigned int* ticket, cudaStream_t st) {
-    if (L.nparts == 0) return;
-    const SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
+              unsigned int* ticket, cudaStream_t st, int64_t c0, int64_t c1) {
+    if (c1 < 0) c1 = L.nparts;
+    if (c1 <= c0) return;
+    if (dot_out && (c0 != 0 || c1 != L.nparts)) fail(MEMXCT_ERR_UNSUPPORTED, "internal: fused dot on a partial launch");
+    SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
+    a.cta_base = c0;
     const size_t smem = sizeof(float) * (size_t)L.B;
     const bool nat = L.out_idx.p() != nullptr, dot = dot_out != nullptr;
     auto kern = nat ? (dot ? spmv_f32_kernel<true, 1> : spmv_f32_kernel<true, 0>)
                     : (dot ? spmv_f32_kernel<false, 1> : spmv_f32_kernel<false, 0>);
-    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, y, PeerArgs{});
+    kern<<<(unsigned)(c1 - c0), L.R, smem, st>>>(a, x, y, PeerArgs{});
     MX_LAUNCHED();
 }
 
@@ -593,16 +599,19 @@ void spmv_f32_peer_back(const Layout& L, const float* x, float* y, double* dot_p
 }
 
 void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
-              unsigned int* ticket, bool canonical, cudaStream_t st) {
-    if (L.nparts == 0) return;
-    const SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
+              unsigned int* ticket, bool canonical, cudaStream_t st, int64_t c0, int64_t c1) {
+    if (c1 < 0) c1 = L.nparts;
+    if (c1 <= c0) return;
+    if (dot_out && (c0 != 0 || c1 != L.nparts)) fail(MEMXCT_ERR_UNSUPPORTED, "internal: fused dot on a partial launch");
+    SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
+    a.cta_base = c0;
     const size_t smem = sizeof(double) * (size_t)std::max(L.B, L.R);
     const bool nat = L.out_idx.p() != nullptr;
     const int mode = dot_out == nullptr ? 0 : (canonical ? 2 : 1);
     void (*kern)(SpmvArgs, const double*, double*);
     if (nat) kern = mode == 0 ? spmv_f64_kernel<true, 0> : mode == 1 ? spmv_f64_kernel<true, 1> : spmv_f64_kernel<true, 2>;
     else kern = mode == 0 ? spmv_f64_kernel<false, 0> : mode == 1 ? spmv_f64_kernel<false, 1> : spmv_f64_kernel<false, 2>;
-    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, y);
+    kern<<<(unsigned)(c1 - c0), L.R, smem, st>>>(a, x, y);
     MX_LAUNCHED();
 }
 

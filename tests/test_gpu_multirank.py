@@ -200,3 +200,25 @@ def test_dense_exchange_bit_identical_to_sparse(nranks, prec):
     assert dense[0].get_option("exchange") == 2
     ex = run_ranks(nranks, lambda r: dense[r].exchange_time(3))
     assert all(e["fwd_us"] > 0 and e["back_us"] > 0 for e in ex)
+
+
+@pytest.mark.parametrize("nranks", [2, 3, 4])
+def test_forward_overlap_bit_identical(monkeypatch, nranks):
+    """Sparse collective exchange with the forward overlap (default: partitions holding rows of
+    other owners first, the self-owned partitions concurrently on a side stream while the
+    all-to-allv runs, the self slice copied after the join) against MEMXCT_FWD_OVERLAP=0: the
+    same kernels write the same partials, so projections and CG are bit-identical."""
+    n, m, c = 256, 360, 256
+    _, on = build_group(n, m, c, nranks)
+    monkeypatch.setenv("MEMXCT_FWD_OVERLAP", "0")
+    _, off = build_group(n, m, c, nranks)
+    x = inputs.uniform(n * n, 31)
+    y = inputs.uniform(m * c, 32)
+
+    def run(plans):
+        xs, ys = scatter(plans, x, 0, np.float32), scatter(plans, y, 1, np.float32)
+        fw = run_ranks(nranks, lambda r: plans[r].forward(xs[r]))
+        cg = run_ranks(nranks, lambda r: plans[r].cg(ys[r], 6))
+        return gather(plans, fw, 1, m * c), gather(plans, cg, 0, n * n)
+    for a, b in zip(run(on), run(off)):
+        assert np.array_equal(a, b)
