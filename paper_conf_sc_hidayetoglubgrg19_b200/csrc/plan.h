@@ -173,6 +173,9 @@ struct Exchange {
     // forward overlap (sparse collective exchange): side stream for the self-owned partitions
     cudaStream_t side = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    Exchange() = default;
+    Exchange(const Exchange&) = delete;
+    Exchange& operator=(const Exchange&) = delete;
     ~Exchange() {
         if (ev_fork) cudaEventDestroy(ev_fork);
         if (ev_join) cudaEventDestroy(ev_join);
