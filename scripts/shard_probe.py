@@ -29,6 +29,7 @@ def main():
     ap.add_argument("--which", default="all")
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--ray-block", default="0", help="comma list of MEMXCT_OPT_RAY_BLOCK values (0 = auto)")
+    ap.add_argument("--part-rows", default="0", help="comma list of MEMXCT_OPT_PART_ROWS values (0 = auto)")
     args = ap.parse_args()
     import torch
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, inputs
@@ -36,11 +37,13 @@ def main():
     P = args.ranks
     which = range(P) if args.which == "all" else [int(v) for v in args.which.split(",")]
     rows = []
-    cases = [(r, rb) for r in which for rb in [int(v) for v in args.ray_block.split(",")]]
-    for r, rb in cases:
+    cases = [(r, rb, pr) for r in which for rb in [int(v) for v in args.ray_block.split(",")]
+             for pr in [int(v) for v in args.part_rows.split(",")]]
+    for r, rb, pr in cases:
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        sp = MemXCT(n, m, c, rank=r, nranks=P, shard=True, vector_order="plan", ray_block=rb).build()
+        sp = MemXCT(n, m, c, rank=r, nranks=P, shard=True, vector_order="plan", ray_block=rb,
+                    part_rows=pr or None).build()
         torch.cuda.synchronize()
         build_s = time.perf_counter() - t0
         t = sp.spmv_time(args.reps)
