@@ -197,7 +197,7 @@ def run_reference(args, rank, world):
     line = {
         "impl": "reference", "metric": "CG iter/s", "value": value, "unit": "CG iter/s",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True, "scaling": "weak",
+        "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": workload_name(cfg, args.iters) + " (oracle: 2% ray sample, "
                    "forward + back SpMV per step, extrapolated to full nnz)"},
