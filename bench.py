@@ -320,9 +320,9 @@ def bench_exchange_variant(args, rank, world, kind):
     cmd = [sys.executable, os.path.abspath(__file__), "--variant", kind, "--config", str(args.config),
            "--iters", str(args.iters), "--steps", str(args.steps), "--warmup", str(args.warmup)]
     try:
-        r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=900)
+        r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=300)
     except subprocess.TimeoutExpired:
-        return {"error": "timed out after 900 s"}
+        return {"error": "timed out after 300 s"}
     if rank != 0:
         return None
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]

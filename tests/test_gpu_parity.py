@@ -317,17 +317,23 @@ def test_degenerate_geometries(orc):
 
 
 @pytest.mark.slow
-def test_cfg3_sampled_rows(orc):
-    """Full size (BASELINE configs[2]), the launch configuration bench.py times: 2000 sampled
-    rays of y = A x and 12 sampled pixels of x = A^T y, each against the oracle's own trace."""
-    n, m, c = inputs.CONFIGS[3]
+@pytest.mark.parametrize("cfg", [3, 4])
+def test_full_size_sampled_rows(orc, cfg):
+    """Full size: config 3 (BASELINE configs[2], the launch configuration bench.py times) and
+    config 4 (configs[3], 2048^2 x 2400 x 2048, 1.2e10 nonzeros per direction: its one-GPU fit,
+    ~150 GB): 2000 sampled rays of y = A x and 12 sampled pixels of x = A^T y, each against the
+    oracle's own trace."""
+    import gc
+    gc.collect()                       # earlier tests' plans release their device memory
+    torch.cuda.empty_cache()
+    n, m, c = inputs.CONFIGS[cfg]
     plan = make_plan(n, m, c)
     st = plan.stats()
     assert abs(st["nnz"] / (m * n * n) - 1.1953) < 2e-3
-    x = torch.from_numpy(inputs.uniform(n * n, inputs.seed_for(3))).cuda()
+    x = torch.from_numpy(inputs.uniform(n * n, inputs.seed_for(cfg))).cuda()
     y = plan.forward(x).cpu().numpy()
     xh = x.cpu().numpy().astype(np.float64)
-    rng = np.random.default_rng(3)
+    rng = np.random.default_rng(cfg)
     rays = rng.choice(m * c, 2000, replace=False)
     got, exp = [], []
     for r in rays:
@@ -335,7 +341,7 @@ def test_cfg3_sampled_rows(orc):
         got.append(y[r])
         exp.append(float(ln @ xh[pix]))
     assert rel_l2(np.array(got), np.array(exp)) <= 1e-5
-    ysino = torch.from_numpy(inputs.uniform(m * c, inputs.seed_for(3) + 1)).cuda()
+    ysino = torch.from_numpy(inputs.uniform(m * c, inputs.seed_for(cfg) + 1)).cuda()
     xb = plan.back(ysino).cpu().numpy()
     yh = ysino.cpu().numpy().astype(np.float64)
     pixels = rng.choice(n * n, 12, replace=False)
@@ -343,6 +349,7 @@ def test_cfg3_sampled_rows(orc):
     for p, (rr, ll) in zip(pixels, orc.sampled_back_rows(n, m, c, pixels)):
         got.append(xb[p])
         exp.append(float(ll @ yh[rr]))
+    plan.close()
     assert rel_l2(np.array(got), np.array(exp)) <= 1e-5
 
 
