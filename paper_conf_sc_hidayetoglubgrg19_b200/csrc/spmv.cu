@@ -188,6 +188,42 @@ __device__ __forceinline__ void prefetch_map_l2(const int32_t* mp, int cnt) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"((unsigned)(a1 - a0)) : "memory");
 }
 
+// One warp's slots of stage g (its 32-row slice block): acc += buf[ind] * val, streamed with
+// 16 B evict-first loads (6 B per nonzero from HBM).
+__device__ __forceinline__ void stream_stage(float& acc, const float* __restrict__ sbuf, const SpmvArgs& a,
+                                             int64_t g, int warp, int lane, unsigned lt, uint64_t pol) {
+    const int64_t blk = g * a.SPP + warp;
+    const int64_t base = a.slot_off[blk];
+    const int nch = a.lane_chunks[blk * 32 + lane];
+    const int maxc = __reduce_max_sync(0xffffffffu, nch);
+    const uint4* ib = reinterpret_cast<const uint4*>(a.ind + base);
+    const float4* vb = reinterpret_cast<const float4*>(a.val + base);
+    // phase 1: chunks every lane has -- plain SELL addressing, branch-free, unrolled so
+    // several 16 B loads per lane are in flight
+    const int minc = __reduce_min_sync(0xffffffffu, nch);
+#pragma unroll 4
+    for (int c = 0; c < minc; ++c) {
+        const uint4 iv = ld_stream_u4(ib + c * 32 + lane, pol);
+        const float4 v0 = ld_stream_f4(vb + c * 64 + lane, pol);
+        const float4 v1 = ld_stream_f4(vb + c * 64 + 32 + lane, pol);
+        fma8(acc, sbuf, iv, v0, v1);
+    }
+    // phase 2: the ragged tail, stored only for the lanes that have it (jagged SELL)
+    int64_t pref = (int64_t)minc * 32;
+    for (int c = minc; c < maxc; ++c) {
+        const unsigned act = __ballot_sync(0xffffffffu, nch > c);
+        const int na = __popc(act);
+        if (nch > c) {
+            const int r = __popc(act & lt);
+            const uint4 iv = ld_stream_u4(ib + pref + r, pol);
+            const float4 v0 = ld_stream_f4(vb + 2 * pref + r, pol);
+            const float4 v1 = ld_stream_f4(vb + 2 * pref + na + r, pol);
+            fma8(acc, sbuf, iv, v0, v1);
+        }
+        pref += na;
+    }
+}
+
 // Fused exchange epilogue (P > 1): every footprint row's partial is stored
 // straight into its owner's receive buffer (peer memory over NVLink), then the last CTA bumps
 // this rank's forward epoch and publishes it to every owner's arrival flag (release, system
@@ -266,36 +302,7 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
         if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B));
         stage_gather<16>(sbuf, x, mp, cnt);
         __syncthreads();
-        const int64_t blk = g * a.SPP + warp;
-        const int64_t base = a.slot_off[blk];
-        const int nch = a.lane_chunks[blk * 32 + lane];
-        const int maxc = __reduce_max_sync(0xffffffffu, nch);
-        const uint4* ib = reinterpret_cast<const uint4*>(a.ind + base);
-        const float4* vb = reinterpret_cast<const float4*>(a.val + base);
-        // phase 1: chunks every lane has -- plain SELL addressing, branch-free, unrolled so
-        // several 16 B loads per lane are in flight
-        const int minc = __reduce_min_sync(0xffffffffu, nch);
-#pragma unroll 4
-        for (int c = 0; c < minc; ++c) {
-            const uint4 iv = ld_stream_u4(ib + c * 32 + lane, pol);
-            const float4 v0 = ld_stream_f4(vb + c * 64 + lane, pol);
-            const float4 v1 = ld_stream_f4(vb + c * 64 + 32 + lane, pol);
-            fma8(acc, sbuf, iv, v0, v1);
-        }
-        // phase 2: the ragged tail, stored only for the lanes that have it (jagged SELL)
-        int64_t pref = (int64_t)minc * 32;
-        for (int c = minc; c < maxc; ++c) {
-            const unsigned act = __ballot_sync(0xffffffffu, nch > c);
-            const int na = __popc(act);
-            if (nch > c) {
-                const int r = __popc(act & lt);
-                const uint4 iv = ld_stream_u4(ib + pref + r, pol);
-                const float4 v0 = ld_stream_f4(vb + 2 * pref + r, pol);
-                const float4 v1 = ld_stream_f4(vb + 2 * pref + na + r, pol);
-                fma8(acc, sbuf, iv, v0, v1);
-            }
-            pref += na;
-        }
+        stream_stage(acc, sbuf, a, g, warp, lane, lt, pol);
     }
     const int64_t row = a.prow0[p] + threadIdx.x;
     const bool valid = row < a.prow0[p + 1];
@@ -569,8 +576,8 @@ void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, doubl
     if (dot_out && (c0 != 0 || c1 != L.nparts)) fail(MEMXCT_ERR_UNSUPPORTED, "internal: fused dot on a partial launch");
     SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
     a.cta_base = c0;
-    const size_t smem = sizeof(float) * (size_t)L.B;
     const bool nat = L.out_idx.p() != nullptr, dot = dot_out != nullptr;
+    const size_t smem = sizeof(float) * (size_t)L.B;
     auto kern = nat ? (dot ? spmv_f32_kernel<true, 1> : spmv_f32_kernel<true, 0>)
                     : (dot ? spmv_f32_kernel<false, 1> : spmv_f32_kernel<false, 0>);
     kern<<<(unsigned)(c1 - c0), L.R, smem, st>>>(a, x, y, PeerArgs{});
