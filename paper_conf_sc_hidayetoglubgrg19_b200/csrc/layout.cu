@@ -625,6 +625,17 @@ void set_part_order(Layout& L, const std::vector<int64_t>& row0, const std::vect
 //    more CG iter/s than 256.
 //  * B (stage buffer entries): 36 fp32 entries per row for one slice (144 KB at R = 1024); for
 //    k-slice plans 192 KB of k-wide entries (a 200 KB buffer leaves 28 KB of L1 for the gathers).
+// Drifting stages (spmv_f32_drift_kernel): MEMXCT_DRIFT=1 selects it, MEMXCT_DRIFT_B sets its
+// auto stage size (3 buffers of B entries share the CTA's shared memory).
+static bool drift_requested() {
+    const char* e = std::getenv("MEMXCT_DRIFT");
+    return e && atoi(e) != 0;
+}
+static int32_t drift_auto_b() {
+    const char* e = std::getenv("MEMXCT_DRIFT_B");
+    return e ? std::max(256, atoi(e)) : 16384;
+}
+
 void resolve_tuning(const Plan& P, int64_t rows, int32_t* R_out, int32_t* B_out) {
     int dev = 0, sms = 148;
     MX_CUDA(cudaGetDevice(&dev));
@@ -647,7 +658,8 @@ void resolve_tuning(const Plan& P, int64_t rows, int32_t* R_out, int32_t* B_out)
     if (B == 0) {
         int32_t k = 1;
         while (k < P.opt.slices) k *= 2;  // batched calls stage k slices per buffer entry
-        B = (k == 1) ? std::min<int32_t>(57344, 36 * R) : std::min<int32_t>(49152, 144 * R) / k;
+        B = (k == 1) ? std::min<int32_t>(drift_requested() ? drift_auto_b() : 57344, 36 * R)
+                     : std::min<int32_t>(49152, 144 * R) / k;
         B = std::max<int32_t>(256, B - B % 256);
     }
     *R_out = R;
@@ -676,6 +688,7 @@ void build_direction(Layout& L, int64_t nrows, int64_t ncols, const Partitions& 
     L.B = B;
     L.nparts = (int64_t)parts.row0.size() - 1;
     L.balanced = parts.balanced;
+    L.drift = drift_requested() && 12 * (int64_t)B <= 224 * 1024;
     L.bank_ordered = bank_classes > 0;
     const int64_t nparts = L.nparts;
     const std::vector<int64_t>& part_nnz = parts.nnz;
@@ -987,6 +1000,17 @@ void build_matrices(Plan& P, cudaStream_t st) {
     // forward rows grouped into projection x channel blocks (MEMXCT_OPT_RAY_BLOCK), or the
     // footprint's Hilbert order; the A_p^T build below keeps the footprint order for its columns
     P.ray_block = resolve_ray_block(P, npix, R);
+    // drifting stages (spmv_f32_drift_kernel) for the forward operator of projection-block plans:
+    // three stage buffers of 16384 entries instead of one of 36 R.  Config-5 shard forward 7.99 ->
+    // 7.73 ms although the smaller stages add 2.2 % slab padding; the balanced back operator and
+    // the Hilbert-row geometries (configs 1-4) gain nothing and keep the plain kernel
+    // (profiles/r01i_drift_*.jsonl).  MEMXCT_DRIFT=1 forces it for both directions.
+    const bool fwd_drift = drift_requested() || (P.ray_block > 0 && P.opt.buffer_entries == 0 &&
+                                                 P.opt.precision == 0 && P.opt.slices <= 1);
+    if (fwd_drift && P.opt.buffer_entries == 0) {
+        B = std::min(B, drift_auto_b());
+        P.buffer_entries = B;
+    }
     DevArr<int32_t> hray_b, len_b, out_b;
     const int32_t* fwd_hray = hray;
     const int32_t* fwd_len = fp_len.p();
@@ -1131,6 +1155,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
     };
     build_direction(P.fwd, nrows, npix, fwd_parts, R, B, gen_fwd, natural ? P.tomo_nat_of_h.p() : nullptr,
                     fwd_out, budget, bank, st, kinv.p(), part_class.p());
+    P.fwd.drift = fwd_drift && 12 * (int64_t)B <= 224 * 1024;
     kfwd.reset();
     kinv.reset();
     part_class.reset();

@@ -38,6 +38,7 @@ struct Layout {
     int32_t max_stages = 0;
     bool bank_ordered = false;   // runs in bank-aware order instead of ascending local index
     bool balanced = false;       // partitions cut for equal work (else fixed R rows each)
+    bool drift = false;          // FP32 single-slice launches use spmv_f32_drift_kernel
     DevArr<int64_t> prow0;       // nparts + 1: first row of each partition (<= R rows each)
     DevArr<int64_t> stage_base;  // nparts + 1
     DevArr<int64_t> map_off;     // nparts + 1

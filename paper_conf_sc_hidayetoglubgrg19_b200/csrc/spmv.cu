@@ -316,6 +316,77 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
     if ((kEpi & 4) && pa.fold) peer_back_epilogue(pa);
 }
 
+// ---- drifting stages (Layout::drift) ------------------------------------------------------------
+// The plain kernel ends every stage with a CTA barrier, so all 32 warps wait for the warp with
+// the most slots in that stage (config-5 shard forward: 0.84 barrier efficiency, ncu "barrier"
+// stalls 4x the back operator's, profiles/r01i_cfg5_forward.md).  Here three stage buffers
+// rotate and two mbarrier rings replace the barrier: full[b] completes when every thread has
+// gathered its share of the stage in buffer b, done[b] when every thread has streamed it.  After
+// streaming stage s a thread waits only for done of stage s-1 (whose buffer stage s+2 reuses),
+// gathers its share of stage s+2 and moves on, so warps drift up to about one stage apart and a
+// warp that is heavy in one stage catches up in the next.  Same layout, same per-row fma order:
+// bit-identical to spmv_f32_kernel for the same stage size B.
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* b, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
+    const uint32_t a = smem_addr(b);
+    const long long t0 = clock64();
+    for (;;) {
+        uint32_t ok;
+        asm volatile("{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+                     "selp.u32 %0, 1, 0, P;\n\t}"
+                     : "=r"(ok) : "r"(a), "r"(parity) : "memory");
+        if (ok) return;
+        if (clock64() - t0 > 20000000000LL) __trap();  // ~10 s: a broken phase, not a slow stage
+    }
+}
+
+template <bool kNatOut, int kEpi>
+__global__ void __launch_bounds__(kMaxThreads, 1)
+spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) {
+    extern __shared__ __align__(16) float sbuf[];  // [3][B]
+    __shared__ __align__(8) uint64_t full[3], done[3];
+    if (threadIdx.x == 0)
+        for (int b = 0; b < 3; ++b) {
+            mbar_init(&full[b], blockDim.x);
+            mbar_init(&done[b], blockDim.x);
+        }
+    __syncthreads();
+    const int64_t p = part_of_cta(a);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    const int64_t g0 = a.stage_base[p], ns = a.stage_base[p + 1] - g0;
+    const int64_t m0 = a.map_off[p], D = a.map_off[p + 1] - m0;
+    const uint64_t pol = evict_first_policy();
+    auto gather = [&](int64_t s) {  // this thread's share of stage s into buffer s % 3
+        const int cnt = (int)min((int64_t)a.B, D - s * a.B);
+        stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt);
+        mbar_arrive(&full[s % 3]);
+    };
+    if (ns > 0) gather(0);
+    if (ns > 1) gather(1);
+    float acc = 0.f;
+    for (int64_t s = 0; s < ns; ++s) {
+        mbar_wait(&full[s % 3], (unsigned)((s / 3) & 1));
+        stream_stage(acc, sbuf + (s % 3) * a.B, a, g0 + s, warp, lane, lt, pol);
+        mbar_arrive(&done[s % 3]);
+        if (s + 2 < ns) {
+            if (s >= 1) mbar_wait(&done[(s + 2) % 3], (unsigned)(((s - 1) / 3) & 1));
+            gather(s + 2);
+        }
+    }
+    const int64_t row = a.prow0[p] + threadIdx.x;
+    const bool valid = row < a.prow0[p + 1];
+    const int64_t o = (kNatOut && valid) ? (int64_t)a.out_idx[row] : row;
+    if (valid) y[o] = acc;
+    if (kEpi & 1) finish_dot_tree<kMaxThreads>(a, valid ? (double)acc * (double)acc : 0.0);
+}
+
 // MIXED precision: fp64 stage buffer, fp64 input/output, one fp64 fma chain per row in ascending
 // Hilbert input order (stages ascend, slots within a stage ascend by local index; padding slots
 // are fma(0, finite, acc) = acc).  This is the canonical row sum of reading R16.
@@ -577,6 +648,14 @@ void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, doubl
     SpmvArgs a = make_args(L, dot_part, dot_out, ticket);
     a.cta_base = c0;
     const bool nat = L.out_idx.p() != nullptr, dot = dot_out != nullptr;
+    if (L.drift) {
+        const size_t smem = 3 * sizeof(float) * (size_t)L.B;
+        auto kern = nat ? (dot ? spmv_f32_drift_kernel<true, 1> : spmv_f32_drift_kernel<true, 0>)
+                        : (dot ? spmv_f32_drift_kernel<false, 1> : spmv_f32_drift_kernel<false, 0>);
+        kern<<<(unsigned)(c1 - c0), L.R, smem, st>>>(a, x, y);
+        MX_LAUNCHED();
+        return;
+    }
     const size_t smem = sizeof(float) * (size_t)L.B;
     auto kern = nat ? (dot ? spmv_f32_kernel<true, 1> : spmv_f32_kernel<true, 0>)
                     : (dot ? spmv_f32_kernel<false, 1> : spmv_f32_kernel<false, 0>);
@@ -697,6 +776,10 @@ __global__ void __launch_bounds__(1024) read_probe_kernel(const uint4* __restric
 void spmv_init() {
     static bool done = false;
     if (done) return;
+    set_smem(spmv_f32_drift_kernel<true, 1>);
+    set_smem(spmv_f32_drift_kernel<true, 0>);
+    set_smem(spmv_f32_drift_kernel<false, 1>);
+    set_smem(spmv_f32_drift_kernel<false, 0>);
     set_smem(spmv_f32_kernel<true, 1>);
     set_smem(spmv_f32_kernel<true, 0>);
     set_smem(spmv_f32_kernel<false, 1>);
