@@ -320,8 +320,8 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
 // The plain kernel ends every stage with a CTA barrier, so all 32 warps wait for the warp with
 // the most slots in that stage (config-5 shard forward: 0.84 barrier efficiency, ncu "barrier"
 // stalls 4x the back operator's, profiles/r01i_cfg5_forward.md).  Here three stage buffers
-// rotate and two mbarrier rings replace the barrier: full[b] completes when every thread has
-// gathered its share of the stage in buffer b, done[b] when every thread has streamed it.  After
+// rotate and two mbarrier rings replace the barrier: full[b] completes when every warp has
+// gathered its share of the stage in buffer b, done[b] when every warp has streamed it.  After
 // streaming stage s a thread waits only for done of stage s-1 (whose buffer stage s+2 reuses),
 // gathers its share of stage s+2 and moves on, so warps drift up to about one stage apart and a
 // warp that is heavy in one stage catches up in the next.  Same layout, same per-row fma order:
@@ -351,10 +351,10 @@ __global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) {
     extern __shared__ __align__(16) float sbuf[];  // [3][B]
     __shared__ __align__(8) uint64_t full[3], done[3];
-    if (threadIdx.x == 0)
+    if (threadIdx.x == 0)  // one arrival per warp (after __syncwarp, which orders the lanes' accesses)
         for (int b = 0; b < 3; ++b) {
-            mbar_init(&full[b], blockDim.x);
-            mbar_init(&done[b], blockDim.x);
+            mbar_init(&full[b], blockDim.x >> 5);
+            mbar_init(&done[b], blockDim.x >> 5);
         }
     __syncthreads();
     const int64_t p = part_of_cta(a);
@@ -366,7 +366,8 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     auto gather = [&](int64_t s) {  // this thread's share of stage s into buffer s % 3
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
         stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt);
-        mbar_arrive(&full[s % 3]);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&full[s % 3]);
     };
     if (ns > 0) gather(0);
     if (ns > 1) gather(1);
@@ -374,7 +375,8 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     for (int64_t s = 0; s < ns; ++s) {
         mbar_wait(&full[s % 3], (unsigned)((s / 3) & 1));
         stream_stage(acc, sbuf + (s % 3) * a.B, a, g0 + s, warp, lane, lt, pol);
-        mbar_arrive(&done[s % 3]);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&done[s % 3]);
         if (s + 2 < ns) {
             if (s >= 1) mbar_wait(&done[(s + 2) % 3], (unsigned)(((s - 1) / 3) & 1));
             gather(s + 2);
