@@ -494,6 +494,11 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
 // slices' inputs interleaved ([B][K] fp32), so every slot read from HBM feeds K fmas and one
 // matrix stream serves K slices.  Each slice's fma sequence is exactly the single-slice kernel's,
 // so every slice's result is bit-identical to spmv_f32 on the same plan.
+#ifndef MEMXCT_SPMM_GATHER_LOADS
+#define MEMXCT_SPMM_GATHER_LOADS 8
+#endif
+constexpr int kSpmmGatherLoads = MEMXCT_SPMM_GATHER_LOADS;  // stage-gather input loads in flight per thread
+
 template <int K>
 __device__ __forceinline__ void load_k(const float* __restrict__ buf, uint32_t i, float (&b)[K]) {
     if constexpr (K == 2) {
@@ -549,7 +554,7 @@ spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __r
         const int32_t* __restrict__ mp = a.map + m0 + st * a.B;
         if (g != g0) __syncthreads();
         if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (st + 1) * a.B));
-        constexpr int U = K >= 8 ? 1 : 8 / K;  // 8 input loads in flight per thread (stage_gather)
+        constexpr int U = K >= kSpmmGatherLoads ? 1 : kSpmmGatherLoads / K;  // input loads in flight per thread
         const int bd = blockDim.x;
         for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
             int64_t col[U];
