@@ -29,7 +29,7 @@ int64_t Plan::device_bytes() const {
                      sino_h_of_nat.buf.bytes() + cg_r.bytes() + cg_q.bytes() + cg_s.bytes() + cg_p.bytes() +
                      cg_ax.bytes() + part_fwd.buf.bytes() + part_back.buf.bytes() + part_vec.buf.bytes() +
                      scal.buf.bytes() + tickets.buf.bytes() + h_in.bytes() + h_out.bytes() +
-                     fp_rays.buf.bytes()) +
+                     fp_rays.buf.bytes() + spmm_xi.bytes()) +
            ex.device_bytes();
 }
 

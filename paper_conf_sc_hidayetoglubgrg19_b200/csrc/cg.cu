@@ -312,6 +312,7 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, int32_t K, cudaStrea
         P.scal.alloc(nd);
         MX_CUDA(cudaMemsetAsync(P.scal.p(), 0, 8 * nd, st));
     }
+    if (K > 1) prepare_batch_scratch(P, st);
     if (P.dist && !P.comm->capturable()) {  // virtual ranks: eager launches
         cg_enqueue_any(P, y, x, iters, K, st);
         return;

@@ -502,30 +502,55 @@ int group_size(const Plan& P, int remaining) {
     return k;
 }
 
-void ensure_batch_buffers(Plan& P, int k) {
+// Sized for the largest group (not the call's), so a buffer allocated here never moves under a
+// graph captured by an earlier call with fewer slices.
+void ensure_batch_scratch(Plan& P) {
+    const int kmax = group_size(P, 8);
+    if (kmax <= 1) return;
+    const int64_t ncols = std::max({P.fwd.ncols, P.back.ncols, (int64_t)1});
+    const size_t xi_bytes = sizeof(float) * (size_t)ncols * kmax;
+    if (P.spmm_xi.bytes() < xi_bytes) P.spmm_xi.alloc(xi_bytes);
     Exchange& X = P.ex;
-    if (k <= X.batch_cap) return;
-    X.y_fp_b.alloc(sizeof(float) * std::max<int64_t>(P.nfp, 1) * k);
-    X.recv_b.alloc(sizeof(float) * std::max<int64_t>(X.nrecv, 1) * k);
-    X.batch_cap = k;
+    if (P.dist && X.batch_cap < kmax) {
+        X.y_fp_b.alloc(sizeof(float) * std::max<int64_t>(P.nfp, 1) * kmax);
+        X.recv_b.alloc(sizeof(float) * std::max<int64_t>(X.nrecv, 1) * kmax);
+        X.batch_cap = kmax;
+    }
 }
 
 }  // namespace
 
+// (Re)allocation invalidates every captured solve that used the old buffers.  No-op under capture:
+// cg_run calls this before it captures.
+void prepare_batch_scratch(Plan& P, cudaStream_t st) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    MX_CUDA(cudaStreamIsCapturing(st, &cs));
+    if (cs != cudaStreamCaptureStatusNone) return;  // under capture: cg_run allocated them already
+    const int kmax = group_size(P, 8);
+    const int64_t ncols = std::max({P.fwd.ncols, P.back.ncols, (int64_t)1});
+    if (kmax <= 1 || (P.spmm_xi.bytes() >= sizeof(float) * (size_t)ncols * kmax &&
+                      (!P.dist || P.ex.batch_cap >= kmax)))
+        return;
+    MX_CUDA(cudaDeviceSynchronize());
+    P.graphs.clear();
+    ensure_batch_scratch(P);
+}
+
 void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t st) {
     const int64_t nx = P.local_len(0), ny = P.local_len(1);
+    prepare_batch_scratch(P, st);
+    float* xi = P.spmm_xi.as<float>();
     for (int s0 = 0; s0 < K;) {
         const int k = group_size(P, K - s0);
         const float* xs = x + s0 * nx;
         float* ys = y + s0 * ny;
         if (!P.dist) {
-            spmm_f32(P.fwd, k, xs, nx, ys, ny, st);
+            spmm_f32(P.fwd, k, xs, nx, ys, ny, xi, st);
         } else {
-            ensure_batch_buffers(P, k);
             Exchange& X = P.ex;
             float* yfp = X.y_fp_b.as<float>();
             float* rb = X.recv_b.as<float>();
-            spmm_f32(P.fwd, k, xs, nx, yfp, P.nfp, st);                       // A_p, k slices
+            spmm_f32(P.fwd, k, xs, nx, yfp, P.nfp, xi, st);                       // A_p, k slices
             for (int s = 0; s < k; ++s)
                 exchange_fwd<float>(P, yfp + s * P.nfp, rb + s * X.nrecv, ys + s * ny, st);  // R C
         }
@@ -535,20 +560,21 @@ void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t 
 
 void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st) {
     const int64_t nx = P.local_len(0), ny = P.local_len(1);
+    prepare_batch_scratch(P, st);
+    float* xi = P.spmm_xi.as<float>();
     for (int s0 = 0; s0 < K;) {
         const int k = group_size(P, K - s0);
         const float* ys = y + s0 * ny;
         float* xs = x + s0 * nx;
         if (!P.dist) {
-            spmm_f32(P.back, k, ys, ny, xs, nx, st);
+            spmm_f32(P.back, k, ys, ny, xs, nx, xi, st);
         } else {
-            ensure_batch_buffers(P, k);
             Exchange& X = P.ex;
             float* yfp = X.y_fp_b.as<float>();
             float* rb = X.recv_b.as<float>();
             for (int s = 0; s < k; ++s)
                 exchange_back<float>(P, ys + s * ny, rb + s * X.nrecv, yfp + s * P.nfp, st);  // C^T R^T
-            spmm_f32(P.back, k, yfp, P.nfp, xs, nx, st);                      // A_p^T, k slices
+            spmm_f32(P.back, k, yfp, P.nfp, xs, nx, xi, st);                      // A_p^T, k slices
         }
         s0 += k;
     }

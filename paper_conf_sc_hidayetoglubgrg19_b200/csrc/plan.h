@@ -251,6 +251,10 @@ struct Plan {
     DevArr<unsigned int> tickets;                   // last-block counters
     int64_t scal_iters = -1;
     int32_t scal_slices = 0, cg_slices = 0;
+    // multi-slice SpMM input, slice-interleaved ([ncols][k] fp32, spmm_f32): sized once for the
+    // largest slice group the stage buffers admit (ensure_spmm_scratch), so captured graphs never
+    // see it move
+    DevBuf spmm_xi;
     // staging for *_host calls
     DevBuf h_in, h_out;
     std::map<std::tuple<const void*, void*, int32_t, cudaStream_t>, std::unique_ptr<CgGraph>> graphs;
@@ -310,6 +314,9 @@ void peer_allreduce(Plan& P, double* v, int K, int64_t stride, cudaStream_t st);
 // K slices, slice-major [K][local_len] fp32 vectors
 void apply_forward_batch(Plan& P, int K, const float* x, float* y, cudaStream_t st);
 void apply_back_batch(Plan& P, int K, const float* y, float* x, cudaStream_t st);
+// allocates the batched-call buffers for the largest slice group; call outside graph capture
+// (a no-op under capture); clears the captured solves when a buffer moves
+void prepare_batch_scratch(Plan& P, cudaStream_t st);
 
 // spmv.cu
 void spmv_init();
@@ -324,8 +331,11 @@ void spmv_f32_remote(const Layout& L, const float* x, const PeerArgs& pa, cudaSt
 // pa.fold the kernel waits for their arrival flags and its last CTA returns the credits
 void spmv_f32_peer_back(const Layout& L, const float* x, float* y, double* dot_part, double* dot_out,
                         unsigned int* dot_ticket, const PeerArgs& pa, cudaStream_t st);
-// K in {1, 2, 4, 8} slices at once: x[s*ldx + i], y[s*ldy + r]
-void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int64_t ldy, cudaStream_t st);
+// K in {1, 2, 4, 8} slices at once: x[s*ldx + i], y[s*ldy + r].  k > 1: x is first interleaved
+// into xi ([L.ncols][k], >= L.ncols * k floats) so that the stage gather fetches one slice group
+// per map entry with a single 8/16/32 B load
+void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int64_t ldy, float* xi,
+              cudaStream_t st);
 int spmm_max_slices(const Layout& L);
 
 inline void spmv_any(Plan&, const Layout& L, const float* in, float* out, cudaStream_t st) {

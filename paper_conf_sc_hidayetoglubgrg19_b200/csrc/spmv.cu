@@ -494,10 +494,10 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
 // slices' inputs interleaved ([B][K] fp32), so every slot read from HBM feeds K fmas and one
 // matrix stream serves K slices.  Each slice's fma sequence is exactly the single-slice kernel's,
 // so every slice's result is bit-identical to spmv_f32 on the same plan.
-#ifndef MEMXCT_SPMM_GATHER_LOADS
-#define MEMXCT_SPMM_GATHER_LOADS 8
-#endif
-constexpr int kSpmmGatherLoads = MEMXCT_SPMM_GATHER_LOADS;  // stage-gather input loads in flight per thread
+// K >= 4: the stage gather reads slice-interleaved inputs (interleave_kernel below); at K = 2 the
+// extra pass costs more than the gather saves (cfg3: +0.5 %, profiles/r01l_spmm_xi.jsonl), so
+// the gather reads the slice-major input directly
+template <int K> constexpr bool kSpmmInterleaved = K >= 4;
 
 template <int K>
 __device__ __forceinline__ void load_k(const float* __restrict__ buf, uint32_t i, float (&b)[K]) {
@@ -554,7 +554,8 @@ spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __r
         const int32_t* __restrict__ mp = a.map + m0 + st * a.B;
         if (g != g0) __syncthreads();
         if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (st + 1) * a.B));
-        constexpr int U = K >= kSpmmGatherLoads ? 1 : kSpmmGatherLoads / K;  // input loads in flight per thread
+        // 8 input words in flight per thread (16 measured no faster at K = 2/4/8, r01k_spmm_ab.jsonl)
+        constexpr int U = K >= 8 ? 1 : 8 / K;
         const int bd = blockDim.x;
         for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
             int64_t col[U];
@@ -564,7 +565,12 @@ spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __r
 #pragma unroll
             for (int u = 0; u < U; ++u)
 #pragma unroll
-                for (int s = 0; s < K; ++s) v[u][s] = col[u] >= 0 ? __ldg(x + s * ldx + col[u]) : 0.f;
+                if constexpr (kSpmmInterleaved<K>) {
+                    if (col[u] >= 0) load_k<K>(x, (uint32_t)col[u], v[u]);
+                    else for (int s = 0; s < K; ++s) v[u][s] = 0.f;
+                } else {
+                    for (int s = 0; s < K; ++s) v[u][s] = col[u] >= 0 ? __ldg(x + s * ldx + col[u]) : 0.f;
+                }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const int i = i0 + u * bd;
@@ -616,12 +622,48 @@ spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __r
     }
 }
 
+// xi[c][s] = x[s * ldx + c]: the K slices' inputs of column c side by side, so the stage gather
+// fetches them with one 16/32 B load per map entry instead of K 4 B loads to K lines (cfg3,
+// interleave included: K = 4 SpMM 2.014 -> 1.965 ms forward, 2.056 -> 2.018 back; K = 8
+// 5.02 -> 4.81 ms, profiles/r01l_spmm_xi.jsonl).  Coalesced on both sides:
+// thread c reads K strided-by-ldx words (each a coalesced warp row) and writes one K-vector.
 template <int K>
-void launch_spmm(const Layout& L, const float* x, int64_t ldx, float* y, int64_t ldy, cudaStream_t st) {
+__global__ void __launch_bounds__(256) interleave_kernel(const float* __restrict__ x, int64_t ldx, int64_t n,
+                                                         float* __restrict__ xi) {
+    for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
+        float v[K];
+#pragma unroll
+        for (int s = 0; s < K; ++s) v[s] = __ldg(x + s * ldx + c);
+        if constexpr (K == 2) {
+            reinterpret_cast<float2*>(xi)[c] = make_float2(v[0], v[1]);
+        } else if constexpr (K == 4) {
+            reinterpret_cast<float4*>(xi)[c] = make_float4(v[0], v[1], v[2], v[3]);
+        } else {
+            reinterpret_cast<float4*>(xi)[2 * c] = make_float4(v[0], v[1], v[2], v[3]);
+            reinterpret_cast<float4*>(xi)[2 * c + 1] = make_float4(v[4], v[5], v[6], v[7]);
+        }
+    }
+}
+
+template <int K>
+void launch_spmm(const Layout& L, const float* x, int64_t ldx, float* y, int64_t ldy, float* xi, cudaStream_t st) {
+    if (L.ncols > ldx) fail(MEMXCT_ERR_INVALID_ARG, "internal: SpMM input stride below the column count");
+    if constexpr (kSpmmInterleaved<K>) {
+        if (!xi) fail(MEMXCT_ERR_INVALID_ARG, "internal: multi-slice SpMM without its interleave buffer");
+        int dev = 0, sms = 0;
+        MX_CUDA(cudaGetDevice(&dev));
+        MX_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        const int64_t blocks = std::min<int64_t>(ceil_div(L.ncols, 256), (int64_t)sms * 8);
+        if (blocks > 0) {
+            interleave_kernel<K><<<(unsigned)blocks, 256, 0, st>>>(x, ldx, L.ncols, xi);
+            MX_LAUNCHED();
+        }
+    }
     const SpmvArgs a = make_args(L, nullptr, nullptr, nullptr);
     const size_t smem = sizeof(float) * (size_t)L.B * K;
     auto kern = L.out_idx.p() ? spmm_f32_kernel<K, true> : spmm_f32_kernel<K, false>;
-    kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, ldx, y, ldy);
+    if constexpr (kSpmmInterleaved<K>) kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, xi, (int64_t)K, y, ldy);
+    else kern<<<(unsigned)L.nparts, L.R, smem, st>>>(a, x, ldx, y, ldy);
     MX_LAUNCHED();
 }
 
@@ -636,13 +678,14 @@ int spmm_max_slices(const Layout& L) {
     return k;
 }
 
-void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int64_t ldy, cudaStream_t st) {
+void spmm_f32(const Layout& L, int k, const float* x, int64_t ldx, float* y, int64_t ldy, float* xi,
+              cudaStream_t st) {
     if (L.nparts == 0) return;
     switch (k) {
         case 1: spmv_f32(L, x, y, nullptr, nullptr, nullptr, st); break;
-        case 2: launch_spmm<2>(L, x, ldx, y, ldy, st); break;
-        case 4: launch_spmm<4>(L, x, ldx, y, ldy, st); break;
-        case 8: launch_spmm<8>(L, x, ldx, y, ldy, st); break;
+        case 2: launch_spmm<2>(L, x, ldx, y, ldy, xi, st); break;
+        case 4: launch_spmm<4>(L, x, ldx, y, ldy, xi, st); break;
+        case 8: launch_spmm<8>(L, x, ldx, y, ldy, xi, st); break;
         default: fail(MEMXCT_ERR_INVALID_ARG, "internal: slice group must be 1, 2, 4 or 8");
     }
 }

@@ -222,3 +222,29 @@ def test_forward_overlap_bit_identical(monkeypatch, nranks):
         return gather(plans, fw, 1, m * c), gather(plans, cg, 0, n * n)
     for a, b in zip(run(on), run(off)):
         assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("nranks", [2, 3])
+def test_batched_multirank_bit_identical_to_single(nranks):
+    """Multi-slice calls on virtual ranks (A_p SpMM over slice-interleaved inputs, then the
+    per-slice exchange): every slice equals its single-slice projection / CG on the same plans.
+    The group of 5 runs as 4 + 1 slices, so the batched scratch is sized for the largest group
+    and the 1-slice remainder takes the single-slice path."""
+    n, m, c, k = 64, 90, 64, 5
+    _, plans = build_group(n, m, c, nranks, slices=4)
+    xs = [inputs.uniform(n * n, 40 + s) for s in range(k)]
+    ys = [inputs.uniform(m * c, 50 + s) for s in range(k)]
+    X = [torch.stack(v) for v in zip(*[scatter(plans, x, 0, np.float32) for x in xs])]
+    Y = [torch.stack(v) for v in zip(*[scatter(plans, y, 1, np.float32) for y in ys])]
+    fb = run_ranks(nranks, lambda r: plans[r].forward_batch(X[r]))
+    bb = run_ranks(nranks, lambda r: plans[r].back_batch(Y[r]))
+    cb = run_ranks(nranks, lambda r: plans[r].cg_batch(Y[r], 6, residuals=True))
+    for s in range(k):
+        f1 = run_ranks(nranks, lambda r: plans[r].forward(X[r][s].contiguous()))
+        b1 = run_ranks(nranks, lambda r: plans[r].back(Y[r][s].contiguous()))
+        c1 = run_ranks(nranks, lambda r: plans[r].cg(Y[r][s].contiguous(), 6, residuals=True))
+        for r in range(nranks):
+            assert torch.equal(fb[r][s], f1[r]), (s, r)
+            assert torch.equal(bb[r][s], b1[r]), (s, r)
+            assert torch.equal(cb[r][0][s], c1[r][0]), (s, r)
+            assert np.array_equal(cb[r][1][s], c1[r][1]), (s, r)
