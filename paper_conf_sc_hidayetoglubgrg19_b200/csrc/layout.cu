@@ -658,8 +658,11 @@ void resolve_tuning(const Plan& P, int64_t rows, int32_t* R_out, int32_t* B_out)
     if (B == 0) {
         int32_t k = 1;
         while (k < P.opt.slices) k *= 2;  // batched calls stage k slices per buffer entry
+        // k >= 2: 192 KB of fp32 slice groups at k >= 4; k = 2 stages as many entries as k = 4
+        // (96 KB): cfg3 K = 2 SpMM 1.742 ms at B = 12288 vs 1.795 at 24576, and every size
+        // above 192 KB falls off a cliff (K = 4 at 14336: 2.49 ms), profiles/r01n_spmm_bigB.jsonl
         B = (k == 1) ? std::min<int32_t>(drift_requested() ? drift_auto_b() : 57344, 36 * R)
-                     : std::min<int32_t>(49152, 144 * R) / k;
+                     : std::min<int32_t>(49152, 144 * R) / std::max<int32_t>(k, 4);
         B = std::max<int32_t>(256, B - B % 256);
     }
     *R_out = R;
