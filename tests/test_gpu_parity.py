@@ -372,6 +372,23 @@ def test_batched_projections_bit_identical_to_single(orc, coo_cache, k):
         assert torch.equal(XB[s], plan.back(Yin[s].contiguous()))
 
 
+@pytest.mark.parametrize("n,m,c,k", [(64, 90, 64, 8), (64, 90, 64, 13), (33, 17, 33, 8), (256, 360, 256, 9)])
+def test_spmm_eight_wide_bit_identical(n, m, c, k):
+    """K = 8 slice groups (slices=8 plan, B small enough for 32 B entries): the interleaved
+    input pass and the 8-wide gather, with a ragged remainder group (k = 9, 13), against the
+    single-slice SpMV on the same plan, every slice bit-identical."""
+    plan = make_plan(n, m, c, slices=8, buffer_entries=2048)
+    assert plan.get_option("slices") == 8
+    rng = np.random.default_rng(k)
+    X = torch.from_numpy(rng.random((k, n * n), dtype=np.float32)).cuda()
+    Y = plan.forward_batch(X)
+    Yin = torch.from_numpy(rng.random((k, m * c), dtype=np.float32)).cuda()
+    XB = plan.back_batch(Yin)
+    for s in range(k):
+        assert torch.equal(Y[s], plan.forward(X[s].contiguous())), s
+        assert torch.equal(XB[s], plan.back(Yin[s].contiguous())), s
+
+
 def test_batched_cg_bit_identical_to_single(orc, coo_cache):
     n, m, c = 64, 90, 64
     plan = make_plan(n, m, c, slices=4)
