@@ -563,14 +563,17 @@ spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __r
             for (int u = 0; u < U; ++u) col[u] = (i0 + u * bd < cnt) ? (int64_t)__ldg(mp + i0 + u * bd) : -1;
             float v[U][K];
 #pragma unroll
-            for (int u = 0; u < U; ++u)
-#pragma unroll
+            for (int u = 0; u < U; ++u) {
                 if constexpr (kSpmmInterleaved<K>) {
                     if (col[u] >= 0) load_k<K>(x, (uint32_t)col[u], v[u]);
-                    else for (int s = 0; s < K; ++s) v[u][s] = 0.f;
+                    else
+#pragma unroll
+                        for (int s = 0; s < K; ++s) v[u][s] = 0.f;
                 } else {
+#pragma unroll
                     for (int s = 0; s < K; ++s) v[u][s] = col[u] >= 0 ? __ldg(x + s * ldx + col[u]) : 0.f;
                 }
+            }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const int i = i0 + u * bd;
