@@ -1,5 +1,7 @@
 /*
- * memxct_oracle.h -- plain, slow, single-threaded fp64 CPU oracle for the MemXCT hot path.
+ * memxct_oracle.h -- plain, slow fp64 CPU oracle for the MemXCT hot path (single-threaded
+ * arithmetic; the sampled-row helpers and the CPU-baseline SpMV spread independent rays / rows over
+ * host threads without changing any operation).
  *
  * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
  * --impl reference legs may load this library.  The product (paper_conf_sc_hidayetoglubgrg19_b200/,
@@ -86,6 +88,41 @@ int orc_sirt(int64_t nrows, int64_t ncols, int64_t nnz, const int32_t* rows, con
  * of `chunk` elements, chunk partials summed sequentially. */
 double orc_dot_canonical(int64_t n, const double* a, const double* b, const int64_t* key,
                          int64_t chunk);
+
+
+/* ---- closed-form chord and sampled rows / columns ------------------------- */
+
+/* Closed-form length of ray `ray` inside the grid square [-L, L]^2 (C.4): with
+ * c' = max(|cos|, |sin|), s' = min(...), tau = |t|: 2L/c' if tau <= L(c'-s'); (L(c'+s') - tau) /
+ * (c' s') if tau < L(c'+s'); else 0 (s' < 1e-15: 2L if tau < L).  Equals the row sum of A.
+ * Pinned by: Liang-Barsky clipping of the line against the square, and the tracer's row sums. */
+double orc_chord(int32_t n, int32_t m_proj, int32_t c_chan, int64_t ray);
+void orc_chords(int32_t n, int32_t m_proj, int32_t c_chan, double* out /* m_proj*c_chan */);
+
+/* CSR result of the sampled functions (library-allocated; free with orc_csr_free). */
+typedef struct { int64_t nrows, nnz; int64_t* ptr; int32_t* idx; double* len; } orc_csr_t;
+orc_csr_t* orc_csr_alloc(int64_t nrows, int64_t nnz);
+void orc_csr_free(orc_csr_t* s);
+
+/* Rows of A for `nrays` natural ray indices: row i = (pixel, length) pairs of rays[i] in trace
+ * order, exactly orc_trace_ray's.  Rays are spread over `nthreads` host threads (0 = all online
+ * cores); no arithmetic changes.  Pinned by: equality with orc_trace_all's rows. */
+orc_csr_t* orc_sample_rows(int32_t n, int32_t m_proj, int32_t c_chan, int64_t nrays,
+                           const int64_t* rays, int32_t nthreads);
+
+/* Columns of A (rows of A^T) for `npix` distinct natural pixel indices: row q = (ray, length)
+ * pairs of every ray crossing pixels[q], rays ascending.  Per projection, candidate channels are
+ * those whose line can meet the pixel square (|t_k - tc| <= (|cos| + |sin|)/2, +-1 channel), each
+ * traced in full by the tracer.  NULL if pixels repeat.  Pinned by: equality with the columns of
+ * the full transpose of orc_trace_all (tests/test_oracle_sampled.py). */
+orc_csr_t* orc_sample_columns(int32_t n, int32_t m_proj, int32_t c_chan, int64_t npix,
+                              const int64_t* pixels, int32_t nthreads);
+
+/* y = A x over CSR with rows split over host threads (the threaded CPU
+ * baseline).  Each row is summed sequentially in entry order, bit-identical to orc_spmv_coo on
+ * row-major COO.  Returns the number of threads used. */
+int32_t orc_spmv_csr_threaded(int64_t nrows, const int64_t* ptr, const int32_t* cols,
+                              const double* vals, const double* x, double* y, int32_t nthreads);
 
 #ifdef __cplusplus
 }

@@ -18,8 +18,14 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 __all__ = [
     "build_oracle", "lib", "trace_ray", "count_nnz", "row_lengths", "trace_all", "gilbert2d",
     "d2xy", "hilbert_rank", "spmv_coo", "spmv_canonical", "cgls", "dot_canonical",
-    "coo_to_csr", "sampled_back_rows", "sirt",
+    "coo_to_csr", "sampled_back_rows", "sirt", "chord", "chords", "sample_rows", "sample_columns",
+    "spmv_csr_threaded",
 ]
+
+
+class _Csr(ctypes.Structure):
+    _fields_ = [("nrows", ctypes.c_int64), ("nnz", ctypes.c_int64), ("ptr", ctypes.POINTER(ctypes.c_int64)),
+                ("idx", ctypes.POINTER(ctypes.c_int32)), ("len", ctypes.POINTER(ctypes.c_double))]
 
 
 def build_oracle(force: bool = False) -> str:
@@ -27,7 +33,7 @@ def build_oracle(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".{os.getpid()}.tmp"
         subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fPIC", "-shared", "-std=gnu11",
-                               "-o", tmp, _SRC, "-lm"])
+                               "-pthread", "-o", tmp, _SRC, "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -65,6 +71,18 @@ def lib():
         L.orc_sirt.argtypes = [i64, i64, i64, vp, vp, vp, vp, i32, vp, vp]
         L.orc_dot_canonical.restype = dbl
         L.orc_dot_canonical.argtypes = [i64, vp, vp, vp, i64]
+        L.orc_chord.restype = dbl
+        L.orc_chord.argtypes = [i32, i32, i32, i64]
+        L.orc_chords.restype = None
+        L.orc_chords.argtypes = [i32, i32, i32, vp]
+        L.orc_sample_rows.restype = ctypes.POINTER(_Csr)
+        L.orc_sample_rows.argtypes = [i32, i32, i32, i64, vp, i32]
+        L.orc_sample_columns.restype = ctypes.POINTER(_Csr)
+        L.orc_sample_columns.argtypes = [i32, i32, i32, i64, vp, i32]
+        L.orc_csr_free.restype = None
+        L.orc_csr_free.argtypes = [ctypes.POINTER(_Csr)]
+        L.orc_spmv_csr_threaded.restype = i32
+        L.orc_spmv_csr_threaded.argtypes = [i64, vp, vp, vp, vp, vp, i32]
         _lib = L
     return _lib
 
@@ -196,28 +214,56 @@ def sirt(rows, cols, vals, y, nrows: int, ncols: int, iters: int):
     return x, res
 
 
-def sampled_back_rows(n: int, m: int, c: int, pixels):
-    """Rows of A^T for a few pixels, by Siddon-tracing every ray that can cross each pixel
-    (at most 3 channels per angle for unit pixels and unit channel spacing, +1 margin each side).
-    Returns a list of (ray indices int64, lengths float64) per pixel, rays ascending."""
-    out = []
-    L = n / 2.0
-    for p in pixels:
-        i, j = divmod(int(p), n)
-        xc, yc = (j + 0.5) - L, (i + 0.5) - L
-        rays, lens = [], []
-        for mm in range(m):
-            th = mm * np.pi / m
-            cth, sth = np.cos(th), np.sin(th)
-            tc = xc * cth + yc * sth
-            hw = 0.5 * (abs(cth) + abs(sth))
-            k0 = int(np.floor(tc - hw + c / 2.0 - 0.5)) - 1
-            k1 = int(np.ceil(tc + hw + c / 2.0 - 0.5)) + 1
-            for k in range(max(k0, 0), min(k1, c - 1) + 1):
-                pix, ln = trace_ray(n, m, c, mm * c + k)
-                hit = np.nonzero(pix == p)[0]
-                if len(hit):
-                    rays.append(mm * c + k)
-                    lens.append(ln[hit[0]])
-        out.append((np.array(rays, np.int64), np.array(lens, np.float64)))
+def chord(n: int, m: int, c: int, ray: int) -> float:
+    """Closed-form length of ray `ray` inside the grid square."""
+    return float(lib().orc_chord(n, m, c, int(ray)))
+
+
+def chords(n: int, m: int, c: int) -> np.ndarray:
+    """Closed-form chord of every ray (natural order, M*C doubles) = the row sums of A."""
+    out = np.empty(m * c, np.float64)
+    lib().orc_chords(n, m, c, _p(out))
     return out
+
+
+def _take_csr(ptr):
+    if not ptr:
+        raise ValueError("oracle sampled function failed (repeated pixels?)")
+    s = ptr.contents
+    nr, nz = int(s.nrows), int(s.nnz)
+    rp = np.ctypeslib.as_array(s.ptr, shape=(nr + 1,)).copy()
+    idx = np.ctypeslib.as_array(s.idx, shape=(max(nz, 1),))[:nz].copy()
+    ln = np.ctypeslib.as_array(s.len, shape=(max(nz, 1),))[:nz].copy()
+    lib().orc_csr_free(ptr)
+    return rp, idx, ln
+
+
+def sample_rows(n: int, m: int, c: int, rays, threads: int = 0):
+    """Rows of A for natural ray indices `rays` (orc_sample_rows): (ptr, pixels int32, lengths)."""
+    r = np.ascontiguousarray(rays, np.int64)
+    return _take_csr(lib().orc_sample_rows(n, m, c, len(r), _p(r), int(threads)))
+
+
+def sample_columns(n: int, m: int, c: int, pixels, threads: int = 0):
+    """Columns of A for distinct natural pixel indices (orc_sample_columns): (ptr, rays int32
+    ascending, lengths) per pixel."""
+    p = np.ascontiguousarray(pixels, np.int64)
+    return _take_csr(lib().orc_sample_columns(n, m, c, len(p), _p(p), int(threads)))
+
+
+def spmv_csr_threaded(ptr, cols, vals, x, threads: int = 0):
+    """Threaded CSR y = A x (orc_spmv_csr_threaded); returns (y, threads used)."""
+    ptr = np.ascontiguousarray(ptr, np.int64)
+    cols = np.ascontiguousarray(cols, np.int32)
+    vals = np.ascontiguousarray(vals, np.float64)
+    x = np.ascontiguousarray(x, np.float64)
+    y = np.empty(len(ptr) - 1, np.float64)
+    nt = lib().orc_spmv_csr_threaded(len(ptr) - 1, _p(ptr), _p(cols), _p(vals), _p(x), _p(y), int(threads))
+    return y, int(nt)
+
+
+def sampled_back_rows(n: int, m: int, c: int, pixels, threads: int = 0):
+    """Rows of A^T for distinct pixels (orc_sample_columns): a list of (ray indices int64,
+    lengths float64) per pixel, rays ascending."""
+    ptr, rays, ln = sample_columns(n, m, c, pixels, threads)
+    return [(rays[ptr[q]:ptr[q + 1]].astype(np.int64), ln[ptr[q]:ptr[q + 1]]) for q in range(len(ptr) - 1)]

@@ -245,13 +245,14 @@ def test_cg_fp32_recovers_phantom(orc, coo_cache, n, m, c):
     print("fp32 CG drift vs fp64 oracle", rel_l2(x_gpu, x_orc), "phantom error", e_gpu, e_orc)
 
 
-def test_cg_explicit_residual_variant(orc, coo_cache):
+@pytest.mark.parametrize("n,m,c,gate", [(64, 90, 64, 1.15), (256, 360, 256, 1.1)])
+def test_cg_explicit_residual_variant(orc, coo_cache, n, m, c, gate):
     """CG_VARIANT = 1 (r = y - A x every iteration, reading R13).  MIXED (fp64 vectors): the
     image matches the fp64 oracle's CGLS (the two variants agree in exact arithmetic, R13) and its
-    error to the phantom.  FP32: finite-precision CG amplifies rounding (R16: fp32 drift 0.5-3e-2
-    from iteration 8 on, phantom error 0.110 vs 0.104 in fp64), so the FP32 gate is the band that
-    noise spans (1.2x the oracle's phantom error) plus a monotone true residual."""
-    n, m, c = 64, 90, 64
+    error to the phantom.  FP32: the phantom error within `gate` x the oracle's plus a monotone
+    true residual.  The gate is SURVEY R16's 1.1x except at config 1, where reading R16b
+    (tests/test_reading_cg_fp32.py, measured without GPU code) shows that fp32 explicit-residual
+    CG spans 1.08-1.11x over summation orders, so 1.1x there is a lottery and the gate is 1.15x."""
     rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
     x_orc = orc.cgls(rows, cols, vals.astype(np.float32).astype(np.float64), y32.astype(np.float64),
                      m * c, n * n, 30)[0]
@@ -261,7 +262,9 @@ def test_cg_explicit_residual_variant(orc, coo_cache):
     assert rel_l2(x_mix, xt) <= 1.01 * rel_l2(x_orc, xt)
     plan = make_plan(n, m, c, cg_variant=1)
     x_gpu, res = plan.cg(torch.from_numpy(y32).cuda(), 30, residuals=True)
-    assert rel_l2(x_gpu.cpu().numpy(), xt) <= 1.2 * rel_l2(x_orc, xt)
+    ratio = rel_l2(x_gpu.cpu().numpy(), xt) / rel_l2(x_orc, xt)
+    print(f"explicit-residual FP32 CG phantom error ratio {ratio:.4f} (gate {gate})")
+    assert ratio <= gate
     assert np.all(np.diff(res) <= 1e-6 * res[0])
 
 
@@ -321,36 +324,46 @@ def test_degenerate_geometries(orc):
 def test_full_size_sampled_rows(orc, cfg):
     """Full size: config 3 (BASELINE configs[2], the launch configuration bench.py times) and
     config 4 (configs[3], 2048^2 x 2400 x 2048, 1.2e10 nonzeros per direction: its one-GPU fit,
-    ~150 GB): 2000 sampled rays of y = A x and 12 sampled pixels of x = A^T y, each against the
-    oracle's own trace."""
+    ~150 GB).  SURVEY C.4 "large configs": 1e4 random rays of y = A x and 1024 pixels (16 random
+    8 x 8 blocks) of x = A^T y against the oracle's own traces (<= 1e-5 relative L2), and the
+    row sums of the GPU-built A on EVERY ray against the closed-form chord (forward of ones:
+    FP32 <= 1e-5 relative L2 and <= 1e-4 per ray; MIXED -- fp64 sums of the same fp32 values --
+    <= 2e-7 per ray, i.e. only the fp32 rounding of the stored lengths, so no entry of any row is
+    missing or wrong)."""
     import gc
+    from fullsize import N_RAYS, chord_errors, pick_pixels, sampled_back_error, sampled_forward_error
     gc.collect()                       # earlier tests' plans release their device memory
     torch.cuda.empty_cache()
     n, m, c = inputs.CONFIGS[cfg]
     plan = make_plan(n, m, c)
     st = plan.stats()
     assert abs(st["nnz"] / (m * n * n) - 1.1953) < 2e-3
+    ones = torch.ones(n * n, device="cuda")
+    l2, per = chord_errors(orc, n, m, c, plan.forward(ones).cpu().numpy())
+    print(f"cfg{cfg} FP32 chord sums: rel L2 {l2:.2e}, worst ray {per:.2e}")
+    assert l2 <= 1e-5 and per <= 1e-4, (l2, per)
     x = torch.from_numpy(inputs.uniform(n * n, inputs.seed_for(cfg))).cuda()
     y = plan.forward(x).cpu().numpy()
     xh = x.cpu().numpy().astype(np.float64)
     rng = np.random.default_rng(cfg)
-    rays = rng.choice(m * c, 2000, replace=False)
-    got, exp = [], []
-    for r in rays:
-        pix, ln = orc.trace_ray(n, m, c, int(r))
-        got.append(y[r])
-        exp.append(float(ln @ xh[pix]))
-    assert rel_l2(np.array(got), np.array(exp)) <= 1e-5
+    rays = rng.choice(m * c, N_RAYS, replace=False)
+    e_fwd = sampled_forward_error(orc, n, m, c, rays, y[rays], xh)
     ysino = torch.from_numpy(inputs.uniform(m * c, inputs.seed_for(cfg) + 1)).cuda()
     xb = plan.back(ysino).cpu().numpy()
     yh = ysino.cpu().numpy().astype(np.float64)
-    pixels = rng.choice(n * n, 12, replace=False)
-    got, exp = [], []
-    for p, (rr, ll) in zip(pixels, orc.sampled_back_rows(n, m, c, pixels)):
-        got.append(xb[p])
-        exp.append(float(ll @ yh[rr]))
+    pixels = pick_pixels(rng, n)
+    e_back = sampled_back_error(orc, n, m, c, pixels, xb[pixels], lambda r: yh[r])
+    print(f"cfg{cfg} sampled rows: {len(rays)} rays {e_fwd:.2e}, {len(pixels)} pixels {e_back:.2e}")
+    assert e_fwd <= 1e-5 and e_back <= 1e-5, (e_fwd, e_back)
     plan.close()
-    assert rel_l2(np.array(got), np.array(exp)) <= 1e-5
+    del plan
+    gc.collect()
+    torch.cuda.empty_cache()
+    mixed = make_plan(n, m, c, precision="mixed")
+    l2, per = chord_errors(orc, n, m, c, mixed.forward(ones.double()).cpu().numpy())
+    print(f"cfg{cfg} MIXED chord sums: rel L2 {l2:.2e}, worst ray {per:.2e}")
+    assert per <= 2e-7, per
+    mixed.close()
 
 
 # ---- multi-slice (SURVEY 8(f) NEXT-1) ---------------------------------------------------------
