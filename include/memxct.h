@@ -59,7 +59,11 @@ typedef enum {
     MEMXCT_ERR_STATE = 2,        /* plan used before build, option set after build, ... */
     MEMXCT_ERR_OUT_OF_MEMORY = 3,/* device or host allocation failed */
     MEMXCT_ERR_CUDA = 4,         /* CUDA runtime / launch error, or no device */
-    MEMXCT_ERR_NCCL = 5,         /* NCCL error (P > 1) */
+    MEMXCT_ERR_NCCL = 5,         /* P > 1 communication error: an NCCL error (including an
+                                  * asynchronous one, polled with ncclCommGetAsyncError at every call
+                                  * on a decomposed plan), or a fused-exchange wait on the device
+                                  * that timed out (~20 s: a peer is gone; reported at the next call,
+                                  * the interrupted call's results are undefined) */
     MEMXCT_ERR_UNSUPPORTED = 6   /* valid request this build does not implement */
 } memxct_status_t;
 

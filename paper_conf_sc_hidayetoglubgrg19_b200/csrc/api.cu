@@ -5,7 +5,9 @@
 #include <cmath>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <string>
+#include <vector>
 
 #include "plan.h"
 
@@ -23,6 +25,17 @@ static std::atomic<int64_t> g_launches{0};
 void count_launch(int64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 int64_t launch_count() { return g_launches.load(std::memory_order_relaxed); }
 
+int num_sms() {
+    static std::mutex mu;
+    static std::vector<int> cache;
+    int dev = 0;
+    MX_CUDA(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(mu);
+    if ((int)cache.size() <= dev) cache.resize(dev + 1, 0);
+    if (!cache[dev]) MX_CUDA(cudaDeviceGetAttribute(&cache[dev], cudaDevAttrMultiProcessorCount, dev));
+    return cache[dev];
+}
+
 int64_t Plan::device_bytes() const {
     return fwd.device_bytes() + back.device_bytes() +
            (int64_t)(tomo_nat_of_h.buf.bytes() + tomo_h_of_nat.buf.bytes() + sino_nat_of_h.buf.bytes() +
@@ -30,6 +43,7 @@ int64_t Plan::device_bytes() const {
                      cg_ax.bytes() + part_fwd.buf.bytes() + part_back.buf.bytes() + part_vec.buf.bytes() +
                      scal.buf.bytes() + tickets.buf.bytes() + h_in.bytes() + h_out.bytes() +
                      fp_rays.buf.bytes() + spmm_xi.bytes()) +
+           [this] { int64_t b = 0; for (const DevBuf& r : retired) b += (int64_t)r.bytes(); return b; }() +
            ex.device_bytes();
 }
 
@@ -68,6 +82,10 @@ mx::Plan& built_plan(memxct_plan_t plan) {
     mx::Plan& P = plan_of(plan);
     if (!P.built) mx::fail(MEMXCT_ERR_STATE, "plan used before memxct_build");
     if (P.device >= 0) MX_CUDA(cudaSetDevice(P.device));
+    if (P.dist) {  // errors of earlier asynchronous work: NCCL, or a peer wait that gave up
+        if (P.comm) P.comm->check_async();
+        if (P.ex.peer) mx::check_peer_abort();
+    }
     return P;
 }
 

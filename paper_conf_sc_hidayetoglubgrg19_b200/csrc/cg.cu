@@ -24,8 +24,9 @@ constexpr int kVT = 256;
 // Vector steps are HBM streams of a few MB: 8 CTAs x 256 threads per SM and 4 independent
 // elements per thread per pass keep ~10 MB of loads in flight (296 CTAs with one element per
 // pass ran at ~1 TB/s: 32 us for the 30 MB of the x/r update at cfg3).
-constexpr int kVecBlocks = 8 * 148;
+constexpr int kVecCtasPerSm = 8;
 constexpr int kU = 4;
+int vec_blocks_max() { return kVecCtasPerSm * num_sms(); }
 
 // scalar slots of slice s: gam[s*n1 + k], del[...], res2[...]; stop flags per slice
 struct Scal {
@@ -181,7 +182,7 @@ dot_kernel(const T* __restrict__ v, int64_t n, double* out, int64_t stride, doub
 }
 
 unsigned vec_blocks(int64_t n) {
-    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(kVecBlocks, ceil_div(n, (int64_t)kVT * kU)));
+    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(vec_blocks_max(), ceil_div(n, (int64_t)kVT * kU)));
 }
 
 // CG dots at P > 1: one fp64 per slice summed over the ranks -- over peer memory with the fused
@@ -288,28 +289,31 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, int32_t K, cudaStrea
     if (K < 1 || K > 64) fail(MEMXCT_ERR_INVALID_ARG, "slices must be in [1, 64]");
     if (K > 1 && P.esize != 4) fail(MEMXCT_ERR_UNSUPPORTED, "multi-slice CG is FP32 only");
     const int64_t nx = P.local_len(0), nr = P.local_len(1);
+    // grow-only (common.h: grow): no cudaFree while peers' kernels may wait on this rank
     if (K > P.cg_slices) {
         MX_CUDA(cudaStreamSynchronize(st));
-        P.graphs.clear();
-        P.cg_r.alloc(P.esize * std::max<int64_t>(nr, 1) * K);
-        P.cg_q.alloc(P.esize * std::max<int64_t>(nr, 1) * K);
-        P.cg_s.alloc(P.esize * std::max<int64_t>(nx, 1) * K);
-        P.cg_p.alloc(P.esize * std::max<int64_t>(nx, 1) * K);
-        if (P.opt.cg_variant == 1) P.cg_ax.alloc(P.esize * std::max<int64_t>(nr, 1) * K);
-        P.part_fwd.alloc(std::max<int64_t>(P.fwd.nparts, 1));
-        P.part_back.alloc(std::max<int64_t>(P.back.nparts, 1));
-        P.part_vec.alloc((int64_t)kVecBlocks * K);
-        P.tickets.alloc(128);
-        MX_CUDA(cudaMemsetAsync(P.tickets.p(), 0, 128 * sizeof(unsigned int), st));
+        grow(P.retired, P.cg_r, P.esize * std::max<int64_t>(nr, 1) * K);
+        grow(P.retired, P.cg_q, P.esize * std::max<int64_t>(nr, 1) * K);
+        grow(P.retired, P.cg_s, P.esize * std::max<int64_t>(nx, 1) * K);
+        grow(P.retired, P.cg_p, P.esize * std::max<int64_t>(nx, 1) * K);
+        if (P.opt.cg_variant == 1) grow(P.retired, P.cg_ax, P.esize * std::max<int64_t>(nr, 1) * K);
+        grow(P.retired, P.part_fwd, std::max<int64_t>(P.fwd.nparts, 1));
+        grow(P.retired, P.part_back, std::max<int64_t>(P.back.nparts, 1));
+        grow(P.retired, P.part_vec, (int64_t)vec_blocks_max() * K);
+        if (!P.tickets.p()) {
+            P.tickets.alloc(128);
+            MX_CUDA(cudaMemsetAsync(P.tickets.p(), 0, 128 * sizeof(unsigned int), st));
+        }
         P.cg_slices = K;
+        P.graphs.clear();  // captured against the previous buffers (still allocated)
     }
     if (iters > P.scal_iters || K > P.scal_slices) {
         MX_CUDA(cudaStreamSynchronize(st));
-        P.graphs.clear();
+        P.graphs.clear();  // the scalar layout (stride iters + 1) changes
         P.scal_iters = std::max<int64_t>(iters, P.scal_iters);
         P.scal_slices = std::max<int32_t>(K, P.scal_slices);
         const int64_t nd = scal_doubles((int32_t)P.scal_iters, P.scal_slices);
-        P.scal.alloc(nd);
+        grow(P.retired, P.scal, nd);
         MX_CUDA(cudaMemsetAsync(P.scal.p(), 0, 8 * nd, st));
     }
     if (K > 1) prepare_batch_scratch(P, st);
@@ -320,6 +324,13 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, int32_t K, cudaStrea
     auto key = std::make_tuple(y, x, iters * 64 + K, st);
     auto it = P.graphs.find(key);
     if (it == P.graphs.end()) {
+        if (P.graphs.size() >= kMaxGraphs) {  // evict the least recently used solve
+            auto lru = P.graphs.begin();
+            for (auto g = P.graphs.begin(); g != P.graphs.end(); ++g)
+                if (g->second->last_used < lru->second->last_used) lru = g;
+            MX_CUDA(cudaStreamSynchronize(st));
+            P.graphs.erase(lru);
+        }
         // capture the whole solve once on a private stream, replay it on the caller's stream
         MX_CUDA(cudaStreamSynchronize(st));
         cudaStream_t cap;
@@ -346,6 +357,7 @@ void cg_run(Plan& P, const void* y, void* x, int32_t iters, int32_t K, cudaStrea
         MX_CUDA(e);
         it = P.graphs.emplace(key, std::move(cgg)).first;
     }
+    it->second->last_used = ++P.graph_clock;
     MX_CUDA(cudaGraphLaunch(it->second->exec, st));
     count_launch(it->second->nkernels);
     MX_CUDA(cudaGetLastError());

@@ -33,6 +33,7 @@ struct NcclApi {
     decltype(&ncclGroupStart) GroupStart = nullptr;
     decltype(&ncclGroupEnd) GroupEnd = nullptr;
     decltype(&ncclGetErrorString) GetErrorString = nullptr;
+    decltype(&ncclCommGetAsyncError) GetAsyncError = nullptr;
     std::string error;
 
     static NcclApi& get() {
@@ -58,6 +59,7 @@ struct NcclApi {
         MX_SYM(GroupStart, "ncclGroupStart");
         MX_SYM(GroupEnd, "ncclGroupEnd");
         MX_SYM(GetErrorString, "ncclGetErrorString");
+        MX_SYM(GetAsyncError, "ncclCommGetAsyncError");
 #undef MX_SYM
         if (!a.GetUniqueId || !a.CommInitRank || !a.AllReduce || !a.Send || !a.Recv || !a.GroupStart ||
             !a.GroupEnd || !a.AllGather || !a.ReduceScatter || !a.CommDestroy)
@@ -99,6 +101,13 @@ public:
         if (comm_) NcclApi::get().CommDestroy(comm_);
     }
     bool capturable() const override { return true; }
+    void check_async() override {
+        NcclApi& a = nccl();
+        if (!a.GetAsyncError || !comm_) return;
+        ncclResult_t r = ncclSuccess;
+        a.check(a.GetAsyncError(comm_, &r), "ncclCommGetAsyncError");
+        if (r != ncclSuccess && r != ncclInProgress) a.check(r, "NCCL asynchronous error");
+    }
     void allreduce_sum(void* buf, int64_t count, DType t, cudaStream_t st) override {
         if (count == 0) return;
         nccl().check(nccl().AllReduce(buf, buf, (size_t)count, nccl_type(t), ncclSum, comm_, st), "ncclAllReduce");

@@ -46,6 +46,9 @@ public:
     // a pointer this rank's kernels can load/store (NVLink peer mapping via CUDA IPC for NCCL
     // ranks, the plain pointer for virtual ranks).  Collective.  Throws if peers are unreachable.
     virtual std::vector<void*> map_peers(void* local, cudaStream_t st) = 0;
+    // Host poll of asynchronous transport errors (NCCL: ncclCommGetAsyncError); throws
+    // MEMXCT_ERR_NCCL.  Called at the start of every library call on a decomposed plan.
+    virtual void check_async() {}
 };
 
 std::unique_ptr<Comm> make_nccl_comm(int rank, int nranks, const void* unique_id);

@@ -8,6 +8,7 @@
 #include <stdexcept>
 #include <string>
 #include <utility>
+#include <vector>
 
 #include "memxct.h"
 
@@ -89,5 +90,23 @@ template <class T> struct DevArr {
 };
 
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Streaming multiprocessors of the current device (148 on B200), for grid sizing.
+int num_sms();
+
+// Grow-only reallocation: the previous buffer moves to `retired` (kept until the plan is
+// destroyed) instead of being freed.  cudaFree synchronises the whole device, and with the
+// fused peer exchange another rank's kernels may be spinning on this rank's next launch; CUDA
+// graphs captured against the previous buffer also stay valid.
+inline void grow(std::vector<DevBuf>& retired, DevBuf& b, size_t bytes) {
+    if (b.bytes() >= bytes) return;
+    if (b.get()) retired.push_back(std::move(b));
+    b.alloc(bytes);
+}
+template <class T> inline void grow(std::vector<DevBuf>& retired, DevArr<T>& a, int64_t count) {
+    if (a.n >= count && a.p()) return;
+    if (a.p()) retired.push_back(std::move(a.buf));
+    a.alloc(count);
+}
 
 }  // namespace mx

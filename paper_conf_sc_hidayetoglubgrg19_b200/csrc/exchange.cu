@@ -66,7 +66,7 @@ reduce_dot_kernel(const T* __restrict__ recv, const int64_t* __restrict__ ptr, c
     __shared__ bool am_last;
     if (pa.fold) {
         if (threadIdx.x == 0)
-            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.notrap);
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
         __syncthreads();
     }
     double d = 0.0;
@@ -362,7 +362,7 @@ void build_exchange(Plan& P, cudaStream_t st) {
     X.recv_buf.alloc(P.esize * std::max<int64_t>(X.nrecv, 1));
     X.tickets.alloc(8);
     MX_CUDA(cudaMemsetAsync(X.tickets.p(), 0, 32, st));
-    X.dot_part.alloc(std::max<int64_t>({P.back.nparts, (int64_t)nblocks(nown), 4 * 148}));
+    X.dot_part.alloc(std::max<int64_t>({P.back.nparts, (int64_t)nblocks(nown), 4 * num_sms()}));
     if (P.opt.exchange == 0 && !P.shard) setup_forward_overlap(P, st);
     if (P.opt.exchange == 2) {  // dense collectives: footprint row i -> [owner][owned-local index]
         X.maxown = 0;
@@ -509,19 +509,20 @@ void ensure_batch_scratch(Plan& P) {
     if (kmax <= 1) return;
     const int64_t ncols = std::max({P.fwd.ncols, P.back.ncols, (int64_t)1});
     const size_t xi_bytes = sizeof(float) * (size_t)ncols * kmax;
-    if (P.spmm_xi.bytes() < xi_bytes) P.spmm_xi.alloc(xi_bytes);
+    grow(P.retired, P.spmm_xi, xi_bytes);
     Exchange& X = P.ex;
     if (P.dist && X.batch_cap < kmax) {
-        X.y_fp_b.alloc(sizeof(float) * std::max<int64_t>(P.nfp, 1) * kmax);
-        X.recv_b.alloc(sizeof(float) * std::max<int64_t>(X.nrecv, 1) * kmax);
+        grow(P.retired, X.y_fp_b, sizeof(float) * std::max<int64_t>(P.nfp, 1) * kmax);
+        grow(P.retired, X.recv_b, sizeof(float) * std::max<int64_t>(X.nrecv, 1) * kmax);
         X.batch_cap = kmax;
     }
 }
 
 }  // namespace
 
-// (Re)allocation invalidates every captured solve that used the old buffers.  No-op under capture:
-// cg_run calls this before it captures.
+// Grow-only (common.h: grow), so solves captured against earlier buffers stay valid and nothing
+// is freed (no device-wide synchronisation while virtual ranks' peer kernels spin).  No-op under
+// capture: cg_run calls this before it captures.
 void prepare_batch_scratch(Plan& P, cudaStream_t st) {
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     MX_CUDA(cudaStreamIsCapturing(st, &cs));
@@ -531,8 +532,6 @@ void prepare_batch_scratch(Plan& P, cudaStream_t st) {
     if (kmax <= 1 || (P.spmm_xi.bytes() >= sizeof(float) * (size_t)ncols * kmax &&
                       (!P.dist || P.ex.batch_cap >= kmax)))
         return;
-    MX_CUDA(cudaDeviceSynchronize());
-    P.graphs.clear();
     ensure_batch_scratch(P);
 }
 

@@ -12,8 +12,8 @@
 //            waits for all owners, then runs A_p^T.
 // Credit flags make buffer reuse safe for any call sequence: a rank writes into a peer's buffer
 // only after that peer has finished consuming the previous contents.  All waits are one-thread
-// kernels (a spinning CTA never blocks a co-resident rank's kernels), with a time-out that traps
-// instead of hanging.
+// kernels (a spinning CTA never blocks a co-resident rank's kernels), with a time-out that sets
+// the process's abort word and returns instead of hanging (plan.h: peer_abort_word).
 #include "plan.h"
 
 namespace mx {
@@ -26,17 +26,9 @@ __device__ __forceinline__ void st_release(unsigned long long* p, unsigned long 
 
 // wait until flags[base + q] >= flags[target_index] for every q < P
 __global__ void wait_kernel(const unsigned long long* flags, int P, int base, int target_index, int me,
-                            int notrap) {
+                            unsigned int* abort) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
-    wait_flags(flags, base, P, ld_acquire_sys(flags + target_index), me, notrap);
-}
-
-int notrap_env() {
-    static const int v = [] {
-        const char* e = std::getenv("MEMXCT_PEER_NOTRAP");
-        return e && e[0] == '1' ? 1 : 0;
-    }();
-    return v;
+    wait_flags(flags, base, P, ld_acquire_sys(flags + target_index), me, abort);
 }
 
 // peer_flags[q][slot] = flags[value_index] for every q (credit: "done with what you sent me")
@@ -58,7 +50,7 @@ __global__ void pack_remote_kernel(const float* __restrict__ y, const int32_t* _
     __shared__ bool am_last;
     if (pa.fold) {
         if (threadIdx.x == 0)
-            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.notrap);
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
         __syncthreads();
     }
     for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
@@ -95,7 +87,8 @@ struct DotArgs {
     const double* mine;                  // my value array
     unsigned long long* my_flags;        // my flag array: [P arrivals | epoch]
 };
-__global__ void peer_allreduce_kernel(DotArgs da, int P, int me, double* v, int K, int64_t stride, int notrap) {
+__global__ void peer_allreduce_kernel(DotArgs da, int P, int me, double* v, int K, int64_t stride,
+                                      unsigned int* abort) {
     if (threadIdx.x != 0 || blockIdx.x != 0) return;
     const unsigned long long e = da.my_flags[P] + 1;
     da.my_flags[P] = e;
@@ -104,7 +97,7 @@ __global__ void peer_allreduce_kernel(DotArgs da, int P, int me, double* v, int 
         for (int s = 0; s < K; ++s) da.dst[q][((int64_t)par * P + me) * kMaxDotSlices + s] = v[s * stride];
     __threadfence_system();
     for (int q = 0; q < P; ++q) st_release(da.flag[q] + me, e);
-    wait_flags(da.my_flags, 0, P, e, me, notrap);
+    wait_flags(da.my_flags, 0, P, e, me, abort);
     for (int s = 0; s < K; ++s) {
         const volatile double* m = da.mine + (int64_t)par * P * kMaxDotSlices + s;
         double acc = m[0];
@@ -113,7 +106,7 @@ __global__ void peer_allreduce_kernel(DotArgs da, int P, int me, double* v, int 
     }
 }
 
-unsigned nblocks(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 4 * 148)); }
+unsigned nblocks(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 4 * num_sms())); }
 
 SignalArgs signal_args(const Plan& P) {
     SignalArgs sa{};
@@ -122,6 +115,24 @@ SignalArgs signal_args(const Plan& P) {
 }
 
 }  // namespace
+
+unsigned int* peer_abort_word() {
+    static unsigned int* word = [] {
+        void* p = nullptr;
+        MX_CUDA(cudaHostAlloc(&p, sizeof(unsigned int), cudaHostAllocMapped | cudaHostAllocPortable));
+        *static_cast<volatile unsigned int*>(p) = 0u;
+        void* d = nullptr;
+        MX_CUDA(cudaHostGetDevicePointer(&d, p, 0));
+        return static_cast<unsigned int*>(d);  // = p under unified addressing
+    }();
+    return word;
+}
+
+void check_peer_abort() {
+    if (*static_cast<volatile unsigned int*>(peer_abort_word()))
+        fail(MEMXCT_ERR_NCCL, "a peer-exchange wait timed out on the device (a peer rank is gone); results of "
+                              "the interrupted call are undefined");
+}
 
 void peer_setup(Plan& P, cudaStream_t st) {
     Exchange& X = P.ex;
@@ -172,7 +183,7 @@ PeerArgs base_args(const Plan& P) {
     pa.me = P.rank;
     pa.my_flags = P.ex.flags.p();
     pa.fold = P.ex.fold ? 1 : 0;
-    pa.notrap = notrap_env();
+    pa.abort = peer_abort_word();
     for (int q = 0; q < P.nranks; ++q) pa.flag[q] = static_cast<unsigned long long*>(P.ex.peer_flags[q]);
     return pa;
 }
@@ -190,7 +201,7 @@ void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream
     const int np = P.nranks;
     unsigned long long* fl = X.flags.p();
     if (!X.fold) {
-        wait_kernel<<<1, 32, 0, st>>>(fl, np, 2 * np, 4 * np, P.rank, notrap_env());
+        wait_kernel<<<1, 32, 0, st>>>(fl, np, 2 * np, 4 * np, P.rank, peer_abort_word());
         MX_LAUNCHED();
     }
     PeerArgs pa = base_args(P);
@@ -205,7 +216,7 @@ void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream
     pa.wait_base = 2 * np;
     spmv_f32_remote(P.fwd, x, pa, st);
     if (!X.fold) {
-        wait_kernel<<<1, 32, 0, st>>>(fl, np, 0, 4 * np, P.rank, notrap_env());
+        wait_kernel<<<1, 32, 0, st>>>(fl, np, 0, 4 * np, P.rank, peer_abort_word());
         MX_LAUNCHED();
     }
     PeerArgs ra = base_args(P);
@@ -229,7 +240,7 @@ void peer_back(Plan& P, const float* y, float* x, double* dot_out, cudaStream_t 
     const int np = P.nranks;
     unsigned long long* fl = X.flags.p();
     if (!X.fold) {
-        wait_kernel<<<1, 32, 0, st>>>(fl, np, 3 * np, 4 * np + 1, P.rank, notrap_env());
+        wait_kernel<<<1, 32, 0, st>>>(fl, np, 3 * np, 4 * np + 1, P.rank, peer_abort_word());
         MX_LAUNCHED();
     }
     PeerArgs pa = base_args(P);
@@ -245,7 +256,7 @@ void peer_back(Plan& P, const float* y, float* x, double* dot_out, cudaStream_t 
     pack_remote_kernel<<<nblocks(X.nrecv), kT, 0, st>>>(y, X.recv_idx.p(), X.nrecv, pa);
     MX_LAUNCHED();
     if (!X.fold) {
-        wait_kernel<<<1, 32, 0, st>>>(fl, np, np, 4 * np + 1, P.rank, notrap_env());
+        wait_kernel<<<1, 32, 0, st>>>(fl, np, np, 4 * np + 1, P.rank, peer_abort_word());
         MX_LAUNCHED();
     }
     PeerArgs ba = base_args(P);
@@ -272,7 +283,7 @@ void peer_allreduce(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) 
     }
     da.mine = X.dotx.p();
     da.my_flags = X.dflags.p();
-    peer_allreduce_kernel<<<1, 32, 0, st>>>(da, P.nranks, P.rank, v, K, stride, notrap_env());
+    peer_allreduce_kernel<<<1, 32, 0, st>>>(da, P.nranks, P.rank, v, K, stride, peer_abort_word());
     MX_LAUNCHED();
 }
 

@@ -102,8 +102,15 @@ struct PeerArgs {
     // ever being scheduled.
     int32_t fold = 0;
     int32_t wait_base = 0;
-    int32_t notrap = 0;
+    unsigned int* abort = nullptr;               // peer_abort_word(): set by a timed-out wait
 };
+
+// A process-wide word in mapped (device-visible) host memory: a peer-flag wait that times out
+// (a peer is gone) sets it and returns instead of trapping, every other wait then gives up at
+// once, and the host reports MEMXCT_ERR_NCCL at the next call on a decomposed plan
+// (check_peer_abort).  The results of the interrupted call are undefined.
+unsigned int* peer_abort_word();
+void check_peer_abort();
 
 #ifdef __CUDACC__
 __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
@@ -116,20 +123,25 @@ __device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned l
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// One thread: wait until flags[base + q] >= target for q < P; after ~20 s print and trap (a peer
-// is gone) instead of hanging, unless notrap.
+// One thread: wait until flags[base + q] >= target for q < P.  After ~20 s (a peer is gone), or
+// as soon as another wait has given up, set / see *abort and return instead of hanging (the
+// host turns it into MEMXCT_ERR_NCCL; check_peer_abort).
 __device__ inline void wait_flags(const unsigned long long* flags, int base, int P, unsigned long long target,
-                                  int me, int notrap) {
+                                  int me, unsigned int* abort) {
     const long long t0 = clock64();
+    unsigned polls = 0;
     for (int q = 0; q < P; ++q) {
         while (ld_acquire_sys(flags + base + q) < target) {
             __nanosleep(64);
+            if ((++polls & 4095u) == 0 && abort && *(volatile unsigned int*)abort) return;
             if (clock64() - t0 > 40000000000LL) {
                 printf("memxct peer wait timeout: rank %d base %d q %d target %llu value %llu\n", me, base, q,
                        target, ld_acquire_sys(flags + base + q));
-                for (int i = 0; i < 4 * P + 2; ++i) printf("  rank %d flag[%d] = %llu\n", me, i, flags[i]);
-                if (notrap) return;
-                __trap();
+                if (abort) {
+                    *(volatile unsigned int*)abort = 1u;
+                    __threadfence_system();
+                }
+                return;
             }
         }
     }
@@ -200,9 +212,11 @@ struct SirtState {
     }
 };
 
+constexpr size_t kMaxGraphs = 8;
 struct CgGraph {
     cudaGraphExec_t exec = nullptr;
     int64_t nkernels = 0;
+    int64_t last_used = 0;
     ~CgGraph() { if (exec) cudaGraphExecDestroy(exec); }
 };
 
@@ -257,7 +271,12 @@ struct Plan {
     DevBuf spmm_xi;
     // staging for *_host calls
     DevBuf h_in, h_out;
+    // captured CG solves, keyed on (y, x, iters * 64 + slices, stream); least recently used evicted
+    // beyond kMaxGraphs
     std::map<std::tuple<const void*, void*, int32_t, cudaStream_t>, std::unique_ptr<CgGraph>> graphs;
+    int64_t graph_clock = 0;
+    // buffers replaced by grow() (common.h): kept until destroy, never freed while peers may spin
+    std::vector<DevBuf> retired;
 
     int64_t local_len(int domain) const { return domain == 0 ? t1 - t0 : s1 - s0; }
     int64_t device_bytes() const;

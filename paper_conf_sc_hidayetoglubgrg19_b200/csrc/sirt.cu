@@ -14,7 +14,7 @@ namespace {
 
 constexpr int kT = 256;
 
-unsigned nb(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 4 * 148)); }
+unsigned nb(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 4 * num_sms())); }
 
 template <class T> __global__ void fill_kernel(T* v, int64_t n, T a) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) v[i] = a;
@@ -74,7 +74,7 @@ void sirt_t(Plan& P, const T* y, T* x, int32_t iters, double* res2_dev, cudaStre
         S.ax.alloc(P.esize * std::max<int64_t>(nr, 1));
         S.s.alloc(P.esize * std::max<int64_t>(nx, 1));
         S.ones.alloc(P.esize * std::max<int64_t>(std::max(nx, nr), 1));
-        S.part.alloc(4 * 148);
+        S.part.alloc(4 * num_sms());
         fill_kernel<T><<<nb(std::max(nx, nr)), kT, 0, st>>>(S.ones.as<T>(), std::max(nx, nr), T(1));
         MX_LAUNCHED();
         apply_forward(P, S.ones.get(), S.rinv.get(), st);  // row sums of A

@@ -16,6 +16,8 @@
 //
 // Optional epilogue: per-CTA partial of <y, y> (fp64) and a last-CTA reduction in fixed
 // partition order -> deterministic dot products for CG without a second pass over y.
+#include <mutex>
+
 #include "plan.h"
 
 namespace mx {
@@ -87,11 +89,11 @@ struct SpmvArgs {
     unsigned int* ticket;
 };
 
-// Partition processed by this CTA.  Partitions differ in work (forward: rays near the detector
-// edge are short chords), so they are launched heaviest first (longest-processing-time order):
-// the last wave then holds the lightest partitions and the tail in which few SMs stream is short.
-// Per-partition results (rows, dot partials) are indexed by partition, so the order changes no
-// result.
+// Partition processed by this CTA: a.order maps launch positions to partitions when a launch
+// order is set -- heaviest first (longest-processing-time order, opt-in: MEMXCT_PART_ORDER=1,
+// measured +-1 %) or the remote-first split of the forward-overlap exchange; otherwise the
+// partition (Hilbert) order.  Per-partition results (rows, dot partials) are indexed by
+// partition, so the order changes no result.
 __device__ __forceinline__ int64_t part_of_cta(const SpmvArgs& a) {
     const int64_t b = a.cta_base + blockIdx.x;
     return a.order ? (int64_t)__ldg(a.order + b) : b;
@@ -236,7 +238,7 @@ __device__ void remote_epilogue(const PeerArgs& pa, int64_t o, bool valid, float
     __shared__ bool am_last;
     if (pa.fold) {
         if (threadIdx.x == 0)
-            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.notrap);
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
         __syncthreads();
     }
     if (valid) {  // o = footprint position of the row
@@ -284,7 +286,7 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
     extern __shared__ __align__(16) float sbuf[];
     if ((kEpi & 4) && pa.fold) {  // the owners' values for this footprint have arrived
         if (threadIdx.x == 0)
-            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.notrap);
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
         __syncthreads();
     }
     const int64_t p = part_of_cta(a);
@@ -824,11 +826,17 @@ __global__ void __launch_bounds__(1024) read_probe_kernel(const uint4* __restric
     if (acc == 0x9e3779b9u) sink[0] = acc;  // keeps the loads live; never true for a zero buffer
 }
 
-// Raise the dynamic shared-memory limit of every SpMV instantiation once (outside any stream
-// capture): stage buffers go up to 227 KB per CTA.
+// Raise the dynamic shared-memory limit of every SpMV instantiation once per device (the
+// attribute belongs to the current device's context; outside any stream capture): stage buffers
+// go up to 227 KB per CTA.  Thread-safe: virtual ranks build concurrently.
 void spmv_init() {
-    static bool done = false;
-    if (done) return;
+    static std::mutex mu;
+    static std::vector<char> done_dev;
+    int dev = 0;
+    MX_CUDA(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(mu);
+    if ((int)done_dev.size() <= dev) done_dev.resize(dev + 1, 0);
+    if (done_dev[dev]) return;
     set_smem(spmv_f32_drift_kernel<true, 1>);
     set_smem(spmv_f32_drift_kernel<true, 0>);
     set_smem(spmv_f32_drift_kernel<false, 1>);
@@ -855,7 +863,7 @@ void spmv_init() {
     set_smem(spmm_f32_kernel<4, false>);
     set_smem(spmm_f32_kernel<8, true>);
     set_smem(spmm_f32_kernel<8, false>);
-    done = true;
+    done_dev[dev] = 1;
 }
 
 void export_coo(const Layout& L, int32_t* rows, int32_t* cols, float* vals, cudaStream_t st) {

@@ -105,11 +105,20 @@ def case_projections(nranks, n, m, c, ray_block=None):
     for r in range(nranks):
         for k in range(6):
             assert torch.equal(res["coll"][r][k], res["peer"][r][k]), (r, k)
-    rows, cols, vals = oracle.trace_all(n, m, c)
     yf = gather(peer, [o[0] for o in res["peer"]], 1, m * c)
-    assert rel_l2(yf, oracle.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)) <= 1e-5
     xb = gather(peer, [o[3] for o in res["peer"]], 0, n * n)
-    assert rel_l2(xb, oracle.spmv_coo(cols, rows, vals, y.astype(np.float64), n * n)) <= 1e-5
+    if n * n * m <= 256 * 256 * 360:
+        rows, cols, vals = oracle.trace_all(n, m, c)
+        assert rel_l2(yf, oracle.spmv_coo(rows, cols, vals, x.astype(np.float64), m * c)) <= 1e-5
+        assert rel_l2(xb, oracle.spmv_coo(cols, rows, vals, y.astype(np.float64), n * n)) <= 1e-5
+    else:  # full size: sampled rows against the oracle's traces
+        from fullsize import N_RAYS, pick_pixels, sampled_back_error, sampled_forward_error
+        rng = np.random.default_rng(n)
+        rays = rng.choice(m * c, N_RAYS, replace=False)
+        assert sampled_forward_error(oracle, n, m, c, rays, yf[rays], x.astype(np.float64)) <= 1e-5
+        pixels = pick_pixels(rng, n)
+        yh = y.astype(np.float64)
+        assert sampled_back_error(oracle, n, m, c, pixels, xb[pixels], lambda r: yh[r]) <= 1e-5
 
 
 def case_cg(nranks, n, m, c):
@@ -126,10 +135,15 @@ def case_cg(nranks, n, m, c):
     out = {}
     for name, plans in (("coll", coll), ("peer", peer)):
         ys = scatter(plans, y32, 1, np.float32)
+        xa = [torch.empty(p.local_size(0), device="cuda") for p in plans]
         xs = [torch.empty(p.local_size(0), device="cuda") for p in plans]
         torch.cuda.synchronize()
-        out[name] = run_ranks(nranks, lambda r, plans=plans, ys=ys, xs=xs: plans[r].cg(ys[r], 30, x=xs[r]))
-    for a, b in zip(out["coll"], out["peer"]):
+        # a short solve, then a longer one: the second grows the CG scalars (grow-only, no
+        # cudaFree while peers' waits spin -- a device-wide sync there would deadlock)
+        out[name] = run_ranks(nranks, lambda r, plans=plans, ys=ys, xa=xa, xs=xs: (
+            plans[r].cg(ys[r], 10, x=xa[r]), plans[r].cg(ys[r], 30, x=xs[r]))[1])
+        out[name + "10"] = xa
+    for a, b in zip(out["coll"] + out["coll10"], out["peer"] + out["peer10"]):
         assert torch.equal(a, b)
     xr = gather(peer, out["peer"], 0, n * n)
     x_orc = oracle.cgls(rows, cols, vals, y32.astype(np.float64), m * c, n * n, 30)[0]
