@@ -220,6 +220,26 @@ memxct_status_t memxct_footprint_back(memxct_plan_t plan, const void* y_footprin
  * `cuda_stream` may be NULL. */
 memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream);
 
+/* Per-phase wall-clock seconds of the last memxct_build (preprocessing throughput, SURVEY 8(f)
+ * NEXT-3; the paper's preprocessing, timed at 4.00 s for ADS2 and 139 s for RDS1 per
+ * KNL node).  `seconds` (host) receives MEMXCT_BUILD_PHASES doubles, in
+ * this order:
+ *   0 hilbert     two-level pseudo-Hilbert permutations of both domains
+ *   1 decompose   domain decomposition: column-count histogram + tile ranges (P > 1)
+ *   2 count       Siddon count pass of every ray (row lengths; footprint at P > 1)
+ *   3 trace_fwd   Siddon emit pass of A / A_p
+ *   4 sort_fwd    per-row ordering of A's entries (segmented sort; slab order)
+ *   5 layout_fwd  partitions, stage cut, 16-bit SELL layout of A, row grouping
+ *   6 trace_back  pixel histogram + count + emit passes of the transposition's chunks
+ *   7 transpose   order-preserving stable radix sort by pixel
+ *   8 layout_back partitions, stage cut, layout of A^T
+ *   9 exchange    exchange maps (P > 1)
+ *  10 total       the whole memxct_build call
+ * Phases are separated by synchronisations the build performs anyway (CUDA events inside the
+ * chunk loops), so they add up to the total up to host bookkeeping.  STATE before build. */
+#define MEMXCT_BUILD_PHASES 11
+memxct_status_t memxct_build_phases(memxct_plan_t plan, double* seconds);
+
 /* Number of locally owned entries of a domain (0 = tomogram pixels, 1 = sinogram rays) and
  * their natural indices in plan order (host array of `count` int64).  At P = 1 the plan order is
  * the two-level pseudo-Hilbert order, i.e. natural_idx[h] = natural index of Hilbert position h. */

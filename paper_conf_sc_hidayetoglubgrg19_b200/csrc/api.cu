@@ -318,6 +318,15 @@ memxct_status_t memxct_exchange_info(memxct_plan_t plan, int64_t* footprint_rays
     });
 }
 
+memxct_status_t memxct_build_phases(memxct_plan_t plan, double* seconds) {
+    return guarded([&] {
+        mx::Plan& P = built_plan(plan);
+        need(seconds, "seconds");
+        static_assert(mx::kNumPhases == MEMXCT_BUILD_PHASES, "phase table");
+        for (int i = 0; i < mx::kNumPhases; ++i) seconds[i] = P.build_s[i];
+    });
+}
+
 memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
     return guarded([&] {
         mx::Plan& P = plan_of(plan);
@@ -335,6 +344,9 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
         else MX_CUDA(cudaGetDevice(&P.device));
         mx::spmv_init();
         cudaStream_t st = stream_of(cuda_stream);
+        for (double& v : P.build_s) v = 0.0;
+        mx::PhaseClock clk(P.build_s, st);
+        const auto t_build = clk.t;
         P.tile_tomo = (int32_t)(P.opt.tile_tomo ? P.opt.tile_tomo : mx::default_tile(P.n, P.n));
         P.tile_sino = (int32_t)(P.opt.tile_sino ? P.opt.tile_sino : mx::default_tile(P.m, P.c));
         const int64_t npix = (int64_t)P.n * P.n, nrays = (int64_t)P.m * P.c;
@@ -344,6 +356,7 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
         P.sino_h_of_nat.alloc(nrays);
         mx::build_hilbert(P.n, P.n, P.tile_tomo, P.tomo_nat_of_h.p(), P.tomo_h_of_nat.p(), &P.tomo_tile_off, st);
         mx::build_hilbert(P.m, P.c, P.tile_sino, P.sino_nat_of_h.p(), P.sino_h_of_nat.p(), &P.sino_tile_off, st);
+        clk.mark(mx::kPhHilbert);
         P.esize = P.opt.precision == 1 ? 8 : 4;
         if (P.dist) {
             if (P.opt.canonical) mx::fail(MEMXCT_ERR_UNSUPPORTED, "CANONICAL mode is single-GPU only");
@@ -359,6 +372,8 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
         P.fused_dot = !(fd && fd[0] == '0');
         mx::build_matrices(P, st);
         MX_CUDA(cudaStreamSynchronize(st));
+        P.build_s[mx::kPhTotal] =
+            std::chrono::duration<double>(std::chrono::steady_clock::now() - t_build).count();
         P.built = true;
     });
 }

@@ -981,13 +981,16 @@ void build_matrices(Plan& P, cudaStream_t st) {
     G.cos_t = dc.p();
     G.sin_t = ds.p();
 
+    PhaseClock clk(P.build_s, st);
     // a3: this rank's tomogram and sinogram subdomains (whole domains at P = 1)
     decompose(P, G, st);
     const int64_t npix = P.t1 - P.t0;
+    clk.mark(kPhDecompose);
 
     // rows of A_p = footprint rays (every ray at P = 1) and their lengths
     DevArr<int32_t> fp_len;
     const int64_t nrows = P.nfp = footprint(P, G, fp_len, st);
+    clk.mark(kPhCount);
     const int32_t* hray = !P.dist ? nullptr : P.fp_rays.p();
     const bool natural = (P.opt.vector_order == 0);  // P = 1 only
     int32_t R, B, Rb, Bb;
@@ -1123,7 +1126,9 @@ void build_matrices(Plan& P, cudaStream_t st) {
     const int32_t bank = (P.opt.precision == 0 && P.opt.slices > 1) ? (P.opt.slices > 2 ? 8 : 16) : 0;
 
     // ---- A_p: rows = footprint rays; entries of each ray sorted by local pixel --------------
+    double gen_s = 0.0;  // generator time inside build_direction (charged to trace / sort)
     Generator gen_fwd = [&](int64_t ra, int64_t rb, Entries& E, cudaStream_t s) {
+        EventSplit ev;
         const int64_t nr = rb - ra;
         DevArr<int64_t> len64, rp;
         len64.alloc(nr + 1);
@@ -1137,7 +1142,9 @@ void build_matrices(Plan& P, cudaStream_t st) {
         col.alloc(std::max<int64_t>(E.n, 1));
         val.alloc(std::max<int64_t>(E.n, 1));
         E.row.alloc(std::max<int64_t>(E.n, 1));
+        ev.rec(0, s);
         trace_emit(P, G, fwd_hray, ra, nr, P.t0, P.t1, rp.p(), col.p(), val.p(), E.row.p(), s);
+        ev.rec(1, s);
         if (kfwd.p() && E.n > 0) {  // slab stage order: sort each row by its partition's class order
             apply_class_order_kernel<<<blocks_for(E.n), kThreads, 0, s>>>(E.row.p(), E.n, row_class.p(), kfwd.p(),
                                                                           npix, col.p());
@@ -1154,10 +1161,16 @@ void build_matrices(Plan& P, cudaStream_t st) {
                                                         (int)E.n, (int)nr, rp.p(), rp.p() + 1, s));
             MX_LAUNCHED();
         }
+        ev.rec(2, s);
         MX_CUDA(cudaStreamSynchronize(s));
+        const double before = P.build_s[kPhTraceFwd] + P.build_s[kPhSortFwd];
+        ev.charge(P.build_s, kPhTraceFwd, kPhSortFwd);
+        gen_s += P.build_s[kPhTraceFwd] + P.build_s[kPhSortFwd] - before;
     };
     build_direction(P.fwd, nrows, npix, fwd_parts, R, B, gen_fwd, natural ? P.tomo_nat_of_h.p() : nullptr,
                     fwd_out, budget, bank, st, kinv.p(), part_class.p());
+    clk.mark(kPhLayoutFwd);
+    P.build_s[kPhLayoutFwd] -= gen_s;  // the generator's share is in trace / sort
     P.fwd.drift = fwd_drift && 12 * (int64_t)B <= 224 * 1024;
     kfwd.reset();
     kinv.reset();
@@ -1173,9 +1186,13 @@ void build_matrices(Plan& P, cudaStream_t st) {
     pix_cnt.alloc(std::max<int64_t>(npix, 1));
     MX_CUDA(cudaMemsetAsync(pix_cnt.p(), 0, 4 * std::max<int64_t>(npix, 1), st));
     trace_hist(P, G, hray, 0, nrows, P.t0, P.t1, true, pix_cnt.p(), st);
+    clk.mark(kPhTraceBack);
     const Partitions back_parts = make_partitions(pix_cnt.p(), npix, Rb, balance, st);
     pix_cnt.reset();
+    gen_s = 0.0;
     Generator gen_back = [&](int64_t ra, int64_t rb, Entries& E, cudaStream_t s) {
+        EventSplit ev;
+        ev.rec(0, s);
         const int64_t lo = P.t0 + ra, hi = P.t0 + rb;
         DevArr<int32_t> len;
         len.alloc(std::max<int64_t>(nrows, 1));
@@ -1195,6 +1212,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
         ray.alloc(std::max<int64_t>(E.n, 1));
         val.alloc(std::max<int64_t>(E.n, 1));
         trace_emit(P, G, hray, 0, nrows, lo, hi, rp.p(), pix.p(), val.p(), ray.p(), s);
+        ev.rec(1, s);
         rp.reset();
         DevArr<uint32_t> perm;
         E.row.alloc(std::max<int64_t>(E.n, 1));
@@ -1209,14 +1227,21 @@ void build_matrices(Plan& P, cudaStream_t st) {
             offset_u32_kernel<<<blocks_for(E.n), kThreads, 0, s>>>(E.row.p(), E.n, (uint32_t)ra);
             MX_LAUNCHED();
         }
+        ev.rec(2, s);
         MX_CUDA(cudaStreamSynchronize(s));
+        const double before = P.build_s[kPhTraceBack] + P.build_s[kPhTranspose];
+        ev.charge(P.build_s, kPhTraceBack, kPhTranspose);
+        gen_s += P.build_s[kPhTraceBack] + P.build_s[kPhTranspose] - before;
     };
     build_direction(P.back, npix, nrows, back_parts, Rb, Bb, gen_back, natural ? P.sino_nat_of_h.p() : nullptr,
                     natural ? P.tomo_nat_of_h.p() : nullptr, chunk_budget(nnz), bank, st);
+    clk.mark(kPhLayoutBack);
+    P.build_s[kPhLayoutBack] -= gen_s;
 
     // a6: exchange maps of the sparse all-to-allv (P > 1)
     if (P.shard) shard_receive_maps(P, G, st);
     build_exchange(P, st);
+    clk.mark(kPhExchange);
 }
 
 }  // namespace mx

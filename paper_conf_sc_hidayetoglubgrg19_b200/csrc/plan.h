@@ -1,6 +1,7 @@
 // plan.h -- internal plan and layout structures of libmemxct.
 #pragma once
 
+#include <chrono>
 #include <map>
 #include <memory>
 #include <tuple>
@@ -220,8 +221,45 @@ struct CgGraph {
     ~CgGraph() { if (exec) cudaGraphExecDestroy(exec); }
 };
 
+// Wall-clock seconds of the build phases (memxct_build_phases; NEXT-3).  Phases are
+// separated by stream synchronisations the build has anyway, and inside the chunk generators by
+// CUDA events, so timing adds no synchronisation.
+enum BuildPhase {
+    kPhHilbert = 0, kPhDecompose, kPhCount, kPhTraceFwd, kPhSortFwd, kPhLayoutFwd, kPhTraceBack,
+    kPhTranspose, kPhLayoutBack, kPhExchange, kPhTotal, kNumPhases
+};
+struct PhaseClock {
+    double* acc;
+    cudaStream_t st;
+    std::chrono::steady_clock::time_point t;
+    PhaseClock(double* a, cudaStream_t s) : acc(a), st(s), t(std::chrono::steady_clock::now()) {}
+    // synchronise, charge the time since the last mark to `phase`
+    void mark(int phase) {
+        MX_CUDA(cudaStreamSynchronize(st));
+        const auto now = std::chrono::steady_clock::now();
+        acc[phase] += std::chrono::duration<double>(now - t).count();
+        t = now;
+    }
+};
+// events around one step of a chunk generator: [e0, e1) charged to phase a, [e1, e2) to b
+struct EventSplit {
+    cudaEvent_t e[3] = {};
+    EventSplit() { for (auto& v : e) MX_CUDA(cudaEventCreate(&v)); }
+    ~EventSplit() { for (auto& v : e) if (v) cudaEventDestroy(v); }
+    void rec(int i, cudaStream_t st) { MX_CUDA(cudaEventRecord(e[i], st)); }
+    // after the stream is synchronised
+    void charge(double* acc, int a, int b) {
+        float ms = 0.f;
+        MX_CUDA(cudaEventElapsedTime(&ms, e[0], e[1]));
+        acc[a] += 1e-3 * ms;
+        MX_CUDA(cudaEventElapsedTime(&ms, e[1], e[2]));
+        acc[b] += 1e-3 * ms;
+    }
+};
+
 struct Plan {
     int32_t n = 0, m = 0, c = 0;
+    double build_s[kNumPhases] = {};
     Options opt;
     bool built = false;
     int32_t rank = 0, nranks = 1, device = -1;

@@ -35,8 +35,12 @@ SYMBOLS = [
     "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
     "memxct_sirt", "memxct_spmv_time", "memxct_plan_set_shard", "memxct_exchange_counts",
     "memxct_footprint_rays", "memxct_footprint_forward", "memxct_footprint_back", "memxct_layout_rows",
-    "memxct_read_ceiling", "memxct_export_coo",
+    "memxct_read_ceiling", "memxct_export_coo", "memxct_build_phases",
 ]
+
+#: memxct_build_phases order (include/memxct.h)
+BUILD_PHASES = ["hilbert", "decompose", "count", "trace_fwd", "sort_fwd", "layout_fwd", "trace_back",
+                "transpose", "layout_back", "exchange", "total"]
 
 
 def read_ceiling(nbytes: int = 11_600_000_000, reps: int = 10, stream=None) -> float:
@@ -107,6 +111,7 @@ def lib():
             "memxct_layout_rows": [vp, i32, vp],
             "memxct_read_ceiling": [i64, i32, ctypes.POINTER(ctypes.c_double), vp],
             "memxct_export_coo": [vp, i32, vp, vp, vp, vp],
+            "memxct_build_phases": [vp, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -260,6 +265,12 @@ class MemXCT:
     def dtype(self):
         import torch
         return torch.float32 if self.precision == "fp32" else torch.float64
+
+    def build_phases(self) -> dict:
+        """Seconds per preprocessing phase of the build (memxct_build_phases)."""
+        out = np.empty(len(BUILD_PHASES), np.float64)
+        _check(lib().memxct_build_phases(self._h, out.ctypes.data_as(ctypes.c_void_p)), "memxct_build_phases")
+        return dict(zip(BUILD_PHASES, out.tolist()))
 
     def local_size(self, domain: int) -> int:
         v = ctypes.c_int64()

@@ -82,11 +82,19 @@ def test_cfg2_p68_mixed_vs_oracle(orc, coo_cache, nranks):
     xt = inputs.shepp_logan(n)
     ysino = orc.spmv_coo(rows, cols, vals, xt, m * c).astype(np.float32).astype(np.float64)
     yss = scatter(plans, ysino, 1, np.float64)
-    res = run_ranks(nranks, lambda r: plans[r].cg(yss[r], 30, residuals=True))
+    # 10 iterations: fp64 iterates with another summation order agree to ~1e-8 (R16 table);
+    # by iteration 28-30 the order decides up to ~2e-3 (R16: the 1e-3 x_30 gate binds the
+    # single-GPU MIXED + CANONICAL mode), so 30 iterations are gated on the reconstruction
+    res = run_ranks(nranks, lambda r: plans[r].cg(yss[r], 10, residuals=True))
     xr = gather(plans, [v[0] for v in res], 0, n * n)
-    x_orc, res_orc, _, _ = orc.cgls(rows, cols, v32, ysino, m * c, n * n, 30)
+    x_orc, res_orc, _, _ = orc.cgls(rows, cols, v32, ysino, m * c, n * n, 10)
     assert rel_l2(xr, x_orc) <= 1e-6
     assert np.allclose(res[0][1], res_orc, rtol=1e-9)
+    res = run_ranks(nranks, lambda r: plans[r].cg(yss[r], 30, residuals=True))
+    xr = gather(plans, [v[0] for v in res], 0, n * n)
+    x_orc = orc.cgls(rows, cols, v32, ysino, m * c, n * n, 30)[0]
+    print(f"P={nranks} MIXED CG x_30 drift {rel_l2(xr, x_orc):.2e}")
+    assert rel_l2(xr, xt) <= 1.01 * rel_l2(x_orc, xt)
 
 
 @pytest.mark.slow

@@ -490,3 +490,14 @@ def test_export_coo_is_the_oracle_matrix(orc, coo_cache, vector_order):
         assert np.array_equal(key[o], expect)
         ko = np.argsort(rows.astype(np.int64) * (n * n) + cols)
         assert np.array_equal(v[o], vals[ko].astype(np.float32))
+
+
+def test_build_phases_account_for_the_build():
+    """memxct_build_phases (NEXT-3): every phase non-negative, the phases add up to the build's
+    wall time (host bookkeeping aside), and the decomposition / exchange phases are empty at P = 1."""
+    plan = make_plan(256, 360, 256)
+    ph = plan.build_phases()
+    parts = {k: v for k, v in ph.items() if k != "total"}
+    assert all(v >= 0 for v in parts.values()), ph
+    assert ph["total"] > 0 and 0.8 * ph["total"] <= sum(parts.values()) <= 1.05 * ph["total"], ph
+    assert ph["trace_fwd"] > 0 and ph["transpose"] > 0 and ph["layout_fwd"] > 0, ph
