@@ -49,6 +49,12 @@ def parse():
     ap.add_argument("--part-rows", type=int, default=None)
     ap.add_argument("--buffer", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-extras", action="store_true",
+                    help="skip the MIXED+CANONICAL, preprocessing and multi-slice side measurements")
+    ap.add_argument("--cpu-sample", type=float, default=0.05,
+                    help="fraction of the config's rays the oracle baseline traces and times")
+    ap.add_argument("--cpu-full", action="store_true",
+                    help="oracle baseline on the WHOLE config (cfg3: ~30 GB host RAM, minutes)")
     ap.add_argument("--spmv-reps", type=int, default=20)
     ap.add_argument("--slices", type=int, default=4, help="multi-slice batch measured beside the headline (1 = off)")
     ap.add_argument("--variant", default=None, choices=["peer", "dense"], help=argparse.SUPPRESS)
@@ -130,35 +136,50 @@ class Clocks:
 # ------------------------------------------------------------------------------------------
 # the oracle (CPU baseline / reference arm): bounded sample of the same workload
 # ------------------------------------------------------------------------------------------
-def oracle_sample(cfg, frac=0.02, seed=0):
-    """Trace a random `frac` of the config's rays with the oracle (untimed); returns the COO."""
+def host_info():
+    """Host cores and CPU model (nproc / lscpu) of the box the oracle runs on."""
+    model = ""
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.lower().startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
+def oracle_sample(cfg, frac, seed=0):
+    """Trace a random `frac` of the config's rays with the oracle (orc_sample_rows, untimed) and
+    build the CSR of those rows of A and of their transpose (rows = pixels); returns a dict."""
     import oracle
     from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
     n, m, c = inputs.CONFIGS[cfg]
     rng = np.random.default_rng(seed)
-    rays = np.sort(rng.choice(m * c, max(1, int(frac * m * c)), replace=False))
-    rows, cols, vals = [], [], []
-    for i, r in enumerate(rays):
-        pix, ln = oracle.trace_ray(n, m, c, int(r))
-        rows.append(np.full(len(pix), i, np.int32))
-        cols.append(pix)
-        vals.append(ln)
-    return (np.concatenate(rows), np.concatenate(cols), np.concatenate(vals), len(rays), n * n)
-
-
-def oracle_step(sample, nnz_full):
-    """One oracle 'step' on the sample: forward + back SpMV (orc_spmv_coo).  Returns the
-    extrapolated CG iterations per second (1 forward + 1 back per iteration, nnz-proportional)."""
-    import oracle
-    rows, cols, vals, nr, nc = sample
-    x = np.ones(nc)
-    y = np.ones(nr)
+    if frac >= 1.0:
+        rays = np.arange(m * c, dtype=np.int64)
+    else:
+        rays = np.sort(rng.choice(m * c, max(1, int(frac * m * c)), replace=False)).astype(np.int64)
     t0 = time.perf_counter()
-    oracle.spmv_coo(rows, cols, vals, x, nr)
-    oracle.spmv_coo(cols, rows, vals, y, nc)
-    dt = time.perf_counter() - t0
-    t_full = dt * nnz_full / len(rows)
-    return 1.0 / t_full, dt
+    ptr, pix, ln = oracle.sample_rows(n, m, c, rays)
+    t_trace = time.perf_counter() - t0
+    rows = np.repeat(np.arange(len(rays), dtype=np.int32), np.diff(ptr))
+    tp, tc, tv = oracle.coo_to_csr(pix, rows, ln, n * n)     # A^T restricted to the sampled rays
+    return {"ptr": ptr, "cols": pix, "vals": ln, "tptr": tp, "tcols": tc, "tvals": tv,
+            "nrays": len(rays), "npix": n * n, "nnz": len(pix), "trace_s": t_trace, "frac": frac}
+
+
+def oracle_step(sample, threads):
+    """One oracle step on the sample: forward + back threaded CSR SpMV (orc_spmv_csr_threaded,
+    rows split over `threads` host threads; 1 = the plain single-thread product).  Returns
+    (seconds, threads used)."""
+    import oracle
+    x = np.ones(sample["npix"])
+    y = np.ones(sample["nrays"])
+    t0 = time.perf_counter()
+    _, nt = oracle.spmv_csr_threaded(sample["ptr"], sample["cols"], sample["vals"], x, threads)
+    oracle.spmv_csr_threaded(sample["tptr"], sample["tcols"], sample["tvals"], y, threads)
+    return time.perf_counter() - t0, nt
 
 
 def nnz_model(cfg):
@@ -167,42 +188,64 @@ def nnz_model(cfg):
     return int(round(1.1953 * m * n * n))
 
 
-def cpu_baseline(cfg, nnz_full, steps=3):
-    t0 = time.perf_counter()
-    sample = oracle_sample(cfg)
-    t_trace = time.perf_counter() - t0
-    vals = [oracle_step(sample, nnz_full)[0] for _ in range(steps)]
-    return {"value": float(np.median(vals)), "unit": "CG iter/s", "cores": 1, "kind": "oracle",
-            "sample": (f"oracle Siddon-traced {sample[3]} random rays (2%) of cfg{cfg} "
-                       f"({len(sample[0])} nonzeros, {t_trace:.1f} s untimed); timed orc_spmv_coo "
-                       f"forward + back on them (single thread), median of {steps}; CG iter/s "
-                       f"extrapolated by nnz_full/nnz_sample = {nnz_full / len(sample[0]):.1f}")}
+def cpu_baseline(cfg, nnz_full, frac=0.05, reps=3):
+    """the oracle on the box's host cores -- a threaded CSR SpMV over all cores and
+    the single-thread product -- on a bounded random ray sample of the workload, forward + back
+    per CG iteration, extrapolated by nnz (the work is proportional to nnz)."""
+    sample = oracle_sample(cfg, frac)
+    scale = nnz_full / max(1, sample["nnz"])
+    res = {}
+    for threads in (0, 1):
+        best, nt = None, 1
+        for _ in range(reps):
+            dt, nt = oracle_step(sample, threads)
+            best = dt if best is None else min(best, dt)
+        res[threads] = (1.0 / (best * scale), nt, best)
+    hi = host_info()
+    full = sample["frac"] >= 1.0
+    return {"value": res[0][0], "unit": "CG iter/s", "cores": res[0][1], "kind": "oracle",
+            "single_thread": {"value": res[1][0], "unit": "CG iter/s", "cores": 1,
+                              "fwd_back_s_sample": res[1][2]},
+            "threaded_fwd_back_s_sample": res[0][2],
+            "host": hi,
+            "sample": (f"{'all' if full else 'a random %.0f%% of the' % (100 * sample['frac'])} rays of cfg{cfg} "
+                       f"({sample['nrays']} rays, {sample['nnz']} nonzeros) traced by orc_sample_rows "
+                       f"({sample['trace_s']:.1f} s, untimed); timed: forward + back orc_spmv_csr_threaded "
+                       f"on them, best of {reps}, all {res[0][1]} host threads (value) and 1 thread "
+                       f"(single_thread); CG iter/s = 1 / (t x nnz_full / nnz_sample)"
+                       + ("" if full else f", x{scale:.1f}"))}
 
 
 def run_reference(args, rank, world):
+    """The reference arm: the oracle as it stands (threaded CSR SpMV on all host cores) on a
+    bounded sample of the workload; rank 0 only."""
     if rank != 0:
         return
-    from paper_conf_sc_hidayetoglubgrg19_b200 import inputs  # noqa: F401
     cfg = args.config
     nnz_full = nnz_model(cfg)
-    sample = oracle_sample(cfg)
+    sample = oracle_sample(cfg, args.cpu_sample)
+    nt = 1
     for _ in range(args.warmup):
-        oracle_step(sample, nnz_full)
+        oracle_step(sample, 0)
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        oracle_step(sample, nnz_full)
+        _, nt = oracle_step(sample, 0)
     dt = time.perf_counter() - t0
-    # each step processes nnz_sample of the 2*nnz_full work of one CG iteration
-    value = args.steps * len(sample[0]) / nnz_full / dt
+    # each step does forward + back over nnz_sample of the nnz_full of one CG iteration
+    value = args.steps * sample["nnz"] / nnz_full / dt
+    hi = host_info()
+    desc = (f"{sample['nrays']} random rays ({100 * sample['frac']:.0f}%) of cfg{cfg}, {sample['nnz']} "
+            f"nonzeros; forward + back orc_spmv_csr_threaded per step on {nt} host threads "
+            f"({hi['cpu_model']}), extrapolated to full nnz")
     line = {
         "impl": "reference", "metric": "CG iter/s", "value": value, "unit": "CG iter/s",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": workload_name(cfg, args.iters) + " (oracle: 2% ray sample, "
+        "config": {"workload": workload_name(cfg, args.iters) + " (oracle: ray sample, "
                    "forward + back SpMV per step, extrapolated to full nnz)"},
-        "cpu_baseline": {"value": value, "unit": "CG iter/s", "cores": 1, "kind": "oracle",
-                         "sample": f"{sample[3]} random rays of cfg{cfg}, {len(sample[0])} nonzeros"},
+        "cpu_baseline": {"value": value, "unit": "CG iter/s", "cores": nt, "kind": "oracle",
+                         "sample": desc, "host": hi},
         "e2e": {"value": value, "unit": "CG iter/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -263,6 +306,69 @@ def bench_multislice(args, plan1, y1, n, m, c, stream):
            "note": "K independent 30-iteration CGLS solves per step sharing one matrix stream per "
                    "SpMM; each slice bit-identical to its single-slice solve (tests)"}
     plan.close()
+    return out
+
+
+def bench_mixed_canonical(args, n, m, c, ph, stream):
+    """The parity-gated mode (reading R16: PRECISION = MIXED, CANONICAL = 1 -- fp64 vectors and
+    one fp64 fma chain per row in Hilbert order, dots as fixed chains; its 30-iteration image is
+    bit-identical to the canonical oracle's), timed like the headline: `steps` CGLS solves of the
+    same slice.  The matrix stream is the same 6 B per nonzero as FP32."""
+    import torch
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
+    plan = MemXCT(n, m, c, precision="mixed", canonical=True).build()
+    y = plan.forward(torch.from_numpy(ph.astype(np.float64)).cuda())
+    x = torch.empty(plan.local_size(0), dtype=torch.float64, device=y.device)
+    for _ in range(max(1, args.warmup)):
+        plan.cg(y, args.iters, x=x, stream=stream)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        plan.cg(y, args.iters, x=x, stream=stream)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    sp = plan.spmv_time(10, stream=stream)
+    fi, bi = plan.layout_info(0), plan.layout_info(1)
+    out = {"value": args.iters * args.steps / (ms * 1e-3), "unit": "CG iter/s", "ms_per_step": ms / args.steps,
+           "spmv_fwd_ms": sp["fwd_us"] * 1e-3, "spmv_back_ms": sp["back_us"] * 1e-3,
+           "spmv_gbs": (spmv_bytes(fi) + spmv_bytes(bi)) / ((sp["fwd_us"] + sp["back_us"]) * 1e-6) / 1e9,
+           "buffer_entries_fp64": [fi["buffer_entries"], bi["buffer_entries"]],
+           "note": "PRECISION=MIXED, CANONICAL=1: the mode the 1e-3 x_30 gate binds (bit-identical to "
+                   "the canonical oracle in tests); same matrix bytes as FP32"}
+    plan.close()
+    return out
+
+
+PAPER_PREPROC = {  # per node, the paper's Tables 4-5 (P:935-941, P:972-983): context, other hardware
+    "ADS2": {"shape": (512, 750, 512), "paper_s": 4.00, "paper_hw": "1 KNL (Theta), Table 4"},
+    "RDS1": {"shape": (2048, 1501, 2048), "paper_s": 139.0, "paper_hw": "1 KNL (Theta), Table 5 (146.3 s in Table 4)"},
+}
+
+
+def bench_preprocessing(args, plan, build_s):
+    """preprocessing throughput (memxct_build: Hilbert ordering, Siddon
+    tracing, transposition, buffered layouts) per phase -- the bench config's build, and fresh
+    builds at the paper's ADS2 (750 x 512) and RDS1 (1501 x 2048) shapes, whose single-node
+    preprocessing the paper times at 4.00 s and 139 s on one KNL."""
+    import torch
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT
+    out = {f"cfg{args.config}": {"build_s": build_s, "phases_s": plan.build_phases(),
+                                 "nnz": plan.stats()["nnz"]}}
+    for name, d in PAPER_PREPROC.items():
+        n, m, c = d["shape"]
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        p = MemXCT(n, m, c).build()
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - t0
+        out[name] = {"shape": {"n": n, "projections": m, "channels": c}, "build_s": wall,
+                     "phases_s": p.build_phases(), "nnz": p.stats()["nnz"],
+                     "nnz_per_s": p.stats()["nnz"] / wall,
+                     "paper_s": d["paper_s"], "paper_hw": d["paper_hw"]}
+        p.close()
+        del p
     return out
 
 
@@ -392,22 +498,38 @@ def run_ours(args, rank, world):
     launches = kernel_launch_count() - k0
     ms = ev0.elapsed_time(ev1)
 
-    # SpMV kernels alone, each launch bracketed by events on the launching stream
+    # SpMV kernels alone, each launch bracketed by events on the launching stream.  N > 1: the
+    # rank's A_p / A_p^T kernels without the exchange (memxct_spmv_time, CUDA events on this
+    # stream), so the roofline is the kernel's; the exchange is timed separately below.
     fwd_ms, back_ms = [], []
-    yb = torch.empty_like(y)
-    xb = torch.empty_like(x)
-    evs = [torch.cuda.Event(enable_timing=True) for _ in range(2 * args.spmv_reps + 1)]
-    evs[0].record(stream)
-    for i in range(args.spmv_reps):
-        plan.forward(x, yb, stream=stream)
-        evs[2 * i + 1].record(stream)
-        plan.back(y, xb, stream=stream)
-        evs[2 * i + 2].record(stream)
-    torch.cuda.synchronize()
-    for i in range(args.spmv_reps):
-        fwd_ms.append(evs[2 * i].elapsed_time(evs[2 * i + 1]))
-        back_ms.append(evs[2 * i + 1].elapsed_time(evs[2 * i + 2]))
+    if dist_mode:
+        sp_t = plan.spmv_time(args.spmv_reps, stream=stream)
+        fwd_ms, back_ms = [sp_t["fwd_us"] * 1e-3], [sp_t["back_us"] * 1e-3]
+    else:
+        yb = torch.empty_like(y)
+        xb = torch.empty_like(x)
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(2 * args.spmv_reps + 1)]
+        evs[0].record(stream)
+        for i in range(args.spmv_reps):
+            plan.forward(x, yb, stream=stream)
+            evs[2 * i + 1].record(stream)
+            plan.back(y, xb, stream=stream)
+            evs[2 * i + 2].record(stream)
+        torch.cuda.synchronize()
+        for i in range(args.spmv_reps):
+            fwd_ms.append(evs[2 * i].elapsed_time(evs[2 * i + 1]))
+            back_ms.append(evs[2 * i + 1].elapsed_time(evs[2 * i + 2]))
     clk = clocks.stop()
+    # per-rank kernel times and algorithmic bytes (one row per rank at N > 1)
+    per_rank = torch.tensor([float(np.median(fwd_ms)), float(np.median(back_ms)),
+                             spmv_bytes(fi), spmv_bytes(bi), fi["nnz"], bi["nnz"]],
+                            dtype=torch.float64, device=dev)
+    if dist_mode:
+        gathered = [torch.empty_like(per_rank) for _ in range(world)]
+        dist.all_gather(gathered, per_rank)
+        per_rank_all = torch.stack(gathered).cpu().numpy()
+    else:
+        per_rank_all = per_rank.cpu().numpy()[None, :]
 
     t = torch.tensor([ms], dtype=torch.float64, device=dev)
     if dist_mode:
@@ -433,14 +555,14 @@ def run_ours(args, rank, world):
     exch_t = None
     if dist_mode:
         exch_t = plan.exchange_time(20, stream=stream)
-        sp_t = plan.spmv_time(20, stream=stream)
-        et = torch.tensor([exch_t["fwd_us"], exch_t["back_us"], sp_t["fwd_us"], sp_t["back_us"]],
-                          dtype=torch.float64, device=dev)
+        et = torch.tensor([exch_t["fwd_us"], exch_t["back_us"]], dtype=torch.float64, device=dev)
         dist.all_reduce(et, op=dist.ReduceOp.MAX)
         exch_t = {"fwd_us": float(et[0]), "back_us": float(et[1]),
                   "per_cg_iter_us": float(et[0] + et[1]),
-                  "local_spmv_fwd_us": float(et[2]), "local_spmv_back_us": float(et[3]),
-                  "how": "max over ranks, CUDA events, 20 reps; local_spmv = A_p / A_p^T kernels alone"}
+                  "local_spmv_fwd_us": float(per_rank_all[:, 0].max() * 1e3),
+                  "local_spmv_back_us": float(per_rank_all[:, 1].max() * 1e3),
+                  "how": "max over ranks, CUDA events, 20 reps (memxct_exchange_time: C + R forward, "
+                         "R^T + C^T back, no SpMV); local_spmv = A_p / A_p^T kernels alone"}
 
     peer = dense = None
     if dist_mode:
@@ -449,17 +571,23 @@ def run_ours(args, rank, world):
         dense = bench_exchange_variant(args, rank, world, "dense")
         dist.barrier()
 
-    multislice = None
-    if args.slices > 1 and not dist_mode:
-        multislice = bench_multislice(args, plan, y, n, m, c, stream)
+    multislice = mixed = prep = None
+    if not dist_mode and not args.no_extras:
+        prep = bench_preprocessing(args, plan, build_s)
+        mixed = bench_mixed_canonical(args, n, m, c, ph, stream)
+        if args.slices > 1:
+            multislice = bench_multislice(args, plan, y, n, m, c, stream)
 
     if rank != 0:
         return
     from paper_conf_sc_hidayetoglubgrg19_b200.memxct import read_ceiling
     read_gbs = read_ceiling(8_000_000_000, 20, stream=stream)  # live, same GPU, after the timed region
     hbm_peak, peak_src = peaks()
-    fb, bb = spmv_bytes(fi), spmv_bytes(bi)
-    tf, tb = float(np.median(fwd_ms)) * 1e-3, float(np.median(back_ms)) * 1e-3
+    # dominant kernel = the SpMV pair of the slowest rank (the one every CG iteration waits for)
+    slow = int(np.argmax(per_rank_all[:, 0] + per_rank_all[:, 1]))
+    tf, tb = per_rank_all[slow, 0] * 1e-3, per_rank_all[slow, 1] * 1e-3
+    fb, bb = per_rank_all[slow, 2], per_rank_all[slow, 3]
+    fnnz, bnnz = per_rank_all[slow, 4], per_rank_all[slow, 5]
     achieved = (fb + bb) / (tf + tb) / 1e9
     traffic = None
     prof = os.path.join(ROOT, "profiles", f"ncu_spmv_cfg{cfg}.json")
@@ -482,7 +610,10 @@ def run_ours(args, rank, world):
                    "parallelism": (f"domain decomposition over {world} GPUs (A = R C A_p, NCCL all-to-allv)"
                                    if dist_mode else "single GPU")},
         "spmv": {"fwd_ms": tf * 1e3, "back_ms": tb * 1e3,
-                 "fwd_gflops": 2 * fi["nnz"] / tf / 1e9, "back_gflops": 2 * bi["nnz"] / tb / 1e9,
+                 "fwd_gflops": 2 * fnnz / tf / 1e9, "back_gflops": 2 * bnnz / tb / 1e9,
+                 "rank": slow,
+                 "how": ("slowest rank's A_p / A_p^T kernels alone (memxct_spmv_time), exchange excluded"
+                         if dist_mode else "forward / back SpMV launches, CUDA events, median"),
                  "fwd_gbs": fb / tf / 1e9, "back_gbs": bb / tb / 1e9,
                  "nnz": st["nnz"], "stored_slots_per_dir": [fi["slots"], bi["slots"]],
                  "padding": [fi["slots"] / fi["nnz"] - 1, bi["slots"] / bi["nnz"] - 1],
@@ -491,7 +622,8 @@ def run_ours(args, rank, world):
                                           6 * bi["slots"] + 4 * bi["map_entries"]]},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
                      "frac": achieved / hbm_peak, "traffic": traffic, "peak_source": peak_src,
-                     "kernel": "spmv_f32_kernel (forward A + back A^T, per launch)",
+                     "kernel": "spmv_f32_kernel (forward A + back A^T, per launch)" +
+                               (f"; rank {slow}'s A_p + A_p^T, the slowest of {world}" if dist_mode else ""),
                      "algorithmic_bytes_per_launch": [fb, bb],
                      "read_ceiling": {"gbs": read_gbs, "frac": achieved / read_gbs,
                                       "how": "memxct_read_ceiling: 8 GB read-only stream with the SpMV's "
@@ -506,6 +638,13 @@ def run_ours(args, rank, world):
     }
     if dist_mode:
         line["exchange"] = {**plan.exchange_info(), **exch_t}
+        line["spmv"]["per_rank_ms"] = [[float(a), float(b)] for a, b in per_rank_all[:, :2]]
+        line["spmv"]["aggregate_gflops"] = float(2 * (per_rank_all[:, 4].sum() + per_rank_all[:, 5].sum())
+                                                 / ((tf + tb)) / 1e9)
+    if prep is not None:
+        line["preprocessing"] = prep
+    if mixed is not None:
+        line["mixed_canonical"] = {**mixed, "ratio_to_fp32": mixed["value"] / value}
     if multislice is not None:
         line["multislice"] = multislice
     if peer is not None:
@@ -513,8 +652,24 @@ def run_ours(args, rank, world):
     if dense is not None:
         line["dense_exchange"] = dense
     if not args.no_cpu_baseline and world == 1:
-        line["cpu_baseline"] = cpu_baseline(cfg, st["nnz"])
+        line["cpu_baseline"] = cpu_baseline(cfg, st["nnz"], 1.0 if args.cpu_full else args.cpu_sample)
     print(json.dumps(line), flush=True)
+
+
+def self_launch(args):
+    """`--gpus N` (N > 1) without a torchrun environment: start N ranks of this script with
+    torch.distributed.run on this node (127.0.0.1); exit non-zero if the node has fewer than N
+    GPUs.  Returns the launcher's exit code."""
+    import torch
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        print(f"bench.py: --gpus {args.gpus} needs {args.gpus} CUDA devices, this node has {have}",
+              file=sys.stderr, flush=True)
+        return 2
+    port = os.environ.get("MASTER_PORT", str(29400 + os.getpid() % 500))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", port, os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
 
 
 def main():
@@ -522,8 +677,13 @@ def main():
     if args.variant:
         variant_child(args)
         return
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1 and args.impl == "ours":
+        sys.exit(self_launch(args))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
+    if args.impl == "ours" and world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr, flush=True)
+        sys.exit(2)
     if world == 1 and args.distributed and args.impl == "ours":
         for k, v in (("MASTER_ADDR", "127.0.0.1"), ("MASTER_PORT", "29533"), ("RANK", "0"),
                      ("WORLD_SIZE", "1"), ("LOCAL_RANK", "0")):

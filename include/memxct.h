@@ -164,6 +164,21 @@ memxct_status_t memxct_local_group_create(int32_t nranks, memxct_group_t* out);
 memxct_status_t memxct_local_group_destroy(memxct_group_t group);
 memxct_status_t memxct_plan_set_comm_local(memxct_plan_t plan, memxct_group_t group, int32_t rank);
 
+/* Host transport (processes of one node, possibly sharing one GPU): rank in [0, nranks <= 16) of
+ * a job whose processes rendezvous through the POSIX shared-memory segment `name` ("/<token>",
+ * unique per job and plan; rank 0 creates it at build, the others attach, rank 0 unlinks it once
+ * all are attached -- the caller broadcasts the name, e.g. over torch.distributed gloo).  The
+ * build's collectives and the collective exchanges (EXCHANGE = 0, 2) move device data between the
+ * processes through CUDA-IPC-mapped device mailboxes with host barriers; the fused exchange
+ * (EXCHANGE = 1) maps the peers' buffers with cudaIpcOpenMemHandle and synchronises through
+ * system-scope flags exactly as NCCL ranks do (waits in one-thread kernels when the ranks share a
+ * GPU).  Same decomposition, kernels and results as NCCL ranks / virtual ranks (sums over ranks in
+ * rank order); not graph-captured.  The multi-process form of the virtual ranks: it runs the
+ * cross-process data plane where NCCL cannot (NCCL rejects two ranks on one device).  Before
+ * build.  Errors: INVALID_ARG (rank, name), NCCL (a peer process never arrives: ~300 s). */
+memxct_status_t memxct_plan_set_comm_host(memxct_plan_t plan, int32_t rank, int32_t nranks,
+                                          const char* name, int32_t cuda_device);
+
 /* Shard probe: build on this device only rank `rank`'s part of a `nranks`-way decomposition
  * -- the same tile ranges (R12), footprint rays, A_p, A_p^T and exchange counts /
  * maps that rank would build inside a real P-rank job, with no peers and no communicator (the

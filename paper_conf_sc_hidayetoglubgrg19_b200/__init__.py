@@ -7,5 +7,5 @@
 The CUDA library (libmemxct.so, built by build_ext.py) is loaded on first use; there is no CPU
 fallback.  ``inputs`` holds the seeded synthetic-input generators.
 """
-from .memxct import (LocalGroup, MemXCT, MemXCTError, bootstrap_unique_id,  # noqa: F401
+from .memxct import (LocalGroup, MemXCT, MemXCTError, bootstrap_host_comm_name, bootstrap_unique_id,  # noqa: F401
                      get_unique_id, kernel_launch_count, lib, partition_ranges)

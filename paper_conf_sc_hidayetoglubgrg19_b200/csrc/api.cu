@@ -225,6 +225,27 @@ memxct_status_t memxct_plan_set_comm(memxct_plan_t plan, int32_t rank, int32_t n
         P.shard = false;
         P.device = cuda_device;
         P.local_group.reset();
+        P.host_comm.clear();
+    });
+}
+
+memxct_status_t memxct_plan_set_comm_host(memxct_plan_t plan, int32_t rank, int32_t nranks, const char* name,
+                                          int32_t cuda_device) {
+    return guarded([&] {
+        mx::Plan& P = plan_of(plan);
+        if (P.built) mx::fail(MEMXCT_ERR_STATE, "set_comm must precede memxct_build");
+        if (nranks < 1 || nranks > 16 || rank < 0 || rank >= nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank / nranks");
+        need(name, "name");
+        if (name[0] != '/' || std::strlen(name) < 2 || std::strlen(name) > 200 || std::strchr(name + 1, '/'))
+            mx::fail(MEMXCT_ERR_INVALID_ARG, "name must be \"/<token>\" (a POSIX shared-memory name)");
+        P.unique_id.clear();
+        P.local_group.reset();
+        P.host_comm = name;
+        P.rank = rank;
+        P.nranks = nranks;
+        P.dist = true;
+        P.shard = false;
+        P.device = cuda_device;
     });
 }
 
@@ -235,6 +256,7 @@ memxct_status_t memxct_plan_set_shard(memxct_plan_t plan, int32_t rank, int32_t 
         if (nranks < 1 || rank < 0 || rank >= nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank / nranks");
         P.unique_id.clear();
         P.local_group.reset();
+        P.host_comm.clear();
         P.rank = rank;
         P.nranks = nranks;
         P.dist = true;
@@ -273,6 +295,7 @@ memxct_status_t memxct_plan_set_comm_local(memxct_plan_t plan, memxct_group_t gr
         P.dist = true;
         P.shard = false;
         P.local_group = group->g;
+        P.host_comm.clear();
     });
 }
 
@@ -363,6 +386,7 @@ memxct_status_t memxct_build(memxct_plan_t plan, void* cuda_stream) {
             if (P.shard && P.opt.exchange == 1) mx::fail(MEMXCT_ERR_UNSUPPORTED, "a shard probe has no peers to map");
             if (P.shard) P.comm.reset();
             else if (P.local_group) P.comm = mx::make_local_comm(P.local_group, P.rank);
+            else if (!P.host_comm.empty()) P.comm = mx::make_host_comm(P.host_comm, P.rank, P.nranks);
             else P.comm = mx::make_nccl_comm(P.rank, P.nranks, P.unique_id.data());
         }
         // CG dots fused into the SpMV epilogue (per-CTA tree + last-CTA sum, deterministic):

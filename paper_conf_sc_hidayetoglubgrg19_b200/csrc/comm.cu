@@ -236,6 +236,7 @@ public:
         nranks = g_->nranks;
     }
     bool capturable() const override { return false; }
+    bool shares_device() const override { return true; }
 
     void allreduce_sum(void* buf, int64_t count, DType t, cudaStream_t st) override {
         MX_CUDA(cudaStreamSynchronize(st));

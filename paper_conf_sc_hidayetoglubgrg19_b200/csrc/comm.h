@@ -13,6 +13,7 @@
 #include <condition_variable>
 #include <memory>
 #include <mutex>
+#include <string>
 #include <vector>
 
 #include "common.h"
@@ -49,9 +50,15 @@ public:
     // Host poll of asynchronous transport errors (NCCL: ncclCommGetAsyncError); throws
     // MEMXCT_ERR_NCCL.  Called at the start of every library call on a decomposed plan.
     virtual void check_async() {}
+    // true when every rank runs on this rank's device (virtual ranks, or host-transport processes
+    // sharing a GPU): the fused exchange then keeps its waits in one-thread kernels
+    virtual bool shares_device() const { return false; }
 };
 
 std::unique_ptr<Comm> make_nccl_comm(int rank, int nranks, const void* unique_id);
+// processes of one node (possibly sharing a GPU) over a named POSIX shared-memory segment and
+// CUDA IPC device mailboxes (proccomm.cu); not graph-capturable
+std::unique_ptr<Comm> make_host_comm(const std::string& name, int rank, int nranks);
 void nccl_unique_id(void* out);
 
 // shared state of a group of virtual ranks

@@ -153,7 +153,7 @@ void peer_setup(Plan& P, cudaStream_t st) {
     X.flags.alloc(4 * np + 2);
     MX_CUDA(cudaMemsetAsync(X.flags.p(), 0, 8 * (4 * np + 2), st));
     // folded waits only where every rank has its own GPU (see PeerArgs::fold); MEMXCT_PEER_FOLD=0/1
-    X.fold = !P.local_group;
+    X.fold = !C.shares_device();
     if (const char* e = std::getenv("MEMXCT_PEER_FOLD")) X.fold = e[0] == '1';
     MX_CUDA(cudaStreamSynchronize(st));
     // where my rows land in every owner's receive buffer, and my values in every peer's footprint

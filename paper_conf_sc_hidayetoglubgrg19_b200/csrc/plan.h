@@ -280,6 +280,7 @@ struct Plan {
     std::unique_ptr<Comm> comm;
     std::shared_ptr<LocalGroup> local_group;
     std::vector<uint8_t> unique_id;
+    std::string host_comm;  // memxct_plan_set_comm_host: shared-memory segment name
     int64_t t0 = 0, t1 = 0, s0 = 0, s1 = 0;
     std::vector<int64_t> tomo_bounds, sino_bounds;      // per rank, Hilbert index ranges
     std::vector<int64_t> tomo_tile_off, sino_tile_off;  // Hilbert offset of every tile (+ total)

@@ -35,7 +35,7 @@ SYMBOLS = [
     "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
     "memxct_sirt", "memxct_spmv_time", "memxct_plan_set_shard", "memxct_exchange_counts",
     "memxct_footprint_rays", "memxct_footprint_forward", "memxct_footprint_back", "memxct_layout_rows",
-    "memxct_read_ceiling", "memxct_export_coo", "memxct_build_phases",
+    "memxct_read_ceiling", "memxct_export_coo", "memxct_build_phases", "memxct_plan_set_comm_host",
 ]
 
 #: memxct_build_phases order (include/memxct.h)
@@ -112,6 +112,7 @@ def lib():
             "memxct_read_ceiling": [i64, i32, ctypes.POINTER(ctypes.c_double), vp],
             "memxct_export_coo": [vp, i32, vp, vp, vp, vp],
             "memxct_build_phases": [vp, vp],
+            "memxct_plan_set_comm_host": [vp, i32, i32, ctypes.c_char_p, i32],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -185,6 +186,16 @@ class LocalGroup:
             pass
 
 
+def bootstrap_host_comm_name(rank: int, group=None) -> str:
+    """Rank 0 draws a fresh shared-memory segment name for memxct_plan_set_comm_host; every rank
+    receives it through torch.distributed (gloo is enough)."""
+    import torch.distributed as dist
+    import uuid
+    obj = ["/memxct-" + uuid.uuid4().hex[:20] if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
 def bootstrap_unique_id(rank: int, group=None) -> bytes:
     """Rank 0 makes an ncclUniqueId; every rank receives it through torch.distributed."""
     import torch.distributed as dist
@@ -206,7 +217,7 @@ class MemXCT:
                  cg_variant: int = 0, rank: int = 0, nranks: int = 1, unique_id: bytes = None,
                  device: int = None, group: "LocalGroup" = None, slices: int = None,
                  exchange: str = None, shard: bool = False, ray_block: int = None,
-                 stage_order: int = None):
+                 stage_order: int = None, host_comm: str = None):
         self.n, self.m, self.c = int(n), int(projections), int(channels)
         self._h = ctypes.c_void_p()
         _check(lib().memxct_plan_create(self.n, self.m, self.c, ctypes.byref(self._h)),
@@ -228,6 +239,10 @@ class MemXCT:
                    "memxct_plan_set_shard")
         elif group is not None:
             _check(lib().memxct_plan_set_comm_local(self._h, group._h, int(rank)), "memxct_plan_set_comm_local")
+        elif host_comm is not None:
+            _check(lib().memxct_plan_set_comm_host(self._h, self.rank, int(nranks), host_comm.encode(),
+                                                   -1 if device is None else int(device)),
+                   "memxct_plan_set_comm_host")
         elif nranks > 1 or device is not None or unique_id is not None:
             uid = None if unique_id is None else ctypes.create_string_buffer(unique_id, 128)
             _check(lib().memxct_plan_set_comm(self._h, rank, nranks, uid,
