@@ -61,7 +61,8 @@ std::vector<int64_t> to_host_i64(const int64_t* d, int64_t n, cudaStream_t st) {
 template <class T>
 __global__ void __launch_bounds__(kT)
 reduce_dot_kernel(const T* __restrict__ recv, const int64_t* __restrict__ ptr, const int32_t* __restrict__ pos,
-                  int64_t nown, T* __restrict__ y, double* part, double* dot_out, unsigned int* ticket, PeerArgs pa) {
+                  int64_t nown, T* __restrict__ y, double* part, double* dot_out, unsigned int* ticket, PeerArgs pa,
+                  const T* __restrict__ self, int64_t self_lo, int64_t self_hi) {
     __shared__ double red[kT / 32];
     __shared__ bool am_last;
     if (pa.fold) {
@@ -74,7 +75,12 @@ reduce_dot_kernel(const T* __restrict__ recv, const int64_t* __restrict__ ptr, c
         T acc;
         if (ptr) {
             acc = T(0);
-            for (int64_t k = ptr[i]; k < ptr[i + 1]; ++k) acc += recv[pos[k]];  // peer order
+            for (int64_t k = ptr[i]; k < ptr[i + 1]; ++k) {  // peer order
+                const int64_t q = pos[k];
+                // this rank's own partial is read in place from its footprint slice (`self`):
+                // no copy into the receive buffer
+                acc += (q >= self_lo && q < self_hi) ? self[q - self_lo] : recv[q];
+            }
         } else {
             acc = recv[i];
         }
@@ -125,6 +131,18 @@ template <class T>
 __global__ void pack_kernel(const T* __restrict__ y, const int32_t* __restrict__ idx, int64_t n, T* __restrict__ out) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         out[i] = y[idx[i]];
+}
+
+// R^T with the self slice [lo, hi) of the pack order written straight into this rank's
+// footprint slice `self` (no copy through the receive buffer and the all-to-allv)
+template <class T>
+__global__ void pack_self_kernel(const T* __restrict__ y, const int32_t* __restrict__ idx, int64_t n,
+                                 T* __restrict__ out, T* __restrict__ self, int64_t lo, int64_t hi) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const T v = y[idx[i]];
+        if (i >= lo && i < hi) self[i - lo] = v;
+        else out[i] = v;
+    }
 }
 
 template <class T>
@@ -381,14 +399,24 @@ void build_exchange(Plan& P, cudaStream_t st) {
     if (P.opt.exchange == 1) peer_setup(P, st);  // fused peer-memory exchange (peer.cu)
 }
 
+// self (nullable): this rank's footprint partials; the receive positions [rdispl[me],
+// rdispl[me + 1]) are then read from self instead of `recv` (the self slice is not copied)
 template <class T>
-void launch_reduce_dot(Plan& P, const T* recv, bool csr, T* y, double* dot_out, const PeerArgs& pa, cudaStream_t st) {
+void launch_reduce_dot(Plan& P, const T* recv, bool csr, T* y, double* dot_out, const PeerArgs& pa, cudaStream_t st,
+                       const T* self = nullptr) {
     Exchange& X = P.ex;
     const int64_t nown = P.s1 - P.s0;
+    const int64_t lo = self ? X.rdispl[P.rank] : 0, hi = self ? X.rdispl[P.rank + 1] : 0;
     reduce_dot_kernel<T><<<nblocks(nown), kT, 0, st>>>(recv, csr ? X.red_ptr.p() : nullptr, X.red_pos.p(), nown, y,
-                                                       X.dot_part.p(), dot_out, X.tickets.p() + 2, pa);
+                                                       X.dot_part.p(), dot_out, X.tickets.p() + 2, pa, self, lo, hi);
     MX_LAUNCHED();
 }
+
+// the all-to-allv counts without this rank's own slice (it stays in place, see above)
+struct RemoteCounts {
+    std::vector<int64_t> sc, rc;
+    RemoteCounts(const Exchange& X, int me) : sc(X.scount), rc(X.rcount) { sc[me] = rc[me] = 0; }
+};
 
 // Forward communication: footprint partials `yfp` (nfp) -> owned ray values `yown` (nown).
 // Sparse (default): C = all-to-allv of the per-owner slices into `rb` (nrecv), R = per owned ray
@@ -410,8 +438,9 @@ static void exchange_fwd(Plan& P, const T* yfp, T* rb, T* yown, cudaStream_t st,
         launch_reduce_dot<T>(P, X.dense_own.as<T>(), false, yown, dot_out, PeerArgs{}, st);  // copy (+ dot)
         return;
     }
-    P.comm->alltoallv(yfp, X.scount.data(), X.sdispl.data(), rb, X.rcount.data(), X.rdispl.data(), t, st);  // C
-    launch_reduce_dot<T>(P, rb, true, yown, dot_out, PeerArgs{}, st);                                      // R
+    const RemoteCounts rcnt(X, P.rank);
+    P.comm->alltoallv(yfp, rcnt.sc.data(), X.sdispl.data(), rb, rcnt.rc.data(), X.rdispl.data(), t, st);  // C
+    launch_reduce_dot<T>(P, rb, true, yown, dot_out, PeerArgs{}, st, yfp + X.sdispl[P.rank]);            // R
 }
 
 // Back communication: owned ray values `yown` -> every footprint ray's value in `yfp`.  Sparse:
@@ -433,11 +462,13 @@ static void exchange_back(Plan& P, const T* yown, T* rb, T* yfp, cudaStream_t st
         }
         return;
     }
-    if (X.nrecv > 0) {
-        pack_kernel<T><<<nblocks(X.nrecv), kT, 0, st>>>(yown, X.recv_idx.p(), X.nrecv, rb);  // R^T
+    if (X.nrecv > 0) {  // R^T (own slice straight into the footprint buffer)
+        pack_self_kernel<T><<<nblocks(X.nrecv), kT, 0, st>>>(yown, X.recv_idx.p(), X.nrecv, rb, yfp + X.sdispl[P.rank],
+                                                             X.rdispl[P.rank], X.rdispl[P.rank + 1]);
         MX_LAUNCHED();
     }
-    P.comm->alltoallv(rb, X.rcount.data(), X.rdispl.data(), yfp, X.scount.data(), X.sdispl.data(), t, st);  // C^T
+    const RemoteCounts rcnt(X, P.rank);
+    P.comm->alltoallv(rb, rcnt.rc.data(), X.rdispl.data(), yfp, rcnt.sc.data(), X.sdispl.data(), t, st);  // C^T
 }
 
 // P > 1 with dot_out: the CG dot of the rank's output part is fused into the reduction
@@ -462,15 +493,10 @@ static void forward_t(Plan& P, const T* x, T* y, double* dot_out, cudaStream_t s
         if constexpr (sizeof(T) == 4) spmv_f32(L, x, yfp, nullptr, nullptr, nullptr, X.side, L.n_first, L.nparts);
         else spmv_f64(L, x, yfp, nullptr, nullptr, nullptr, false, X.side, L.n_first, L.nparts);
         MX_CUDA(cudaEventRecord(X.ev_join, X.side));
-        const int me = P.rank;
-        std::vector<int64_t> sc(X.scount), rc(X.rcount);  // the self slice moves after the join
-        sc[me] = rc[me] = 0;
-        P.comm->alltoallv(yfp, sc.data(), X.sdispl.data(), rb, rc.data(), X.rdispl.data(), t, st);  // C (remote)
+        const RemoteCounts rcnt(X, P.rank);  // the self slice is read in place after the join
+        P.comm->alltoallv(yfp, rcnt.sc.data(), X.sdispl.data(), rb, rcnt.rc.data(), X.rdispl.data(), t, st);  // C
         MX_CUDA(cudaStreamWaitEvent(st, X.ev_join, 0));
-        if (X.scount[me] > 0)
-            MX_CUDA(cudaMemcpyAsync(rb + X.rdispl[me], yfp + X.sdispl[me], sizeof(T) * X.scount[me],
-                                    cudaMemcpyDeviceToDevice, st));
-        launch_reduce_dot<T>(P, rb, true, y, dot_out, PeerArgs{}, st);      // R
+        launch_reduce_dot<T>(P, rb, true, y, dot_out, PeerArgs{}, st, yfp + X.sdispl[P.rank]);  // R
         return;
     }
     spmv_any(P, P.fwd, x, yfp, st);                                         // A_p
@@ -657,6 +683,7 @@ void preload_exchange_kernels() {
     MX_CUDA(cudaFuncGetAttributes(&fa, reduce_dot_kernel<float>));
     MX_CUDA(cudaFuncGetAttributes(&fa, reduce_dot_kernel<double>));
     MX_CUDA(cudaFuncGetAttributes(&fa, pack_kernel<float>));
+    MX_CUDA(cudaFuncGetAttributes(&fa, pack_self_kernel<float>));
 }
 
 void reduce_partials(Plan& P, const float* recv, float* y, double* dot_out, const PeerArgs& pa, cudaStream_t st) {

@@ -30,6 +30,31 @@ __device__ __forceinline__ uint64_t evict_first_policy() {
     return pol;
 }
 
+__device__ __forceinline__ uint64_t evict_last_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+
+// Stage-gather loads with L2 priorities (SpmvArgs::l2hint): the map is read once per partition
+// (evict-first, like the slot stream), the input vector is re-read by every partition whose rays
+// cross its pixels (evict-last, so neither the stream nor the maps push it out of L2).
+__device__ __forceinline__ int32_t ld_map_hint(const int32_t* p, uint64_t pol) {
+    int32_t r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ float ld_x_hint(const float* p, uint64_t pol) {
+    float r;
+    asm volatile("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(r) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ double ld_x_hint(const double* p, uint64_t pol) {
+    double r;
+    asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(r) : "l"(p), "l"(pol));
+    return r;
+}
+
 __device__ __forceinline__ uint4 ld_stream_u4(const void* p, uint64_t pol) {
     uint4 r;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
@@ -87,6 +112,7 @@ struct SpmvArgs {
     double* dot_part;
     double* dot_out;
     unsigned int* ticket;
+    int32_t l2hint;        // stage gather: map evict-first, input evict-last (MEMXCT_L2HINT)
 };
 
 // Partition processed by this CTA: a.order maps launch positions to partitions when a launch
@@ -163,8 +189,23 @@ constexpr int kMaxThreads = 1024;
 // time here, profiles/r01b: while an SM gathers it streams nothing from HBM).
 template <int U, class T>
 __device__ __forceinline__ void stage_gather(T* __restrict__ buf, const T* __restrict__ x,
-                                             const int32_t* __restrict__ mp, int cnt) {
+                                             const int32_t* __restrict__ mp, int cnt, int hint) {
     const int bd = blockDim.x;
+    if (hint) {
+        const uint64_t pm = evict_first_policy(), px = evict_last_policy();
+        for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+            int32_t j[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) j[u] = (i0 + u * bd < cnt) ? ld_map_hint(mp + i0 + u * bd, pm) : -1;
+            T v[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) v[u] = (j[u] >= 0) ? ld_x_hint(x + j[u], px) : T(0);
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (i0 + u * bd < cnt) buf[i0 + u * bd] = v[u];
+        }
+        return;
+    }
     for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
         int32_t j[U];
 #pragma unroll
@@ -183,11 +224,15 @@ __device__ __forceinline__ void stage_gather(T* __restrict__ buf, const T* __res
 // stages, and the gather (a dependent map -> input chain) is the part of a stage during which the
 // SM streams nothing.  The range is widened to 16 B alignment (inside the map allocation's
 // 256 B granularity); a prefetch never faults.
-__device__ __forceinline__ void prefetch_map_l2(const int32_t* mp, int cnt) {
+__device__ __forceinline__ void prefetch_map_l2(const int32_t* mp, int cnt, int hint = 0) {
     if (cnt <= 0) return;
     const uintptr_t a0 = reinterpret_cast<uintptr_t>(mp) & ~(uintptr_t)15;
     const uintptr_t a1 = (reinterpret_cast<uintptr_t>(mp + cnt) + 15) & ~(uintptr_t)15;
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"((unsigned)(a1 - a0)) : "memory");
+    if (hint)
+        asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;"
+                     ::"l"(a0), "r"((unsigned)(a1 - a0)), "l"(evict_first_policy()) : "memory");
+    else
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"((unsigned)(a1 - a0)) : "memory");
 }
 
 // One warp's slots of stage g (its 32-row slice block): acc += buf[ind] * val, streamed with
@@ -301,8 +346,8 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();  // previous stage fully consumed
-        if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B));
-        stage_gather<16>(sbuf, x, mp, cnt);
+        if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
+        stage_gather<16>(sbuf, x, mp, cnt, a.l2hint);
         __syncthreads();
         stream_stage(acc, sbuf, a, g, warp, lane, lt, pol);
     }
@@ -367,7 +412,7 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     const uint64_t pol = evict_first_policy();
     auto gather = [&](int64_t s) {  // this thread's share of stage s into buffer s % 3
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
-        stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt);
+        stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt, a.l2hint);
         __syncwarp();
         if (lane == 0) mbar_arrive(&full[s % 3]);
     };
@@ -410,8 +455,8 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();
-        if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B));
-        stage_gather<4>(dbuf, x, mp, cnt);
+        if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
+        stage_gather<4>(dbuf, x, mp, cnt, a.l2hint);
         __syncthreads();
         const int64_t blk = g * a.SPP + warp;
         const int64_t base = a.slot_off[blk];
@@ -488,6 +533,11 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.dot_part = dot_part;
     a.dot_out = dot_out;
     a.ticket = ticket;
+    static const int hint = [] {
+        const char* e = std::getenv("MEMXCT_L2HINT");
+        return e ? atoi(e) : 0;
+    }();
+    a.l2hint = hint;
     return a;
 }
 
