@@ -51,9 +51,16 @@ def up_to_date() -> bool:
     return os.path.exists(OUT) and os.path.getmtime(OUT) >= _deps_mtime()
 
 
+# experiment builds only (scripts/build_variant.sh): extra nvcc flags and another output name
+VARIANT_FLAGS = os.environ.get("MEMXCT_VARIANT_FLAGS", "").split()
+if os.environ.get("MEMXCT_VARIANT"):
+    OUT = os.path.join(PKG, f"libmemxct_{os.environ['MEMXCT_VARIANT']}.so")
+    BUILD = os.path.join(PKG, "build", os.environ["MEMXCT_VARIANT"])
+
+
 def _compile(src: str) -> str:
     obj = os.path.join(BUILD, src.replace(".cu", ".o"))
-    cmd = [NVCC, "-c", "-O3", "-lineinfo", "-std=c++17", *ARCH, "-Xcompiler", "-fPIC",
+    cmd = [NVCC, "-c", "-O3", "-lineinfo", "-std=c++17", *ARCH, "-Xcompiler", "-fPIC", *VARIANT_FLAGS,
            "-Xptxas", "-v", "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(), *EXTRA.get(src, []),
            os.path.join(CSRC, src), "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)

@@ -123,11 +123,14 @@ __device__ __forceinline__ float upd(float a, double s, float b) { return (float
 __device__ __forceinline__ double upd(double a, double s, double b) { return __fma_rn(s, a, b); }
 
 // alpha = gam[k-1] / del[k]; x = fma(alpha, p, x); r = fma(-alpha, q, r); res2[k] = <r, r>
-template <class T, bool kUpdateR>
+// kPack (P > 1, sparse collective exchange): also the R^T pack of the next back projection --
+// the new r[i] goes to every pack position of owned ray i (pk.red_pos[pk.red_ptr[i] ..]), its own
+// slice in place in the footprint buffer.  Same grid and element map, so the dot is unchanged.
+template <class T, bool kUpdateR, bool kPack = false>
 __global__ void __launch_bounds__(kVT)
 cg_update_xr_kernel(T* __restrict__ x, const T* __restrict__ p, int64_t nx, T* __restrict__ r,
                     const T* __restrict__ q, int64_t nr, Scal sc, int32_t k, double* part,
-                    unsigned int* ticket) {
+                    unsigned int* ticket, PackTargets pk = PackTargets{}) {
     const int s = blockIdx.y;
     const int64_t o = (int64_t)s * sc.n1;
     x += s * nx; p += s * nx; r += s * nr; q += s * nr;
@@ -140,7 +143,17 @@ cg_update_xr_kernel(T* __restrict__ x, const T* __restrict__ p, int64_t nx, T* _
     MX_GRID_LOOP_U(i, nx, x[i] = upd(p[i], alpha, x[i]);)
     if (kUpdateR) {
         double acc = 0.0;
-        MX_GRID_LOOP_U(i, nr, const T v = upd(q[i], -alpha, r[i]); r[i] = v; acc += (double)v * (double)v;)
+        if constexpr (kPack) {
+            T* rb = static_cast<T*>(pk.rb);
+            T* self = static_cast<T*>(pk.self);
+            MX_GRID_LOOP_U(i, nr, const T v = upd(q[i], -alpha, r[i]); r[i] = v; acc += (double)v * (double)v;
+                           for (int64_t e = pk.red_ptr[i]; e < pk.red_ptr[i + 1]; ++e) {
+                               const int64_t j = pk.red_pos[e];
+                               if (j >= pk.lo && j < pk.hi) self[j - pk.lo] = v; else rb[j] = v;
+                           })
+        } else {
+            MX_GRID_LOOP_U(i, nr, const T v = upd(q[i], -alpha, r[i]); r[i] = v; acc += (double)v * (double)v;)
+        }
         vec_dot_finish(acc, part, sc.res2 + o + k, ticket);
     }
 }
@@ -206,7 +219,7 @@ void allreduce_slices(Plan& P, double* v, int K, int64_t stride, cudaStream_t st
 // and summed over the ranks.  Batched: separate dot kernels.
 template <class T>
 void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, int64_t dot_stride,
-            cudaStream_t st) {
+            cudaStream_t st, bool prepacked = false) {
     // P > 1: the rank's local dot is fused into the reduction R (forward) or into A_p^T's
     // epilogue (back) for every exchange, then summed over the ranks (allreduce_slices)
     const bool fused = dot_out && K == 1 && (P.dist || P.opt.canonical != 0 || P.fused_dot);
@@ -219,7 +232,7 @@ void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, 
             spmv_f64(L, in, out, part, fused ? dot_out : nullptr, P.tickets.p(), P.opt.canonical != 0, st);
     } else if (K == 1) {
         if (forward) apply_forward(P, in, out, st, fused ? dot_out : nullptr);
-        else apply_back(P, in, out, st, fused ? dot_out : nullptr);
+        else apply_back(P, in, out, st, fused ? dot_out : nullptr, prepacked);
     } else {
         if constexpr (sizeof(T) == 4) {
             if (forward) apply_forward_batch(P, K, in, out, st);
@@ -249,6 +262,8 @@ void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, int K, cudaStream_t st
     double* vpart = P.part_vec.p();
     unsigned int* tick = P.tickets.p() + 32;
     const unsigned gb = vec_blocks(std::max(nx, nr));
+    // sparse collective exchange, one slice: the back projection's R^T pack rides on the r update
+    const bool packed = K == 1 && P.opt.cg_variant == 0 && cg_fused_pack(P);
     cg_init_kernel<T><<<dim3(gb, K), kVT, 0, st>>>(y, r, nr, x, nx, sc, vpart, tick);
     MX_LAUNCHED();
     op_dir<T>(P, false, K, r, s, sc.gam, sc.n1, st);                    // s = A^T r, gamma_0
@@ -263,11 +278,15 @@ void cg_enqueue(Plan& P, const T* y, T* x, int32_t iters, int K, cudaStream_t st
             op_dir<T>(P, true, K, x, ax, nullptr, 0, st);                // ax = A x
             cg_explicit_r_kernel<T><<<dim3(vec_blocks(nr), K), kVT, 0, st>>>(y, ax, r, nr, sc, k, vpart, tick);
             MX_LAUNCHED();
+        } else if (packed) {  // + the R^T pack of the back projection below
+            cg_update_xr_kernel<T, true, true><<<dim3(gb, K), kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k, vpart, tick,
+                                                                            pack_targets(P));
+            MX_LAUNCHED();
         } else {
             cg_update_xr_kernel<T, true><<<dim3(gb, K), kVT, 0, st>>>(x, p, nx, r, q, nr, sc, k, vpart, tick);
             MX_LAUNCHED();
         }
-        op_dir<T>(P, false, K, r, s, sc.gam + k, sc.n1, st);            // s = A^T r, gamma_k
+        op_dir<T>(P, false, K, r, s, sc.gam + k, sc.n1, st, packed);    // s = A^T r, gamma_k
         cg_update_p_kernel<T><<<dim3(vec_blocks(nx), K), kVT, 0, st>>>(p, s, nx, sc, k);
         MX_LAUNCHED();
     }

@@ -448,7 +448,7 @@ static void exchange_fwd(Plan& P, const T* yfp, T* rb, T* yown, cudaStream_t st,
 // all-to-allv straight into the footprint slices.  Dense: allgather of the owned values into the
 // [P][maxown] sinogram, gather of the footprint rays.
 template <class T>
-static void exchange_back(Plan& P, const T* yown, T* rb, T* yfp, cudaStream_t st) {
+static void exchange_back(Plan& P, const T* yown, T* rb, T* yfp, cudaStream_t st, bool prepacked = false) {
     Exchange& X = P.ex;
     const DType t = sizeof(T) == 4 ? DType::F32 : DType::F64;
     if (X.dense) {
@@ -462,7 +462,7 @@ static void exchange_back(Plan& P, const T* yown, T* rb, T* yfp, cudaStream_t st
         }
         return;
     }
-    if (X.nrecv > 0) {  // R^T (own slice straight into the footprint buffer)
+    if (X.nrecv > 0 && !prepacked) {  // R^T (own slice straight into the footprint buffer)
         pack_self_kernel<T><<<nblocks(X.nrecv), kT, 0, st>>>(yown, X.recv_idx.p(), X.nrecv, rb, yfp + X.sdispl[P.rank],
                                                              X.rdispl[P.rank], X.rdispl[P.rank + 1]);
         MX_LAUNCHED();
@@ -504,14 +504,14 @@ static void forward_t(Plan& P, const T* x, T* y, double* dot_out, cudaStream_t s
 }
 
 template <class T>
-static void back_t(Plan& P, const T* y, T* x, double* dot_out, cudaStream_t st) {
+static void back_t(Plan& P, const T* y, T* x, double* dot_out, cudaStream_t st, bool prepacked = false) {
     if (!P.dist) {
         spmv_any(P, P.back, y, x, st);
         return;
     }
     Exchange& X = P.ex;
     T* yfp = X.y_fp.as<T>();
-    exchange_back<T>(P, y, X.recv_buf.as<T>(), yfp, st);                    // C^T R^T
+    exchange_back<T>(P, y, X.recv_buf.as<T>(), yfp, st, prepacked);         // C^T R^T
     double* part = dot_out ? X.dot_part.p() : nullptr;                      // A_p^T
     if constexpr (sizeof(T) == 4) spmv_f32(P.back, yfp, x, part, dot_out, X.tickets.p() + 4, st);
     else spmv_f64(P.back, yfp, x, part, dot_out, X.tickets.p() + 4, false, st);
@@ -696,10 +696,30 @@ void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st, double* dot
     else forward_t<double>(P, (const double*)x, (double*)y, dot_out, st);
 }
 
-void apply_back(Plan& P, const void* y, void* x, cudaStream_t st, double* dot_out) {
+void apply_back(Plan& P, const void* y, void* x, cudaStream_t st, double* dot_out, bool prepacked) {
     if (P.ex.peer) peer_back(P, (const float*)y, (float*)x, dot_out, st);
-    else if (P.esize == 4) back_t<float>(P, (const float*)y, (float*)x, dot_out, st);
-    else back_t<double>(P, (const double*)y, (double*)x, dot_out, st);
+    else if (P.esize == 4) back_t<float>(P, (const float*)y, (float*)x, dot_out, st, prepacked);
+    else back_t<double>(P, (const double*)y, (double*)x, dot_out, st, prepacked);
+}
+
+bool cg_fused_pack(const Plan& P) {
+    static const bool on = [] {
+        const char* e = std::getenv("MEMXCT_CG_FUSED_PACK");
+        return !(e && e[0] == '0');
+    }();
+    return on && P.dist && !P.shard && !P.ex.peer && !P.ex.dense && P.ex.nrecv > 0;
+}
+
+PackTargets pack_targets(Plan& P) {
+    Exchange& X = P.ex;
+    PackTargets t;
+    t.red_ptr = X.red_ptr.p();
+    t.red_pos = X.red_pos.p();
+    t.rb = X.recv_buf.get();
+    t.self = static_cast<char*>(X.y_fp.get()) + P.esize * X.sdispl[P.rank];
+    t.lo = X.rdispl[P.rank];
+    t.hi = X.rdispl[P.rank + 1];
+    return t;
 }
 
 }  // namespace mx

@@ -354,7 +354,21 @@ void shard_receive_maps(Plan& P, const Geometry& G, cudaStream_t st);
 void build_exchange(Plan& P, cudaStream_t st);
 // dot_out (nullable, P > 1): the CG dot of this rank's output part, fused into the last kernel
 void apply_forward(Plan& P, const void* x, void* y, cudaStream_t st, double* dot_out = nullptr);
-void apply_back(Plan& P, const void* y, void* x, cudaStream_t st, double* dot_out = nullptr);
+void apply_back(Plan& P, const void* y, void* x, cudaStream_t st, double* dot_out = nullptr,
+                bool prepacked = false);
+// CG at P > 1 with the sparse collective exchange: the R^T pack of the back projection is fused
+// into the x / r update (cg.cu), which scatters every updated owned ray r[i] to its pack positions
+// (the reduction map R lists them: {j : recv_idx[j] = i}); apply_back(..., prepacked) then
+// starts at the all-to-allv.  Destinations: recv_buf, and this rank's own slice in place.
+struct PackTargets {
+    const int64_t* red_ptr = nullptr;
+    const int32_t* red_pos = nullptr;
+    void* rb = nullptr;        // receive / pack buffer
+    void* self = nullptr;      // y_fp + sdispl[me]
+    int64_t lo = 0, hi = 0;    // pack positions of the own slice: [rdispl[me], rdispl[me + 1])
+};
+bool cg_fused_pack(const Plan& P);  // the sparse collective path (not dense, not peer)
+PackTargets pack_targets(Plan& P);
 void time_exchange(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 void time_spmv(Plan& P, int reps, double* us_fwd, double* us_back, cudaStream_t st);
 double read_ceiling_gbs(int64_t bytes, int reps, cudaStream_t st);  // memxct_read_ceiling

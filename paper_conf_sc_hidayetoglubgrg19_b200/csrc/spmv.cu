@@ -182,6 +182,9 @@ __device__ void finish_dot_canonical(const SpmvArgs& a, const double* rows_val, 
 }
 
 constexpr int kMaxThreads = 1024;
+#ifndef MX_F64_GATHER_U
+#define MX_F64_GATHER_U 4   // fp64 stage gather: map / input loads in flight per thread
+#endif
 
 // Stage gather buf[i] = x[map[i]]: U entries per thread in flight -- all U map loads
 // first, then the U dependent input loads (mostly L2 hits) -- so a stage costs ~cnt / (U * bd)
@@ -456,7 +459,7 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();
         if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
-        stage_gather<4>(dbuf, x, mp, cnt, a.l2hint);
+        stage_gather<MX_F64_GATHER_U>(dbuf, x, mp, cnt, a.l2hint);
         __syncthreads();
         const int64_t blk = g * a.SPP + warp;
         const int64_t base = a.slot_off[blk];
@@ -560,9 +563,21 @@ __device__ __forceinline__ void load_k(const float* __restrict__ buf, uint32_t i
         const float4 v = reinterpret_cast<const float4*>(buf)[i];
         b[0] = v.x; b[1] = v.y; b[2] = v.z; b[3] = v.w;
     } else {
-        const float4 u = reinterpret_cast<const float4*>(buf)[2 * i];
-        const float4 v = reinterpret_cast<const float4*>(buf)[2 * i + 1];
-        b[0] = u.x; b[1] = u.y; b[2] = u.z; b[3] = u.w; b[4] = v.x; b[5] = v.y; b[6] = v.z; b[7] = v.w;
+        // 32 B entry = two 16 B halves in bank groups 2i and 2i + 1 (mod 8).  Loading the low half
+        // first would confine a warp's first LDS.128 to the 4 even groups (and the second to the 4
+        // odd ones): 2-way conflicts even when the lanes' local indices hit all 8 classes i mod 8.
+        // The half loaded first is h = bit 2 of i, so the first load's group 2 (i mod 4) + h and
+        // the second's 2 (i mod 4) + 1 - h are both bijections of i mod 8 -- the bank-aware run
+        // order (layout.cu, 8 classes) then keeps both loads conflict-free.  Per-slice sums are
+        // unchanged (each slice's fma chain is independent of the load order).
+#ifndef MX_K8_SWIZZLE
+#define MX_K8_SWIZZLE 1
+#endif
+        const uint32_t h = MX_K8_SWIZZLE ? ((i >> 2) & 1u) : 0u;
+        const float4 u = reinterpret_cast<const float4*>(buf)[2 * i + h];
+        const float4 v = reinterpret_cast<const float4*>(buf)[2 * i + 1 - h];
+        const float4 lo = h ? v : u, hi = h ? u : v;
+        b[0] = lo.x; b[1] = lo.y; b[2] = lo.z; b[3] = lo.w; b[4] = hi.x; b[5] = hi.y; b[6] = hi.z; b[7] = hi.w;
     }
 }
 
