@@ -56,7 +56,7 @@ def parse():
     ap.add_argument("--cpu-full", action="store_true",
                     help="oracle baseline on the WHOLE config (cfg3: ~30 GB host RAM, minutes)")
     ap.add_argument("--spmv-reps", type=int, default=20)
-    ap.add_argument("--slices", type=int, default=4, help="multi-slice batch measured beside the headline (1 = off)")
+    ap.add_argument("--slices", type=int, default=8, help="multi-slice batch measured beside the headline (1 = off)")
     ap.add_argument("--variant", default=None, choices=["peer", "dense"], help=argparse.SUPPRESS)
     ap.add_argument("--distributed", action="store_true",
                     help="run the decomposed path (NCCL communicator, exchange, allreduce) even at N = 1")

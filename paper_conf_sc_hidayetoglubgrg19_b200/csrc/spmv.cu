@@ -113,6 +113,7 @@ struct SpmvArgs {
     double* dot_out;
     unsigned int* ticket;
     int32_t l2hint;        // stage gather: map evict-first, input evict-last (MEMXCT_L2HINT)
+    int32_t jitter;        // drifting-stage kernel: test-only per-warp delays (MEMXCT_DRIFT_JITTER)
 };
 
 // Partition processed by this CTA: a.order maps launch positions to partitions when a launch
@@ -424,6 +425,9 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     float acc = 0.f;
     for (int64_t s = 0; s < ns; ++s) {
         mbar_wait(&full[s % 3], (unsigned)((s / 3) & 1));
+        // test-only: pseudo-random per-warp delays stretch the drift between warps, so the
+        // buffer-reuse protocol is exercised at its limits (tests/test_gpu_drift.py)
+        if (a.jitter && ((warp * 7 + (int)s) % 5 == 0)) __nanosleep(2000 + 131 * warp);
         stream_stage(acc, sbuf + (s % 3) * a.B, a, g0 + s, warp, lane, lt, pol);
         __syncwarp();
         if (lane == 0) mbar_arrive(&done[s % 3]);
@@ -515,6 +519,14 @@ template <class K> void set_smem(K kern) {
                                  optin - (int)fa.sharedSizeBytes));
 }
 
+int l2hint_env() {
+    static const int v = [] {
+        const char* e = std::getenv("MEMXCT_L2HINT");
+        return e ? atoi(e) : -1;
+    }();
+    return v;
+}
+
 SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned int* ticket) {
     SpmvArgs a;
     a.stage_base = L.stage_base.p();
@@ -536,11 +548,13 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.dot_part = dot_part;
     a.dot_out = dot_out;
     a.ticket = ticket;
-    static const int hint = [] {
-        const char* e = std::getenv("MEMXCT_L2HINT");
-        return e ? atoi(e) : 0;
-    }();
-    a.l2hint = hint;
+    // L2 priorities of the stage gather (map evict-first, input evict-last): on by default for
+    // the plain / fp64 / SpMM kernels (cfg3 forward 1.694 -> 1.660 ms, back 1.711 -> 1.695 ms,
+    // ABAB r02e), off for the drifting-stage kernel (config-5 forward 7.92 -> 8.01 ms);
+    // MEMXCT_L2HINT=0/1 forces it for every kernel
+    a.l2hint = l2hint_env() < 0 ? 1 : l2hint_env();
+    const char* jit = std::getenv("MEMXCT_DRIFT_JITTER");  // read per launch: tests toggle it
+    a.jitter = jit ? atoi(jit) : 0;
     return a;
 }
 
@@ -769,6 +783,7 @@ void spmv_f32(const Layout& L, const float* x, float* y, double* dot_part, doubl
     a.cta_base = c0;
     const bool nat = L.out_idx.p() != nullptr, dot = dot_out != nullptr;
     if (L.drift) {
+        if (l2hint_env() < 0) a.l2hint = 0;
         const size_t smem = 3 * sizeof(float) * (size_t)L.B;
         auto kern = nat ? (dot ? spmv_f32_drift_kernel<true, 1> : spmv_f32_drift_kernel<true, 0>)
                         : (dot ? spmv_f32_drift_kernel<false, 1> : spmv_f32_drift_kernel<false, 0>);

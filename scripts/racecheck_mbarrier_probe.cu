@@ -5,7 +5,8 @@
 //   mode 0  the drift protocol (full / done rings, warp arrivals after __syncwarp)
 //   mode 1  the same with a __syncthreads() before every gather (racecheck's native barrier)
 //   mode 2  a real race: the wait on `done` before the gather is removed
-// and checks the result on the host.  nvcc -gencode arch=compute_100a,code=sm_100a -o probe probe.cu
+// and checks the result on the host; argument 2 = 1 adds per-warp delays so a broken handoff
+// shows up as wrong sums (r02e: racecheck reports hazards for all three modes alike).  nvcc -gencode arch=compute_100a,code=sm_100a -o probe probe.cu
 #include <cstdio>
 #include <cstdint>
 
@@ -26,7 +27,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
 }
 
 constexpr int B = 256;
-__global__ void probe(const float* __restrict__ x, int ns, int mode, float* out) {
+__global__ void probe(const float* __restrict__ x, int ns, int mode, float* out, int jitter) {
     __shared__ float buf[3][B];
     __shared__ __align__(8) uint64_t full[3], done[3];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
@@ -43,6 +44,7 @@ __global__ void probe(const float* __restrict__ x, int ns, int mode, float* out)
     float acc = 0.f;
     for (int s = 0; s < ns; ++s) {
         mbar_wait(&full[s % 3], (s / 3) & 1);
+        if (jitter && ((warp * 7 + s) % 5 == 0)) __nanosleep(2000 + 131 * warp);
         for (int i = lane; i < B; i += 32) acc += buf[s % 3][(i * 7 + warp) % B];   // read other warps' slots
         __syncwarp();
         if (lane == 0) mbar_arrive(&done[s % 3]);
@@ -56,12 +58,12 @@ __global__ void probe(const float* __restrict__ x, int ns, int mode, float* out)
 }
 
 int main(int argc, char** argv) {
-    const int mode = argc > 1 ? atoi(argv[1]) : 0, ns = 12, nt = 256;
+    const int mode = argc > 1 ? atoi(argv[1]) : 0, jitter = argc > 2 ? atoi(argv[2]) : 0, ns = 12, nt = 256;
     float *x, *out;
     cudaMallocManaged(&x, sizeof(float) * ns * B);
     cudaMallocManaged(&out, sizeof(float) * nt);
     for (int i = 0; i < ns * B; ++i) x[i] = (float)(i % 97);
-    probe<<<1, nt>>>(x, ns, mode, out);
+    probe<<<1, nt>>>(x, ns, mode, out, jitter);
     cudaDeviceSynchronize();
     // expected: every thread sums 8 reads per stage of its warp's slots
     int bad = 0;
@@ -72,6 +74,6 @@ int main(int argc, char** argv) {
             for (int i = lane; i < B; i += 32) e += x[s * B + (i * 7 + warp) % B];
         bad += (out[t] != e);
     }
-    printf("mode %d: %s (%d threads wrong)\n", mode, bad ? "WRONG" : "correct", bad);
+    printf("mode %d jitter %d: %s (%d threads wrong)\n", mode, jitter, bad ? "WRONG" : "correct", bad);
     return 0;
 }

@@ -97,3 +97,24 @@ def test_ray_block_forward_uses_drift_by_default(orc, coo_cache):
     rows, cols, vals = coo_cache(n, m, c)
     y_ref = orc.spmv_coo(rows, cols, vals, x.cpu().numpy().astype(np.float64), m * c)
     assert rel_l2(y1.cpu().numpy(), y_ref) <= 1e-5
+
+
+@pytest.mark.parametrize("n,m,c,B", [(256, 360, 256, 256), (256, 360, 256, 1024), (64, 90, 64, 256)])
+def test_drift_under_jitter_bit_identical(monkeypatch, n, m, c, B):
+    """The buffer-reuse protocol at its limits: MEMXCT_DRIFT_JITTER=1 makes warps sleep
+    pseudo-randomly (1-6 us) before streaming some stages, so they drift as far apart as the
+    mbarrier rings allow while stage buffers are regathered.  compute-sanitizer racecheck does not
+    model mbarrier synchronisation (it flags the correct protocol and a deliberately broken one
+    alike, scripts/racecheck_mbarrier_probe.cu), so this is the protocol's stress test: many
+    stages per partition (small B), repeated launches, every output bit-identical to the plain
+    kernel's."""
+    plain, drift = _plans(monkeypatch, n, m, c, buffer_entries=B)
+    rng = np.random.default_rng(B)
+    x = torch.from_numpy(rng.random(n * n, dtype=np.float32)).cuda()
+    y = torch.from_numpy(rng.random(m * c, dtype=np.float32)).cuda()
+    yf0, xb0 = plain.forward(x), plain.back(y)
+    monkeypatch.setenv("MEMXCT_DRIFT_JITTER", "1")
+    for _ in range(3):
+        assert torch.equal(drift.forward(x), yf0)
+        assert torch.equal(drift.back(y), xb0)
+    monkeypatch.delenv("MEMXCT_DRIFT_JITTER")
