@@ -45,6 +45,13 @@ constexpr int kT = 256;
 
 unsigned nblocks(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, kT), 1 << 20)); }
 
+// grid of the reduction R and the packs R^T: 8 CTAs of kT threads per SM, kRedU elements per thread
+// per pass (one element per thread over ~6000 CTAs ran the config-3 reduction at ~1.3 TB/s)
+constexpr int kRedU = 4;
+unsigned red_blocks(int64_t n) {
+    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(n, (int64_t)kT * kRedU), 8 * num_sms()));
+}
+
 std::vector<int64_t> to_host_i64(const int64_t* d, int64_t n, cudaStream_t st) {
     std::vector<int64_t> h(n);
     MX_CUDA(cudaMemcpyAsync(h.data(), d, 8 * n, cudaMemcpyDeviceToHost, st));
@@ -71,21 +78,29 @@ reduce_dot_kernel(const T* __restrict__ recv, const int64_t* __restrict__ ptr, c
         __syncthreads();
     }
     double d = 0.0;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nown; i += (int64_t)gridDim.x * blockDim.x) {
-        T acc;
-        if (ptr) {
-            acc = T(0);
-            for (int64_t k = ptr[i]; k < ptr[i + 1]; ++k) {  // peer order
-                const int64_t q = pos[k];
-                // this rank's own partial is read in place from its footprint slice (`self`):
-                // no copy into the receive buffer
-                acc += (q >= self_lo && q < self_hi) ? self[q - self_lo] : recv[q];
+    // kRedU independent owned rays per thread per pass (a fixed element -> thread map, so the
+    // dot's summation order depends only on the grid)
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i0 < nown; i0 += kRedU * stride) {
+#pragma unroll
+        for (int u = 0; u < kRedU; ++u) {
+            const int64_t i = i0 + u * stride;
+            if (i >= nown) break;
+            T acc;
+            if (ptr) {
+                acc = T(0);
+                for (int64_t k = ptr[i]; k < ptr[i + 1]; ++k) {  // peer order
+                    const int64_t q = pos[k];
+                    // this rank's own partial is read in place from its footprint slice (`self`):
+                    // no copy into the receive buffer
+                    acc += (q >= self_lo && q < self_hi) ? self[q - self_lo] : recv[q];
+                }
+            } else {
+                acc = recv[i];
             }
-        } else {
-            acc = recv[i];
+            y[i] = acc;
+            d += (double)acc * (double)acc;
         }
-        y[i] = acc;
-        d += (double)acc * (double)acc;
     }
     if (!dot_out && !pa.fold) return;
     if (dot_out) {
@@ -138,10 +153,16 @@ __global__ void pack_kernel(const T* __restrict__ y, const int32_t* __restrict__
 template <class T>
 __global__ void pack_self_kernel(const T* __restrict__ y, const int32_t* __restrict__ idx, int64_t n,
                                  T* __restrict__ out, T* __restrict__ self, int64_t lo, int64_t hi) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const T v = y[idx[i]];
-        if (i >= lo && i < hi) self[i - lo] = v;
-        else out[i] = v;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i0 < n; i0 += kRedU * stride) {
+#pragma unroll
+        for (int u = 0; u < kRedU; ++u) {
+            const int64_t i = i0 + u * stride;
+            if (i >= n) break;
+            const T v = y[idx[i]];
+            if (i >= lo && i < hi) self[i - lo] = v;
+            else out[i] = v;
+        }
     }
 }
 
@@ -380,7 +401,7 @@ void build_exchange(Plan& P, cudaStream_t st) {
     X.recv_buf.alloc(P.esize * std::max<int64_t>(X.nrecv, 1));
     X.tickets.alloc(8);
     MX_CUDA(cudaMemsetAsync(X.tickets.p(), 0, 32, st));
-    X.dot_part.alloc(std::max<int64_t>({P.back.nparts, (int64_t)nblocks(nown), 4 * num_sms()}));
+    X.dot_part.alloc(std::max<int64_t>({P.back.nparts, (int64_t)red_blocks(nown), 8 * num_sms()}));
     if (P.opt.exchange == 0 && !P.shard) setup_forward_overlap(P, st);
     if (P.opt.exchange == 2) {  // dense collectives: footprint row i -> [owner][owned-local index]
         X.maxown = 0;
@@ -407,7 +428,7 @@ void launch_reduce_dot(Plan& P, const T* recv, bool csr, T* y, double* dot_out, 
     Exchange& X = P.ex;
     const int64_t nown = P.s1 - P.s0;
     const int64_t lo = self ? X.rdispl[P.rank] : 0, hi = self ? X.rdispl[P.rank + 1] : 0;
-    reduce_dot_kernel<T><<<nblocks(nown), kT, 0, st>>>(recv, csr ? X.red_ptr.p() : nullptr, X.red_pos.p(), nown, y,
+    reduce_dot_kernel<T><<<red_blocks(nown), kT, 0, st>>>(recv, csr ? X.red_ptr.p() : nullptr, X.red_pos.p(), nown, y,
                                                        X.dot_part.p(), dot_out, X.tickets.p() + 2, pa, self, lo, hi);
     MX_LAUNCHED();
 }
@@ -463,7 +484,7 @@ static void exchange_back(Plan& P, const T* yown, T* rb, T* yfp, cudaStream_t st
         return;
     }
     if (X.nrecv > 0 && !prepacked) {  // R^T (own slice straight into the footprint buffer)
-        pack_self_kernel<T><<<nblocks(X.nrecv), kT, 0, st>>>(yown, X.recv_idx.p(), X.nrecv, rb, yfp + X.sdispl[P.rank],
+        pack_self_kernel<T><<<red_blocks(X.nrecv), kT, 0, st>>>(yown, X.recv_idx.p(), X.nrecv, rb, yfp + X.sdispl[P.rank],
                                                              X.rdispl[P.rank], X.rdispl[P.rank + 1]);
         MX_LAUNCHED();
     }

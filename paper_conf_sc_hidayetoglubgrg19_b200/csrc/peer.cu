@@ -44,7 +44,10 @@ __global__ void signal_kernel(SignalArgs sa, int P, int slot, const unsigned lon
 
 // R^T + C^T: value j (recv order, peer g = the range containing j) goes to g's footprint buffer
 // (pa.fold: thread 0 of every CTA first waits for the peers' credits -- footprint buffers
-// consumed -- reading the epoch before this CTA's ticket, i.e. before the last CTA bumps it)
+// consumed -- reading the epoch before this CTA's ticket, i.e. before the last CTA bumps it).
+// Each CTA packs one contiguous range of the recv order, so only CTAs whose range reaches
+// another rank's slice pay a system-scope fence; the others' stores stay on this GPU (own
+// footprint slice) and a device-scope fence orders them before the ticket.
 __global__ void pack_remote_kernel(const float* __restrict__ y, const int32_t* __restrict__ idx, int64_t n,
                                    PeerArgs pa) {
     __shared__ bool am_last;
@@ -53,14 +56,19 @@ __global__ void pack_remote_kernel(const float* __restrict__ y, const int32_t* _
             wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
         __syncthreads();
     }
-    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t per = (n + gridDim.x - 1) / gridDim.x;
+    const int64_t chunk = (per + blockDim.x - 1) / blockDim.x * blockDim.x;
+    const int64_t j0 = (int64_t)blockIdx.x * chunk, j1 = min(n, j0 + chunk);
+    for (int64_t j = j0 + threadIdx.x; j < j1; j += blockDim.x) {
         int g = 0;
         while (g + 1 < pa.P && j >= pa.bound[g + 1]) ++g;
         pa.dst[g][pa.off[g] + j] = y[idx[j]];
     }
     __syncthreads();
     if (threadIdx.x == 0) {
-        __threadfence_system();
+        const bool remote = j0 < j1 && (j0 < pa.bound[pa.me] || j1 > pa.bound[pa.me + 1]);
+        if (remote) __threadfence_system();
+        else __threadfence();
         am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
     }
     __syncthreads();

@@ -290,14 +290,19 @@ __device__ void remote_epilogue(const PeerArgs& pa, int64_t o, bool valid, float
             wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
         __syncthreads();
     }
+    int h = pa.me;
     if (valid) {  // o = footprint position of the row
-        int h = 0;
+        h = 0;
         while (h + 1 < pa.P && o >= pa.bound[h + 1]) ++h;
         pa.dst[h][pa.off[h] + o] = acc;
     }
-    __syncthreads();
+    // only a CTA that stored into another rank's buffer needs the system-scope fence; stores to
+    // this rank's own receive buffer stay on this GPU (the last CTA fences at system scope before
+    // it publishes the epoch)
+    const int remote = __syncthreads_or(h != pa.me);
     if (threadIdx.x == 0) {
-        __threadfence_system();
+        if (remote) __threadfence_system();
+        else __threadfence();
         am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
     }
     __syncthreads();

@@ -20,6 +20,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", type=int, default=3)
     ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--rounds", type=int, default=5)
     a = ap.parse_args()
     import torch
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, get_unique_id, inputs
@@ -36,24 +37,33 @@ def main():
         torch.cuda.synchronize()
         return e0.elapsed_time(e1) / reps * 1e3  # us
 
+    plans = {}
     for kind in ("plain", "collective", "peer", "dense"):
         if kind == "plain":
-            plan = MemXCT(n, m, c, vector_order="plan").build()
+            plans[kind] = MemXCT(n, m, c, vector_order="plan").build()
         else:
-            plan = MemXCT(n, m, c, rank=0, nranks=1, unique_id=get_unique_id(), device=0,
-                          vector_order="plan", exchange=kind).build()
-        x = torch.rand(plan.local_size(0), device="cuda")
-        y = torch.rand(plan.local_size(1), device="cuda")
-        q, s = torch.empty_like(y), torch.empty_like(x)
-        fwd = timed(lambda: plan.forward(x, q), a.reps)
-        back = timed(lambda: plan.back(y, s), a.reps)
-        c10 = timed(lambda: plan.cg(y, 10, x=s), 3)
-        c40 = timed(lambda: plan.cg(y, 40, x=s), 3)
-        print(json.dumps({"config": a.config, "exchange": kind, "fwd_us": round(fwd, 1), "back_us": round(back, 1),
-                          "cg_iter_us": round((c40 - c10) / 30, 1)}), flush=True)
-        plan.close()
-        del plan
-        torch.cuda.empty_cache()
+            plans[kind] = MemXCT(n, m, c, rank=0, nranks=1, unique_id=get_unique_id(), device=0,
+                                 vector_order="plan", exchange=kind).build()
+    res = {k: {"fwd": [], "back": [], "cg": []} for k in plans}
+    # interleaved rounds (ABCD ABCD ...): clock drift of the power-capped box hits every kind alike
+    for _ in range(a.rounds):
+        for kind, plan in plans.items():
+            x = torch.rand(plan.local_size(0), device="cuda")
+            y = torch.rand(plan.local_size(1), device="cuda")
+            q, s = torch.empty_like(y), torch.empty_like(x)
+            res[kind]["fwd"].append(timed(lambda: plan.forward(x, q), a.reps))
+            res[kind]["back"].append(timed(lambda: plan.back(y, s), a.reps))
+            c10 = timed(lambda: plan.cg(y, 10, x=s), 3)
+            c40 = timed(lambda: plan.cg(y, 40, x=s), 3)
+            res[kind]["cg"].append((c40 - c10) / 30)
+    import numpy as np
+    base = float(np.median(res["plain"]["cg"]))
+    for kind in plans:
+        med = {k: float(np.median(v)) for k, v in res[kind].items()}
+        print(json.dumps({"config": a.config, "exchange": kind, "fwd_us": round(med["fwd"], 1),
+                          "back_us": round(med["back"], 1), "cg_iter_us": round(med["cg"], 1),
+                          "cg_iter_minus_plain_us": round(med["cg"] - base, 1), "rounds": a.rounds,
+                          "cg_iter_samples": [round(v, 1) for v in res[kind]["cg"]]}), flush=True)
 
 
 if __name__ == "__main__":
