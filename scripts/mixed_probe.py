@@ -19,12 +19,18 @@ def main():
     ap.add_argument("--canonical", type=int, default=1)
     ap.add_argument("--iters", type=int, default=30)
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--buffers", default="0", help="comma list of BUFFER_ENTRIES (fp32 units; 0 = auto)")
     a = ap.parse_args()
-    import numpy as np
+    from paper_conf_sc_hidayetoglubgrg19_b200 import inputs
+    n, m, c = inputs.CONFIGS[a.config]
+    for b in map(int, a.buffers.split(",")):
+        run(a, n, m, c, b or None)
+
+
+def run(a, n, m, c, buf):
     import torch
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, inputs
-    n, m, c = inputs.CONFIGS[a.config]
-    plan = MemXCT(n, m, c, precision="mixed", canonical=bool(a.canonical)).build()
+    plan = MemXCT(n, m, c, precision="mixed", canonical=bool(a.canonical), buffer_entries=buf).build()
     y = plan.forward(torch.from_numpy(inputs.shepp_logan(n)).cuda())
     x = torch.empty(n * n, dtype=torch.float64, device="cuda")
     plan.cg(y, a.iters, x=x)
@@ -40,6 +46,7 @@ def main():
                       "fwd_ms": sp["fwd_us"] / 1e3, "back_ms": sp["back_us"] / 1e3,
                       "buffer_entries": [plan.layout_info(0)["buffer_entries"], plan.layout_info(1)["buffer_entries"]]}),
           flush=True)
+    plan.close()
 
 
 if __name__ == "__main__":
