@@ -22,7 +22,7 @@ OUT = os.path.join(PKG, "libmemxct.so")
 BUILD = os.path.join(PKG, "build")
 
 SOURCES = ["api.cu", "hilbert.cu", "trace.cu", "layout.cu", "spmv.cu", "cg.cu", "comm.cu", "exchange.cu",
-           "sirt.cu", "peer.cu", "proccomm.cu"]
+           "sirt.cu", "peer.cu", "proccomm.cu", "rle.cu"]
 EXTRA = {"trace.cu": ["--fmad=false"]}
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

@@ -1172,6 +1172,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
     clk.mark(kPhLayoutFwd);
     P.build_s[kPhLayoutFwd] -= gen_s;  // the generator's share is in trace / sort
     P.fwd.drift = fwd_drift && 12 * (int64_t)B <= 224 * 1024;
+    if (rle_requested()) encode_map_runs(P.fwd, st);
     kfwd.reset();
     kinv.reset();
     part_class.reset();
@@ -1235,6 +1236,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
     };
     build_direction(P.back, npix, nrows, back_parts, Rb, Bb, gen_back, natural ? P.sino_nat_of_h.p() : nullptr,
                     natural ? P.tomo_nat_of_h.p() : nullptr, chunk_budget(nnz), bank, st);
+    if (rle_requested()) encode_map_runs(P.back, st);
     clk.mark(kPhLayoutBack);
     P.build_s[kPhLayoutBack] -= gen_s;
 

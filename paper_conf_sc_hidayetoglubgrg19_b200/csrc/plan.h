@@ -52,10 +52,21 @@ struct Layout {
     DevArr<int32_t> part_order;  // nparts, optional: partition run by CTA b (launch order)
     int64_t n_first = -1;        // P > 1 forward: the first n_first CTAs hold every partition with
                                  // rows owned by other ranks (exchange overlap), else -1
+    // Run-length stage maps (rle.cu, MEMXCT_RLE): every 32-slot block of a stage's map as one
+    // 16 B record of up to 4 runs of consecutive input indices -- start | (first slot << 27) per
+    // run -- instead of 32 int32 entries; blocks with more runs hold (1 << 27) | overflow block
+    // and keep their 32 entries in `ovf`.  The stage gather reads a record (broadcast) per 32
+    // slots: 0.5 B per map entry plus overflow instead of 4 B.
+    bool rle = false;
+    DevArr<int64_t> blk_base;    // nstages + 1: first 32-slot block of every stage
+    DevArr<int4> blk_rec;        // one record per block
+    DevArr<int32_t> ovf;         // 32 entries per overflow block
+    int64_t n_ovf = 0;
     int64_t device_bytes() const {
         return (int64_t)(prow0.buf.bytes() + stage_base.buf.bytes() + map_off.buf.bytes() + map.buf.bytes() +
                          slot_off.buf.bytes() + ind.buf.bytes() + val.buf.bytes() +
-                         lane_chunks.buf.bytes() + out_idx.buf.bytes() + part_order.buf.bytes());
+                         lane_chunks.buf.bytes() + out_idx.buf.bytes() + part_order.buf.bytes() +
+                         blk_base.buf.bytes() + blk_rec.buf.bytes() + ovf.buf.bytes());
     }
 };
 
@@ -337,6 +348,11 @@ void trace_emit(const Plan& P, const Geometry& G, const int32_t* hray, int64_t r
                 cudaStream_t st);
 void trace_hist(const Plan& P, const Geometry& G, const int32_t* hray, int64_t r0, int64_t nrows, int64_t lo,
                 int64_t hi, bool filter, int32_t* hist, cudaStream_t st);
+
+// rle.cu: block-record encoding of a built layout's stage maps (Layout::rle); returns false (and
+// leaves the layout alone) when the encoding does not apply (input indices >= 2^27)
+bool encode_map_runs(Layout& L, cudaStream_t st);
+bool rle_requested();
 
 // layout.cu: chunked device build of both directions' staged jagged-SELL layouts
 void build_matrices(Plan& P, cudaStream_t st);

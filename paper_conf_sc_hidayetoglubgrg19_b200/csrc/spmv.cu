@@ -114,6 +114,11 @@ struct SpmvArgs {
     unsigned int* ticket;
     int32_t l2hint;        // stage gather: map evict-first, input evict-last (MEMXCT_L2HINT)
     int32_t jitter;        // drifting-stage kernel: test-only per-warp delays (MEMXCT_DRIFT_JITTER)
+    // run-length stage maps (Layout::rle, rle.cu): records per 32-slot block instead of map
+    int32_t rle;
+    const int64_t* blk_base;
+    const int4* blk_rec;
+    const int32_t* ovf;
 };
 
 // Partition processed by this CTA: a.order maps launch positions to partitions when a launch
@@ -217,6 +222,57 @@ __device__ __forceinline__ void stage_gather(T* __restrict__ buf, const T* __res
         T v[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) v[u] = (j[u] >= 0) ? __ldg(x + j[u]) : T(0);
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if (i0 + u * bd < cnt) buf[i0 + u * bd] = v[u];
+    }
+}
+
+// The same gather from run-length maps (Layout::rle): slot i of the stage belongs to 32-slot
+// block i / 32 (one warp instruction's slots: lane = i mod 32); the block's 16 B record (one
+// broadcast load per warp) gives the runs, so the input index is start + (lane - first slot of
+// the run) -- two dependent loads per slot as with the plain map (record, input), 0.5 B of map
+// per slot instead of 4.  Blocks of more than 4 runs read their 32 entries from `ovf`.
+__device__ __forceinline__ int4 ld_rec(const int4* p, uint64_t pol) {
+    int4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ int32_t decode_rec(const int4& r, int lane, const int32_t* __restrict__ ovf) {
+    constexpr int32_t M = (1 << 27) - 1;
+    const unsigned t0 = (unsigned)r.x >> 27;
+    if (t0 == 1u) return __ldg(ovf + (int64_t)(r.x & M) * 32 + lane);
+    int32_t st = r.x & M;
+    int d = 0;
+    const int d1 = (int)((unsigned)r.y >> 27), d2 = (int)((unsigned)r.z >> 27), d3 = (int)((unsigned)r.w >> 27);
+    if (d1 && lane >= d1) { st = r.y & M; d = d1; }
+    if (d2 && lane >= d2) { st = r.z & M; d = d2; }
+    if (d3 && lane >= d3) { st = r.w & M; d = d3; }
+    return st + (lane - d);
+}
+template <int U, class T, class A>
+__device__ __forceinline__ void stage_gather_rle(T* __restrict__ buf, const T* __restrict__ x, const A& a,
+                                                 int64_t g, int cnt) {
+    const int bd = blockDim.x, lane = threadIdx.x & 31;
+    const int4* __restrict__ rb = a.blk_rec + a.blk_base[g];
+    const uint64_t pm = evict_first_policy();
+    for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+        int32_t j[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int i = i0 + u * bd;
+            j[u] = i < cnt ? decode_rec(ld_rec(rb + (i >> 5), pm), lane, a.ovf) : -1;
+        }
+        T v[U];
+        if (a.l2hint) {
+            const uint64_t px = evict_last_policy();
+#pragma unroll
+            for (int u = 0; u < U; ++u) v[u] = (j[u] >= 0) ? ld_x_hint(x + j[u], px) : T(0);
+        } else {
+#pragma unroll
+            for (int u = 0; u < U; ++u) v[u] = (j[u] >= 0) ? __ldg(x + j[u]) : T(0);
+        }
 #pragma unroll
         for (int u = 0; u < U; ++u)
             if (i0 + u * bd < cnt) buf[i0 + u * bd] = v[u];
@@ -355,8 +411,12 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();  // previous stage fully consumed
-        if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
-        stage_gather<16>(sbuf, x, mp, cnt, a.l2hint);
+        if (a.rle) {
+            stage_gather_rle<8>(sbuf, x, a, g, cnt);
+        } else {
+            if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
+            stage_gather<16>(sbuf, x, mp, cnt, a.l2hint);
+        }
         __syncthreads();
         stream_stage(acc, sbuf, a, g, warp, lane, lt, pol);
     }
@@ -421,7 +481,8 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     const uint64_t pol = evict_first_policy();
     auto gather = [&](int64_t s) {  // this thread's share of stage s into buffer s % 3
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
-        stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt, a.l2hint);
+        if (a.rle) stage_gather_rle<8>(sbuf + (s % 3) * a.B, x, a, g0 + s, cnt);
+        else stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt, a.l2hint);
         __syncwarp();
         if (lane == 0) mbar_arrive(&full[s % 3]);
     };
@@ -467,8 +528,12 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();
-        if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
-        stage_gather<MX_F64_GATHER_U>(dbuf, x, mp, cnt, a.l2hint);
+        if (a.rle) {
+            stage_gather_rle<4>(dbuf, x, a, g, cnt);
+        } else {
+            if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
+            stage_gather<MX_F64_GATHER_U>(dbuf, x, mp, cnt, a.l2hint);
+        }
         __syncthreads();
         const int64_t blk = g * a.SPP + warp;
         const int64_t base = a.slot_off[blk];
@@ -560,6 +625,10 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.l2hint = l2hint_env() < 0 ? 1 : l2hint_env();
     const char* jit = std::getenv("MEMXCT_DRIFT_JITTER");  // read per launch: tests toggle it
     a.jitter = jit ? atoi(jit) : 0;
+    a.rle = L.rle ? 1 : 0;
+    a.blk_base = L.blk_base.p();
+    a.blk_rec = L.blk_rec.p();
+    a.ovf = L.ovf.p();
     return a;
 }
 
