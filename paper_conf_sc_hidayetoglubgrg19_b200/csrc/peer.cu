@@ -56,13 +56,23 @@ __global__ void pack_remote_kernel(const float* __restrict__ y, const int32_t* _
             wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
         __syncthreads();
     }
+    // destination table in shared memory (no dynamic indexing of the kernel parameters)
+    __shared__ int64_t bound[kMaxPeers + 1], off[kMaxPeers];
+    __shared__ float* dst[kMaxPeers];
+    if (threadIdx.x <= (unsigned)pa.P) bound[threadIdx.x] = pa.bound[threadIdx.x];
+    if (threadIdx.x < (unsigned)pa.P) {
+        dst[threadIdx.x] = pa.dst[threadIdx.x];
+        off[threadIdx.x] = pa.off[threadIdx.x];
+    }
+    __syncthreads();
     const int64_t per = (n + gridDim.x - 1) / gridDim.x;
     const int64_t chunk = (per + blockDim.x - 1) / blockDim.x * blockDim.x;
     const int64_t j0 = (int64_t)blockIdx.x * chunk, j1 = min(n, j0 + chunk);
+    int g = 0;
+    while (g + 1 < pa.P && j0 + (int64_t)threadIdx.x >= bound[g + 1]) ++g;
     for (int64_t j = j0 + threadIdx.x; j < j1; j += blockDim.x) {
-        int g = 0;
-        while (g + 1 < pa.P && j >= pa.bound[g + 1]) ++g;
-        pa.dst[g][pa.off[g] + j] = y[idx[j]];
+        while (g + 1 < pa.P && j >= bound[g + 1]) ++g;   // ranges ascend with j
+        dst[g][off[g] + j] = y[idx[j]];
     }
     __syncthreads();
     if (threadIdx.x == 0) {

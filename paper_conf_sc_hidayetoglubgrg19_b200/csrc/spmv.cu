@@ -335,22 +335,32 @@ __device__ __forceinline__ void stream_stage(float& acc, const float* __restrict
 // straight into its owner's receive buffer (peer memory over NVLink), then the last CTA bumps
 // this rank's forward epoch and publishes it to every owner's arrival flag (release, system
 // scope).  Replaces the separate all-to-allv of C in A = R C A_p.
-// With pa.fold the owners' credits (receive buffers consumed) are awaited here, by thread 0 of
-// every CTA before the CTA's stores, instead of by a wait kernel ahead of the SpMV: the epoch is
-// read before this CTA's ticket, so before the last CTA bumps it.  One system-scope fence per CTA
-// (after the barrier) orders all of the CTA's remote stores before its ticket.
-__device__ void remote_epilogue(const PeerArgs& pa, int64_t o, bool valid, float acc) {
-    __shared__ bool am_last;
-    if (pa.fold) {
-        if (threadIdx.x == 0)
-            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
-        __syncthreads();
+// With pa.fold the owners' credits (receive buffers consumed) are awaited by thread 0 of every
+// CTA at the CTA's START (spmv_f32_kernel), overlapped with the stage work, instead of a wait
+// kernel ahead of the SpMV; the epoch is read before this CTA's ticket, so before the last CTA
+// bumps it.  (Waiting at the CTA's end kept every SM idle for a system-scope load per partition:
+// +39 us per config-3 forward on one rank, r02g.)  The destination table (owner ranges, buffers,
+// offsets) is read from shared memory, not by dynamic indexing of the kernel parameters.  Only a
+// CTA that stored into another rank's buffer pays a system-scope fence before its ticket.
+struct PeerDst {
+    int64_t bound[kMaxPeers + 1];
+    float* dst[kMaxPeers];
+    int64_t off[kMaxPeers];
+};
+__device__ __forceinline__ void load_peer_dst(PeerDst& t, const PeerArgs& pa) {
+    if (threadIdx.x <= (unsigned)pa.P) t.bound[threadIdx.x] = pa.bound[threadIdx.x];
+    if (threadIdx.x < (unsigned)pa.P) {
+        t.dst[threadIdx.x] = pa.dst[threadIdx.x];
+        t.off[threadIdx.x] = pa.off[threadIdx.x];
     }
+}
+__device__ void remote_epilogue(const PeerArgs& pa, const PeerDst& t, int64_t o, bool valid, float acc) {
+    __shared__ bool am_last;
     int h = pa.me;
     if (valid) {  // o = footprint position of the row
         h = 0;
-        while (h + 1 < pa.P && o >= pa.bound[h + 1]) ++h;
-        pa.dst[h][pa.off[h] + o] = acc;
+        while (h + 1 < pa.P && o >= t.bound[h + 1]) ++h;
+        t.dst[h][t.off[h] + o] = acc;
     }
     // only a CTA that stored into another rank's buffer needs the system-scope fence; stores to
     // this rank's own receive buffer stay on this GPU (the last CTA fences at system scope before
@@ -366,7 +376,7 @@ __device__ void remote_epilogue(const PeerArgs& pa, int64_t o, bool valid, float
     __threadfence_system();
     const unsigned long long e = pa.my_flags[pa.epoch_index] + 1;
     pa.my_flags[pa.epoch_index] = e;
-    for (int h = 0; h < pa.P; ++h) st_release_sys(pa.flag[h] + pa.slot + pa.me, e);
+    for (int h2 = 0; h2 < pa.P; ++h2) st_release_sys(pa.flag[h2] + pa.slot + pa.me, e);
     *pa.ticket = 0u;
 }
 
@@ -394,10 +404,18 @@ template <bool kNatOut, int kEpi>
 __global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, PeerArgs pa) {
     extern __shared__ __align__(16) float sbuf[];
+    __shared__ PeerDst pdst;
     if ((kEpi & 4) && pa.fold) {  // the owners' values for this footprint have arrived
         if (threadIdx.x == 0)
             wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
         __syncthreads();
+    }
+    if (kEpi & 2) {
+        // the owners have consumed my previous partials (credits); ordered before this CTA's
+        // stores by the stage barriers below
+        if (pa.fold && threadIdx.x == 0)
+            wait_flags(pa.my_flags, pa.wait_base, pa.P, pa.my_flags[pa.epoch_index], pa.me, pa.abort);
+        load_peer_dst(pdst, pa);
     }
     const int64_t p = part_of_cta(a);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -424,7 +442,8 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
     const bool valid = row < a.prow0[p + 1];
     const int64_t o = (kNatOut && valid) ? (int64_t)a.out_idx[row] : row;
     if (kEpi & 2) {
-        remote_epilogue(pa, o, valid, acc);
+        if (g0 == g1) __syncthreads();  // no stage barrier ordered the start (credit wait, table)
+        remote_epilogue(pa, pdst, o, valid, acc);
         return;
     }
     if (valid) y[o] = acc;
