@@ -251,12 +251,25 @@ __device__ __forceinline__ int32_t decode_rec(const int4& r, int lane, const int
     if (d3 && lane >= d3) { st = r.w & M; d = d3; }
     return st + (lane - d);
 }
+#ifndef MX_RLE_U
+#define MX_RLE_U 8
+#endif
+#ifndef MX_RLE_PREFETCH
+#define MX_RLE_PREFETCH 1
+#endif
 template <int U, class T, class A>
 __device__ __forceinline__ void stage_gather_rle(T* __restrict__ buf, const T* __restrict__ x, const A& a,
-                                                 int64_t g, int cnt) {
+                                                 int64_t g, int cnt, bool has_next) {
     const int bd = blockDim.x, lane = threadIdx.x & 31;
     const int4* __restrict__ rb = a.blk_rec + a.blk_base[g];
     const uint64_t pm = evict_first_policy();
+    if (MX_RLE_PREFETCH && has_next && threadIdx.x == 0) {  // the next stage's records into L2
+        const int4* n0 = a.blk_rec + a.blk_base[g + 1];
+        const int64_t nb = a.blk_base[g + 2] - a.blk_base[g + 1];
+        if (nb > 0)
+            asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;"
+                         ::"l"(n0), "r"((unsigned)(16 * nb)), "l"(pm) : "memory");
+    }
     for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
         int32_t j[U];
 #pragma unroll
@@ -430,7 +443,7 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();  // previous stage fully consumed
         if (a.rle) {
-            stage_gather_rle<8>(sbuf, x, a, g, cnt);
+            stage_gather_rle<MX_RLE_U>(sbuf, x, a, g, cnt, g + 1 < g1);
         } else {
             if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
             stage_gather<16>(sbuf, x, mp, cnt, a.l2hint);
@@ -500,7 +513,7 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     const uint64_t pol = evict_first_policy();
     auto gather = [&](int64_t s) {  // this thread's share of stage s into buffer s % 3
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
-        if (a.rle) stage_gather_rle<8>(sbuf + (s % 3) * a.B, x, a, g0 + s, cnt);
+        if (a.rle) stage_gather_rle<MX_RLE_U>(sbuf + (s % 3) * a.B, x, a, g0 + s, cnt, s + 1 < ns);
         else stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt, a.l2hint);
         __syncwarp();
         if (lane == 0) mbar_arrive(&full[s % 3]);
@@ -548,7 +561,7 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
         if (g != g0) __syncthreads();
         if (a.rle) {
-            stage_gather_rle<4>(dbuf, x, a, g, cnt);
+            stage_gather_rle<4>(dbuf, x, a, g, cnt, g + 1 < g1);
         } else {
             if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
             stage_gather<MX_F64_GATHER_U>(dbuf, x, mp, cnt, a.l2hint);
