@@ -42,6 +42,14 @@ __global__ void signal_kernel(SignalArgs sa, int P, int slot, const unsigned lon
     for (int q = 0; q < P; ++q) st_release(sa.flag[q] + slot, v);
 }
 
+__global__ void publish_epoch_kernel(SignalArgs sa, int P, int slot, unsigned long long* flags, int epoch_index) {
+    if (threadIdx.x != 0 || blockIdx.x != 0) return;
+    __threadfence_system();
+    const unsigned long long e = flags[epoch_index] + 1;
+    flags[epoch_index] = e;
+    for (int q = 0; q < P; ++q) st_release(sa.flag[q] + slot, e);
+}
+
 // R^T + C^T: value j (recv order, peer g = the range containing j) goes to g's footprint buffer
 // (pa.fold: thread 0 of every CTA first waits for the peers' credits -- footprint buffers
 // consumed -- reading the epoch before this CTA's ticket, i.e. before the last CTA bumps it).
@@ -70,9 +78,21 @@ __global__ void pack_remote_kernel(const float* __restrict__ y, const int32_t* _
     const int64_t j0 = (int64_t)blockIdx.x * chunk, j1 = min(n, j0 + chunk);
     int g = 0;
     while (g + 1 < pa.P && j0 + (int64_t)threadIdx.x >= bound[g + 1]) ++g;
-    for (int64_t j = j0 + threadIdx.x; j < j1; j += blockDim.x) {
-        while (g + 1 < pa.P && j >= bound[g + 1]) ++g;   // ranges ascend with j
-        dst[g][off[g] + j] = y[idx[j]];
+    constexpr int kU = 4;  // independent (index, value) loads in flight per thread
+    for (int64_t j = j0 + threadIdx.x; j < j1; j += kU * (int64_t)blockDim.x) {
+        float v[kU];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t jj = j + u * (int64_t)blockDim.x;
+            v[u] = jj < j1 ? y[idx[jj]] : 0.f;
+        }
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int64_t jj = j + u * (int64_t)blockDim.x;
+            if (jj >= j1) break;
+            while (g + 1 < pa.P && jj >= bound[g + 1]) ++g;   // ranges ascend with j
+            dst[g][off[g] + jj] = v[u];
+        }
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -161,6 +181,7 @@ void peer_setup(Plan& P, cudaStream_t st) {
         cudaFuncAttributes fa;
         MX_CUDA(cudaFuncGetAttributes(&fa, wait_kernel));
         MX_CUDA(cudaFuncGetAttributes(&fa, signal_kernel));
+        MX_CUDA(cudaFuncGetAttributes(&fa, publish_epoch_kernel));
         MX_CUDA(cudaFuncGetAttributes(&fa, pack_remote_kernel));
         MX_CUDA(cudaFuncGetAttributes(&fa, peer_allreduce_kernel));
         preload_exchange_kernels();
@@ -210,10 +231,10 @@ PeerArgs base_args(const Plan& P) {
 // Flags of rank g ([4P + 2]): arrivals fwd [0, P) | arrivals back [P, 2P) | credits fwd [2P, 3P) |
 // credits back [3P, 4P) | my fwd epoch 4P | my back epoch 4P + 1.
 // Forward: (1) owners have consumed my previous partials (credits fwd >= my epoch); (2) A_p
-// stores the partials into the owners' receive buffers, last CTA bumps the epoch and publishes
-// it to every owner; (3) every peer's partials for my rays have arrived; (4) R (+ dot); (5)
-// credits back to every peer.  Folded (NCCL ranks): (1) runs inside A_p's epilogue, (3) and (5)
-// inside the reduction kernel -- two kernels per forward instead of five.
+// stores the partials into the owners' receive buffers; a one-thread kernel then bumps the epoch
+// and publishes it to every owner; (3) every peer's partials for my rays have arrived; (4) R (+
+// dot); (5) credits back to every peer.  Folded (NCCL ranks): (1) runs at the start of A_p's
+// CTAs, (3) and (5) inside the reduction kernel.
 void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream_t st) {
     Exchange& X = P.ex;
     const int np = P.nranks;
@@ -233,6 +254,8 @@ void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream
     pa.epoch_index = 4 * np;
     pa.wait_base = 2 * np;
     spmv_f32_remote(P.fwd, x, pa, st);
+    publish_epoch_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 0 + P.rank, fl, 4 * np);  // arrivals fwd
+    MX_LAUNCHED();
     if (!X.fold) {
         wait_kernel<<<1, 32, 0, st>>>(fl, np, 0, 4 * np, P.rank, peer_abort_word());
         MX_LAUNCHED();
@@ -251,8 +274,8 @@ void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream
 // Back: (1) every peer has finished reading my previous values from its footprint buffer
 // (credits back); (2) R^T + C^T: the owned ray values stored straight into the peers' footprint
 // buffers, last CTA publishes the back epoch; (3) every owner's values for my footprint have
-// arrived; (4) A_p^T (+ dot); (5) credits to every peer.  Folded: (1) in the pack kernel's
-// prologue, (3) in A_p^T's prologue, (5) from A_p^T's last CTA.
+// arrived; (4) A_p^T (+ dot); (5) credits to every peer (one-thread kernel).  Folded: (1) in the
+// pack kernel's prologue, (3) in A_p^T's prologue.
 void peer_back(Plan& P, const float* y, float* x, double* dot_out, cudaStream_t st) {
     Exchange& X = P.ex;
     const int np = P.nranks;
@@ -284,10 +307,9 @@ void peer_back(Plan& P, const float* y, float* x, double* dot_out, cudaStream_t 
     ba.wait_base = np;         // arrivals back
     spmv_f32_peer_back(P.back, X.y_fp.as<float>(), x, dot_out ? X.dot_part.p() : nullptr, dot_out,
                        X.tickets.p() + 4, ba, st);
-    if (!X.fold) {
-        signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 3 * np + P.rank, fl, 4 * np + 1);
-        MX_LAUNCHED();
-    }
+    // credits to every peer (footprint buffer consumed), after the kernel boundary
+    signal_kernel<<<1, 32, 0, st>>>(signal_args(P), np, 3 * np + P.rank, fl, 4 * np + 1);
+    MX_LAUNCHED();
 }
 
 void peer_allreduce(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) {

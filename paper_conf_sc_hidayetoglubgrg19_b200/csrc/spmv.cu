@@ -345,16 +345,15 @@ __device__ __forceinline__ void stream_stage(float& acc, const float* __restrict
 }
 
 // Fused exchange epilogue (P > 1): every footprint row's partial is stored
-// straight into its owner's receive buffer (peer memory over NVLink), then the last CTA bumps
-// this rank's forward epoch and publishes it to every owner's arrival flag (release, system
-// scope).  Replaces the separate all-to-allv of C in A = R C A_p.
+// straight into its owner's receive buffer (peer memory over NVLink); a one-thread kernel after
+// the SpMV bumps this rank's forward epoch and publishes it to every owner's arrival flag
+// (release, system scope).  Replaces the separate all-to-allv of C in A = R C A_p.
 // With pa.fold the owners' credits (receive buffers consumed) are awaited by thread 0 of every
 // CTA at the CTA's START (spmv_f32_kernel), overlapped with the stage work, instead of a wait
 // kernel ahead of the SpMV; the epoch is read before this CTA's ticket, so before the last CTA
 // bumps it.  (Waiting at the CTA's end kept every SM idle for a system-scope load per partition:
 // +39 us per config-3 forward on one rank, r02g.)  The destination table (owner ranges, buffers,
-// offsets) is read from shared memory, not by dynamic indexing of the kernel parameters.  Only a
-// CTA that stored into another rank's buffer pays a system-scope fence before its ticket.
+// offsets) is read from shared memory, not by dynamic indexing of the kernel parameters.
 struct PeerDst {
     int64_t bound[kMaxPeers + 1];
     float* dst[kMaxPeers];
@@ -367,52 +366,21 @@ __device__ __forceinline__ void load_peer_dst(PeerDst& t, const PeerArgs& pa) {
         t.off[threadIdx.x] = pa.off[threadIdx.x];
     }
 }
-__device__ void remote_epilogue(const PeerArgs& pa, const PeerDst& t, int64_t o, bool valid, float acc) {
-    __shared__ bool am_last;
-    int h = pa.me;
+__device__ __forceinline__ void remote_epilogue(const PeerArgs& pa, const PeerDst& t, int64_t o, bool valid,
+                                                float acc) {
     if (valid) {  // o = footprint position of the row
-        h = 0;
+        int h = 0;
         while (h + 1 < pa.P && o >= t.bound[h + 1]) ++h;
         t.dst[h][t.off[h] + o] = acc;
     }
-    // only a CTA that stored into another rank's buffer needs the system-scope fence; stores to
-    // this rank's own receive buffer stay on this GPU (the last CTA fences at system scope before
-    // it publishes the epoch)
-    const int remote = __syncthreads_or(h != pa.me);
-    if (threadIdx.x == 0) {
-        if (remote) __threadfence_system();
-        else __threadfence();
-        am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
-    }
-    __syncthreads();
-    if (!am_last || threadIdx.x != 0) return;
-    __threadfence_system();
-    const unsigned long long e = pa.my_flags[pa.epoch_index] + 1;
-    pa.my_flags[pa.epoch_index] = e;
-    for (int h2 = 0; h2 < pa.P; ++h2) st_release_sys(pa.flag[h2] + pa.slot + pa.me, e);
-    *pa.ticket = 0u;
+    // the epoch is published by publish_kernel after this kernel (peer.cu): the kernel boundary
+    // orders every CTA's stores before its system-scope fence and flag release, so no CTA pays
+    // a barrier + fence + ticket tail here (that tail cost ~10 us per config-3 forward)
 }
 
-// A_p^T of the fused exchange with pa.fold: after every CTA has finished reading the footprint
-// input, the last CTA tells every peer that its footprint buffer may be overwritten again
-// (credits, slot pa.slot + me, value = the back epoch the owners' pack kernels published).
-__device__ void peer_back_epilogue(const PeerArgs& pa) {
-    __shared__ bool am_last;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        am_last = (atomicAdd(pa.ticket, 1u) == gridDim.x - 1);
-    }
-    __syncthreads();
-    if (!am_last || threadIdx.x != 0) return;
-    __threadfence_system();
-    const unsigned long long e = pa.my_flags[pa.epoch_index];
-    for (int h = 0; h < pa.P; ++h) st_release_sys(pa.flag[h] + pa.slot + pa.me, e);
-    *pa.ticket = 0u;
-}
-
-// kEpi bits: 1 = fused dot (last-CTA tree), 2 = fused exchange (remote_epilogue), 4 = A_p^T of the
-// fused exchange (folded arrival wait before the first gather, credits from the last CTA)
+// kEpi bits: 1 = fused dot (last-CTA tree), 2 = fused exchange (remote_epilogue; folded credit
+// wait at the CTA start), 4 = A_p^T of the fused exchange (folded arrival wait before the first
+// gather; the credits go out from a one-thread kernel after it, peer.cu)
 template <bool kNatOut, int kEpi>
 __global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, PeerArgs pa) {
@@ -461,7 +429,6 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
     }
     if (valid) y[o] = acc;
     if (kEpi & 1) finish_dot_tree<kMaxThreads>(a, valid ? (double)acc * (double)acc : 0.0);
-    if ((kEpi & 4) && pa.fold) peer_back_epilogue(pa);
 }
 
 // ---- drifting stages (Layout::drift) ------------------------------------------------------------
