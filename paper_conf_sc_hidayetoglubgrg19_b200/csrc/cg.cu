@@ -200,8 +200,8 @@ unsigned vec_blocks(int64_t n) {
 
 // CG dots at P > 1: one fp64 per slice summed over the ranks -- over peer memory with the fused
 // exchange (peer_allreduce, rank order), else by the transport's allreduce (NCCL / virtual ranks).
-void allreduce_slices(Plan& P, double* v, int K, int64_t stride, cudaStream_t st) {
-    if (!P.dist) return;
+void allreduce_slices(Plan& P, double* v, int K, int64_t stride, cudaStream_t st, bool in_kernel = false) {
+    if (!P.dist || in_kernel) return;
     if (P.ex.peer) {
         peer_allreduce(P, v, K, stride, st);
         return;
@@ -247,7 +247,10 @@ void op_dir(Plan& P, bool forward, int K, const T* in, T* out, double* dot_out, 
                                                               P.tickets.p() + 64);
         MX_LAUNCHED();
     }
-    if (dot_out && P.dist) allreduce_slices(P, dot_out, K, dot_stride, st);
+    // fused peer exchange with folded waits: the last kernel of the projection already summed
+    // the dot over the ranks (peer_dot_allreduce)
+    const bool summed = fused && P.ex.peer && P.ex.fold;
+    if (dot_out && P.dist) allreduce_slices(P, dot_out, K, dot_stride, st, summed);
 }
 
 template <class T>

@@ -138,6 +138,8 @@ reduce_dot_kernel(const T* __restrict__ recv, const int64_t* __restrict__ ptr, c
         __threadfence_system();
         const unsigned long long e = pa.my_flags[pa.epoch_index];
         for (int q = 0; q < pa.P; ++q) st_release_sys(pa.flag[q] + pa.slot + pa.me, e);
+        // the CG dot over the ranks (credits are out first: peers may be waiting on them)
+        if (dot_out && pa.dot_fold) peer_dot_allreduce(pa, dot_out);
     }
     *ticket = 0u;
 }

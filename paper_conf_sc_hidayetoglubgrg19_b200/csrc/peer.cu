@@ -226,6 +226,18 @@ PeerArgs base_args(const Plan& P) {
     for (int q = 0; q < P.nranks; ++q) pa.flag[q] = static_cast<unsigned long long*>(P.ex.peer_flags[q]);
     return pa;
 }
+// the CG dot of this projection summed over the ranks inside its last kernel (fold mode only:
+// a spinning last CTA on a GPU of its own never blocks a peer's kernels)
+void set_dot_fold(const Plan& P, PeerArgs& pa) {
+    const Exchange& X = P.ex;
+    pa.dot_fold = 1;
+    for (int q = 0; q < P.nranks; ++q) {
+        pa.dot_dst[q] = static_cast<double*>(X.peer_dotx[q]);
+        pa.dot_flag[q] = static_cast<unsigned long long*>(X.peer_dflags[q]);
+    }
+    pa.dot_mine = X.dotx.p();
+    pa.dot_my_flags = X.dflags.p();
+}
 }  // namespace
 
 // Flags of rank g ([4P + 2]): arrivals fwd [0, P) | arrivals back [P, 2P) | credits fwd [2P, 3P) |
@@ -239,11 +251,12 @@ void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream
     Exchange& X = P.ex;
     const int np = P.nranks;
     unsigned long long* fl = X.flags.p();
-    if (!X.fold) {
-        wait_kernel<<<1, 32, 0, st>>>(fl, np, 2 * np, 4 * np, P.rank, peer_abort_word());
-        MX_LAUNCHED();
-    }
+    // (1) credits: a one-thread wait kernel in both modes -- folded into A_p's CTAs, the
+    // system-scope wait delayed every partition (+26 us per config-3 forward, r02j)
+    wait_kernel<<<1, 32, 0, st>>>(fl, np, 2 * np, 4 * np, P.rank, peer_abort_word());
+    MX_LAUNCHED();
     PeerArgs pa = base_args(P);
+    pa.fold = 0;  // the credits are awaited above
     for (int h = 0; h <= np; ++h) pa.bound[h] = X.sdispl[h];
     for (int h = 0; h < np; ++h) {
         pa.dst[h] = static_cast<float*>(X.peer_recv[h]);
@@ -261,6 +274,7 @@ void peer_forward(Plan& P, const float* x, float* y, double* dot_out, cudaStream
         MX_LAUNCHED();
     }
     PeerArgs ra = base_args(P);
+    if (X.fold && dot_out) set_dot_fold(P, ra);
     ra.slot = 2 * np;          // credits fwd in the senders' arrays
     ra.epoch_index = 4 * np;
     ra.wait_base = 0;          // arrivals fwd
@@ -301,6 +315,7 @@ void peer_back(Plan& P, const float* y, float* x, double* dot_out, cudaStream_t 
         MX_LAUNCHED();
     }
     PeerArgs ba = base_args(P);
+    if (X.fold && dot_out) set_dot_fold(P, ba);
     ba.ticket = X.tickets.p() + 3;
     ba.slot = 3 * np;          // credits back in the owners' arrays
     ba.epoch_index = 4 * np + 1;

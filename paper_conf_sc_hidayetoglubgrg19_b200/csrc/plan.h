@@ -115,6 +115,13 @@ struct PeerArgs {
     int32_t fold = 0;
     int32_t wait_base = 0;
     unsigned int* abort = nullptr;               // peer_abort_word(): set by a timed-out wait
+    // CG dot summed over the ranks by the kernel's last CTA (folded peer dot, one slice): the
+    // peer_allreduce protocol of peer.cu on one value, in place of its one-thread kernel
+    int32_t dot_fold = 0;
+    double* dot_dst[kMaxPeers] = {};               // rank q's dot slots (peer pointer)
+    unsigned long long* dot_flag[kMaxPeers] = {};  // rank q's dot flags (peer pointer)
+    const double* dot_mine = nullptr;              // my dot slots
+    unsigned long long* dot_my_flags = nullptr;    // my dot flags: [P arrivals | epoch]
 };
 
 // A process-wide word in mapped (device-visible) host memory: a peer-flag wait that times out
@@ -157,6 +164,25 @@ __device__ inline void wait_flags(const unsigned long long* flags, int base, int
             }
         }
     }
+}
+#endif
+
+#ifdef __CUDACC__
+// One thread (a kernel's last CTA): *v summed over the ranks in rank order through peer memory
+// (the protocol of peer.cu: peer_allreduce_kernel, kMaxDotSlices slots per parity).
+__device__ inline void peer_dot_allreduce(const PeerArgs& pa, double* v) {
+    const unsigned long long e = pa.dot_my_flags[pa.P] + 1;
+    pa.dot_my_flags[pa.P] = e;
+    const int par = (int)(e & 1ull);
+    const double mine = *v;
+    for (int q = 0; q < pa.P; ++q) pa.dot_dst[q][((int64_t)par * pa.P + pa.me) * kMaxDotSlices] = mine;
+    __threadfence_system();
+    for (int q = 0; q < pa.P; ++q) st_release_sys(pa.dot_flag[q] + pa.me, e);
+    wait_flags(pa.dot_my_flags, 0, pa.P, e, pa.me, pa.abort);
+    const volatile double* m = pa.dot_mine + (int64_t)par * pa.P * kMaxDotSlices;
+    double acc = m[0];
+    for (int q = 1; q < pa.P; ++q) acc += m[(int64_t)q * kMaxDotSlices];
+    *v = acc;
 }
 #endif
 
