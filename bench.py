@@ -60,7 +60,38 @@ def parse():
     ap.add_argument("--variant", default=None, choices=["peer", "dense"], help=argparse.SUPPRESS)
     ap.add_argument("--distributed", action="store_true",
                     help="run the decomposed path (NCCL communicator, exchange, allreduce) even at N = 1")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "host"],
+                    help="N > 1 transport: nccl (one GPU per rank) or host (memxct_plan_set_comm_host: "
+                         "processes may share a GPU -- exercises the multi-rank bench on one GPU; "
+                         "its times are not multi-GPU numbers)")
     return ap.parse_args()
+
+
+def _dist_allreduce_max(t):
+    """MAX over ranks of a CUDA tensor (through the CPU on gloo)."""
+    import torch.distributed as dist
+    if dist.get_backend() == "gloo":
+        c = t.cpu()
+        dist.all_reduce(c, op=dist.ReduceOp.MAX)
+        t.copy_(c)
+    else:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return t
+
+
+def _dist_allgather(t):
+    import torch
+    import torch.distributed as dist
+    src = t.cpu() if dist.get_backend() == "gloo" else t
+    out = [torch.empty_like(src) for _ in range(dist.get_world_size())]
+    dist.all_gather(out, src)
+    return torch.stack(out).cpu()
+
+
+def _device_index(args):
+    import torch
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    return local % max(1, torch.cuda.device_count()) if args.transport == "host" else local
 
 
 def workload_name(cfg, iters):
@@ -378,15 +409,18 @@ def variant_child(args):
     JSON line."""
     import torch
     import torch.distributed as dist
-    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, bootstrap_unique_id, inputs
-    local = int(os.environ.get("LOCAL_RANK", 0))
+    from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, bootstrap_host_comm_name, bootstrap_unique_id, inputs
+    local = _device_index(args)
     torch.cuda.set_device(local)
-    dist.init_process_group("nccl")
+    dist.init_process_group("gloo" if args.transport == "host" else "nccl")
     rank, world = dist.get_rank(), dist.get_world_size()
     n, m, c = inputs.CONFIGS[args.config]
-    uid = bootstrap_unique_id(rank)
-    plan = MemXCT(n, m, c, rank=rank, nranks=world, unique_id=uid, device=local,
-                  vector_order="plan", exchange=args.variant).build()
+    if args.transport == "host":
+        comm = {"host_comm": bootstrap_host_comm_name(rank)}
+    else:
+        comm = {"unique_id": bootstrap_unique_id(rank)}
+    plan = MemXCT(n, m, c, rank=rank, nranks=world, device=local, vector_order="plan", exchange=args.variant,
+                  **comm).build()
     ph = np.ascontiguousarray(inputs.shepp_logan(n).astype(np.float32)[plan.local_indices(0)])
     stream = torch.cuda.current_stream()
     y = plan.forward(torch.from_numpy(ph).cuda())
@@ -403,7 +437,7 @@ def variant_child(args):
     torch.cuda.synchronize()
     ex = plan.exchange_time(20, stream=stream) if args.variant == "dense" else {"fwd_us": 0.0, "back_us": 0.0}
     t = torch.tensor([e0.elapsed_time(e1), ex["fwd_us"], ex["back_us"]], dtype=torch.float64, device=y.device)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    _dist_allreduce_max(t)
     out = {"value": args.iters * args.steps / (float(t[0]) * 1e-3), "unit": "CG iter/s",
            "ms_per_step": float(t[0]) / args.steps}
     if args.variant == "dense":
@@ -424,7 +458,8 @@ def bench_exchange_variant(args, rank, world, kind):
     env = dict(os.environ)
     env["MASTER_PORT"] = str(int(os.environ.get("MASTER_PORT", "29500")) + (17 if kind == "peer" else 23))
     cmd = [sys.executable, os.path.abspath(__file__), "--variant", kind, "--config", str(args.config),
-           "--iters", str(args.iters), "--steps", str(args.steps), "--warmup", str(args.warmup)]
+           "--iters", str(args.iters), "--steps", str(args.steps), "--warmup", str(args.warmup),
+           "--transport", args.transport]
     try:
         r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=300)
     except subprocess.TimeoutExpired:
@@ -443,7 +478,7 @@ def run_ours(args, rank, world):
 
     from paper_conf_sc_hidayetoglubgrg19_b200 import MemXCT, inputs, kernel_launch_count
 
-    local = int(os.environ.get("LOCAL_RANK", 0))
+    local = _device_index(args)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     cfg = args.config
@@ -457,10 +492,12 @@ def run_ours(args, rank, world):
     t0 = time.perf_counter()
     if dist_mode:
         # domain decomposition over the ranks (A = R C A_p), NCCL exchange
-        from paper_conf_sc_hidayetoglubgrg19_b200 import bootstrap_unique_id
-        uid = bootstrap_unique_id(rank)
-        plan = MemXCT(n, m, c, rank=rank, nranks=world, unique_id=uid, device=local,
-                      vector_order="plan", **kw).build()
+        from paper_conf_sc_hidayetoglubgrg19_b200 import bootstrap_host_comm_name, bootstrap_unique_id
+        if args.transport == "host":
+            kw["host_comm"] = bootstrap_host_comm_name(rank)
+        else:
+            kw["unique_id"] = bootstrap_unique_id(rank)
+        plan = MemXCT(n, m, c, rank=rank, nranks=world, device=local, vector_order="plan", **kw).build()
     else:
         plan = MemXCT(n, m, c, **kw).build()
     torch.cuda.synchronize()
@@ -525,15 +562,13 @@ def run_ours(args, rank, world):
                              spmv_bytes(fi), spmv_bytes(bi), fi["nnz"], bi["nnz"]],
                             dtype=torch.float64, device=dev)
     if dist_mode:
-        gathered = [torch.empty_like(per_rank) for _ in range(world)]
-        dist.all_gather(gathered, per_rank)
-        per_rank_all = torch.stack(gathered).cpu().numpy()
+        per_rank_all = _dist_allgather(per_rank).numpy()
     else:
         per_rank_all = per_rank.cpu().numpy()[None, :]
 
     t = torch.tensor([ms], dtype=torch.float64, device=dev)
     if dist_mode:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        _dist_allreduce_max(t)
     ms_max = float(t.item())
 
     # e2e through the C ABI with host buffers (pinned sinogram in, tomogram out)
@@ -549,14 +584,14 @@ def run_ours(args, rank, world):
     te = time.perf_counter() - te0
     te_t = torch.tensor([te], dtype=torch.float64, device=dev)
     if dist_mode:
-        dist.all_reduce(te_t, op=dist.ReduceOp.MAX)
+        _dist_allreduce_max(te_t)
     te = float(te_t.item())
 
     exch_t = None
     if dist_mode:
         exch_t = plan.exchange_time(20, stream=stream)
         et = torch.tensor([exch_t["fwd_us"], exch_t["back_us"]], dtype=torch.float64, device=dev)
-        dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        _dist_allreduce_max(et)
         exch_t = {"fwd_us": float(et[0]), "back_us": float(et[1]),
                   "per_cg_iter_us": float(et[0] + et[1]),
                   "local_spmv_fwd_us": float(per_rank_all[:, 0].max() * 1e3),
@@ -607,7 +642,10 @@ def run_ours(args, rank, world):
                          (6 * st["stored_slots"] / 2 / 1e9),
                    "part_rows": plan.get_option("part_rows"),
                    "buffer_entries": plan.get_option("buffer_entries"),
-                   "parallelism": (f"domain decomposition over {world} GPUs (A = R C A_p, NCCL all-to-allv)"
+                   "parallelism": ((f"domain decomposition over {world} GPUs (A = R C A_p, NCCL all-to-allv)"
+                                    if args.transport == "nccl" else
+                                    f"domain decomposition over {world} processes sharing "
+                                    f"{torch.cuda.device_count()} GPU(s) (host transport; NOT a multi-GPU timing)")
                                    if dist_mode else "single GPU")},
         "spmv": {"fwd_ms": tf * 1e3, "back_ms": tb * 1e3,
                  "fwd_gflops": 2 * fnnz / tf / 1e9, "back_gflops": 2 * bnnz / tb / 1e9,
@@ -662,7 +700,7 @@ def self_launch(args):
     GPUs.  Returns the launcher's exit code."""
     import torch
     have = torch.cuda.device_count()
-    if have < args.gpus:
+    if have < args.gpus and args.transport != "host":
         print(f"bench.py: --gpus {args.gpus} needs {args.gpus} CUDA devices, this node has {have}",
               file=sys.stderr, flush=True)
         return 2
@@ -690,7 +728,7 @@ def main():
             os.environ.setdefault(k, v)
     if world > 1 or (args.distributed and args.impl == "ours"):
         import torch.distributed as dist
-        if args.impl == "ours":
+        if args.impl == "ours" and args.transport == "nccl":
             import torch
             torch.cuda.set_device(int(os.environ.get("LOCAL_RANK", 0)))
             dist.init_process_group("nccl")

@@ -900,6 +900,38 @@ void spmv_f32_peer_back(const Layout& L, const float* x, float* y, double* dot_p
     MX_LAUNCHED();
 }
 
+// Canonical dot (reading R16) after the SpMV instead of inside it: one thread per partition runs
+// the partition's fma chain over its rows in row (Hilbert) order -- the same operations in the
+// same order as finish_dot_canonical -- and the last block adds the partials in partition order.
+// Inside the SpMV the chain held each CTA's SM idle for ~1024 dependent fma (~5 us per
+// partition); here all chains run at once.
+__global__ void __launch_bounds__(128)
+canonical_dot_kernel(const double* __restrict__ y, const int32_t* __restrict__ out_idx, const int64_t* __restrict__ prow0,
+                     int64_t nparts, double* __restrict__ part, double* dot_out, unsigned int* ticket) {
+    __shared__ bool am_last;
+    const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p < nparts) {
+        double acc = 0.0;
+        for (int64_t r = prow0[p]; r < prow0[p + 1]; ++r) {
+            const double v = y[out_idx ? (int64_t)out_idx[r] : r];
+            acc = __fma_rn(v, v, acc);
+        }
+        part[p] = acc;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        am_last = (atomicAdd(ticket, 1u) == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!am_last || threadIdx.x != 0) return;
+    __threadfence();
+    double tot = 0.0;
+    for (int64_t i = 0; i < nparts; ++i) tot = __dadd_rn(tot, ((volatile double*)part)[i]);
+    *dot_out = tot;
+    *ticket = 0u;
+}
+
 void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, double* dot_out,
               unsigned int* ticket, bool canonical, cudaStream_t st, int64_t c0, int64_t c1) {
     if (c1 < 0) c1 = L.nparts;
@@ -909,12 +941,24 @@ void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, dou
     a.cta_base = c0;
     const size_t smem = sizeof(double) * (size_t)std::max(L.B, L.R);
     const bool nat = L.out_idx.p() != nullptr;
-    const int mode = dot_out == nullptr ? 0 : (canonical ? 2 : 1);
+    // canonical dot: a chain per partition after the SpMV (canonical_dot_kernel), unless
+    // MEMXCT_CANONICAL_DOT_INLINE=1 keeps it in the SpMV's CTAs (spmv_f64_kernel<., 2>)
+    static const bool inline_dot = [] {
+        const char* e = std::getenv("MEMXCT_CANONICAL_DOT_INLINE");
+        return e && e[0] == '1';
+    }();
+    const bool after = dot_out && canonical && !inline_dot;
+    const int mode = (dot_out == nullptr || after) ? 0 : (canonical ? 2 : 1);
     void (*kern)(SpmvArgs, const double*, double*);
     if (nat) kern = mode == 0 ? spmv_f64_kernel<true, 0> : mode == 1 ? spmv_f64_kernel<true, 1> : spmv_f64_kernel<true, 2>;
     else kern = mode == 0 ? spmv_f64_kernel<false, 0> : mode == 1 ? spmv_f64_kernel<false, 1> : spmv_f64_kernel<false, 2>;
     kern<<<(unsigned)(c1 - c0), L.R, smem, st>>>(a, x, y);
     MX_LAUNCHED();
+    if (after) {
+        canonical_dot_kernel<<<(unsigned)ceil_div(L.nparts, 128), 128, 0, st>>>(y, L.out_idx.p(), L.prow0.p(), L.nparts,
+                                                                              dot_part, dot_out, ticket);
+        MX_LAUNCHED();
+    }
 }
 
 // ---- layout export to COO on the device (memxct_export_coo) --------------------------------
