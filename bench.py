@@ -457,6 +457,10 @@ def bench_exchange_variant(args, rank, world, kind):
     hanging) is reported without taking down the headline's process."""
     env = dict(os.environ)
     env["MASTER_PORT"] = str(int(os.environ.get("MASTER_PORT", "29500")) + (17 if kind == "peer" else 23))
+    # under torchrun the ranks' env:// rendezvous is a client of the agent's store; the children's
+    # fresh rendezvous needs its own store, hosted by child rank 0 (else every child waits for a
+    # server that never starts -- the r02l host-transport run timed out exactly so)
+    env.pop("TORCHELASTIC_USE_AGENT_STORE", None)
     cmd = [sys.executable, os.path.abspath(__file__), "--variant", kind, "--config", str(args.config),
            "--iters", str(args.iters), "--steps", str(args.steps), "--warmup", str(args.warmup),
            "--transport", args.transport]

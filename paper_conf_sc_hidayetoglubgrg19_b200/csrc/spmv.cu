@@ -941,13 +941,15 @@ void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, dou
     a.cta_base = c0;
     const size_t smem = sizeof(double) * (size_t)std::max(L.B, L.R);
     const bool nat = L.out_idx.p() != nullptr;
-    // canonical dot: a chain per partition after the SpMV (canonical_dot_kernel), unless
-    // MEMXCT_CANONICAL_DOT_INLINE=1 keeps it in the SpMV's CTAs (spmv_f64_kernel<., 2>)
-    static const bool inline_dot = [] {
-        const char* e = std::getenv("MEMXCT_CANONICAL_DOT_INLINE");
+    // canonical dot: in the SpMV's CTAs (spmv_f64_kernel<., 2>, default), or with
+    // MEMXCT_CANONICAL_DOT_AFTER=1 as one chain per partition in a kernel after the SpMV --
+    // measured slower (config-3 MIXED + CANONICAL CG 227 vs 235 iter/s, r02l: 1500 threads each
+    // walking 1024 dependent rows)
+    static const bool after_env = [] {
+        const char* e = std::getenv("MEMXCT_CANONICAL_DOT_AFTER");
         return e && e[0] == '1';
     }();
-    const bool after = dot_out && canonical && !inline_dot;
+    const bool after = dot_out && canonical && after_env;
     const int mode = (dot_out == nullptr || after) ? 0 : (canonical ? 2 : 1);
     void (*kern)(SpmvArgs, const double*, double*);
     if (nat) kern = mode == 0 ? spmv_f64_kernel<true, 0> : mode == 1 ? spmv_f64_kernel<true, 1> : spmv_f64_kernel<true, 2>;
