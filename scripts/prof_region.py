@@ -3,7 +3,8 @@
 selected call between cudaProfilerStart / Stop.
 
     ncu --profile-from-start off ... python scripts/prof_region.py --kind collective --what cg --iters 3
-kinds: plain | collective | peer | dense (one-rank NCCL communicator) | mixed (MIXED + CANONICAL)
+kinds: plain | bench (natural order, the bench's plan) | collective | peer | dense (one-rank NCCL
+communicator) | mixed (MIXED + CANONICAL)
 what:  cg (a CG solve of --iters iterations) | fwd | back | pair
 """
 import argparse
@@ -26,6 +27,8 @@ def main():
     n, m, c = inputs.CONFIGS[a.config]
     if a.kind == "plain":
         plan = MemXCT(n, m, c, vector_order="plan").build()
+    elif a.kind == "bench":  # the bench's plan: natural vector order, default options
+        plan = MemXCT(n, m, c).build()
     elif a.kind == "mixed":
         plan = MemXCT(n, m, c, vector_order="plan", precision="mixed", canonical=True).build()
     else:
