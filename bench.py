@@ -194,8 +194,7 @@ def oracle_sample(cfg, frac, seed=0):
     t0 = time.perf_counter()
     ptr, pix, ln = oracle.sample_rows(n, m, c, rays)
     t_trace = time.perf_counter() - t0
-    rows = np.repeat(np.arange(len(rays), dtype=np.int32), np.diff(ptr))
-    tp, tc, tv = oracle.coo_to_csr(pix, rows, ln, n * n)     # A^T restricted to the sampled rays
+    tp, tc, tv = oracle.csr_transpose(ptr, pix, ln, n * n)    # A^T restricted to the sampled rays
     return {"ptr": ptr, "cols": pix, "vals": ln, "tptr": tp, "tcols": tc, "tvals": tv,
             "nrays": len(rays), "npix": n * n, "nnz": len(pix), "trace_s": t_trace, "frac": frac}
 

@@ -118,6 +118,11 @@ orc_csr_t* orc_sample_rows(int32_t n, int32_t m_proj, int32_t c_chan, int64_t nr
 orc_csr_t* orc_sample_columns(int32_t n, int32_t m_proj, int32_t c_chan, int64_t npix,
                               const int64_t* pixels, int32_t nthreads);
 
+/* Stable transpose of a CSR (nrows x ncols): output row c lists the input rows holding column c
+ * in ascending input-row order.  Pinned by: equality with the sort-based coo_to_csr. */
+orc_csr_t* orc_csr_transpose(int64_t nrows, const int64_t* ptr, const int32_t* idx, const double* len,
+                             int64_t ncols);
+
 /* y = A x over CSR with rows split over host threads (the threaded CPU
  * baseline).  Each row is summed sequentially in entry order, bit-identical to orc_spmv_coo on
  * row-major COO.  Returns the number of threads used. */

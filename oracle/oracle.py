@@ -19,7 +19,7 @@ __all__ = [
     "build_oracle", "lib", "trace_ray", "count_nnz", "row_lengths", "trace_all", "gilbert2d",
     "d2xy", "hilbert_rank", "spmv_coo", "spmv_canonical", "cgls", "dot_canonical",
     "coo_to_csr", "sampled_back_rows", "sirt", "chord", "chords", "sample_rows", "sample_columns",
-    "spmv_csr_threaded",
+    "spmv_csr_threaded", "csr_transpose",
 ]
 
 
@@ -81,6 +81,8 @@ def lib():
         L.orc_sample_columns.argtypes = [i32, i32, i32, i64, vp, i32]
         L.orc_csr_free.restype = None
         L.orc_csr_free.argtypes = [ctypes.POINTER(_Csr)]
+        L.orc_csr_transpose.restype = ctypes.POINTER(_Csr)
+        L.orc_csr_transpose.argtypes = [i64, vp, vp, vp, i64]
         L.orc_spmv_csr_threaded.restype = i32
         L.orc_spmv_csr_threaded.argtypes = [i64, vp, vp, vp, vp, vp, i32]
         _lib = L
@@ -249,6 +251,14 @@ def sample_columns(n: int, m: int, c: int, pixels, threads: int = 0):
     ascending, lengths) per pixel."""
     p = np.ascontiguousarray(pixels, np.int64)
     return _take_csr(lib().orc_sample_columns(n, m, c, len(p), _p(p), int(threads)))
+
+
+def csr_transpose(ptr, idx, vals, ncols: int):
+    """Stable CSR transpose (orc_csr_transpose): (ptr, row indices, values) per column."""
+    ptr = np.ascontiguousarray(ptr, np.int64)
+    idx = np.ascontiguousarray(idx, np.int32)
+    vals = np.ascontiguousarray(vals, np.float64)
+    return _take_csr(lib().orc_csr_transpose(len(ptr) - 1, _p(ptr), _p(idx), _p(vals), int(ncols)))
 
 
 def spmv_csr_threaded(ptr, cols, vals, x, threads: int = 0):

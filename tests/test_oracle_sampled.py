@@ -125,3 +125,12 @@ def test_threaded_spmv_bit_identical_to_coo(orc, coo_cache, threads):
     yt = np.random.default_rng(2).standard_normal(m * c)
     xb, _ = orc.spmv_csr_threaded(tp, tc, tv, yt, threads)
     assert np.array_equal(xb, orc.spmv_coo(cols, rows, vals, yt, n * n))
+
+
+def test_csr_transpose_equals_sort_based(orc, coo_cache):
+    n, m, c = 33, 17, 33
+    rows, cols, vals = coo_cache(n, m, c)
+    ptr = np.searchsorted(rows, np.arange(m * c + 1)).astype(np.int64)
+    tp, tc, tv = orc.csr_transpose(ptr, cols, vals, n * n)
+    rp, rc, rv = orc.coo_to_csr(cols, rows, vals, n * n)
+    assert np.array_equal(tp, rp) and np.array_equal(tc, rc) and np.array_equal(tv, rv)
