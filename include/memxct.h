@@ -352,7 +352,7 @@ memxct_status_t memxct_layout_info(memxct_plan_t plan, int32_t dir, int64_t* par
  * arrays of memxct_layout_info's `slots` entries.  Entry = (output index, input index, value) in
  * the plan's vector order (natural indices with VECTOR_ORDER = 0); padding slots are written as
  * (-1, -1, 0).  Stream-ordered on `cuda_stream`.  For interoperability -- e.g. handing the same
- * matrix to a library SpMV (scripts/cusparse_compare.py) -- not part of the hot path.
+ * matrix to another SpMV implementation -- not part of the hot path.
  * Errors: STATE before build, INVALID_ARG for dir or NULL arrays. */
 memxct_status_t memxct_export_coo(memxct_plan_t plan, int32_t dir, int32_t* rows, int32_t* cols,
                                   float* vals, void* cuda_stream);

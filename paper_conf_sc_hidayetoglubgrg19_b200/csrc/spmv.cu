@@ -465,7 +465,9 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
                      "selp.u32 %0, 1, 0, P;\n\t}"
                      : "=r"(ok) : "r"(a), "r"(parity) : "memory");
         if (ok) return;
-        if (clock64() - t0 > 20000000000LL) __trap();  // ~10 s: a broken phase, not a slow stage
+        // ~10 s: a broken phase (an internal invariant of this CTA -- every warp arrives once per
+        // phase -- not a peer), so a trap rather than the peer waits' abort word
+        if (clock64() - t0 > 20000000000LL) __trap();
     }
 }
 
