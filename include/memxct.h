@@ -179,6 +179,13 @@ memxct_status_t memxct_plan_set_comm_local(memxct_plan_t plan, memxct_group_t gr
 memxct_status_t memxct_plan_set_comm_host(memxct_plan_t plan, int32_t rank, int32_t nranks,
                                           const char* name, int32_t cuda_device);
 
+/* Host-only round trip of the host transport (no device needed): rendezvous on `name` (as in
+ * memxct_plan_set_comm_host), a host allgather of one int64 per rank into gathered[0..nranks)
+ * (host), a barrier, teardown.  For checking the processes' rendezvous (e.g. the CPU gloo tests).
+ * The rendezvous gives up after MEMXCT_HOST_COMM_TIMEOUT_S seconds (default 300): NCCL status. */
+memxct_status_t memxct_host_comm_probe(const char* name, int32_t rank, int32_t nranks, int64_t value,
+                                       int64_t* gathered);
+
 /* Shard probe: build on this device only rank `rank`'s part of a `nranks`-way decomposition
  * -- the same tile ranges (R12), footprint rays, A_p, A_p^T and exchange counts /
  * maps that rank would build inside a real P-rank job, with no peers and no communicator (the

@@ -249,6 +249,19 @@ memxct_status_t memxct_plan_set_comm_host(memxct_plan_t plan, int32_t rank, int3
     });
 }
 
+memxct_status_t memxct_host_comm_probe(const char* name, int32_t rank, int32_t nranks, int64_t value,
+                                       int64_t* gathered) {
+    return guarded([&] {
+        need(name, "name");
+        need(gathered, "gathered");
+        if (nranks < 1 || nranks > 16 || rank < 0 || rank >= nranks) mx::fail(MEMXCT_ERR_INVALID_ARG, "bad rank / nranks");
+        if (name[0] != '/' || std::strlen(name) < 2 || std::strlen(name) > 200 || std::strchr(name + 1, '/'))
+            mx::fail(MEMXCT_ERR_INVALID_ARG, "name must be \"/<token>\" (a POSIX shared-memory name)");
+        const auto v = mx::host_comm_probe(name, rank, nranks, value);
+        for (int q = 0; q < nranks; ++q) gathered[q] = v[q];
+    });
+}
+
 memxct_status_t memxct_plan_set_shard(memxct_plan_t plan, int32_t rank, int32_t nranks, int32_t cuda_device) {
     return guarded([&] {
         mx::Plan& P = plan_of(plan);

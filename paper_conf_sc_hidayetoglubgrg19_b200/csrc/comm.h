@@ -59,6 +59,8 @@ std::unique_ptr<Comm> make_nccl_comm(int rank, int nranks, const void* unique_id
 // processes of one node (possibly sharing a GPU) over a named POSIX shared-memory segment and
 // CUDA IPC device mailboxes (proccomm.cu); not graph-capturable
 std::unique_ptr<Comm> make_host_comm(const std::string& name, int rank, int nranks);
+// host-only round trip of the host transport (rendezvous, barriers, host allgather): no device
+std::vector<int64_t> host_comm_probe(const std::string& name, int rank, int nranks, int64_t value);
 void nccl_unique_id(void* out);
 
 // shared state of a group of virtual ranks

@@ -41,7 +41,14 @@ namespace {
 constexpr int kMaxRanks = 16;                    // kMaxPeers of the fused exchange
 constexpr int64_t kSlotWords = 1 << 14;          // host allgather slot: 128 KB per rank (~2 MB segment)
 constexpr uint64_t kMagic = 0x4d454d5843543031ull;  // "MEMXCT01"
-constexpr double kTimeoutS = 300.0;
+// rendezvous / barrier time-out: 300 s, or MEMXCT_HOST_COMM_TIMEOUT_S (tests)
+double timeout_s() {
+    static const double v = [] {
+        const char* e = std::getenv("MEMXCT_HOST_COMM_TIMEOUT_S");
+        return e ? std::max(0.1, atof(e)) : 300.0;
+    }();
+    return v;
+}
 
 struct Shared {
     std::atomic<uint64_t> magic;
@@ -88,12 +95,12 @@ public:
             }
         } else {
             while ((fd = shm_open(name.c_str(), O_RDWR, 0600)) < 0) {
-                if (elapsed(t0) > kTimeoutS) fail(MEMXCT_ERR_NCCL, "host transport: rank 0 never created " + name);
+                if (elapsed(t0) > timeout_s()) fail(MEMXCT_ERR_NCCL, "host transport: rank 0 never created " + name);
                 std::this_thread::sleep_for(std::chrono::milliseconds(2));
             }
             struct stat sb;
             while (fstat(fd, &sb) == 0 && (size_t)sb.st_size < bytes) {
-                if (elapsed(t0) > kTimeoutS) fail(MEMXCT_ERR_NCCL, "host transport: segment never sized");
+                if (elapsed(t0) > timeout_s()) fail(MEMXCT_ERR_NCCL, "host transport: segment never sized");
                 std::this_thread::sleep_for(std::chrono::milliseconds(2));
             }
         }
@@ -108,16 +115,19 @@ public:
             sh_->magic.store(kMagic, std::memory_order_release);
         } else {
             while (sh_->magic.load(std::memory_order_acquire) != kMagic) {
-                if (elapsed(t0) > kTimeoutS) fail(MEMXCT_ERR_NCCL, "host transport: segment never initialised");
+                if (elapsed(t0) > timeout_s()) fail(MEMXCT_ERR_NCCL, "host transport: segment never initialised");
                 std::this_thread::sleep_for(std::chrono::milliseconds(2));
             }
             if (sh_->nranks != n) fail(MEMXCT_ERR_INVALID_ARG, "host transport: nranks differs from rank 0's");
         }
-        cudaDeviceProp prop;
+        // the device's UUID (zeros without a device: the host-only probe, memxct_host_comm_probe)
+        std::memset(sh_->rank[rank].device_uuid, 0, 16);
         int dev = 0;
-        MX_CUDA(cudaGetDevice(&dev));
-        MX_CUDA(cudaGetDeviceProperties(&prop, dev));
-        std::memcpy(sh_->rank[rank].device_uuid, &prop.uuid, 16);
+        cudaDeviceProp prop;
+        if (cudaGetDevice(&dev) == cudaSuccess && cudaGetDeviceProperties(&prop, dev) == cudaSuccess)
+            std::memcpy(sh_->rank[rank].device_uuid, &prop.uuid, 16);
+        else
+            cudaGetLastError();
         barrier();
         if (r == 0) shm_unlink(name.c_str());  // every rank is attached: the name is no longer needed
         same_device_ = true;
@@ -240,7 +250,7 @@ public:
         while (sh_->generation.load(std::memory_order_acquire) == gen) {
             if (++spins > 1000) std::this_thread::sleep_for(std::chrono::microseconds(20));
             else sched_yield();
-            if (spins % 4096 == 0 && elapsed(t0) > kTimeoutS)
+            if (spins % 4096 == 0 && elapsed(t0) > timeout_s())
                 fail(MEMXCT_ERR_NCCL, "host transport: a peer process did not reach the barrier");
         }
     }
@@ -315,6 +325,13 @@ private:
 
 std::unique_ptr<Comm> make_host_comm(const std::string& name, int rank, int nranks) {
     return std::make_unique<ProcComm>(name, rank, nranks);
+}
+
+std::vector<int64_t> host_comm_probe(const std::string& name, int rank, int nranks, int64_t value) {
+    ProcComm c(name, rank, nranks);
+    auto v = c.allgather_host(value, nullptr);
+    c.barrier();
+    return v;
 }
 
 

@@ -35,7 +35,7 @@ SYMBOLS = [
     "memxct_forward_batch", "memxct_back_batch", "memxct_cg_batch", "memxct_exchange_time",
     "memxct_sirt", "memxct_spmv_time", "memxct_plan_set_shard", "memxct_exchange_counts",
     "memxct_footprint_rays", "memxct_footprint_forward", "memxct_footprint_back", "memxct_layout_rows",
-    "memxct_read_ceiling", "memxct_export_coo", "memxct_build_phases", "memxct_plan_set_comm_host",
+    "memxct_read_ceiling", "memxct_export_coo", "memxct_build_phases", "memxct_plan_set_comm_host", "memxct_host_comm_probe",
 ]
 
 #: memxct_build_phases order (include/memxct.h)
@@ -113,6 +113,7 @@ def lib():
             "memxct_export_coo": [vp, i32, vp, vp, vp, vp],
             "memxct_build_phases": [vp, vp],
             "memxct_plan_set_comm_host": [vp, i32, i32, ctypes.c_char_p, i32],
+            "memxct_host_comm_probe": [ctypes.c_char_p, i32, i32, i64, vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -184,6 +185,14 @@ class LocalGroup:
             self.close()
         except Exception:
             pass
+
+
+def host_comm_probe(name: str, rank: int, nranks: int, value: int) -> np.ndarray:
+    """memxct_host_comm_probe: host-only rendezvous + allgather of one int64 per rank."""
+    out = np.empty(nranks, np.int64)
+    _check(lib().memxct_host_comm_probe(name.encode(), int(rank), int(nranks), int(value),
+                                        out.ctypes.data_as(ctypes.c_void_p)), "memxct_host_comm_probe")
+    return out
 
 
 def bootstrap_host_comm_name(rank: int, group=None) -> str:

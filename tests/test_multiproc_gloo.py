@@ -64,3 +64,57 @@ def test_partition_ranges_edge_cases():
     assert b.tolist() == [0, 33, 67, 100]
     with pytest.raises(Exception):
         partition_ranges([-1, 2], 2)
+
+
+def _host_comm_worker(rank, world, port, q, rounds):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_sc_hidayetoglubgrg19_b200.memxct import bootstrap_host_comm_name, host_comm_probe
+        out = []
+        for k in range(rounds):   # a fresh segment per round: create, attach, unlink, reuse of names
+            name = bootstrap_host_comm_name(rank)
+            out.append((name, host_comm_probe(name, rank, world, 1000 * k + 7 * rank + 1).tolist()))
+        q.put((rank, out))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_gloo_host_transport_rendezvous(world):
+    """The host transport's host side (memxct_plan_set_comm_host's rendezvous: a shared-memory
+    segment created by rank 0 and attached by the others, process-shared barriers, the host
+    allgather) across `world` processes on CPU, the segment name bootstrapped over gloo."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    rounds = 3
+    procs = [ctx.Process(target=_host_comm_worker, args=(r, world, port, q, rounds)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=180) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for k in range(rounds):
+        names = {res[r][k][0] for r in range(world)}
+        assert len(names) == 1
+        expect = [1000 * k + 7 * r + 1 for r in range(world)]
+        for r in range(world):
+            assert res[r][k][1] == expect
+
+
+def test_host_transport_missing_peer_fails_loudly(monkeypatch):
+    """A rank whose peers never arrive gets MEMXCT_ERR_NCCL after the time-out, not a hang."""
+    import subprocess
+    import sys
+    code = ("import sys; sys.path.insert(0, %r)\n"
+            "from paper_conf_sc_hidayetoglubgrg19_b200.memxct import host_comm_probe, MemXCTError\n"
+            "try:\n    host_comm_probe('/memxct-missing-peer-test', 1, 2, 5)\nexcept MemXCTError as e:\n"
+            "    print('ERR', e)\n") % os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, MEMXCT_HOST_COMM_TIMEOUT_S="1.5")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=120)
+    assert "ERR" in r.stdout and "NCCL" in r.stdout, (r.stdout, r.stderr)
