@@ -488,8 +488,15 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     const int64_t g0 = a.stage_base[p], ns = a.stage_base[p + 1] - g0;
     const int64_t m0 = a.map_off[p], D = a.map_off[p + 1] - m0;
     const uint64_t pol = evict_first_policy();
+#ifndef MX_DRIFT_PREFETCH
+#define MX_DRIFT_PREFETCH 1
+#endif
     auto gather = [&](int64_t s) {  // this thread's share of stage s into buffer s % 3
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
+        // the map of stage s + 2 into L2 (one bulk request by thread 0): a warp gathers a stage
+        // one to two stages after warp 0 gathers this one, so its map loads then hit L2
+        if (MX_DRIFT_PREFETCH && !a.rle && threadIdx.x == 0 && s + 2 < ns)
+            prefetch_map_l2(a.map + m0 + (s + 2) * a.B, (int)min((int64_t)a.B, D - (s + 2) * a.B), a.l2hint);
         if (a.rle) stage_gather_rle<MX_RLE_U>(sbuf + (s % 3) * a.B, x, a, g0 + s, cnt, s + 1 < ns);
         else stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt, a.l2hint);
         __syncwarp();
