@@ -318,17 +318,32 @@ __device__ __forceinline__ void prefetch_map_l2(const int32_t* mp, int cnt, int 
 
 // One warp's slots of stage g (its 32-row slice block): acc += buf[ind] * val, streamed with
 // 16 B evict-first loads (6 B per nonzero from HBM).
-__device__ __forceinline__ void stream_stage(float& acc, const float* __restrict__ sbuf, const SpmvArgs& a,
-                                             int64_t g, int warp, int lane, unsigned lt, uint64_t pol) {
+// The block's head: slot offset and this lane's chunk count.  The fp64 kernel loads it ahead of
+// the stage's gather (MX_HEAD_EARLY), so its latency -- a DRAM round trip: the heads are read
+// once -- overlaps the gather instead of standing between the stage barrier and the first stream
+// load: MIXED config-3 SpMV 2.01 -> 1.94 ms (r02s).  In the fp32 kernels it measured neutral
+// (config 3, config-5 forward) or slower (config-5 back +1 %), so they load it after the barrier.
+struct StageHead {
+    int64_t base;
+    int nch;
+};
+__device__ __forceinline__ StageHead stage_head(const SpmvArgs& a, int64_t g, int warp, int lane) {
     const int64_t blk = g * a.SPP + warp;
-    const int64_t base = a.slot_off[blk];
-    const int nch = a.lane_chunks[blk * 32 + lane];
+    return {a.slot_off[blk], (int)a.lane_chunks[blk * 32 + lane]};
+}
+#ifndef MX_HEAD_EARLY
+#define MX_HEAD_EARLY 1
+#endif
+__device__ __forceinline__ void stream_stage(float& acc, const float* __restrict__ sbuf, const StageHead& h,
+                                             const SpmvArgs& a, int lane, unsigned lt, uint64_t pol) {
+    const int64_t base = h.base;
+    const int nch = h.nch;
     const int maxc = __reduce_max_sync(0xffffffffu, nch);
     const uint4* ib = reinterpret_cast<const uint4*>(a.ind + base);
     const float4* vb = reinterpret_cast<const float4*>(a.val + base);
+    const int minc = __reduce_min_sync(0xffffffffu, nch);
     // phase 1: chunks every lane has -- plain SELL addressing, branch-free, unrolled so
     // several 16 B loads per lane are in flight
-    const int minc = __reduce_min_sync(0xffffffffu, nch);
 #pragma unroll 4
     for (int c = 0; c < minc; ++c) {
         const uint4 iv = ld_stream_u4(ib + c * 32 + lane, pol);
@@ -425,7 +440,7 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
             stage_gather<16>(sbuf, x, mp, cnt, a.l2hint);
         }
         __syncthreads();
-        stream_stage(acc, sbuf, a, g, warp, lane, lt, pol);
+        stream_stage(acc, sbuf, stage_head(a, g, warp, lane), a, lane, lt, pol);
     }
     const int64_t row = a.prow0[p] + threadIdx.x;
     const bool valid = row < a.prow0[p + 1];
@@ -471,14 +486,48 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
     }
 }
 
+// Asynchronous stage gather (MX_DRIFT_ASYNC): the thread's map entries are loaded (16 in
+// flight), then each input is copied global -> shared by a 4-byte cp.async (LDGSTS) that
+// completes in the background, and `cp.async.mbarrier.arrive.noinc` makes full[b]'s phase wait
+// for this thread's copies.  The warp goes back to streaming after ONE L2 round trip (the map)
+// instead of two (map, then the dependent inputs through registers): in the synchronous form
+// the gather held ~24 % of the config-5 forward's warp-state samples (r02p), time in which the
+// warp has no stream loads in flight.
+__device__ __forceinline__ void cp_async4(float* dst, const float* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_addr(dst)),
+                 "l"(__cvta_generic_to_global(src)) : "memory");
+}
+__device__ __forceinline__ void cp_async_mbar_arrive_noinc(uint64_t* b) {
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_addr(b)) : "memory");
+}
+__device__ __forceinline__ void stage_gather_async(float* __restrict__ buf, const float* __restrict__ x,
+                                                   const int32_t* __restrict__ mp, int cnt) {
+    constexpr int U = 16;
+    const int bd = blockDim.x;
+    for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+        int32_t j[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) j[u] = (i0 + u * bd < cnt) ? __ldg(mp + i0 + u * bd) : -1;
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if (j[u] >= 0) cp_async4(buf + i0 + u * bd, x + j[u]);
+    }
+}
+#ifndef MX_DRIFT_ASYNC
+#define MX_DRIFT_ASYNC 1
+#endif
+
 template <bool kNatOut, int kEpi>
 __global__ void __launch_bounds__(kMaxThreads, 1)
 spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y) {
     extern __shared__ __align__(16) float sbuf[];  // [3][B]
     __shared__ __align__(8) uint64_t full[3], done[3];
-    if (threadIdx.x == 0)  // one arrival per warp (after __syncwarp, which orders the lanes' accesses)
+    // full: one arrival per thread with the asynchronous gather (its cp.async completions), else
+    // one per warp; done: one per warp (after __syncwarp, which orders the lanes' accesses)
+    const bool async_gather = MX_DRIFT_ASYNC && !a.rle;
+    if (threadIdx.x == 0)
         for (int b = 0; b < 3; ++b) {
-            mbar_init(&full[b], blockDim.x >> 5);
+            mbar_init(&full[b], async_gather ? blockDim.x : blockDim.x >> 5);
             mbar_init(&done[b], blockDim.x >> 5);
         }
     __syncthreads();
@@ -497,6 +546,11 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
         // one to two stages after warp 0 gathers this one, so its map loads then hit L2
         if (MX_DRIFT_PREFETCH && !a.rle && threadIdx.x == 0 && s + 2 < ns)
             prefetch_map_l2(a.map + m0 + (s + 2) * a.B, (int)min((int64_t)a.B, D - (s + 2) * a.B), a.l2hint);
+        if (async_gather) {
+            stage_gather_async(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt);
+            cp_async_mbar_arrive_noinc(&full[s % 3]);
+            return;
+        }
         if (a.rle) stage_gather_rle<MX_RLE_U>(sbuf + (s % 3) * a.B, x, a, g0 + s, cnt, s + 1 < ns);
         else stage_gather<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt, a.l2hint);
         __syncwarp();
@@ -510,7 +564,7 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
         // test-only: pseudo-random per-warp delays stretch the drift between warps, so the
         // buffer-reuse protocol is exercised at its limits (tests/test_gpu_drift.py)
         if (a.jitter && ((warp * 7 + (int)s) % 5 == 0)) __nanosleep(2000 + 131 * warp);
-        stream_stage(acc, sbuf + (s % 3) * a.B, a, g0 + s, warp, lane, lt, pol);
+        stream_stage(acc, sbuf + (s % 3) * a.B, stage_head(a, g0 + s, warp, lane), a, lane, lt, pol);
         __syncwarp();
         if (lane == 0) mbar_arrive(&done[s % 3]);
         if (s + 2 < ns) {
@@ -543,6 +597,8 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
         const int64_t s = g - g0;
         const int cnt = (int)min((int64_t)a.B, D - s * a.B);
         const int32_t* __restrict__ mp = a.map + m0 + s * a.B;
+        StageHead h;
+        if (MX_HEAD_EARLY) h = stage_head(a, g, warp, lane);
         if (g != g0) __syncthreads();
         if (a.rle) {
             stage_gather_rle<4>(dbuf, x, a, g, cnt, g + 1 < g1);
@@ -551,9 +607,9 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
             stage_gather<MX_F64_GATHER_U>(dbuf, x, mp, cnt, a.l2hint);
         }
         __syncthreads();
-        const int64_t blk = g * a.SPP + warp;
-        const int64_t base = a.slot_off[blk];
-        const int nch = a.lane_chunks[blk * 32 + lane];
+        if (!MX_HEAD_EARLY) h = stage_head(a, g, warp, lane);
+        const int64_t base = h.base;
+        const int nch = h.nch;
         const int maxc = __reduce_max_sync(0xffffffffu, nch);
         const uint4* ib = reinterpret_cast<const uint4*>(a.ind + base);
         const float4* vb = reinterpret_cast<const float4*>(a.val + base);
