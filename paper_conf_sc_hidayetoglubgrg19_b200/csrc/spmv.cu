@@ -471,14 +471,25 @@ __device__ __forceinline__ void mbar_init(uint64_t* b, unsigned count) {
 __device__ __forceinline__ void mbar_arrive(uint64_t* b) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(b)) : "memory");
 }
+#ifndef MX_MBAR_HINT
+#define MX_MBAR_HINT 0
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
     const uint32_t a = smem_addr(b);
     const long long t0 = clock64();
     for (;;) {
         uint32_t ok;
+#if MX_MBAR_HINT
+        // suspend-time hint (ns): the thread sleeps in the try_wait until the phase completes or
+        // the hint expires, instead of re-issuing it (and the time-out check) at the default rate
+        asm volatile("{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2, %3;\n\t"
+                     "selp.u32 %0, 1, 0, P;\n\t}"
+                     : "=r"(ok) : "r"(a), "r"(parity), "r"((unsigned)MX_MBAR_HINT) : "memory");
+#else
         asm volatile("{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
                      "selp.u32 %0, 1, 0, P;\n\t}"
                      : "=r"(ok) : "r"(a), "r"(parity) : "memory");
+#endif
         if (ok) return;
         // ~10 s: a broken phase (an internal invariant of this CTA -- every warp arrives once per
         // phase -- not a peer), so a trap rather than the peer waits' abort word
@@ -513,6 +524,31 @@ __device__ __forceinline__ void stage_gather_async(float* __restrict__ buf, cons
             if (j[u] >= 0) cp_async4(buf + i0 + u * bd, x + j[u]);
     }
 }
+// the same from run-length maps: records (phase 1, all in flight), decode, cp.async per slot
+template <int U, class A>
+__device__ __forceinline__ void stage_gather_rle_async(float* __restrict__ buf, const float* __restrict__ x,
+                                                       const A& a, int64_t g, int cnt, bool has_next) {
+    const int bd = blockDim.x, lane = threadIdx.x & 31;
+    const int4* __restrict__ rb = a.blk_rec + a.blk_base[g];
+    if (MX_RLE_PREFETCH && has_next && threadIdx.x == 0) {  // the next stage's records into L2
+        const int4* n0 = a.blk_rec + a.blk_base[g + 1];
+        const int64_t nb = a.blk_base[g + 2] - a.blk_base[g + 1];
+        if (nb > 0)
+            asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;"
+                         ::"l"(n0), "r"((unsigned)(16 * nb)), "l"(evict_first_policy()) : "memory");
+    }
+    for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+        int4 r[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int i = i0 + u * bd;
+            r[u] = i < cnt ? __ldg(rb + (i >> 5)) : make_int4(0, 0, 0, 0);
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if (i0 + u * bd < cnt) cp_async4(buf + i0 + u * bd, x + decode_rec(r[u], lane, a.ovf));
+    }
+}
 #ifndef MX_DRIFT_ASYNC
 #define MX_DRIFT_ASYNC 1
 #endif
@@ -524,7 +560,7 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     __shared__ __align__(8) uint64_t full[3], done[3];
     // full: one arrival per thread with the asynchronous gather (its cp.async completions), else
     // one per warp; done: one per warp (after __syncwarp, which orders the lanes' accesses)
-    const bool async_gather = MX_DRIFT_ASYNC && !a.rle;
+    const bool async_gather = MX_DRIFT_ASYNC;
     if (threadIdx.x == 0)
         for (int b = 0; b < 3; ++b) {
             mbar_init(&full[b], async_gather ? blockDim.x : blockDim.x >> 5);
@@ -547,7 +583,8 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
         if (MX_DRIFT_PREFETCH && !a.rle && threadIdx.x == 0 && s + 2 < ns)
             prefetch_map_l2(a.map + m0 + (s + 2) * a.B, (int)min((int64_t)a.B, D - (s + 2) * a.B), a.l2hint);
         if (async_gather) {
-            stage_gather_async(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt);
+            if (a.rle) stage_gather_rle_async<MX_RLE_U>(sbuf + (s % 3) * a.B, x, a, g0 + s, cnt, s + 1 < ns);
+            else stage_gather_async(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt);
             cp_async_mbar_arrive_noinc(&full[s % 3]);
             return;
         }
