@@ -170,21 +170,33 @@ __device__ void finish_dot_tree(const SpmvArgs& a, double mine, const PeerArgs* 
 
 // canonical (reading R16): partial = fma chain over the partition's rows in Hilbert order,
 // total = partials added sequentially in partition order, all in IEEE fp64 round-to-nearest.
-__device__ void finish_dot_canonical(const SpmvArgs& a, const double* rows_val, int nvalid) {
+// The last CTA stages the partials in shared memory (`sbuf`, `cap` entries; every thread, one
+// coalesced pass per chunk) and thread 0 adds them from there: the same additions in the same
+// order, but one load round trip per chunk instead of one dependent L2 load per partition (the
+// one-thread loop over volatile global loads cost ~1500 serial round trips per config-3 dot).
+__device__ void finish_dot_canonical(const SpmvArgs& a, double* sbuf, int nvalid, int cap) {
     __shared__ bool am_last;
     if (threadIdx.x == 0) {
         double part = 0.0;
-        for (int i = 0; i < nvalid; ++i) part = __fma_rn(rows_val[i], rows_val[i], part);
+        for (int i = 0; i < nvalid; ++i) part = __fma_rn(sbuf[i], sbuf[i], part);
         a.dot_part[part_of_cta(a)] = part;
         __threadfence();
         const unsigned t = atomicAdd(a.ticket, 1u);
         am_last = (t == (unsigned)(a.nparts - 1));
     }
     __syncthreads();
-    if (!am_last || threadIdx.x != 0) return;
+    if (!am_last) return;
     __threadfence();
-    double tot = 0.0;
-    for (int64_t i = 0; i < a.nparts; ++i) tot = __dadd_rn(tot, ((volatile double*)a.dot_part)[i]);
+    double tot = 0.0;  // thread 0's
+    for (int64_t c0 = 0; c0 < a.nparts; c0 += cap) {
+        const int n = (int)min((int64_t)cap, a.nparts - c0);
+        __syncthreads();  // the previous chunk (first pass: this CTA's row values) consumed
+        for (int i = threadIdx.x; i < n; i += blockDim.x) sbuf[i] = ((volatile double*)a.dot_part)[c0 + i];
+        __syncthreads();
+        if (threadIdx.x == 0)
+            for (int i = 0; i < n; ++i) tot = __dadd_rn(tot, sbuf[i]);
+    }
+    if (threadIdx.x != 0) return;
     *a.dot_out = tot;
     *a.ticket = 0u;
 }
@@ -684,7 +696,7 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
         dbuf[threadIdx.x] = valid ? acc : 0.0;
         __syncthreads();
         const int64_t nvalid = a.prow0[p + 1] - a.prow0[p];
-        finish_dot_canonical(a, dbuf, (int)nvalid);
+        finish_dot_canonical(a, dbuf, (int)nvalid, max(a.B, a.R));
     }
 }
 
@@ -1002,23 +1014,33 @@ void spmv_f32_peer_back(const Layout& L, const float* x, float* y, double* dot_p
     MX_LAUNCHED();
 }
 
-// Canonical dot (reading R16) after the SpMV instead of inside it: one thread per partition runs
-// the partition's fma chain over its rows in row (Hilbert) order -- the same operations in the
-// same order as finish_dot_canonical -- and the last block adds the partials in partition order.
-// Inside the SpMV the chain held each CTA's SM idle for ~1024 dependent fma (~5 us per
-// partition); here all chains run at once.
-__global__ void __launch_bounds__(128)
+// Canonical dot (reading R16) after the SpMV instead of inside it: one WARP per partition stages
+// the partition's row values in shared memory (coalesced, all lanes), then its lane 0 runs the
+// partition's fma chain over them in row (Hilbert) order -- the same operations in the same order
+// as finish_dot_canonical -- and the last block adds the partials in partition order (staged in
+// shared memory likewise).  Inside the SpMV the chain holds the CTA's SM idle for ~1024 dependent
+// fma per partition; here the chains of many partitions run at once.  (The first form of this
+// kernel, one thread per partition walking its rows with global loads, was slower than the
+// in-SpMV chain: 227 vs 235 CG iter/s, r02l.)
+constexpr int kCdWarps = 8;
+__global__ void __launch_bounds__(kCdWarps * 32)
 canonical_dot_kernel(const double* __restrict__ y, const int32_t* __restrict__ out_idx, const int64_t* __restrict__ prow0,
-                     int64_t nparts, double* __restrict__ part, double* dot_out, unsigned int* ticket) {
+                     int64_t nparts, int R, double* __restrict__ part, double* dot_out, unsigned int* ticket) {
+    extern __shared__ __align__(16) double sv[];  // [kCdWarps][R]
     __shared__ bool am_last;
-    const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t p = (int64_t)blockIdx.x * kCdWarps + warp;
     if (p < nparts) {
-        double acc = 0.0;
-        for (int64_t r = prow0[p]; r < prow0[p + 1]; ++r) {
-            const double v = y[out_idx ? (int64_t)out_idx[r] : r];
-            acc = __fma_rn(v, v, acc);
+        const int64_t r0 = prow0[p];
+        const int n = (int)(prow0[p + 1] - r0);
+        double* v = sv + (size_t)warp * R;
+        for (int i = lane; i < n; i += 32) v[i] = y[out_idx ? (int64_t)out_idx[r0 + i] : r0 + i];
+        __syncwarp();
+        if (lane == 0) {
+            double acc = 0.0;
+            for (int i = 0; i < n; ++i) acc = __fma_rn(v[i], v[i], acc);
+            part[p] = acc;
         }
-        part[p] = acc;
     }
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -1026,10 +1048,19 @@ canonical_dot_kernel(const double* __restrict__ y, const int32_t* __restrict__ o
         am_last = (atomicAdd(ticket, 1u) == gridDim.x - 1);
     }
     __syncthreads();
-    if (!am_last || threadIdx.x != 0) return;
+    if (!am_last) return;
     __threadfence();
-    double tot = 0.0;
-    for (int64_t i = 0; i < nparts; ++i) tot = __dadd_rn(tot, ((volatile double*)part)[i]);
+    const int cap = kCdWarps * R;
+    double tot = 0.0;  // thread 0's
+    for (int64_t c0 = 0; c0 < nparts; c0 += cap) {
+        const int n = (int)min((int64_t)cap, nparts - c0);
+        __syncthreads();
+        for (int i = threadIdx.x; i < n; i += blockDim.x) sv[i] = ((volatile double*)part)[c0 + i];
+        __syncthreads();
+        if (threadIdx.x == 0)
+            for (int i = 0; i < n; ++i) tot = __dadd_rn(tot, sv[i]);
+    }
+    if (threadIdx.x != 0) return;
     *dot_out = tot;
     *ticket = 0u;
 }
@@ -1047,10 +1078,8 @@ void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, dou
     // MEMXCT_CANONICAL_DOT_AFTER=1 as one chain per partition in a kernel after the SpMV --
     // measured slower (config-3 MIXED + CANONICAL CG 227 vs 235 iter/s, r02l: 1500 threads each
     // walking 1024 dependent rows)
-    static const bool after_env = [] {
-        const char* e = std::getenv("MEMXCT_CANONICAL_DOT_AFTER");
-        return e && e[0] == '1';
-    }();
+    const char* ae = std::getenv("MEMXCT_CANONICAL_DOT_AFTER");  // read per call (tests switch it)
+    const bool after_env = ae && ae[0] == '1';
     const bool after = dot_out && canonical && after_env;
     const int mode = (dot_out == nullptr || after) ? 0 : (canonical ? 2 : 1);
     void (*kern)(SpmvArgs, const double*, double*);
@@ -1059,8 +1088,9 @@ void spmv_f64(const Layout& L, const double* x, double* y, double* dot_part, dou
     kern<<<(unsigned)(c1 - c0), L.R, smem, st>>>(a, x, y);
     MX_LAUNCHED();
     if (after) {
-        canonical_dot_kernel<<<(unsigned)ceil_div(L.nparts, 128), 128, 0, st>>>(y, L.out_idx.p(), L.prow0.p(), L.nparts,
-                                                                              dot_part, dot_out, ticket);
+        canonical_dot_kernel<<<(unsigned)ceil_div(L.nparts, kCdWarps), kCdWarps * 32,
+                               sizeof(double) * kCdWarps * (size_t)L.R, st>>>(y, L.out_idx.p(), L.prow0.p(), L.nparts,
+                                                                              L.R, dot_part, dot_out, ticket);
         MX_LAUNCHED();
     }
 }
@@ -1166,6 +1196,7 @@ void spmv_init() {
     set_smem(spmv_f64_kernel<false, 0>);
     set_smem(spmv_f64_kernel<false, 1>);
     set_smem(spmv_f64_kernel<false, 2>);
+    set_smem(canonical_dot_kernel);
     set_smem(spmm_f32_kernel<2, true>);
     set_smem(spmm_f32_kernel<2, false>);
     set_smem(spmm_f32_kernel<4, true>);

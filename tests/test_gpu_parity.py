@@ -232,6 +232,21 @@ def test_cg_mixed_canonical_matches_oracle(orc, coo_cache, n, m, c, R):
     assert np.allclose(res_gpu, res_orc, rtol=1e-6, atol=0)
 
 
+@pytest.mark.parametrize("n,m,c,R", [(64, 90, 64, 128), (256, 360, 256, 512)])
+def test_canonical_dot_after_spmv_bit_identical(monkeypatch, orc, coo_cache, n, m, c, R):
+    """The canonical dot run inside the fp64 SpMV's CTAs and in a separate kernel after it
+    (MEMXCT_CANONICAL_DOT_AFTER=1: one warp per partition) perform the same fp64 operations in the
+    same order (reading R16), so the MIXED + CANONICAL CG iterates and residuals are identical."""
+    rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
+    plan = make_plan(n, m, c, precision="mixed", canonical=True, part_rows=R)
+    y = torch.from_numpy(y32.astype(np.float64)).cuda()
+    monkeypatch.setenv("MEMXCT_CANONICAL_DOT_AFTER", "0")
+    x0, r0 = plan.cg(y, 12, residuals=True)
+    monkeypatch.setenv("MEMXCT_CANONICAL_DOT_AFTER", "1")
+    x1, r1 = plan.cg(y, 12, residuals=True)
+    assert torch.equal(x0, x1) and np.array_equal(r0, r1)
+
+
 @pytest.mark.parametrize("n,m,c", [(64, 90, 64), (256, 360, 256)])
 def test_cg_fp32_recovers_phantom(orc, coo_cache, n, m, c):
     rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
