@@ -215,10 +215,13 @@ def _phantom_problem(orc, coo_cache, n, m, c):
     return rows, cols, vals, xt, y32
 
 
-@pytest.mark.parametrize("n,m,c,R", [(64, 90, 64, 512), (64, 90, 64, 128), (256, 360, 256, 512)])
-def test_cg_mixed_canonical_matches_oracle(orc, coo_cache, n, m, c, R):
+# the last case has more partitions (180) than the SpMV's shared buffer holds fp64 partials (64),
+# so the canonical dot's final sum is staged in several chunks
+@pytest.mark.parametrize("n,m,c,R,B", [(64, 90, 64, 512, None), (64, 90, 64, 128, None), (256, 360, 256, 512, None),
+                                       (64, 90, 64, 32, 128)])
+def test_cg_mixed_canonical_matches_oracle(orc, coo_cache, n, m, c, R, B):
     rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
-    plan = make_plan(n, m, c, precision="mixed", canonical=True, part_rows=R)
+    plan = make_plan(n, m, c, precision="mixed", canonical=True, part_rows=R, buffer_entries=B)
     tt, ts = tiles_of(plan)
     v32 = vals.astype(np.float32).astype(np.float64)
     x_orc, res_orc, _, _ = orc.cgls(rows, cols, v32, y32.astype(np.float64), m * c, n * n, 30,
@@ -232,7 +235,7 @@ def test_cg_mixed_canonical_matches_oracle(orc, coo_cache, n, m, c, R):
     assert np.allclose(res_gpu, res_orc, rtol=1e-6, atol=0)
 
 
-@pytest.mark.parametrize("n,m,c,R", [(64, 90, 64, 128), (256, 360, 256, 512)])
+@pytest.mark.parametrize("n,m,c,R", [(64, 90, 64, 128), (256, 360, 256, 512), (256, 360, 256, 32)])
 def test_canonical_dot_after_spmv_bit_identical(monkeypatch, orc, coo_cache, n, m, c, R):
     """The canonical dot run inside the fp64 SpMV's CTAs and in a separate kernel after it
     (MEMXCT_CANONICAL_DOT_AFTER=1: one warp per partition) perform the same fp64 operations in the
