@@ -215,10 +215,10 @@ def _phantom_problem(orc, coo_cache, n, m, c):
     return rows, cols, vals, xt, y32
 
 
-# the last case has more partitions (180) than the SpMV's shared buffer holds fp64 partials (64),
-# so the canonical dot's final sum is staged in several chunks
+# the last case has more forward partitions (180) than the SpMV's shared buffer holds fp64
+# partials (128), so the canonical dot's final sum is staged in two chunks
 @pytest.mark.parametrize("n,m,c,R,B", [(64, 90, 64, 512, None), (64, 90, 64, 128, None), (256, 360, 256, 512, None),
-                                       (64, 90, 64, 32, 128)])
+                                       (64, 90, 64, 32, 256)])
 def test_cg_mixed_canonical_matches_oracle(orc, coo_cache, n, m, c, R, B):
     rows, cols, vals, xt, y32 = _phantom_problem(orc, coo_cache, n, m, c)
     plan = make_plan(n, m, c, precision="mixed", canonical=True, part_rows=R, buffer_entries=B)
