@@ -87,7 +87,9 @@ typedef enum {
     MEMXCT_OPT_PRECISION = 4,
     /* 1 = canonical summation order (reading R16): one fp64 fma chain per row in ascending
      * Hilbert column order, dots as per-partition fma chains summed in partition order.
-     * Requires PRECISION = MIXED.  Default 0. */
+     * Requires PRECISION = MIXED.  Single GPU only (P = 1): at P > 1 a row's sum is split
+     * over the ranks that own its pixels (A = R C A_p), so one chain per row does not
+     * exist; memxct_build on a decomposed plan gives MEMXCT_ERR_UNSUPPORTED.  Default 0. */
     MEMXCT_OPT_CANONICAL = 5,
     /* 0 = recursive-residual CGLS (default, 1 forward + 1 back per iteration, reading R13).
      * 1 = explicit residual r = y - A x each iteration (2 forward + 1 back). */
