@@ -119,6 +119,8 @@ struct SpmvArgs {
     const int64_t* blk_base;
     const int4* blk_rec;
     const int32_t* ovf;
+    int32_t wave;          // CTAs resident at once (one per SM): the launch-order distance to the
+                           // CTA that takes over this SM (MX_NEXT_PREFETCH)
 };
 
 // Partition processed by this CTA: a.order maps launch positions to partitions when a launch
@@ -241,6 +243,71 @@ __device__ __forceinline__ void stage_gather(T* __restrict__ buf, const T* __res
             if (i0 + u * bd < cnt) buf[i0 + u * bd] = v[u];
     }
 }
+
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+// Asynchronous stage gather: the thread's U map entries are loaded (all in flight), then each
+// input is copied global -> shared by a cp.async (LDGSTS, 4 or 8 B) that completes in the
+// background -- no register round trip for the inputs, so the next U map loads issue right away
+// and a stage costs ~cnt / (U * bd) map round trips plus one input round trip at the end, instead
+// of two dependent round trips per U entries.  Completion: cp.async.wait_all + barrier (plain
+// and fp64 kernels) or the stage's `full` mbarrier (drifting kernel).  hint: map evict-first,
+// input evict-last (the L2 priorities of stage_gather).
+__device__ __forceinline__ void cp_async_el(float* dst, const float* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_addr(dst)),
+                 "l"(__cvta_generic_to_global(src)) : "memory");
+}
+__device__ __forceinline__ void cp_async_el(double* dst, const double* src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_addr(dst)),
+                 "l"(__cvta_generic_to_global(src)) : "memory");
+}
+__device__ __forceinline__ void cp_async_el(float* dst, const float* src, uint64_t pol) {
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(smem_addr(dst)),
+                 "l"(__cvta_generic_to_global(src)), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void cp_async_el(double* dst, const double* src, uint64_t pol) {
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 8, %2;" ::"r"(smem_addr(dst)),
+                 "l"(__cvta_generic_to_global(src)), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+template <int U, class T>
+__device__ __forceinline__ void stage_gather_async(T* __restrict__ buf, const T* __restrict__ x,
+                                                   const int32_t* __restrict__ mp, int cnt, int hint) {
+    const int bd = blockDim.x;
+    if (hint) {
+        const uint64_t pm = evict_first_policy(), px = evict_last_policy();
+        for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+            int32_t j[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) j[u] = (i0 + u * bd < cnt) ? ld_map_hint(mp + i0 + u * bd, pm) : -1;
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (j[u] >= 0) cp_async_el(buf + i0 + u * bd, x + j[u], px);
+        }
+        return;
+    }
+    for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+        int32_t j[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) j[u] = (i0 + u * bd < cnt) ? __ldg(mp + i0 + u * bd) : -1;
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if (j[u] >= 0) cp_async_el(buf + i0 + u * bd, x + j[u]);
+    }
+}
+// entries per thread in flight of the plain kernel's asynchronous gather (0 = the synchronous
+// stage_gather): config-3 SpMV 1.650 / 1.686 -> 1.640 / 1.677 ms, config 4 -0.2 / -0.6 % at 16;
+// 32 gains less (r02ac, profiles/r02ac_async_*.jsonl)
+#ifndef MX_PLAIN_ASYNC
+#define MX_PLAIN_ASYNC 16
+#endif
+#ifndef MX_NEXT_PREFETCH
+#define MX_NEXT_PREFETCH 0
+#endif
+// the same for the fp64 kernel: within noise on the MIXED config-3 CG (r02ac), so synchronous
+#ifndef MX_F64_ASYNC
+#define MX_F64_ASYNC 0
+#endif
 
 // The same gather from run-length maps (Layout::rle): slot i of the stage belongs to 32-slot
 // block i / 32 (one warp instruction's slots: lane = i mod 32); the block's 16 B record (one
@@ -449,7 +516,23 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
             stage_gather_rle<MX_RLE_U>(sbuf, x, a, g, cnt, g + 1 < g1);
         } else {
             if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
-            stage_gather<16>(sbuf, x, mp, cnt, a.l2hint);
+#if MX_NEXT_PREFETCH
+            // last stage: the first-stage map of the CTA launched about one wave later (launch
+            // order ~ partition order) into L2, so that CTA's first gather starts with L2 hits
+            if (threadIdx.x == 32 && g + 1 == g1 && !a.order) {
+                const int64_t q = a.cta_base + blockIdx.x + a.wave;
+                if (q < a.nparts) {
+                    const int64_t mq = a.map_off[q];
+                    prefetch_map_l2(a.map + mq, (int)min((int64_t)a.B, a.map_off[q + 1] - mq), a.l2hint);
+                }
+            }
+#endif
+            if (MX_PLAIN_ASYNC) {
+                stage_gather_async<(MX_PLAIN_ASYNC > 0 ? MX_PLAIN_ASYNC : 1)>(sbuf, x, mp, cnt, a.l2hint);
+                cp_async_wait_all();
+            } else {
+                stage_gather<16>(sbuf, x, mp, cnt, a.l2hint);
+            }
         }
         __syncthreads();
         stream_stage(acc, sbuf, stage_head(a, g, warp, lane), a, lane, lt, pol);
@@ -476,7 +559,6 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
 // gathers its share of stage s+2 and moves on, so warps drift up to about one stage apart and a
 // warp that is heavy in one stage catches up in the next.  Same layout, same per-row fma order:
 // bit-identical to spmv_f32_kernel for the same stage size B.
-__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint64_t* b, unsigned count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(b)), "r"(count) : "memory");
 }
@@ -516,25 +598,8 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, unsigned parity) {
 // instead of two (map, then the dependent inputs through registers): in the synchronous form
 // the gather held ~24 % of the config-5 forward's warp-state samples (r02p), time in which the
 // warp has no stream loads in flight.
-__device__ __forceinline__ void cp_async4(float* dst, const float* src) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_addr(dst)),
-                 "l"(__cvta_generic_to_global(src)) : "memory");
-}
 __device__ __forceinline__ void cp_async_mbar_arrive_noinc(uint64_t* b) {
     asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_addr(b)) : "memory");
-}
-__device__ __forceinline__ void stage_gather_async(float* __restrict__ buf, const float* __restrict__ x,
-                                                   const int32_t* __restrict__ mp, int cnt) {
-    constexpr int U = 16;
-    const int bd = blockDim.x;
-    for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
-        int32_t j[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) j[u] = (i0 + u * bd < cnt) ? __ldg(mp + i0 + u * bd) : -1;
-#pragma unroll
-        for (int u = 0; u < U; ++u)
-            if (j[u] >= 0) cp_async4(buf + i0 + u * bd, x + j[u]);
-    }
 }
 // the same from run-length maps: records (phase 1, all in flight), decode, cp.async per slot
 template <int U, class A>
@@ -558,7 +623,7 @@ __device__ __forceinline__ void stage_gather_rle_async(float* __restrict__ buf, 
         }
 #pragma unroll
         for (int u = 0; u < U; ++u)
-            if (i0 + u * bd < cnt) cp_async4(buf + i0 + u * bd, x + decode_rec(r[u], lane, a.ovf));
+            if (i0 + u * bd < cnt) cp_async_el(buf + i0 + u * bd, x + decode_rec(r[u], lane, a.ovf));
     }
 }
 #ifndef MX_DRIFT_ASYNC
@@ -596,7 +661,7 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
             prefetch_map_l2(a.map + m0 + (s + 2) * a.B, (int)min((int64_t)a.B, D - (s + 2) * a.B), a.l2hint);
         if (async_gather) {
             if (a.rle) stage_gather_rle_async<MX_RLE_U>(sbuf + (s % 3) * a.B, x, a, g0 + s, cnt, s + 1 < ns);
-            else stage_gather_async(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt);
+            else stage_gather_async<16>(sbuf + (s % 3) * a.B, x, a.map + m0 + s * a.B, cnt, a.l2hint);
             cp_async_mbar_arrive_noinc(&full[s % 3]);
             return;
         }
@@ -653,7 +718,12 @@ spmv_f64_kernel(SpmvArgs a, const double* __restrict__ x, double* __restrict__ y
             stage_gather_rle<4>(dbuf, x, a, g, cnt, g + 1 < g1);
         } else {
             if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
-            stage_gather<MX_F64_GATHER_U>(dbuf, x, mp, cnt, a.l2hint);
+            if (MX_F64_ASYNC) {
+                stage_gather_async<(MX_F64_ASYNC > 0 ? MX_F64_ASYNC : 1)>(dbuf, x, mp, cnt, a.l2hint);
+                cp_async_wait_all();
+            } else {
+                stage_gather<MX_F64_GATHER_U>(dbuf, x, mp, cnt, a.l2hint);
+            }
         }
         __syncthreads();
         if (!MX_HEAD_EARLY) h = stage_head(a, g, warp, lane);
@@ -739,6 +809,7 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.dot_part = dot_part;
     a.dot_out = dot_out;
     a.ticket = ticket;
+    a.wave = num_sms();
     // L2 priorities of the stage gather (map evict-first, input evict-last): on by default for
     // the plain / fp64 / SpMM kernels (cfg3 forward 1.694 -> 1.660 ms, back 1.711 -> 1.695 ms,
     // ABAB r02e), off for the drifting-stage kernel (config-5 forward 7.92 -> 8.01 ms);
