@@ -119,8 +119,6 @@ struct SpmvArgs {
     const int64_t* blk_base;
     const int4* blk_rec;
     const int32_t* ovf;
-    int32_t wave;          // CTAs resident at once (one per SM): the launch-order distance to the
-                           // CTA that takes over this SM (MX_NEXT_PREFETCH)
 };
 
 // Partition processed by this CTA: a.order maps launch positions to partitions when a launch
@@ -300,9 +298,6 @@ __device__ __forceinline__ void stage_gather_async(T* __restrict__ buf, const T*
 // 32 gains less (r02ac, profiles/r02ac_async_*.jsonl)
 #ifndef MX_PLAIN_ASYNC
 #define MX_PLAIN_ASYNC 16
-#endif
-#ifndef MX_NEXT_PREFETCH
-#define MX_NEXT_PREFETCH 0
 #endif
 // the same for the fp64 kernel: within noise on the MIXED config-3 CG (r02ac), so synchronous
 #ifndef MX_F64_ASYNC
@@ -516,17 +511,6 @@ spmv_f32_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict__ y, 
             stage_gather_rle<MX_RLE_U>(sbuf, x, a, g, cnt, g + 1 < g1);
         } else {
             if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (s + 1) * a.B), a.l2hint);
-#if MX_NEXT_PREFETCH
-            // last stage: the first-stage map of the CTA launched about one wave later (launch
-            // order ~ partition order) into L2, so that CTA's first gather starts with L2 hits
-            if (threadIdx.x == 32 && g + 1 == g1 && !a.order) {
-                const int64_t q = a.cta_base + blockIdx.x + a.wave;
-                if (q < a.nparts) {
-                    const int64_t mq = a.map_off[q];
-                    prefetch_map_l2(a.map + mq, (int)min((int64_t)a.B, a.map_off[q + 1] - mq), a.l2hint);
-                }
-            }
-#endif
             if (MX_PLAIN_ASYNC) {
                 stage_gather_async<(MX_PLAIN_ASYNC > 0 ? MX_PLAIN_ASYNC : 1)>(sbuf, x, mp, cnt, a.l2hint);
                 cp_async_wait_all();
@@ -809,7 +793,6 @@ SpmvArgs make_args(const Layout& L, double* dot_part, double* dot_out, unsigned 
     a.dot_part = dot_part;
     a.dot_out = dot_out;
     a.ticket = ticket;
-    a.wave = num_sms();
     // L2 priorities of the stage gather (map evict-first, input evict-last): on by default for
     // the plain / fp64 / SpMM kernels (cfg3 forward 1.694 -> 1.660 ms, back 1.711 -> 1.695 ms,
     // ABAB r02e), off for the drifting-stage kernel (config-5 forward 7.92 -> 8.01 ms);
@@ -901,10 +884,33 @@ spmm_f32_kernel(SpmvArgs a, const float* __restrict__ x, int64_t ldx, float* __r
         const int32_t* __restrict__ mp = a.map + m0 + st * a.B;
         if (g != g0) __syncthreads();
         if (threadIdx.x == 0 && g + 1 < g1) prefetch_map_l2(mp + a.B, (int)min((int64_t)a.B, D - (st + 1) * a.B));
-        // 8 input words in flight per thread (16 measured no faster at K = 2/4/8, r01k_spmm_ab.jsonl)
-        constexpr int U = K >= 8 ? 1 : 8 / K;
         const int bd = blockDim.x;
-        for (int i0 = threadIdx.x; i0 < cnt; i0 += U * bd) {
+        // asynchronous gather at K >= 4: UA map entries in flight, each entry's K inputs copied to
+        // the stage buffer by 16 B cp.async pieces of the interleaved input (r02af: K = 8 forward
+        // 3.273 -> 3.205 ms at UA = 4, K = 4 2.002 -> 1.971 ms at UA = 8; at K = 2 the synchronous
+        // gather below is as fast)
+        constexpr int UA = K >= 8 ? 4 : (K == 4 ? 8 : 0);
+        if constexpr (UA > 0) {
+            for (int i0 = threadIdx.x; i0 < cnt; i0 += UA * bd) {
+                int32_t col[UA];
+#pragma unroll
+                for (int u = 0; u < UA; ++u) col[u] = (i0 + u * bd < cnt) ? __ldg(mp + i0 + u * bd) : -1;
+#pragma unroll
+                for (int u = 0; u < UA; ++u) {
+                    if (col[u] < 0) continue;
+                    const int i = i0 + u * bd;
+#pragma unroll
+                    for (int h = 0; h < K / 4; ++h)
+                        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;"
+                                     ::"r"(smem_addr(kbuf + (size_t)K * i + 4 * h)),
+                                     "l"(__cvta_generic_to_global(x + (int64_t)K * col[u] + 4 * h)) : "memory");
+                }
+            }
+            cp_async_wait_all();
+        } else
+        // 8 input words in flight per thread (16 measured no faster at K = 2/4/8, r01k_spmm_ab.jsonl)
+        for (int i0 = threadIdx.x; i0 < cnt; i0 += (K >= 8 ? 1 : 8 / K) * bd) {
+            constexpr int U = K >= 8 ? 1 : 8 / K;
             int64_t col[U];
 #pragma unroll
             for (int u = 0; u < U; ++u) col[u] = (i0 + u * bd < cnt) ? (int64_t)__ldg(mp + i0 + u * bd) : -1;
