@@ -3,6 +3,10 @@
 
 #include <cuda_runtime.h>
 
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
+
 #include <cstdint>
 #include <cstdio>
 #include <stdexcept>
@@ -37,6 +41,19 @@ inline void cuda_check(cudaError_t e, const char* what, const char* file, int li
 void count_launch(int64_t n = 1);
 int64_t launch_count();
 
+// MEMXCT_ALLOC_TRACE=1: report every cudaMalloc / cudaFree slower than 20 ms on stderr
+// (diagnostic of the build-time variance)
+inline std::chrono::steady_clock::time_point trace_clock() { return std::chrono::steady_clock::now(); }
+inline void trace_slow(const char* what, size_t bytes, std::chrono::steady_clock::time_point t0) {
+    static const bool on = [] {
+        const char* e = std::getenv("MEMXCT_ALLOC_TRACE");
+        return e && e[0] == '1';
+    }();
+    if (!on) return;
+    const double ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    if (ms > 20.0) fprintf(stderr, "[memxct] %s(%zu B) %.1f ms\n", what, bytes, ms);
+}
+
 // Owning device allocation (cudaMalloc); freed on destruction, so an OOM in the middle of a
 // build leaves the plan destroyable.
 class DevBuf {
@@ -55,7 +72,9 @@ public:
         reset();
         if (bytes == 0) return;
         void* p = nullptr;
+        const auto t0 = trace_clock();
         cudaError_t e = cudaMalloc(&p, bytes);
+        trace_slow("cudaMalloc", bytes, t0);
         if (e != cudaSuccess) {
             cudaGetLastError();
             fail(e == cudaErrorMemoryAllocation ? MEMXCT_ERR_OUT_OF_MEMORY : MEMXCT_ERR_CUDA,
@@ -66,7 +85,12 @@ public:
         g_bytes_ += bytes;
     }
     void reset() {
-        if (p_) { cudaFree(p_); g_bytes_ -= n_; }
+        if (p_) {
+            const auto t0 = trace_clock();
+            cudaFree(p_);
+            trace_slow("cudaFree", n_, t0);
+            g_bytes_ -= n_;
+        }
         p_ = nullptr;
         n_ = 0;
     }
