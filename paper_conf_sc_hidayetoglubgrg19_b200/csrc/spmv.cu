@@ -613,6 +613,11 @@ __device__ __forceinline__ void stage_gather_rle_async(float* __restrict__ buf, 
 #ifndef MX_DRIFT_ASYNC
 #define MX_DRIFT_ASYNC 1
 #endif
+// map loads of stage s + 2 ahead of the wait for its buffer: config-5 forward 7.588 -> 7.553 ms
+// (r02aj, profiles/r02aj_early_map_cfg5.jsonl)
+#ifndef MX_DRIFT_EARLY_MAP
+#define MX_DRIFT_EARLY_MAP 1
+#endif
 
 template <bool kNatOut, int kEpi>
 __global__ void __launch_bounds__(kMaxThreads, 1)
@@ -666,6 +671,34 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
         __syncwarp();
         if (lane == 0) mbar_arrive(&done[s % 3]);
         if (s + 2 < ns) {
+#if MX_DRIFT_EARLY_MAP
+            // the first 16 map entries of this thread's share of stage s + 2 are loaded BEFORE
+            // waiting for that stage's buffer to be released (the map does not live in it), so
+            // their round trip overlaps the wait; the copies are issued after it
+            if (async_gather && !a.rle) {
+                const int64_t s2 = s + 2;
+                const int cnt = (int)min((int64_t)a.B, D - s2 * a.B);
+                const int32_t* __restrict__ mp = a.map + m0 + s2 * a.B;
+                float* __restrict__ buf = sbuf + (s2 % 3) * a.B;
+                if (MX_DRIFT_PREFETCH && threadIdx.x == 0 && s2 + 2 < ns)
+                    prefetch_map_l2(a.map + m0 + (s2 + 2) * a.B, (int)min((int64_t)a.B, D - (s2 + 2) * a.B), a.l2hint);
+                const int bd = blockDim.x;
+                int32_t j[16];
+#pragma unroll
+                for (int u = 0; u < 16; ++u) {
+                    const int i = threadIdx.x + u * bd;
+                    j[u] = i < cnt ? __ldg(mp + i) : -1;
+                }
+                if (s >= 1) mbar_wait(&done[s2 % 3], (unsigned)(((s - 1) / 3) & 1));
+#pragma unroll
+                for (int u = 0; u < 16; ++u)
+                    if (j[u] >= 0) cp_async_el(buf + threadIdx.x + u * bd, x + j[u]);
+                const int rest = threadIdx.x + 16 * bd;  // stages larger than 16 entries per thread
+                if (rest < cnt) stage_gather_async<16>(buf + 16 * bd, x, mp + 16 * bd, cnt - 16 * bd, a.l2hint);
+                cp_async_mbar_arrive_noinc(&full[s2 % 3]);
+                continue;
+            }
+#endif
             if (s >= 1) mbar_wait(&done[(s + 2) % 3], (unsigned)(((s - 1) / 3) & 1));
             gather(s + 2);
         }
