@@ -618,6 +618,12 @@ __device__ __forceinline__ void stage_gather_rle_async(float* __restrict__ buf, 
 #ifndef MX_DRIFT_EARLY_MAP
 #define MX_DRIFT_EARLY_MAP 1
 #endif
+// the next stage's head (slot offset, chunk count) loaded right after streaming a stage, in
+// flight during the gather and the full wait: config-5 forward 7.574 -> 7.534 ms (r02ak; with the
+// synchronous gather it measured neutral, r02s)
+#ifndef MX_DRIFT_HEAD_EARLY
+#define MX_DRIFT_HEAD_EARLY 1
+#endif
 
 template <bool kNatOut, int kEpi>
 __global__ void __launch_bounds__(kMaxThreads, 1)
@@ -662,14 +668,19 @@ spmv_f32_drift_kernel(SpmvArgs a, const float* __restrict__ x, float* __restrict
     if (ns > 0) gather(0);
     if (ns > 1) gather(1);
     float acc = 0.f;
+    StageHead head;
+    if (MX_DRIFT_HEAD_EARLY && ns > 0) head = stage_head(a, g0, warp, lane);
     for (int64_t s = 0; s < ns; ++s) {
         mbar_wait(&full[s % 3], (unsigned)((s / 3) & 1));
         // test-only: pseudo-random per-warp delays stretch the drift between warps, so the
         // buffer-reuse protocol is exercised at its limits (tests/test_gpu_drift.py)
         if (a.jitter && ((warp * 7 + (int)s) % 5 == 0)) __nanosleep(2000 + 131 * warp);
-        stream_stage(acc, sbuf + (s % 3) * a.B, stage_head(a, g0 + s, warp, lane), a, lane, lt, pol);
+        if (!MX_DRIFT_HEAD_EARLY) head = stage_head(a, g0 + s, warp, lane);
+        stream_stage(acc, sbuf + (s % 3) * a.B, head, a, lane, lt, pol);
         __syncwarp();
         if (lane == 0) mbar_arrive(&done[s % 3]);
+        // the next stage's head, in flight during the gather of stage s + 2 and the full wait
+        if (MX_DRIFT_HEAD_EARLY && s + 1 < ns) head = stage_head(a, g0 + s + 1, warp, lane);
         if (s + 2 < ns) {
 #if MX_DRIFT_EARLY_MAP
             // the first 16 map entries of this thread's share of stage s + 2 are loaded BEFORE
