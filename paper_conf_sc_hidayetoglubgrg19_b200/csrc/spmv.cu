@@ -20,8 +20,6 @@
 
 #include "plan.h"
 
-#include <type_traits>
-
 namespace mx {
 
 namespace {
@@ -410,9 +408,6 @@ __device__ __forceinline__ StageHead stage_head(const SpmvArgs& a, int64_t g, in
 #ifndef MX_HEAD_EARLY
 #define MX_HEAD_EARLY 1
 #endif
-#ifndef MX_REM2
-#define MX_REM2 0
-#endif
 __device__ __forceinline__ void stream_stage(float& acc, const float* __restrict__ sbuf, const StageHead& h,
                                              const SpmvArgs& a, int lane, unsigned lt, uint64_t pol) {
     const int64_t base = h.base;
@@ -423,30 +418,6 @@ __device__ __forceinline__ void stream_stage(float& acc, const float* __restrict
     const int minc = __reduce_min_sync(0xffffffffu, nch);
     // phase 1: chunks every lane has -- plain SELL addressing, branch-free, unrolled so
     // several 16 B loads per lane are in flight
-#if MX_REM2
-    // groups of 4 chunks, then one group of 2 and one single: the remainder (< 4 chunks) with at
-    // most two round trips instead of up to three one-chunk iterations
-    auto group = [&](int c, auto kn) {
-        constexpr int N = decltype(kn)::value;
-        uint4 iv[N];
-        float4 v0[N], v1[N];
-#pragma unroll
-        for (int k = 0; k < N; ++k) {
-            iv[k] = ld_stream_u4(ib + (c + k) * 32 + lane, pol);
-            v0[k] = ld_stream_f4(vb + (c + k) * 64 + lane, pol);
-            v1[k] = ld_stream_f4(vb + (c + k) * 64 + 32 + lane, pol);
-        }
-#pragma unroll
-        for (int k = 0; k < N; ++k) fma8(acc, sbuf, iv[k], v0[k], v1[k]);
-    };
-    int c1 = 0;
-    for (; c1 + 4 <= minc; c1 += 4) group(c1, std::integral_constant<int, 4>{});
-    if (c1 + 2 <= minc) {
-        group(c1, std::integral_constant<int, 2>{});
-        c1 += 2;
-    }
-    if (c1 < minc) group(c1, std::integral_constant<int, 1>{});
-#else
 #pragma unroll 4
     for (int c = 0; c < minc; ++c) {
         const uint4 iv = ld_stream_u4(ib + c * 32 + lane, pol);
@@ -454,7 +425,6 @@ __device__ __forceinline__ void stream_stage(float& acc, const float* __restrict
         const float4 v1 = ld_stream_f4(vb + c * 64 + 32 + lane, pol);
         fma8(acc, sbuf, iv, v0, v1);
     }
-#endif
     // phase 2: the ragged tail, stored only for the lanes that have it (jagged SELL)
     int64_t pref = (int64_t)minc * 32;
     for (int c = minc; c < maxc; ++c) {
