@@ -295,7 +295,7 @@ __device__ __forceinline__ void stage_gather_async(T* __restrict__ buf, const T*
 }
 // entries per thread in flight of the plain kernel's asynchronous gather (0 = the synchronous
 // stage_gather): config-3 SpMV 1.650 / 1.686 -> 1.640 / 1.677 ms, config 4 -0.2 / -0.6 % at 16;
-// 32 gains less (r02ac, profiles/r02ac_async_*.jsonl)
+// 32 gains less (r02ac, profiles/r02ac_async_*.jsonl), 8 is neutral (r02an)
 #ifndef MX_PLAIN_ASYNC
 #define MX_PLAIN_ASYNC 16
 #endif
