@@ -631,9 +631,14 @@ static bool drift_requested() {
     const char* e = std::getenv("MEMXCT_DRIFT");
     return e && atoi(e) != 0;
 }
+// Three buffers of 13312 entries (156 KB) are the largest that keep the shared-memory carve-out
+// at 164 KB and so 92 KB of L1 for the stream's loads in flight; 16384 (192 KB) selects the 196 KB
+// carve-out and leaves 60 KB.  Config-5 shard forward (asynchronous gather): 7.54 ms at 16384,
+// 7.42 at 13312, 7.48 at 12288 although the smaller stages raise the slab padding 3.8 -> 4.7 %
+// (r02aw, profiles/r02aw_drift_b_cfg5.jsonl; with the synchronous gather 16384 was best, r01i).
 static int32_t drift_auto_b() {
     const char* e = std::getenv("MEMXCT_DRIFT_B");
-    return e ? std::max(256, atoi(e)) : 16384;
+    return e ? std::max(256, atoi(e)) : 13312;
 }
 
 void resolve_tuning(const Plan& P, int64_t rows, int32_t* R_out, int32_t* B_out) {
@@ -1007,7 +1012,7 @@ void build_matrices(Plan& P, cudaStream_t st) {
     // footprint's Hilbert order; the A_p^T build below keeps the footprint order for its columns
     P.ray_block = resolve_ray_block(P, npix, R);
     // drifting stages (spmv_f32_drift_kernel) for the forward operator of projection-block plans:
-    // three stage buffers of 16384 entries instead of one of 36 R.  Config-5 shard forward 7.99 ->
+    // three stage buffers of 13312 entries (16384 until r02aw) instead of one of 36 R.  Config-5 shard forward 7.99 ->
     // 7.73 ms although the smaller stages add 2.2 % slab padding; the balanced back operator and
     // the Hilbert-row geometries (configs 1-4) gain nothing and keep the plain kernel
     // (profiles/r01i_drift_*.jsonl).  MEMXCT_DRIFT=1 forces it for both directions.
